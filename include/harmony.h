@@ -1,0 +1,205 @@
+/*
+ * harmony.h — C ABI of the B200-native Harmony-DP training step.
+ *
+ * Method: Li, Phanishayee, Murray, Kim, "Doing more with less: Training large
+ * DNN models on commodity servers for the masses", HotOS '21.
+ * Citations "P:a-b" are PAPER.md lines.  The interface follows the paper's
+ * problem statement: the user targets "a single virtual accelerator device with
+ * practically unbounded memory", supplies a model "as if running
+ * sequentially on a single device", a parallelization scheme,
+ * the hardware configuration and a mini-batch size.
+ * Behind these calls the library decomposes the step into per-layer x
+ * per-microbatch forward / backward / update tasks,
+ * late-binds them to streams and HBM slots under a per-GPU memory cap, swaps
+ * state and activations to pinned host RAM, groups
+ * microbatches, runs each layer's update just in time,
+ * and inserts collectives to keep the result that of the plain single-device
+ * step.
+ *
+ * Process model: ONE process per GPU (rank r of world_size).  Every rank calls
+ * the same functions in the same order; collectives (NCCL, loaded with dlopen)
+ * run inside harmony_step / harmony_read_state.
+ *
+ * Conventions for every call:
+ *  - Status codes only; no exception or abort crosses the ABI.  On failure
+ *    harmony_last_error(ctx) returns a NUL-terminated message.  A CUDA or NCCL
+ *    error is sticky: afterwards only harmony_finalize is valid.
+ *  - Pointer arguments are caller-owned and only read/written during the call
+ *    (the library copies what it keeps into its own pinned host store).
+ *  - Buffers may be HOST or DEVICE pointers wherever "host or device" is said;
+ *    the library detects which with cudaPointerGetAttributes.
+ *  - A context is not thread-safe.
+ *  - Row-major everywhere.  Linear weights are W[d_in][d_out], Y = X.W + b.
+ *
+ * Parameter packing (per layer, fp32, canonical order):
+ *  HARMONY_LAYER_MLP:          W[d_in][d_out], b[d_out]
+ *  HARMONY_LAYER_TRANSFORMER:  ln1_g[d], ln1_b[d], W_qkv[d][3d], b_qkv[3d],
+ *     W_o[d][d], b_o[d], ln2_g[d], ln2_b[d], W_fc1[d][4d], b_fc1[4d],
+ *     W_fc2[4d][d], b_fc2[d]            (12 d^2 + 13 d floats; QKV columns are
+ *     [Q | K | V], head h owning columns h*dh .. h*dh+dh-1 of each third).
+ *  The transformer layer is a pre-LN block (reading c1):
+ *     U=LN1(X); QKV=U W_qkv+b_qkv; C=MHA(QKV) (causal optional);
+ *     X2=X+C W_o+b_o; U2=LN2(X2); H=U2 W_fc1+b_fc1; Y=X2+GeLU_tanh(H) W_fc2+b_fc2.
+ *  Loss (reading c2): L = (1/B) sum_b 1/2 ||Y_b - T_b||^2 over the GLOBAL batch B.
+ *  Optimizer (reading c3): Adam [30] with bias correction, t from 1.
+ */
+#ifndef HARMONY_H_
+#define HARMONY_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HARMONY_ABI_VERSION 1
+
+typedef struct harmony_ctx harmony_ctx; /* opaque; owns all device and pinned memory */
+
+typedef enum {
+  HARMONY_OK = 0,
+  HARMONY_E_INVALID_ARG = 1,   /* bad sizes, NULL where required, batch != m*b          */
+  HARMONY_E_BAD_STATE = 2,     /* calls out of order (e.g. step before register_layers)  */
+  HARMONY_E_CAP_TOO_SMALL = 3, /* minimum working set exceeds hbm_cap_bytes               */
+  HARMONY_E_HOST_OOM = 4,      /* pinned host allocation failed                           */
+  HARMONY_E_CUDA = 5,          /* CUDA runtime / driver error (sticky)                    */
+  HARMONY_E_NCCL = 6,          /* NCCL missing or failed (sticky)                         */
+  HARMONY_E_UNSUPPORTED = 7    /* valid request the build does not support (e.g. d%8!=0 on bf16) */
+} harmony_status;
+
+typedef enum { HARMONY_FP32 = 0, HARMONY_BF16_FP32MASTER = 1 } harmony_precision;
+typedef enum { HARMONY_LAYER_MLP = 0, HARMONY_LAYER_TRANSFORMER = 1 } harmony_layer_kind;
+typedef enum { HARMONY_ACT_NONE = 0, HARMONY_ACT_RELU = 1, HARMONY_ACT_GELU_TANH = 2 } harmony_act;
+typedef enum { HARMONY_PARAM = 0, HARMONY_GRAD = 1, HARMONY_ADAM_M = 2, HARMONY_ADAM_V = 3 } harmony_state_kind;
+
+/* Schedules.  HARMONY_SCHED_HARMONY_DP is the paper's Harmony-DP (input-batch
+ * grouping P:537-548 + JIT update P:549-553 + p2p weight shards P:738-748).
+ * HARMONY_SCHED_PER_GPU_VIRT is the baseline the paper compares against
+ * (per-GPU memory virtualization, Fig. 5(b)): each microbatch swaps
+ * the weights in and out for its own forward and backward, and the update runs
+ * after the whole backward.  Both compute the identical result. */
+typedef enum { HARMONY_SCHED_HARMONY_DP = 0, HARMONY_SCHED_PER_GPU_VIRT = 1 } harmony_schedule;
+
+typedef struct {
+  uint32_t struct_size;      /* = sizeof(harmony_config) (ABI versioning)                   */
+  int32_t rank;              /* this process's rank in the data-parallel group, 0..world-1   */
+  int32_t world_size;        /* N GPUs (one process each); 1 = no collectives                */
+  int32_t device;            /* CUDA device ordinal used by this process                     */
+  uint64_t hbm_cap_bytes;    /* per-GPU arena budget in bytes; 0 = uncapped (all resident)   */
+  void* arena;               /* optional caller-owned DEVICE buffer of hbm_cap_bytes (e.g. a
+                                torch tensor); NULL = the library allocates the arena itself */
+  int32_t microbatches;      /* m microbatches per rank per step (the input-batch group)     */
+  int32_t microbatch_size;   /* b samples per microbatch; local batch = m*b, global = N*m*b  */
+  int32_t precision;         /* harmony_precision                                            */
+  int32_t schedule;          /* harmony_schedule                                             */
+  int32_t retain_grads;      /* 1 = keep the last reduced gradients readable (HARMONY_GRAD)  */
+  int32_t stash_policy;      /* 0 = stash every op input (36d+2hS+16 B/token/block);
+                                1 = recompute elementwise outputs (LN outputs, GeLU) in the
+                                backward (24d+2hS+16 B/token/block)                          */
+  float lr, beta1, beta2, eps, weight_decay; /* Adam; weight_decay must be 0 (reading c3)    */
+  uint8_t nccl_id[128];      /* ncclUniqueId from harmony_get_unique_id() on rank 0, broadcast
+                                to all ranks by the caller (ignored when world_size == 1)    */
+} harmony_config;
+
+typedef struct {
+  int32_t kind;      /* harmony_layer_kind                                            */
+  int32_t d_in;      /* input width (transformer: d)                                  */
+  int32_t d_out;     /* output width (transformer: must equal d_in)                   */
+  int32_t n_heads;   /* transformer heads h (d % h == 0)                              */
+  int32_t seq_len;   /* transformer sequence length S (MLP: 1)                        */
+  int32_t causal;    /* transformer: 1 = causal mask                                  */
+  int32_t act;       /* MLP activation (harmony_act)                                  */
+} harmony_layer_desc;
+
+/* Per-step statistics of THIS rank (the copy ledger).  Bytes are what
+ * was actually issued to the copy engines / NCCL during the last step. */
+typedef struct {
+  uint64_t h2d_bytes, d2h_bytes;               /* all host<->device copies            */
+  uint64_t h2d_weight_bytes, d2h_weight_bytes; /* compute-copy weights W (Fig. 5)     */
+  uint64_t h2d_state_bytes, d2h_state_bytes;   /* fp32 master W, Adam m, v (K) */
+  uint64_t h2d_stash_bytes, d2h_stash_bytes;   /* stashed activations    */
+  uint64_t h2d_input_bytes, d2h_output_bytes;  /* X, T in; loss out                   */
+  uint64_t h2d_grad_bytes, d2h_grad_bytes;     /* dW crossing PCIe (Harmony-DP: 0)     */
+  uint64_t nvlink_bytes;                        /* bytes this rank sent through NCCL   */
+  uint64_t peak_arena_bytes;                    /* arena bytes the plan uses           */
+  uint64_t kernel_launches;                     /* kernels launched in the step        */
+  uint64_t n_ops;                               /* ops in the static program           */
+  double step_seconds;                          /* device time of the step (CUDA events)*/
+} harmony_step_stats;
+
+/* Static plan summary (host-only; also available without a GPU via harmony_plan_dry). */
+typedef struct {
+  uint64_t arena_bytes;            /* bytes of arena the plan lays out                   */
+  uint64_t min_working_set_bytes;  /* smallest cap this model/batch can run under        */
+  uint64_t resident_weight_bytes, total_weight_bytes;  /* compute copies                 */
+  uint64_t resident_state_bytes, total_state_bytes;    /* master+m+v shards of this rank */
+  uint64_t resident_stash_bytes, total_stash_bytes;    /* per step                       */
+  uint64_t pred_h2d_bytes, pred_d2h_bytes;             /* per step, this rank            */
+  uint64_t pred_h2d_weight_bytes, pred_d2h_weight_bytes;
+  uint64_t flops_per_step;         /* algorithmic GEMM FLOPs of this rank's step         */
+  int64_t n_params;                /* model parameters                                   */
+  int32_t n_ops, n_compute_ops, n_copy_ops, n_comm_ops;
+  int32_t weight_slots, stash_slots, state_slots;
+  int32_t hazards;                 /* conflicting accesses the independent byte-range validator
+                                      found in the program (must be 0; register refuses otherwise) */
+} harmony_plan_summary;
+
+/* sizeof of the ABI structs as the library was compiled: harmony_config, harmony_layer_desc,
+ * harmony_step_stats, harmony_plan_summary, hk_gemm_args (bindings check their mirrors). */
+void harmony_abi_sizes(uint64_t out[5]);
+
+/* Writes an ncclUniqueId (128 bytes) into out.  Call on rank 0 only, then broadcast. */
+harmony_status harmony_get_unique_id(uint8_t out[128]);
+
+/* Validates cfg, selects cfg->device, creates streams/events, allocates (or adopts)
+ * the arena and, for world_size > 1, the NCCL communicator.  *out owns everything. */
+harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out);
+
+/* Registers the layer stack and its initial fp32 parameters (canonical packing, one
+ * host array per layer, identical on every rank).  Decomposes the step into tasks,
+ * plans residency / slots / swap sets / the per-stream program, and fills the pinned
+ * host store (this rank's shard of master W, m = v = 0, and of the compute copy).
+ * Returns HARMONY_E_CAP_TOO_SMALL when the minimum working set exceeds the cap.
+ * Weight tying is impossible by construction (each layer owns its parameters;
+ * reading c4: no weight is read after its own backward, so JIT updates are exact). */
+harmony_status harmony_register_layers(harmony_ctx* ctx, int32_t n_layers, const harmony_layer_desc* descs,
+                                       const float* const* init_params);
+
+/* One training step on this rank's local batch of m*b samples.
+ *  x:      host or device fp32 [m*b, S, d_in] (MLP: [m*b, d_in]), this rank's rows of
+ *          the global batch (rank r holds global rows r*m*b .. (r+1)*m*b-1, reading c14)
+ *  target: host or device fp32, the output shape
+ *  batch:  must equal m*b
+ *  loss_out (nullable): the GLOBAL loss (rank partials summed in rank order, c22)
+ *  stats (nullable): this rank's ledger for the step
+ * Synchronous: returns when the update of every layer has finished on this GPU. */
+harmony_status harmony_step(harmony_ctx* ctx, const float* x, const float* target, int64_t batch, double* loss_out,
+                            harmony_step_stats* stats);
+
+/* Reads one fp32 state tensor of `layer` (n_floats = the layer's parameter count) into
+ * the host buffer dst.  HARMONY_GRAD needs retain_grads.  For world_size > 1 this is a
+ * collective (all ranks must call it with the same arguments). */
+harmony_status harmony_read_state(harmony_ctx* ctx, int32_t layer, int32_t which, float* dst, uint64_t n_floats);
+
+harmony_status harmony_read_stats(const harmony_ctx* ctx, harmony_step_stats* out);
+harmony_status harmony_plan_info(const harmony_ctx* ctx, harmony_plan_summary* out);
+
+/* Host-only planning (no CUDA call): what register_layers would plan for this
+ * config.  program_text (nullable) receives a textual dump of the per-stream program
+ * (truncated to text_len bytes).  Used by the CPU tests of the scheduler. */
+harmony_status harmony_plan_dry(const harmony_config* cfg, int32_t n_layers, const harmony_layer_desc* descs,
+                                harmony_plan_summary* out, char* program_text, uint64_t text_len);
+
+/* Frees every device and pinned allocation and the communicator; ctx is invalid after. */
+harmony_status harmony_finalize(harmony_ctx* ctx);
+
+/* Last error message of ctx (or of the last failed context-less call when ctx is NULL). */
+const char* harmony_last_error(const harmony_ctx* ctx);
+
+int32_t harmony_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HARMONY_H_ */

@@ -1,0 +1,85 @@
+// common.hpp — shared helpers of libharmony (error plumbing, bf16 conversion, launch helpers).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <cmath>
+#include <string>
+
+#include "harmony.h"
+
+namespace hm {
+
+// Thread-local message of the last failure of a context-less call (kernel ABI).
+void set_global_error(const std::string& msg);
+const char* global_error();
+
+struct Error {
+  harmony_status code;
+  std::string msg;
+};
+
+#define HM_CUDA(expr)                                                                                   \
+  do {                                                                                                  \
+    cudaError_t _e = (expr);                                                                            \
+    if (_e != cudaSuccess) {                                                                            \
+      throw ::hm::Error{HARMONY_E_CUDA, std::string(#expr) + " -> " + cudaGetErrorString(_e) + " at " + \
+                                           __FILE__ + ":" + std::to_string(__LINE__)};                  \
+    }                                                                                                   \
+  } while (0)
+
+#define HM_CHECK(cond, code, msg)                                  \
+  do {                                                             \
+    if (!(cond)) throw ::hm::Error{(code), std::string(msg)};      \
+  } while (0)
+
+// Kernel launch accounting (the ledger counts the kernels a step launches).
+extern thread_local uint64_t g_kernel_launches;
+inline void count_launch() { ++g_kernel_launches; }
+
+inline void check_launch(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) throw Error{HARMONY_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e)};
+  count_launch();
+}
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+// Activation types of the step: fp32 path stores T = float, bf16 path T = __nv_bfloat16.
+template <typename T> struct TypeTag;
+template <> struct TypeTag<float> { static constexpr int id = 0; };
+template <> struct TypeTag<__nv_bfloat16> { static constexpr int id = 1; };
+
+__device__ __forceinline__ float to_f32(float x) { return x; }
+__device__ __forceinline__ float to_f32(__nv_bfloat16 x) { return __bfloat162float(x); }
+template <typename T> __device__ __forceinline__ T from_f32(float x);
+template <> __device__ __forceinline__ float from_f32<float>(float x) { return x; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f32<__nv_bfloat16>(float x) { return __float2bfloat16_rn(x); }
+
+// GeLU (tanh approximation, reading c12) and its derivative, fp32.
+__device__ __forceinline__ float gelu_tanh_f(float x) {
+  const float c = 0.7978845608028654f, a = 0.044715f;
+  float u = c * (x + a * x * x * x);
+  return 0.5f * x * (1.0f + tanhf(u));
+}
+__device__ __forceinline__ float gelu_tanh_grad_f(float x) {
+  const float c = 0.7978845608028654f, a = 0.044715f;
+  float u = c * (x + a * x * x * x);
+  float t = tanhf(u);
+  return 0.5f * (1.0f + t) + 0.5f * x * (1.0f - t * t) * c * (1.0f + 3.0f * a * x * x);
+}
+__device__ __forceinline__ float act_f(int act, float z) {
+  if (act == HARMONY_ACT_RELU) return z > 0.f ? z : 0.f;
+  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_f(z);
+  return z;
+}
+__device__ __forceinline__ float act_grad_f(int act, float z) {
+  if (act == HARMONY_ACT_RELU) return z > 0.f ? 1.f : 0.f;
+  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_grad_f(z);
+  return 1.f;
+}
+
+}  // namespace hm

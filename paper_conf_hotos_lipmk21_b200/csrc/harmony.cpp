@@ -1,0 +1,496 @@
+// harmony.cpp — runtime and C ABI of libharmony (include/harmony.h).
+//
+// Runtime pieces: the capped device arena (one block, laid out by the planner),
+// the pinned host store (this rank's shards of the fp32 master W, Adam m and v, the compute copy
+// of W, and the spilled activation stash), four CUDA streams {compute, h2d, d2h, comm} with the
+// plan's events, the NCCL communicator, and the copy ledger (bytes per tensor class, per step).
+// The executor replays the static program of plan.cpp every step: for each op it waits on the
+// events of its cross-stream dependencies, issues the op on its stream, and records its event.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "comm.hpp"
+#include "harmony_kernels.h"
+#include "common.hpp"
+#include "kernels/kernels.hpp"
+#include "layers.hpp"
+#include "plan.hpp"
+
+namespace hm {
+thread_local uint64_t g_kernel_launches = 0;
+static thread_local std::string g_err;
+void set_global_error(const std::string& msg) { g_err = msg; }
+const char* global_error() { return g_err.c_str(); }
+
+static inline uint16_t f32_to_bf16_rne(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  if ((u & 0x7F800000u) == 0x7F800000u) return (uint16_t)((u >> 16) | ((u & 0xFFFF) ? 0x40 : 0));  // inf / nan
+  return (uint16_t)((u + 0x7FFFu + ((u >> 16) & 1u)) >> 16);
+}
+}  // namespace hm
+
+using namespace hm;
+
+struct harmony_ctx {
+  harmony_config cfg{};
+  std::string err;
+  bool broken = false;
+  cudaStream_t st[S_NUM] = {};
+  std::vector<cudaEvent_t> events;
+  cudaEvent_t ev_begin = nullptr, ev_end[S_NUM] = {};
+  uint8_t* arena = nullptr;
+  bool own_arena = false;
+  ncclComm_t comm = nullptr;
+  bool registered = false;
+  Plan plan;
+  std::vector<uint8_t*> h_wc;     // per layer: compute-copy shard (T)
+  std::vector<float*> h_state;    // per layer: [master | m | v] shard
+  std::vector<uint8_t*> h_stash;  // per (layer, microbatch): spilled stash, nullptr if resident
+  std::vector<float*> h_grad;     // retain_grads: reduced gradient shard
+  double* h_loss = nullptr;
+  int t = 0;
+  harmony_step_stats last{};
+};
+
+namespace {
+
+void free_host(void* p) {
+  if (p) cudaFreeHost(p);
+}
+
+void* alloc_host(size_t bytes) {
+  void* p = nullptr;
+  cudaError_t e = cudaHostAlloc(&p, std::max<size_t>(bytes, 64), cudaHostAllocPortable);
+  if (e != cudaSuccess) throw Error{HARMONY_E_HOST_OOM, std::string("cudaHostAlloc(") + std::to_string(bytes) +
+                                                            ") failed: " + cudaGetErrorString(e)};
+  return p;
+}
+
+void check_nccl(ncclResult_t r, const char* what) {
+  if (r != ncclSuccess)
+    throw Error{HARMONY_E_NCCL, std::string(what) + ": " + (nccl().GetErrorString ? nccl().GetErrorString(r) : "?")};
+}
+
+harmony_status fail(harmony_ctx* ctx, const Error& e) {
+  if (ctx) {
+    ctx->err = e.msg;
+    if (e.code == HARMONY_E_CUDA || e.code == HARMONY_E_NCCL) ctx->broken = true;
+  }
+  set_global_error(e.msg);
+  return e.code;
+}
+
+#define HM_API_BEGIN try {
+#define HM_API_END(ctx)                                               \
+  }                                                                   \
+  catch (const Error& e) {                                            \
+    return fail(ctx, e);                                              \
+  }                                                                   \
+  catch (const std::exception& e) {                                   \
+    return fail(ctx, Error{HARMONY_E_INVALID_ARG, e.what()});         \
+  }                                                                   \
+  return HARMONY_OK;
+
+void destroy(harmony_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->cfg.device);
+  for (int s = 0; s < S_NUM; ++s)
+    if (c->st[s]) cudaStreamSynchronize(c->st[s]);
+  for (auto e : c->events) cudaEventDestroy(e);
+  if (c->ev_begin) cudaEventDestroy(c->ev_begin);
+  for (int s = 0; s < S_NUM; ++s) {
+    if (c->ev_end[s]) cudaEventDestroy(c->ev_end[s]);
+    if (c->st[s]) cudaStreamDestroy(c->st[s]);
+  }
+  if (c->comm && nccl().CommDestroy) nccl().CommDestroy(c->comm);
+  if (c->own_arena && c->arena) cudaFree(c->arena);
+  for (auto p : c->h_wc) free_host(p);
+  for (auto p : c->h_state) free_host(p);
+  for (auto p : c->h_stash) free_host(p);
+  for (auto p : c->h_grad) free_host(p);
+  free_host(c->h_loss);
+  delete c;
+}
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// ---------------------------------------------------------------------------------------- executor
+void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out, harmony_step_stats* out) {
+  Plan& p = c->plan;
+  uint8_t* A = c->arena;
+  const int dt = p.dtype;
+  harmony_step_stats s{};
+  s.n_ops = p.ops.size();
+  s.peak_arena_bytes = p.arena_bytes;
+  g_kernel_launches = 0;
+  c->t += 1;
+  const bool x_dev = is_device_ptr(x), t_dev = is_device_ptr(tg);
+  const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
+
+  HM_CUDA(cudaEventRecord(c->ev_begin, c->st[S_COMPUTE]));
+  for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_begin, 0));
+
+  for (size_t oi = 0; oi < p.ops.size(); ++oi) {
+    const Op& o = p.ops[oi];
+    cudaStream_t st = c->st[o.stream];
+    for (int w : o.waits) HM_CUDA(cudaStreamWaitEvent(st, c->events[p.ops[w].event], 0));
+    switch (o.kind) {
+      case OP_INPUT: {
+        const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)x : (const void*)tg);
+        const bool dev = o.hbuf == HB_USER_X ? x_dev : t_dev;
+        HM_CUDA(cudaMemcpyAsync(A + o.dev, src + o.hoff, o.bytes, cudaMemcpyDefault, st));
+        if (!dev) { s.h2d_bytes += o.bytes; s.h2d_input_bytes += o.bytes; }
+        break;
+      }
+      case OP_H2D:
+      case OP_D2H: {
+        uint8_t* h = nullptr;
+        switch (o.hbuf) {
+          case HB_WC: h = c->h_wc[o.hidx]; break;
+          case HB_STATE: h = reinterpret_cast<uint8_t*>(c->h_state[o.hidx]); break;
+          case HB_STASH: h = c->h_stash[o.hidx]; break;
+          case HB_GRAD: h = reinterpret_cast<uint8_t*>(c->h_grad[o.hidx]); break;
+          default: throw Error{HARMONY_E_INVALID_ARG, "bad host buffer in plan"};
+        }
+        h += o.hoff;
+        if (o.kind == OP_H2D) {
+          HM_CUDA(cudaMemcpyAsync(A + o.dev, h, o.bytes, cudaMemcpyHostToDevice, st));
+          s.h2d_bytes += o.bytes;
+          if (o.cat == CAT_WEIGHT) s.h2d_weight_bytes += o.bytes;
+          else if (o.cat == CAT_STATE) s.h2d_state_bytes += o.bytes;
+          else if (o.cat == CAT_STASH) s.h2d_stash_bytes += o.bytes;
+          else if (o.cat == CAT_GRAD) s.h2d_grad_bytes += o.bytes;
+        } else {
+          HM_CUDA(cudaMemcpyAsync(h, A + o.dev, o.bytes, cudaMemcpyDeviceToHost, st));
+          s.d2h_bytes += o.bytes;
+          if (o.cat == CAT_WEIGHT) s.d2h_weight_bytes += o.bytes;
+          else if (o.cat == CAT_STATE) s.d2h_state_bytes += o.bytes;
+          else if (o.cat == CAT_STASH) s.d2h_stash_bytes += o.bytes;
+          else if (o.cat == CAT_GRAD) s.d2h_grad_bytes += o.bytes;
+        }
+        break;
+      }
+      case OP_FWD: {
+        const LayerPlan& lp = p.layers[o.layer];
+        layer_fwd(lp.g, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
+                  A + o.stash, A + o.ws, st);
+        break;
+      }
+      case OP_LOSS: {
+        mse(p.out_elems_per_mb, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<const float*>(A + o.tgt),
+            inv_batch, reinterpret_cast<float*>(A + o.out), reinterpret_cast<double*>(A + o.loss),
+            reinterpret_cast<double*>(A + p.loss_scratch), st);
+        break;
+      }
+      case OP_BWD: {
+        const LayerPlan& lp = p.layers[o.layer];
+        layer_bwd(lp.g, A + o.w, A + o.stash, reinterpret_cast<const float*>(A + o.in),
+                  reinterpret_cast<float*>(A + o.out), reinterpret_cast<float*>(A + o.dw), o.first, A + o.ws, st);
+        break;
+      }
+      case OP_UPD: {
+        const LayerPlan& lp = p.layers[o.layer];
+        float* state = reinterpret_cast<float*>(A + o.state);
+        const uint64_t sh = (uint64_t)lp.shard;
+        uint8_t* wc = A + o.w + (uint64_t)p.rank * sh * (dt ? 2 : 4);
+        adam(dt, (int64_t)sh, state, state + sh, state + 2 * sh, reinterpret_cast<const float*>(A + o.grad), wc,
+             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->t, st);
+        break;
+      }
+      case OP_ALLGATHER: {
+        const size_t esz = dt ? 2 : 4;
+        uint8_t* buf = A + o.dev;
+        check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * esz, buf, o.count, dt ? ncclBfloat16 : ncclFloat32,
+                                    c->comm, st),
+                   "ncclAllGather");
+        s.nvlink_bytes += o.bytes;
+        break;
+      }
+      case OP_REDUCESCATTER: {
+        check_nccl(nccl().ReduceScatter(A + o.dev, A + o.grad, o.count, ncclFloat32, ncclSum, c->comm, st),
+                   "ncclReduceScatter");
+        s.nvlink_bytes += o.bytes;
+        break;
+      }
+      case OP_LOSS_GATHER: {
+        uint8_t* buf = A + o.dev;
+        check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * 8, buf, o.count, ncclFloat64, c->comm, st),
+                   "ncclAllGather(loss)");
+        s.nvlink_bytes += o.bytes;
+        break;
+      }
+      case OP_LOSS_OUT: {
+        uint8_t* dst = reinterpret_cast<uint8_t*>(c->h_loss) + (p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8);
+        HM_CUDA(cudaMemcpyAsync(dst, A + o.dev + (p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8), o.bytes,
+                                cudaMemcpyDeviceToHost, st));
+        s.d2h_bytes += o.bytes;
+        s.d2h_output_bytes += o.bytes;
+        break;
+      }
+      default:
+        throw Error{HARMONY_E_INVALID_ARG, "unknown op kind in plan"};
+    }
+    if (o.event >= 0) HM_CUDA(cudaEventRecord(c->events[o.event], st));
+  }
+  for (int k = 0; k < S_NUM; ++k) HM_CUDA(cudaEventRecord(c->ev_end[k], c->st[k]));
+  float ms = 0.f;
+  for (int k = 0; k < S_NUM; ++k) {
+    HM_CUDA(cudaEventSynchronize(c->ev_end[k]));
+    float e = 0.f;
+    HM_CUDA(cudaEventElapsedTime(&e, c->ev_begin, c->ev_end[k]));
+    ms = std::max(ms, e);
+  }
+  HM_CUDA(cudaGetLastError());
+  double loss = 0.0;  // rank partials summed in rank order, microbatches in order (reading c22)
+  for (int r = 0; r < p.N; ++r)
+    for (int i = 0; i < p.m; ++i) loss += c->h_loss[r * p.m + i];
+  if (loss_out) *loss_out = loss;
+  s.step_seconds = ms * 1e-3;
+  s.kernel_launches = g_kernel_launches;
+  c->last = s;
+  if (out) *out = s;
+}
+
+}  // namespace
+
+// ============================================================================================ C ABI
+extern "C" {
+
+int32_t harmony_abi_version(void) { return HARMONY_ABI_VERSION; }
+
+void harmony_abi_sizes(uint64_t out[5]) {
+  out[0] = sizeof(harmony_config);
+  out[1] = sizeof(harmony_layer_desc);
+  out[2] = sizeof(harmony_step_stats);
+  out[3] = sizeof(harmony_plan_summary);
+  out[4] = sizeof(hk_gemm_args);
+}
+
+const char* harmony_last_error(const harmony_ctx* ctx) { return ctx ? ctx->err.c_str() : global_error(); }
+
+harmony_status harmony_get_unique_id(uint8_t out[128]) {
+  HM_API_BEGIN
+  HM_CHECK(out != nullptr, HARMONY_E_INVALID_ARG, "out is NULL");
+  HM_CHECK(nccl().load(), HARMONY_E_NCCL, nccl().err);
+  ncclUniqueId id;
+  check_nccl(nccl().GetUniqueId(&id), "ncclGetUniqueId");
+  static_assert(sizeof(id) == 128, "ncclUniqueId size");
+  memcpy(out, &id, 128);
+  HM_API_END(nullptr)
+}
+
+harmony_status harmony_plan_dry(const harmony_config* cfg, int32_t n_layers, const harmony_layer_desc* descs,
+                                harmony_plan_summary* out, char* text, uint64_t text_len) {
+  HM_API_BEGIN
+  HM_CHECK(cfg && descs && out, HARMONY_E_INVALID_ARG, "NULL argument");
+  Plan p = make_plan(*cfg, n_layers, descs);
+  *out = p.summary;
+  if (text && text_len > 0) {
+    std::string d = dump_plan(p);
+    size_t n = std::min<size_t>(d.size(), text_len - 1);
+    memcpy(text, d.data(), n);
+    text[n] = 0;
+  }
+  HM_API_END(nullptr)
+}
+
+harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
+  harmony_ctx* c = nullptr;
+  HM_API_BEGIN
+  HM_CHECK(cfg && out, HARMONY_E_INVALID_ARG, "NULL argument");
+  *out = nullptr;
+  validate_config(*cfg);
+  c = new harmony_ctx();
+  c->cfg = *cfg;
+  int ndev = 0;
+  HM_CUDA(cudaGetDeviceCount(&ndev));
+  HM_CHECK(cfg->device >= 0 && cfg->device < ndev, HARMONY_E_INVALID_ARG, "device ordinal out of range");
+  HM_CUDA(cudaSetDevice(cfg->device));
+  cudaDeviceProp prop;
+  HM_CUDA(cudaGetDeviceProperties(&prop, cfg->device));
+  HM_CHECK(prop.major == 10, HARMONY_E_UNSUPPORTED,
+           std::string("libharmony is built for sm_100a (B200); device is ") + prop.name);
+  for (int s = 0; s < S_NUM; ++s) {
+    HM_CUDA(cudaStreamCreateWithFlags(&c->st[s], cudaStreamNonBlocking));
+    HM_CUDA(cudaEventCreate(&c->ev_end[s]));
+  }
+  HM_CUDA(cudaEventCreate(&c->ev_begin));
+  if (cfg->arena) {
+    HM_CHECK(cfg->hbm_cap_bytes > 0, HARMONY_E_INVALID_ARG, "an adopted arena needs hbm_cap_bytes");
+    HM_CHECK(is_device_ptr(cfg->arena), HARMONY_E_INVALID_ARG, "cfg.arena is not a device pointer");
+    HM_CHECK(reinterpret_cast<uintptr_t>(cfg->arena) % 1024 == 0, HARMONY_E_INVALID_ARG, "cfg.arena must be 1 KiB aligned");
+    c->arena = static_cast<uint8_t*>(cfg->arena);
+  }
+  if (cfg->world_size > 1) {
+    HM_CHECK(nccl().load(), HARMONY_E_NCCL, nccl().err);
+    ncclUniqueId id;
+    memcpy(&id, cfg->nccl_id, 128);
+    check_nccl(nccl().CommInitRank(&c->comm, cfg->world_size, id, cfg->rank), "ncclCommInitRank");
+  }
+  *out = c;
+  c = nullptr;
+  }
+  catch (const Error& e) {
+    harmony_status st = fail(nullptr, e);
+    destroy(c);
+    return st;
+  }
+  return HARMONY_OK;
+}
+
+harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const harmony_layer_desc* descs,
+                                       const float* const* init_params) {
+  HM_API_BEGIN
+  HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
+  HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
+  HM_CHECK(!c->registered, HARMONY_E_BAD_STATE, "layers already registered");
+  HM_CHECK(descs && init_params, HARMONY_E_INVALID_ARG, "NULL argument");
+  HM_CUDA(cudaSetDevice(c->cfg.device));
+  Plan p = make_plan(c->cfg, n_layers, descs);
+  HM_CHECK(p.summary.hazards == 0, HARMONY_E_INVALID_ARG, "internal: planned program has a hazard: " + p.hazard_msg);
+  const int L = n_layers, m = p.m, N = p.N, r = p.rank;
+  const size_t ts = p.dtype ? 2 : 4;
+  for (int l = 0; l < L; ++l) HM_CHECK(init_params[l] != nullptr, HARMONY_E_INVALID_ARG, "init_params[l] is NULL");
+  // arena
+  if (c->arena) {
+    HM_CHECK(p.arena_bytes <= c->cfg.hbm_cap_bytes, HARMONY_E_CAP_TOO_SMALL, "plan exceeds the adopted arena");
+  } else {
+    HM_CUDA(cudaMalloc(&c->arena, p.arena_bytes));
+    c->own_arena = true;
+  }
+  // events of the program
+  c->events.resize(p.n_events);
+  for (auto& e : c->events) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  // pinned host store
+  c->h_wc.assign(L, nullptr);
+  c->h_state.assign(L, nullptr);
+  c->h_stash.assign((size_t)L * m, nullptr);
+  c->h_grad.assign(L, nullptr);
+  c->h_loss = static_cast<double*>(alloc_host((size_t)N * m * 8));
+  std::vector<uint8_t> full;  // staging of a full compute copy for resident layers
+  for (int l = 0; l < L; ++l) {
+    const LayerPlan& lp = p.layers[l];
+    const int64_t sh = lp.shard, P = lp.P;
+    c->h_wc[l] = static_cast<uint8_t*>(alloc_host((size_t)sh * ts));
+    c->h_state[l] = static_cast<float*>(alloc_host((size_t)lp.state_bytes));
+    if (p.retain_grads) c->h_grad[l] = static_cast<float*>(alloc_host((size_t)sh * 4));
+    float* master = c->h_state[l];
+    memset(master, 0, lp.state_bytes);  // m = v = 0 (reading c3), padding = 0
+    const int64_t lo = (int64_t)r * sh, hi = std::min<int64_t>(P, lo + sh);
+    if (hi > lo) memcpy(master, init_params[l] + lo, (size_t)(hi - lo) * 4);
+    if (ts == 2) {
+      uint16_t* w = reinterpret_cast<uint16_t*>(c->h_wc[l]);
+      for (int64_t i = 0; i < sh; ++i) w[i] = f32_to_bf16_rne(master[i]);
+    } else {
+      memcpy(c->h_wc[l], master, (size_t)sh * 4);
+    }
+    for (int i = 0; i < m; ++i)
+      if (lp.stash_res[i] < 0) c->h_stash[(size_t)l * m + i] = static_cast<uint8_t*>(alloc_host(lp.g.st.total));
+    // resident tensors go to HBM now
+    if (lp.wc_res >= 0) {
+      full.assign((size_t)lp.Ppad * ts, 0);
+      if (ts == 2) {
+        uint16_t* w = reinterpret_cast<uint16_t*>(full.data());
+        for (int64_t i = 0; i < P; ++i) w[i] = f32_to_bf16_rne(init_params[l][i]);
+      } else {
+        memcpy(full.data(), init_params[l], (size_t)P * 4);
+      }
+      HM_CUDA(cudaMemcpy(c->arena + lp.wc_res, full.data(), full.size(), cudaMemcpyHostToDevice));
+    }
+    if (lp.state_res >= 0)
+      HM_CUDA(cudaMemcpy(c->arena + lp.state_res, c->h_state[l], lp.state_bytes, cudaMemcpyHostToDevice));
+  }
+  HM_CUDA(cudaDeviceSynchronize());
+  c->plan = std::move(p);
+  c->registered = true;
+  HM_API_END(c)
+}
+
+harmony_status harmony_step(harmony_ctx* c, const float* x, const float* target, int64_t batch, double* loss_out,
+                            harmony_step_stats* stats) {
+  HM_API_BEGIN
+  HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
+  HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
+  HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
+  HM_CHECK(x && target, HARMONY_E_INVALID_ARG, "x/target NULL");
+  HM_CHECK(batch == (int64_t)c->plan.m * c->plan.b, HARMONY_E_INVALID_ARG,
+           "batch must equal microbatches*microbatch_size (this rank's rows)");
+  HM_CUDA(cudaSetDevice(c->cfg.device));
+  run_step(c, x, target, loss_out, stats);
+  HM_API_END(c)
+}
+
+harmony_status harmony_read_state(harmony_ctx* c, int32_t layer, int32_t which, float* dst, uint64_t n) {
+  HM_API_BEGIN
+  HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
+  HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
+  HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
+  const Plan& p = c->plan;
+  HM_CHECK(layer >= 0 && layer < (int)p.layers.size(), HARMONY_E_INVALID_ARG, "layer out of range");
+  const LayerPlan& lp = p.layers[layer];
+  HM_CHECK(dst && n == (uint64_t)lp.P, HARMONY_E_INVALID_ARG, "n_floats must equal the layer's parameter count");
+  HM_CHECK(which >= HARMONY_PARAM && which <= HARMONY_ADAM_V, HARMONY_E_INVALID_ARG, "bad state kind");
+  HM_CHECK(which != HARMONY_GRAD || p.retain_grads, HARMONY_E_BAD_STATE, "HARMONY_GRAD needs retain_grads");
+  HM_CUDA(cudaSetDevice(c->cfg.device));
+  const uint64_t sh = (uint64_t)lp.shard;
+  std::vector<float> mine(sh);
+  if (which == HARMONY_GRAD) {
+    memcpy(mine.data(), c->h_grad[layer], sh * 4);
+  } else {
+    const uint64_t off = (which == HARMONY_PARAM ? 0 : which == HARMONY_ADAM_M ? 1 : 2) * sh * 4;
+    if (lp.state_res >= 0) HM_CUDA(cudaMemcpy(mine.data(), c->arena + lp.state_res + off, sh * 4, cudaMemcpyDeviceToHost));
+    else memcpy(mine.data(), reinterpret_cast<uint8_t*>(c->h_state[layer]) + off, sh * 4);
+  }
+  if (p.N == 1) {
+    memcpy(dst, mine.data(), (size_t)lp.P * 4);
+  } else {
+    float* d = nullptr;
+    HM_CUDA(cudaMalloc(&d, (size_t)lp.Ppad * 4));
+    HM_CUDA(cudaMemcpy(d + (uint64_t)p.rank * sh, mine.data(), sh * 4, cudaMemcpyHostToDevice));
+    ncclResult_t rr = nccl().AllGather(d + (uint64_t)p.rank * sh, d, sh, ncclFloat32, c->comm, c->st[S_COMM]);
+    cudaError_t e1 = cudaStreamSynchronize(c->st[S_COMM]);
+    std::vector<float> all((size_t)lp.Ppad);
+    cudaError_t e2 = cudaMemcpy(all.data(), d, (size_t)lp.Ppad * 4, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    check_nccl(rr, "ncclAllGather(read_state)");
+    HM_CUDA(e1);
+    HM_CUDA(e2);
+    memcpy(dst, all.data(), (size_t)lp.P * 4);
+  }
+  HM_API_END(c)
+}
+
+harmony_status harmony_read_stats(const harmony_ctx* c, harmony_step_stats* out) {
+  if (!c || !out) return HARMONY_E_INVALID_ARG;
+  *out = c->last;
+  return HARMONY_OK;
+}
+
+harmony_status harmony_plan_info(const harmony_ctx* c, harmony_plan_summary* out) {
+  if (!c || !out) return HARMONY_E_INVALID_ARG;
+  if (!c->registered) return HARMONY_E_BAD_STATE;
+  *out = c->plan.summary;
+  return HARMONY_OK;
+}
+
+harmony_status harmony_finalize(harmony_ctx* c) {
+  if (!c) return HARMONY_E_INVALID_ARG;
+  destroy(c);
+  return HARMONY_OK;
+}
+
+}  // extern "C"

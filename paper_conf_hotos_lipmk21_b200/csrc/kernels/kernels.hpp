@@ -1,0 +1,41 @@
+// kernels.hpp — host launchers of the step's kernels (all asynchronous on `st`).
+#pragma once
+#include <cmath>
+#include <algorithm>
+
+#include "../common.hpp"
+#include "harmony_kernels.h"
+
+namespace hm {
+
+void gemm(const hk_gemm_args& a, cudaStream_t st);
+
+void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
+                   float* rstd, cudaStream_t st);
+size_t layernorm_bwd_scratch_bytes(int64_t rows, int d);
+void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                   const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
+                   float* scratch, cudaStream_t st);
+size_t colsum_scratch_bytes(int64_t rows, int n);
+void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float* out, int accumulate, float* scratch,
+            cudaStream_t st);
+void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st);
+void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
+                 cudaStream_t st);
+void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr, float b1, float b2,
+          float eps, int t, cudaStream_t st);
+size_t mse_scratch_bytes();
+void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY, double* loss_out, double* scratch,
+         cudaStream_t st);
+void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st);
+void act_bwd(int dtype, int act, int64_t n, const float* dY, const void* Z, void* dZ, cudaStream_t st);
+void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st);
+
+// Convenience: a GEMM descriptor with defaults (batch 1, alpha 1, no bias/aux).
+inline hk_gemm_args gemm_args(int dtype, int M, int N, int K) {
+  hk_gemm_args a{};
+  a.dtype = dtype; a.M = M; a.N = N; a.K = K; a.nz0 = 1; a.nz1 = 1; a.alpha = 1.f;
+  return a;
+}
+
+}  // namespace hm

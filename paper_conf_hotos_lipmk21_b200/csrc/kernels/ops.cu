@@ -1,0 +1,387 @@
+// ops.cu — the step's HBM-bound kernels (kernels K6-K12).
+//
+// LayerNorm fwd/bwd and softmax fwd/bwd use one warp per row with warp-shuffle reductions
+// (fixed butterfly order).  Column reductions (LN dgamma/dbeta, bias grads) are two-stage
+// and deterministic: fixed row chunks write partials, a second kernel sums them in chunk
+// order — no floating-point atomics anywhere (bit-exact capped == uncapped).
+// Adam, cast and the activation backward are vectorised grid-stride elementwise kernels.
+#include "../common.hpp"
+#include "kernels.hpp"
+
+namespace hm {
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+static int grid_for(int64_t n, int per_block) {
+  int64_t g = ceil_div(n, per_block);
+  int64_t cap = 148 * 16;
+  return (int)(g < 1 ? 1 : (g > cap ? cap : g));
+}
+
+// ------------------------------------------------------------------------------------- LayerNorm fwd
+// Two-pass statistics (mean, then centred sum of squares; reading c10), eps = 1e-5.
+template <typename T>
+__global__ void __launch_bounds__(256) layernorm_fwd_kernel(int64_t rows, int d, const float* __restrict__ X,
+                                                            const T* __restrict__ g, const T* __restrict__ b,
+                                                            T* __restrict__ U, float* __restrict__ mean,
+                                                            float* __restrict__ rstd) {
+  const int lane = threadIdx.x & 31;
+  const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (row >= rows) return;
+  const float* x = X + row * d;
+  float s = 0.f;
+  for (int c = lane; c < d; c += 32) s += x[c];
+  const float mu = warp_sum(s) / (float)d;
+  float q = 0.f;
+  for (int c = lane; c < d; c += 32) {
+    float t = x[c] - mu;
+    q += t * t;
+  }
+  const float var = warp_sum(q) / (float)d;
+  const float rs = rsqrtf(var + 1e-5f);
+  T* u = U + row * d;
+  for (int c = lane; c < d; c += 32) u[c] = from_f32<T>((x[c] - mu) * rs * to_f32(g[c]) + to_f32(b[c]));
+  if (lane == 0) { mean[row] = mu; rstd[row] = rs; }
+}
+
+// ------------------------------------------------------------------------------------- LayerNorm bwd
+constexpr int LN_ROWS_PER_BLOCK = 32;
+
+template <typename T>
+__global__ void __launch_bounds__(256) layernorm_bwd_kernel(int64_t rows, int d, const float* __restrict__ dU,
+                                                            const float* __restrict__ X, const float* __restrict__ mean,
+                                                            const float* __restrict__ rstd, const T* __restrict__ g,
+                                                            const float* __restrict__ dres, float* __restrict__ dX,
+                                                            float* __restrict__ partial) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t r0 = (int64_t)blockIdx.x * LN_ROWS_PER_BLOCK;
+  // phase 1: dX per row (one warp per row)
+  for (int i = warp; i < LN_ROWS_PER_BLOCK; i += 8) {
+    const int64_t row = r0 + i;
+    if (row >= rows) break;
+    const float mu = mean[row], rs = rstd[row];
+    const float* x = X + row * d;
+    const float* du = dU + row * d;
+    float s1 = 0.f, s2 = 0.f;
+    for (int c = lane; c < d; c += 32) {
+      float xh = (x[c] - mu) * rs;
+      float dxh = du[c] * to_f32(g[c]);
+      s1 += dxh;
+      s2 += dxh * xh;
+    }
+    s1 = warp_sum(s1) / (float)d;
+    s2 = warp_sum(s2) / (float)d;
+    float* dx = dX + row * d;
+    const float* dr = dres ? dres + row * d : nullptr;
+    for (int c = lane; c < d; c += 32) {
+      float xh = (x[c] - mu) * rs;
+      float dxh = du[c] * to_f32(g[c]);
+      float v = rs * (dxh - s1 - xh * s2);
+      dx[c] = dr ? dr[c] + v : v;
+    }
+  }
+  // phase 2: this block's column partials of dgamma = sum dU*xh and dbeta = sum dU (rows in order)
+  const int64_t rend = min(rows, r0 + LN_ROWS_PER_BLOCK);
+  float* pg = partial + (int64_t)blockIdx.x * 2 * d;
+  for (int c = threadIdx.x; c < d; c += 256) {
+    float ag = 0.f, ab = 0.f;
+    for (int64_t row = r0; row < rend; ++row) {
+      float du = dU[row * d + c];
+      ag += du * ((X[row * d + c] - mean[row]) * rstd[row]);
+      ab += du;
+    }
+    pg[c] = ag;
+    pg[d + c] = ab;
+  }
+}
+
+// out[c] (+)= sum over chunks j in order of partial[j][c]  (partial row stride `stride`)
+__global__ void colreduce_kernel(int nchunks, int n, const float* __restrict__ partial, int64_t stride,
+                                 float* __restrict__ out, int accumulate) {
+  int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  float s = 0.f;
+  for (int j = 0; j < nchunks; ++j) s += partial[(int64_t)j * stride + c];
+  out[c] = accumulate ? out[c] + s : s;
+}
+
+// ------------------------------------------------------------------------------------- column sums
+constexpr int CS_ROWS = 64;
+template <typename Tin>
+__global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict__ X, int64_t ld,
+                                      float* __restrict__ partial) {
+  int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  int64_t r0 = (int64_t)blockIdx.y * CS_ROWS, r1 = min(rows, r0 + CS_ROWS);
+  float s = 0.f;
+  for (int64_t r = r0; r < r1; ++r) s += to_f32(X[r * ld + c]);
+  partial[(int64_t)blockIdx.y * n + c] = s;
+}
+
+// ------------------------------------------------------------------------------------- softmax
+// P = softmax(scale * Z) over each row; causal rows mask keys j > (row % S) to exactly 0 (c11).
+template <typename T>
+__global__ void __launch_bounds__(256) softmax_fwd_kernel(int64_t rows, int S, int causal, float scale,
+                                                          const float* __restrict__ Z, T* __restrict__ P) {
+  const int lane = threadIdx.x & 31;
+  const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (row >= rows) return;
+  const int lim = causal ? (int)(row % S) + 1 : S;
+  const float* z = Z + row * S;
+  float mx = -INFINITY;
+  for (int c = lane; c < lim; c += 32) mx = fmaxf(mx, scale * z[c]);
+  mx = warp_max(mx);
+  float s = 0.f;
+  for (int c = lane; c < lim; c += 32) s += __expf(scale * z[c] - mx);
+  s = warp_sum(s);
+  const float inv = 1.f / s;
+  T* p = P + row * S;
+  for (int c = lane; c < S; c += 32) p[c] = from_f32<T>(c < lim ? __expf(scale * z[c] - mx) * inv : 0.f);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) softmax_bwd_kernel(int64_t rows, int S, float alpha,
+                                                          const float* __restrict__ dP, const T* __restrict__ P,
+                                                          T* __restrict__ dZ) {
+  const int lane = threadIdx.x & 31;
+  const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (row >= rows) return;
+  const float* dp = dP + row * S;
+  const T* p = P + row * S;
+  float s = 0.f;
+  for (int c = lane; c < S; c += 32) s += dp[c] * to_f32(p[c]);
+  s = warp_sum(s);
+  T* dz = dZ + row * S;
+  for (int c = lane; c < S; c += 32) dz[c] = from_f32<T>(alpha * to_f32(p[c]) * (dp[c] - s));
+}
+
+// ------------------------------------------------------------------------------------- Adam
+// Kingma & Ba [30], Algorithm 1 with bias correction; fp32 master state (reading c3).
+template <typename T>
+__global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict__ m, float* __restrict__ v,
+                            const float* __restrict__ g, T* __restrict__ Wc, float lr, float b1, float b2, float eps,
+                            float inv_bc1, float inv_bc2) {
+  const int64_t n4 = n / 4;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
+    float4 w = reinterpret_cast<float4*>(W)[i];
+    float4 mm = reinterpret_cast<float4*>(m)[i];
+    float4 vv = reinterpret_cast<float4*>(v)[i];
+    float4 gg = reinterpret_cast<const float4*>(g)[i];
+    float* wp = &w.x; float* mp = &mm.x; float* vp = &vv.x; const float* gp = &gg.x;
+    float out[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      mp[j] = b1 * mp[j] + (1.f - b1) * gp[j];
+      vp[j] = b2 * vp[j] + (1.f - b2) * gp[j] * gp[j];
+      wp[j] = wp[j] - lr * (mp[j] * inv_bc1) / (sqrtf(vp[j] * inv_bc2) + eps);
+      out[j] = wp[j];
+    }
+    reinterpret_cast<float4*>(W)[i] = w;
+    reinterpret_cast<float4*>(m)[i] = mm;
+    reinterpret_cast<float4*>(v)[i] = vv;
+    if (sizeof(T) == 2) {
+      __nv_bfloat162 lo = __floats2bfloat162_rn(out[0], out[1]);
+      __nv_bfloat162 hi = __floats2bfloat162_rn(out[2], out[3]);
+      uint2 pk;
+      pk.x = *reinterpret_cast<uint32_t*>(&lo);
+      pk.y = *reinterpret_cast<uint32_t*>(&hi);
+      reinterpret_cast<uint2*>(Wc)[i] = pk;
+    } else {
+      reinterpret_cast<float4*>(Wc)[i] = make_float4(out[0], out[1], out[2], out[3]);
+    }
+  }
+  for (int64_t i = n4 * 4 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    float mi = b1 * m[i] + (1.f - b1) * g[i];
+    float vi = b2 * v[i] + (1.f - b2) * g[i] * g[i];
+    float wi = W[i] - lr * (mi * inv_bc1) / (sqrtf(vi * inv_bc2) + eps);
+    m[i] = mi; v[i] = vi; W[i] = wi;
+    Wc[i] = from_f32<T>(wi);
+  }
+}
+
+// ------------------------------------------------------------------------------------- MSE loss
+constexpr int MSE_BLOCK = 256;
+__global__ void mse_kernel(int64_t n, const float* __restrict__ Y, const float* __restrict__ Tg, float inv_batch,
+                           float* __restrict__ dY, double* __restrict__ partial) {
+  __shared__ double sh[MSE_BLOCK / 32];
+  double acc = 0.0;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    float dlt = Y[i] - Tg[i];
+    dY[i] = dlt * inv_batch;
+    acc += (double)dlt * (double)dlt;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int w = 0; w < MSE_BLOCK / 32; ++w) s += sh[w];
+    partial[blockIdx.x] = s;
+  }
+}
+__global__ void mse_final_kernel(int nblk, const double* __restrict__ partial, double half_inv_batch,
+                                 double* __restrict__ out) {
+  double s = 0.0;
+  for (int j = 0; j < nblk; ++j) s += partial[j];
+  *out = s * half_inv_batch;
+}
+
+// ------------------------------------------------------------------------------------- elementwise
+template <typename T>
+__global__ void cast_kernel(int64_t n, const float* __restrict__ in, T* __restrict__ out) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = from_f32<T>(in[i]);
+}
+template <typename T>
+__global__ void act_bwd_kernel(int act, int64_t n, const float* __restrict__ dY, const T* __restrict__ Z,
+                               T* __restrict__ dZ) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+    dZ[i] = from_f32<T>(dY[i] * act_grad_f(act, to_f32(Z[i])));
+}
+template <typename T>
+__global__ void act_fwd_kernel(int act, int64_t n, const T* __restrict__ Z, T* __restrict__ out) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+    out[i] = from_f32<T>(act_f(act, to_f32(Z[i])));
+}
+__global__ void copy_rows_kernel(int64_t n4, const float4* __restrict__ src, float4* __restrict__ dst) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) dst[i] = src[i];
+}
+
+// ===================================================================================== launchers
+#define HM_DISPATCH_T(dtype, ...)                                 \
+  do {                                                            \
+    if ((dtype) == 1) {                                           \
+      using T = __nv_bfloat16;                                    \
+      __VA_ARGS__;                                                \
+    } else {                                                      \
+      using T = float;                                            \
+      __VA_ARGS__;                                                \
+    }                                                             \
+  } while (0)
+
+void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
+                   float* rstd, cudaStream_t st) {
+  if (rows == 0) return;
+  HM_DISPATCH_T(dtype, (layernorm_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(
+                           rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)));
+  check_launch("layernorm_fwd");
+}
+
+size_t layernorm_bwd_scratch_bytes(int64_t rows, int d) {
+  return (size_t)ceil_div(rows, LN_ROWS_PER_BLOCK) * 2 * d * sizeof(float);
+}
+
+void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                   const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
+                   float* scratch, cudaStream_t st) {
+  if (rows == 0) {
+    return;
+  }
+  int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
+  HM_DISPATCH_T(dtype, (layernorm_bwd_kernel<T><<<nblk, 256, 0, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres,
+                                                                      dX, scratch)));
+  check_launch("layernorm_bwd");
+  colreduce_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
+  check_launch("colreduce(dgamma)");
+  colreduce_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
+  check_launch("colreduce(dbeta)");
+}
+
+size_t colsum_scratch_bytes(int64_t rows, int n) { return (size_t)ceil_div(rows, CS_ROWS) * n * sizeof(float); }
+
+void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float* out, int accumulate, float* scratch,
+            cudaStream_t st) {
+  int nch = (int)ceil_div(rows, CS_ROWS);
+  if (nch == 0) {
+    if (!accumulate) HM_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * n, st));
+    return;
+  }
+  dim3 grid((unsigned)ceil_div(n, 128), (unsigned)nch);
+  HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+  check_launch("colsum_partial");
+  colreduce_kernel<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(nch, n, scratch, n, out, accumulate);
+  check_launch("colsum_reduce");
+}
+
+void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st) {
+  if (rows == 0) return;
+  HM_DISPATCH_T(dtype, (softmax_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, causal, scale, Z,
+                                                                                          (T*)P)));
+  check_launch("softmax_fwd");
+}
+
+void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
+                 cudaStream_t st) {
+  if (rows == 0) return;
+  HM_DISPATCH_T(dtype, (softmax_bwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, alpha, dP,
+                                                                                          (const T*)P, (T*)dZ)));
+  check_launch("softmax_bwd");
+}
+
+void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr, float b1, float b2,
+          float eps, int t, cudaStream_t st) {
+  if (n == 0) return;
+  // bias corrections computed in double on the host, applied as fp32 reciprocals
+  double bc1 = 1.0 - std::pow((double)b1, (double)t), bc2 = 1.0 - std::pow((double)b2, (double)t);
+  HM_CHECK(((uintptr_t)W | (uintptr_t)m | (uintptr_t)v | (uintptr_t)g) % 16 == 0, HARMONY_E_INVALID_ARG,
+           "adam: fp32 state must be 16-byte aligned");
+  HM_DISPATCH_T(dtype, (adam_kernel<T><<<grid_for(ceil_div(n, 4), 256), 256, 0, st>>>(
+                           n, W, m, v, g, (T*)Wc, lr, b1, b2, eps, (float)(1.0 / bc1), (float)(1.0 / bc2))));
+  check_launch("adam");
+}
+
+size_t mse_scratch_bytes() { return 1024 * sizeof(double); }
+
+void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY, double* loss_out, double* scratch,
+         cudaStream_t st) {
+  int nblk = (int)std::min<int64_t>(1024, std::max<int64_t>(1, ceil_div(n, MSE_BLOCK * 8)));
+  mse_kernel<<<nblk, MSE_BLOCK, 0, st>>>(n, Y, Tg, inv_batch, dY, scratch);
+  check_launch("mse");
+  mse_final_kernel<<<1, 1, 0, st>>>(nblk, scratch, 0.5 * (double)inv_batch, loss_out);
+  check_launch("mse_final");
+}
+
+void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st) {
+  if (n == 0) return;
+  HM_DISPATCH_T(dtype, (cast_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(n, in, (T*)out)));
+  check_launch("cast");
+}
+
+void act_bwd(int dtype, int act, int64_t n, const float* dY, const void* Z, void* dZ, cudaStream_t st) {
+  if (n == 0) return;
+  HM_DISPATCH_T(dtype, (act_bwd_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(act, n, dY, (const T*)Z, (T*)dZ)));
+  check_launch("act_bwd");
+}
+
+void act_fwd_T(int dtype, int act, int64_t n, const void* Z, void* out, cudaStream_t st) {
+  if (n == 0) return;
+  HM_DISPATCH_T(dtype, (act_fwd_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(act, n, (const T*)Z, (T*)out)));
+  check_launch("act_fwd");
+}
+
+void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st) {
+  if (n == 0) return;
+  if (n % 4 == 0 && ((uintptr_t)src | (uintptr_t)dst) % 16 == 0) {
+    copy_rows_kernel<<<grid_for(n / 4, 256), 256, 0, st>>>(n / 4, (const float4*)src, (float4*)dst);
+    check_launch("copy_f32");
+  } else {
+    HM_CUDA(cudaMemcpyAsync(dst, src, n * sizeof(float), cudaMemcpyDeviceToDevice, st));
+  }
+}
+
+}  // namespace hm

@@ -1,0 +1,379 @@
+// layers.cu — forward / backward task bodies of the registered layer kinds.
+// Math: oracle-independent restatement of the pre-LN block (reading c1) and the
+// MLP layer; every contraction runs on hk gemm (tcgen05 for bf16, SIMT for fp32).
+#include <cmath>
+
+#include "common.hpp"
+#include "kernels/kernels.hpp"
+#include "layers.hpp"
+
+namespace hm {
+
+void act_fwd_T(int dtype, int act, int64_t n, const void* Z, void* out, cudaStream_t st);
+
+int64_t layer_n_params(const harmony_layer_desc& d) {
+  if (d.kind == HARMONY_LAYER_MLP) return (int64_t)d.d_in * d.d_out + d.d_out;
+  int64_t D = d.d_in;
+  return 12 * D * D + 13 * D;
+}
+
+// scratch of the backward: LN column partials, bias-grad partials, or 2 rows of recomputed LN stats
+static uint64_t bwd_scratch_bytes(int64_t R, int D) {
+  return std::max<uint64_t>(std::max<uint64_t>(layernorm_bwd_scratch_bytes(R, D), colsum_scratch_bytes(R, 4 * D)),
+                            (uint64_t)R * 8);
+}
+
+static uint64_t bump(uint64_t& cur, uint64_t bytes) {
+  uint64_t o = cur;
+  cur = align_up(cur + bytes, 256);
+  return o;
+}
+
+LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_policy) {
+  LayerGeom g;
+  g.desc = desc;
+  g.dtype = dtype;
+  g.ts = dtype == 1 ? 2 : 4;
+  g.stash_policy = stash_policy;
+  g.b = b;
+  g.n_params = layer_n_params(desc);
+  if (desc.kind == HARMONY_LAYER_MLP) {
+    g.S = 1;
+    g.rows = b;
+    g.d = desc.d_in;
+    g.off[P_MLP_W] = 0;
+    g.off[P_MLP_B] = (int64_t)desc.d_in * desc.d_out;
+    uint64_t c = 0;
+    g.st.X = bump(c, (uint64_t)g.rows * desc.d_in * g.ts);  // Xc: the GEMM operand (T)
+    g.st.Z = bump(c, (uint64_t)g.rows * desc.d_out * g.ts); // pre-activation
+    g.st.total = c;
+    uint64_t w = 0;
+    bump(w, (uint64_t)g.rows * desc.d_out * g.ts);  // dZ
+    bump(w, std::max(colsum_scratch_bytes(g.rows, desc.d_out), (size_t)256));
+    g.ws_bwd = w;
+    g.ws_fwd = 256;
+    g.flops_fwd = 2.0 * g.rows * desc.d_in * desc.d_out;
+    return g;
+  }
+  const int64_t D = desc.d_in;
+  g.d = desc.d_in;
+  g.h = desc.n_heads;
+  g.dh = desc.d_in / desc.n_heads;
+  g.S = desc.seq_len;
+  g.rows = (int64_t)b * g.S;
+  int64_t o = 0;
+  const int64_t seg[12] = {D, D, 3 * D * D, 3 * D, D * D, D, D, D, 4 * D * D, 4 * D, 4 * D * D, D};
+  for (int i = 0; i < 12; ++i) { g.off[i] = o; o += seg[i]; }
+  const uint64_t R = (uint64_t)g.rows, ts = (uint64_t)g.ts;
+  const uint64_t SS = (uint64_t)b * g.h * g.S * g.S;
+  uint64_t c = 0;
+  g.st.X = bump(c, R * D * 4);
+  g.st.mean1 = bump(c, R * 4);
+  g.st.rstd1 = bump(c, R * 4);
+  if (stash_policy == 0) g.st.U = bump(c, R * D * ts);
+  g.st.QKV = bump(c, R * 3 * D * ts);
+  g.st.P = bump(c, SS * ts);
+  g.st.C = bump(c, R * D * ts);
+  g.st.X2 = bump(c, R * D * 4);
+  g.st.mean2 = bump(c, R * 4);
+  g.st.rstd2 = bump(c, R * 4);
+  if (stash_policy == 0) g.st.U2 = bump(c, R * D * ts);
+  g.st.H = bump(c, R * 4 * D * ts);
+  if (stash_policy == 0) g.st.G = bump(c, R * 4 * D * ts);
+  g.st.total = c;
+  // forward workspace: scores Z (fp32) [+ recomputable U, U2, G under policy 1]
+  uint64_t wf = 0;
+  bump(wf, SS * 4);
+  if (stash_policy == 1) { bump(wf, R * D * ts); bump(wf, R * D * ts); bump(wf, R * 4 * D * ts); }
+  g.ws_fwd = wf;
+  // backward workspace (see layer_bwd for the aliasing)
+  uint64_t wb = 0;
+  bump(wb, R * D * ts);          // dYc / dX2c
+  bump(wb, R * 4 * D * ts);      // dH / dQKV
+  bump(wb, R * D * 4);           // dU2 / dU (fp32)
+  bump(wb, R * D * 4);           // dX2 (fp32)
+  bump(wb, R * D * ts);          // dC
+  bump(wb, SS * 4);              // dP (fp32)
+  bump(wb, SS * ts);             // dZ
+  bump(wb, bwd_scratch_bytes(g.rows, (int)D));
+  if (stash_policy == 1) bump(wb, R * 4 * D * ts);  // recomputed G / U2 / U
+  g.ws_bwd = wb;
+  g.flops_fwd = 24.0 * (double)R * D * D + 4.0 * (double)b * g.S * g.S * D;
+  return g;
+}
+
+// ------------------------------------------------------------------------------------------------ helpers
+static inline const uint8_t* wseg(const LayerGeom& g, const void* W, int seg) {
+  return static_cast<const uint8_t*>(W) + g.off[seg] * g.ts;
+}
+static inline float* gseg(const LayerGeom& g, float* dW, int seg) { return dW + g.off[seg]; }
+
+// Linear Y[rows][n] = X[rows][k] . W[k][n]  (W stored [k][n]: MN-major B)
+static hk_gemm_args lin_fwd(const LayerGeom& g, int64_t rows, int n, int k, const void* X, const void* W) {
+  hk_gemm_args a = gemm_args(g.dtype, (int)rows, n, k);
+  a.A = X; a.a_mn_major = 0; a.lda = k;
+  a.B = W; a.b_mn_major = 1; a.ldb = n;
+  a.ldc = n;
+  return a;
+}
+// dX[rows][k] = dY[rows][n] . W^T  (W[k][n] read as (n=k-index, k=n-index): K-major B)
+static hk_gemm_args lin_dgrad(const LayerGeom& g, int64_t rows, int n, int k, const void* dY, const void* W) {
+  hk_gemm_args a = gemm_args(g.dtype, (int)rows, k, n);
+  a.A = dY; a.a_mn_major = 0; a.lda = n;
+  a.B = W; a.b_mn_major = 0; a.ldb = n;
+  a.ldc = k;
+  return a;
+}
+// dW[k][n] (+)= X^T . dY  (both MN-major), fp32 accumulate (one writer per element: deterministic)
+static hk_gemm_args lin_wgrad(const LayerGeom& g, int64_t rows, int n, int k, const void* X, const void* dY, float* dW,
+                              int first) {
+  hk_gemm_args a = gemm_args(g.dtype, k, n, (int)rows);
+  a.A = X; a.a_mn_major = 1; a.lda = k;
+  a.B = dY; a.b_mn_major = 1; a.ldb = n;
+  a.C = dW; a.ldc = n;
+  a.epilogue = HK_EPI_ACC_F32;
+  a.accumulate = first ? 0 : 1;
+  return a;
+}
+
+// ------------------------------------------------------------------------------------------------ forward
+void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* stv) {
+  cudaStream_t st = static_cast<cudaStream_t>(stv);
+  const harmony_layer_desc& d = g.desc;
+  if (d.kind == HARMONY_LAYER_MLP) {
+    void* Xc = stash + g.st.X;
+    void* Z = stash + g.st.Z;
+    if (g.dtype == 1) cast(1, g.rows * d.d_in, X, Xc, st);
+    else copy_f32(g.rows * d.d_in, X, static_cast<float*>(Xc), st);
+    hk_gemm_args a = lin_fwd(g, g.rows, d.d_out, d.d_in, Xc, wseg(g, W, P_MLP_W));
+    a.C = Z; a.epilogue = HK_EPI_BIAS_ACT_F32; a.act = d.act; a.bias = wseg(g, W, P_MLP_B); a.aux_out = Y;
+    gemm(a, st);
+    return;
+  }
+  const int64_t R = g.rows;
+  const int D = g.d, S = g.S, H = g.h, dh = g.dh, b = g.b;
+  const size_t ts = g.ts;
+  float* Xs = reinterpret_cast<float*>(stash + g.st.X);
+  float* mean1 = reinterpret_cast<float*>(stash + g.st.mean1);
+  float* rstd1 = reinterpret_cast<float*>(stash + g.st.rstd1);
+  uint8_t* QKV = stash + g.st.QKV;
+  uint8_t* P = stash + g.st.P;
+  uint8_t* C = stash + g.st.C;
+  float* X2 = reinterpret_cast<float*>(stash + g.st.X2);
+  float* mean2 = reinterpret_cast<float*>(stash + g.st.mean2);
+  float* rstd2 = reinterpret_cast<float*>(stash + g.st.rstd2);
+  uint8_t* Hh = stash + g.st.H;
+  uint64_t wc = 0;
+  float* Z = reinterpret_cast<float*>(ws + bump(wc, (uint64_t)b * H * S * S * 4));
+  uint8_t *U, *U2, *G;
+  if (g.stash_policy == 0) {
+    U = stash + g.st.U; U2 = stash + g.st.U2; G = stash + g.st.G;
+  } else {
+    U = ws + bump(wc, R * D * ts); U2 = ws + bump(wc, R * D * ts); G = ws + bump(wc, R * 4 * D * ts);
+  }
+  // stash the layer input (Fig. 5(a) "Stashed X")
+  copy_f32(R * D, X, Xs, st);
+  // U = LN1(X)
+  layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st);
+  // QKV = U W_qkv + b_qkv
+  {
+    hk_gemm_args a = lin_fwd(g, R, 3 * D, D, U, wseg(g, W, P_WQKV));
+    a.C = QKV; a.epilogue = HK_EPI_STORE_T; a.bias = wseg(g, W, P_BQKV);
+    gemm(a, st);
+  }
+  // Z[b,h] = Q_h K_h^T (fp32), batched over heads (z0) and sequences (z1)
+  {
+    hk_gemm_args a = gemm_args(g.dtype, S, S, dh);
+    a.nz0 = H; a.nz1 = b;
+    a.A = QKV; a.a_mn_major = 0; a.lda = 3 * D; a.a_sz0 = dh; a.a_sz1 = (int64_t)S * 3 * D;
+    a.B = QKV + (size_t)D * ts; a.b_mn_major = 0; a.ldb = 3 * D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * D;
+    a.C = Z; a.ldc = S; a.c_sz0 = (int64_t)S * S; a.c_sz1 = (int64_t)H * S * S;
+    a.epilogue = HK_EPI_STORE_F32;
+    gemm(a, st);
+  }
+  // P = softmax(Z / sqrt(dh)) (+ causal mask)
+  softmax_fwd(g.dtype, (int64_t)b * H * S, S, d.causal, 1.0f / std::sqrt((float)dh), Z, P, st);
+  // C_h = P V_h, written head-interleaved into C [R][D]
+  {
+    hk_gemm_args a = gemm_args(g.dtype, S, dh, S);
+    a.nz0 = H; a.nz1 = b;
+    a.A = P; a.a_mn_major = 0; a.lda = S; a.a_sz0 = (int64_t)S * S; a.a_sz1 = (int64_t)H * S * S;
+    a.B = QKV + (size_t)2 * D * ts; a.b_mn_major = 1; a.ldb = 3 * D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * D;
+    a.C = C; a.ldc = D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * D;
+    a.epilogue = HK_EPI_STORE_T;
+    gemm(a, st);
+  }
+  // X2 = X + C W_o + b_o   (fp32 residual stream)
+  {
+    hk_gemm_args a = lin_fwd(g, R, D, D, C, wseg(g, W, P_WO));
+    a.C = X2; a.epilogue = HK_EPI_RESID_F32; a.aux = X; a.bias = wseg(g, W, P_BO);
+    gemm(a, st);
+  }
+  // U2 = LN2(X2)
+  layernorm_fwd(g.dtype, R, D, X2, wseg(g, W, P_LN2_G), wseg(g, W, P_LN2_B), U2, mean2, rstd2, st);
+  // H = U2 W_fc1 + b_fc1 ; G = GeLU(H)
+  {
+    hk_gemm_args a = lin_fwd(g, R, 4 * D, D, U2, wseg(g, W, P_WFC1));
+    a.C = Hh; a.epilogue = HK_EPI_BIAS_ACT; a.act = HARMONY_ACT_GELU_TANH; a.bias = wseg(g, W, P_BFC1); a.aux_out = G;
+    gemm(a, st);
+  }
+  // Y = X2 + G W_fc2 + b_fc2
+  {
+    hk_gemm_args a = lin_fwd(g, R, D, 4 * D, G, wseg(g, W, P_WFC2));
+    a.C = Y; a.epilogue = HK_EPI_RESID_F32; a.aux = X2; a.bias = wseg(g, W, P_BFC2);
+    gemm(a, st);
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ backward
+void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
+               int first, uint8_t* ws, void* stv) {
+  cudaStream_t st = static_cast<cudaStream_t>(stv);
+  const harmony_layer_desc& d = g.desc;
+  const int acc = first ? 0 : 1;
+  if (d.kind == HARMONY_LAYER_MLP) {
+    uint64_t wc = 0;
+    uint8_t* dZ = ws + bump(wc, (uint64_t)g.rows * d.d_out * g.ts);
+    float* scratch = reinterpret_cast<float*>(ws + bump(wc, colsum_scratch_bytes(g.rows, d.d_out)));
+    const uint8_t* Xc = stash + g.st.X;
+    const uint8_t* Z = stash + g.st.Z;
+    act_bwd(g.dtype, d.act, g.rows * d.d_out, dY, Z, dZ, st);
+    gemm(lin_wgrad(g, g.rows, d.d_out, d.d_in, Xc, dZ, gseg(g, dW, P_MLP_W), first), st);
+    colsum(g.dtype, g.rows, d.d_out, dZ, d.d_out, gseg(g, dW, P_MLP_B), acc, scratch, st);
+    if (dX) {
+      hk_gemm_args a = lin_dgrad(g, g.rows, d.d_out, d.d_in, dZ, wseg(g, W, P_MLP_W));
+      a.C = dX; a.epilogue = HK_EPI_STORE_F32;
+      gemm(a, st);
+    }
+    return;
+  }
+  const int64_t R = g.rows;
+  const int D = g.d, S = g.S, H = g.h, dh = g.dh, b = g.b;
+  const size_t ts = g.ts;
+  const int dt = g.dtype;
+  const float* Xs = reinterpret_cast<const float*>(stash + g.st.X);
+  const float* mean1 = reinterpret_cast<const float*>(stash + g.st.mean1);
+  const float* rstd1 = reinterpret_cast<const float*>(stash + g.st.rstd1);
+  const uint8_t* QKV = stash + g.st.QKV;
+  const uint8_t* P = stash + g.st.P;
+  const uint8_t* C = stash + g.st.C;
+  const float* X2 = reinterpret_cast<const float*>(stash + g.st.X2);
+  const float* mean2 = reinterpret_cast<const float*>(stash + g.st.mean2);
+  const float* rstd2 = reinterpret_cast<const float*>(stash + g.st.rstd2);
+  const uint8_t* Hh = stash + g.st.H;
+  const uint64_t SS = (uint64_t)b * H * S * S;
+  uint64_t wc = 0;
+  uint8_t* dYc = ws + bump(wc, R * D * ts);            // later dX2c
+  uint8_t* dHb = ws + bump(wc, R * 4 * D * ts);        // later dQKV
+  float* dUf = reinterpret_cast<float*>(ws + bump(wc, R * D * 4));
+  float* dX2 = reinterpret_cast<float*>(ws + bump(wc, R * D * 4));
+  uint8_t* dC = ws + bump(wc, R * D * ts);
+  float* dP = reinterpret_cast<float*>(ws + bump(wc, SS * 4));
+  uint8_t* dZ = ws + bump(wc, SS * ts);
+  float* scratch = reinterpret_cast<float*>(ws + bump(wc, bwd_scratch_bytes(R, D)));
+  uint8_t* rec = g.stash_policy == 1 ? ws + bump(wc, R * 4 * D * ts) : nullptr;
+
+  // dY as a GEMM operand
+  const void* dYop = dY;
+  if (dt == 1) { cast(1, R * D, dY, dYc, st); dYop = dYc; }
+  // ---- FC2: dG = dY W_fc2^T, fused with GeLU': dH = dG * gelu'(H)
+  {
+    hk_gemm_args a = lin_dgrad(g, R, D, 4 * D, dYop, wseg(g, W, P_WFC2));
+    a.C = dHb; a.epilogue = HK_EPI_ACT_BWD; a.act = HARMONY_ACT_GELU_TANH; a.aux = Hh;
+    gemm(a, st);
+  }
+  const uint8_t* G = g.stash_policy == 0 ? stash + g.st.G : rec;
+  if (g.stash_policy == 1) act_fwd_T(dt, HARMONY_ACT_GELU_TANH, R * 4 * D, Hh, rec, st);
+  gemm(lin_wgrad(g, R, D, 4 * D, G, dYop, gseg(g, dW, P_WFC2), first), st);
+  colsum(0, R, D, dY, D, gseg(g, dW, P_BFC2), acc, scratch, st);
+  // ---- FC1: dU2 = dH W_fc1^T (fp32 for the LN backward); dW_fc1 += U2^T dH
+  {
+    hk_gemm_args a = lin_dgrad(g, R, 4 * D, D, dHb, wseg(g, W, P_WFC1));
+    a.C = dUf; a.epilogue = HK_EPI_STORE_F32;
+    gemm(a, st);
+  }
+  const uint8_t* U2 = stash + g.st.U2;
+  if (g.stash_policy == 1) {
+    // recompute U2 = LN2(X2) from the stashed X2 (identical kernel => identical bits)
+    float* tmp_mean = reinterpret_cast<float*>(scratch);
+    float* tmp_rstd = tmp_mean + R;
+    layernorm_fwd(dt, R, D, X2, wseg(g, W, P_LN2_G), wseg(g, W, P_LN2_B), rec, tmp_mean, tmp_rstd, st);
+    U2 = rec;
+  }
+  gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), st);
+  colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, scratch, st);
+  // ---- LN2 backward: dX2 = dY + LN2'(dU2)
+  layernorm_bwd(dt, R, D, dUf, X2, mean2, rstd2, wseg(g, W, P_LN2_G), dY, dX2, gseg(g, dW, P_LN2_G),
+                gseg(g, dW, P_LN2_B), acc, scratch, st);
+  // ---- O projection: dC = dX2 W_o^T; dW_o += C^T dX2; db_o += sum dX2
+  const void* dX2op = dX2;
+  if (dt == 1) { cast(1, R * D, dX2, dYc, st); dX2op = dYc; }
+  {
+    hk_gemm_args a = lin_dgrad(g, R, D, D, dX2op, wseg(g, W, P_WO));
+    a.C = dC; a.epilogue = HK_EPI_STORE_T;
+    gemm(a, st);
+  }
+  gemm(lin_wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first), st);
+  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, scratch, st);
+  // ---- attention backward (batched over heads z0 and sequences z1)
+  uint8_t* dQKV = dHb;
+  const float scale = 1.0f / std::sqrt((float)dh);
+  {  // dP = dC_h V_h^T
+    hk_gemm_args a = gemm_args(dt, S, S, dh);
+    a.nz0 = H; a.nz1 = b;
+    a.A = dC; a.a_mn_major = 0; a.lda = D; a.a_sz0 = dh; a.a_sz1 = (int64_t)S * D;
+    a.B = QKV + (size_t)2 * D * ts; a.b_mn_major = 0; a.ldb = 3 * D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * D;
+    a.C = dP; a.ldc = S; a.c_sz0 = (int64_t)S * S; a.c_sz1 = (int64_t)H * S * S;
+    a.epilogue = HK_EPI_STORE_F32;
+    gemm(a, st);
+  }
+  {  // dV_h = P^T dC_h
+    hk_gemm_args a = gemm_args(dt, S, dh, S);
+    a.nz0 = H; a.nz1 = b;
+    a.A = P; a.a_mn_major = 1; a.lda = S; a.a_sz0 = (int64_t)S * S; a.a_sz1 = (int64_t)H * S * S;
+    a.B = dC; a.b_mn_major = 1; a.ldb = D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * D;
+    a.C = dQKV + (size_t)2 * D * ts; a.ldc = 3 * D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * 3 * D;
+    a.epilogue = HK_EPI_STORE_T;
+    gemm(a, st);
+  }
+  // dZ = scale * P.(dP - rowsum(dP.P))
+  softmax_bwd(dt, (int64_t)b * H * S, S, scale, dP, P, dZ, st);
+  {  // dQ_h = dZ K_h
+    hk_gemm_args a = gemm_args(dt, S, dh, S);
+    a.nz0 = H; a.nz1 = b;
+    a.A = dZ; a.a_mn_major = 0; a.lda = S; a.a_sz0 = (int64_t)S * S; a.a_sz1 = (int64_t)H * S * S;
+    a.B = QKV + (size_t)D * ts; a.b_mn_major = 1; a.ldb = 3 * D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * D;
+    a.C = dQKV; a.ldc = 3 * D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * 3 * D;
+    a.epilogue = HK_EPI_STORE_T;
+    gemm(a, st);
+  }
+  {  // dK_h = dZ^T Q_h
+    hk_gemm_args a = gemm_args(dt, S, dh, S);
+    a.nz0 = H; a.nz1 = b;
+    a.A = dZ; a.a_mn_major = 1; a.lda = S; a.a_sz0 = (int64_t)S * S; a.a_sz1 = (int64_t)H * S * S;
+    a.B = QKV; a.b_mn_major = 1; a.ldb = 3 * D; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * D;
+    a.C = dQKV + (size_t)D * ts; a.ldc = 3 * D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * 3 * D;
+    a.epilogue = HK_EPI_STORE_T;
+    gemm(a, st);
+  }
+  // ---- QKV projection: dU = dQKV W_qkv^T; dW_qkv += U^T dQKV; db_qkv += sum dQKV
+  {
+    hk_gemm_args a = lin_dgrad(g, R, 3 * D, D, dQKV, wseg(g, W, P_WQKV));
+    a.C = dUf; a.epilogue = HK_EPI_STORE_F32;
+    gemm(a, st);
+  }
+  const uint8_t* U = stash + g.st.U;
+  if (g.stash_policy == 1) {
+    float* tmp_mean = reinterpret_cast<float*>(scratch);
+    float* tmp_rstd = tmp_mean + R;
+    layernorm_fwd(dt, R, D, Xs, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), rec, tmp_mean, tmp_rstd, st);
+    U = rec;
+  }
+  gemm(lin_wgrad(g, R, 3 * D, D, U, dQKV, gseg(g, dW, P_WQKV), first), st);
+  colsum(dt, R, 3 * D, dQKV, 3 * D, gseg(g, dW, P_BQKV), acc, scratch, st);
+  // ---- LN1 backward: dX = dX2 + LN1'(dU)
+  layernorm_bwd(dt, R, D, dUf, Xs, mean1, rstd1, wseg(g, W, P_LN1_G), dX2, dX, gseg(g, dW, P_LN1_G),
+                gseg(g, dW, P_LN1_B), acc, scratch, st);
+}
+
+}  // namespace hm

@@ -1,0 +1,741 @@
+// plan.cpp — decompose + plan (see plan.hpp).  Host-only: runs without a GPU (harmony_plan_dry).
+#include "plan.hpp"
+
+#include <algorithm>
+#include <array>
+#include <deque>
+#include <map>
+#include <sstream>
+#include <unordered_map>
+
+#include "common.hpp"
+#include "kernels/kernels.hpp"
+
+namespace hm {
+
+static const uint64_t ALIGN = 1024;  // every arena buffer 1 KiB aligned: identical code paths capped/uncapped
+
+void validate_config(const harmony_config& c) {
+  HM_CHECK(c.struct_size == sizeof(harmony_config), HARMONY_E_INVALID_ARG, "harmony_config.struct_size mismatch");
+  HM_CHECK(c.world_size >= 1 && c.world_size <= 64, HARMONY_E_INVALID_ARG, "world_size must be in 1..64");
+  HM_CHECK(c.rank >= 0 && c.rank < c.world_size, HARMONY_E_INVALID_ARG, "rank out of range");
+  HM_CHECK(c.microbatches >= 1, HARMONY_E_INVALID_ARG, "microbatches must be >= 1");
+  HM_CHECK(c.microbatch_size >= 1, HARMONY_E_INVALID_ARG, "microbatch_size must be >= 1");
+  HM_CHECK(c.precision == HARMONY_FP32 || c.precision == HARMONY_BF16_FP32MASTER, HARMONY_E_INVALID_ARG,
+           "unknown precision");
+  HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP || c.schedule == HARMONY_SCHED_PER_GPU_VIRT, HARMONY_E_INVALID_ARG,
+           "unknown schedule");
+  HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
+           "the per-GPU-virtualization baseline schedule is not built yet (SURVEY NEXT-3)");
+  HM_CHECK(c.stash_policy == 0 || c.stash_policy == 1, HARMONY_E_INVALID_ARG, "stash_policy must be 0 or 1");
+  HM_CHECK(c.weight_decay == 0.f, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
+  HM_CHECK(c.lr > 0.f && c.beta1 >= 0.f && c.beta1 < 1.f && c.beta2 >= 0.f && c.beta2 < 1.f && c.eps > 0.f,
+           HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
+}
+
+static void validate_layers(const harmony_config& c, int n, const harmony_layer_desc* d) {
+  HM_CHECK(n >= 1 && d != nullptr, HARMONY_E_INVALID_ARG, "need >= 1 layer");
+  for (int l = 0; l < n; ++l) {
+    const harmony_layer_desc& x = d[l];
+    HM_CHECK(x.d_in >= 1 && x.d_out >= 1, HARMONY_E_INVALID_ARG, "layer widths must be >= 1");
+    if (x.kind == HARMONY_LAYER_MLP) {
+      HM_CHECK(x.act >= 0 && x.act <= 2, HARMONY_E_INVALID_ARG, "unknown activation");
+      if (c.precision == HARMONY_BF16_FP32MASTER)
+        HM_CHECK(x.d_in % 8 == 0 && x.d_out % 8 == 0, HARMONY_E_UNSUPPORTED, "bf16 path needs widths % 8 == 0 (c24)");
+    } else if (x.kind == HARMONY_LAYER_TRANSFORMER) {
+      HM_CHECK(x.d_out == x.d_in, HARMONY_E_INVALID_ARG, "transformer layer needs d_out == d_in");
+      HM_CHECK(x.n_heads >= 1 && x.d_in % x.n_heads == 0, HARMONY_E_INVALID_ARG, "d % h must be 0 (c24)");
+      HM_CHECK(x.seq_len >= 1, HARMONY_E_INVALID_ARG, "seq_len must be >= 1");
+      if (c.precision == HARMONY_BF16_FP32MASTER)
+        HM_CHECK(x.d_in % 8 == 0 && (x.d_in / x.n_heads) % 8 == 0 && x.seq_len % 8 == 0, HARMONY_E_UNSUPPORTED,
+                 "bf16 path needs d, d/h and S multiples of 8 (16-byte TMA strides, c24)");
+    } else {
+      HM_CHECK(false, HARMONY_E_INVALID_ARG, "unknown layer kind");
+    }
+    if (l > 0) {
+      HM_CHECK(d[l - 1].d_out == x.d_in, HARMONY_E_INVALID_ARG, "layer widths do not chain");
+      HM_CHECK(d[l - 1].kind == x.kind, HARMONY_E_UNSUPPORTED, "mixed layer kinds in one stack");
+      if (x.kind == HARMONY_LAYER_TRANSFORMER)
+        HM_CHECK(d[l - 1].seq_len == x.seq_len, HARMONY_E_INVALID_ARG, "seq_len must match across layers");
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------ resource tracking
+namespace {
+enum ResKind : uint64_t {
+  R_BND = 1, R_TGT, R_LOSS, R_WSLOT, R_WRES, R_SSLOT, R_SRES, R_STAGE, R_STASHRES, R_DW, R_GSH,
+  H_WC, H_STATE, H_STASH, H_GRAD, R_LOSSALL
+};
+inline uint64_t key(ResKind k, uint64_t a, uint64_t b = 0) { return ((uint64_t)k << 56) | (a << 28) | b; }
+
+struct Tracker {
+  struct Res {
+    int writer = -1;
+    std::vector<int> readers;
+  };
+  std::unordered_map<uint64_t, Res> res;
+  std::vector<Op>* ops;
+
+  int add(Op op, const std::vector<uint64_t>& reads, const std::vector<uint64_t>& writes) {
+    const int idx = (int)ops->size();
+    std::vector<int> deps;
+    for (uint64_t r : reads) {
+      auto it = res.find(r);
+      if (it != res.end() && it->second.writer >= 0) deps.push_back(it->second.writer);
+    }
+    for (uint64_t w : writes) {
+      auto it = res.find(w);
+      if (it == res.end()) continue;
+      if (it->second.writer >= 0) deps.push_back(it->second.writer);
+      for (int rd : it->second.readers) deps.push_back(rd);
+    }
+    // keep only the latest dependency per other stream (streams execute in order)
+    int latest[S_NUM] = {-1, -1, -1, -1};
+    for (int dpi : deps) {
+      int s = (*ops)[dpi].stream;
+      if (s != op.stream) latest[s] = std::max(latest[s], dpi);
+    }
+    op.waits.clear();
+    for (int s = 0; s < S_NUM; ++s)
+      if (latest[s] >= 0) op.waits.push_back(latest[s]);
+    for (uint64_t r : reads) res[r].readers.push_back(idx);
+    for (uint64_t w : writes) {
+      Res& x = res[w];
+      x.writer = idx;
+      x.readers.clear();
+    }
+    ops->push_back(op);
+    return idx;
+  }
+};
+
+struct Arena {
+  uint64_t cur = 0;
+  uint64_t take(uint64_t bytes) {
+    uint64_t o = cur;
+    cur = align_up(cur + std::max<uint64_t>(bytes, 1), ALIGN);
+    return o;
+  }
+};
+}  // namespace
+
+
+// ------------------------------------------------------------------------------------ program validator
+// Independent of the resource keys used to derive the edges: every op's arena (and host-store)
+// byte ranges are recomputed from its operands, happens-before is derived from stream order
+// plus the wait edges (vector clocks), and any two unordered ops touching overlapping bytes,
+// at least one writing, count as a hazard.  (race detection.)
+namespace {
+struct Acc {
+  int space;  // 0 = arena, 1 + host buffer kind
+  int64_t idx;
+  uint64_t lo, hi;
+  bool write;
+};
+}  // namespace
+
+static std::vector<Acc> accesses(const Plan& p, const Op& o) {
+  std::vector<Acc> v;
+  auto ar = [&](uint64_t off, uint64_t bytes, bool w) {
+    if (bytes) v.push_back({0, 0, off, off + bytes, w});
+  };
+  auto hb = [&](int hbuf, int64_t idx, uint64_t off, uint64_t bytes, bool w) {
+    if (bytes) v.push_back({1 + hbuf, idx, off, off + bytes, w});
+  };
+  const uint64_t ts = p.dtype ? 2 : 4;
+  switch (o.kind) {
+    case OP_INPUT: ar(o.dev, o.bytes, true); break;
+    case OP_H2D: ar(o.dev, o.bytes, true); hb(o.hbuf, o.hidx, o.hoff, o.bytes, false); break;
+    case OP_D2H: ar(o.dev, o.bytes, false); hb(o.hbuf, o.hidx, o.hoff, o.bytes, true); break;
+    case OP_FWD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      ar(o.w, (uint64_t)lp.P * ts, false);
+      ar(o.in, (uint64_t)lp.g.rows * lp.g.desc.d_in * 4, false);
+      ar(o.out, (uint64_t)lp.g.rows * lp.g.desc.d_out * 4, true);
+      ar(o.stash, lp.g.st.total, true);
+      ar(o.ws, lp.g.ws_fwd, true);
+      break;
+    }
+    case OP_BWD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      ar(o.w, (uint64_t)lp.P * ts, false);
+      ar(o.stash, lp.g.st.total, false);
+      ar(o.in, (uint64_t)lp.g.rows * lp.g.desc.d_out * 4, false);
+      ar(o.out, (uint64_t)lp.g.rows * lp.g.desc.d_in * 4, true);
+      ar(o.dw, (uint64_t)lp.P * 4, true);
+      ar(o.ws, lp.g.ws_bwd, true);
+      break;
+    }
+    case OP_LOSS:
+      ar(o.in, (uint64_t)p.out_elems_per_mb * 4, false);
+      ar(o.tgt, (uint64_t)p.out_elems_per_mb * 4, false);
+      ar(o.out, (uint64_t)p.out_elems_per_mb * 4, true);
+      ar(o.loss, 8, true);
+      ar(p.loss_scratch, mse_scratch_bytes(), true);
+      break;
+    case OP_UPD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      ar(o.grad, (uint64_t)lp.shard * 4, false);
+      ar(o.state, lp.state_bytes, true);
+      ar(o.w + (uint64_t)p.rank * lp.shard * ts, (uint64_t)lp.shard * ts, true);
+      break;
+    }
+    case OP_ALLGATHER: ar(o.dev, (uint64_t)p.N * o.count * ts, true); break;
+    case OP_REDUCESCATTER: ar(o.dev, (uint64_t)p.N * o.count * 4, false); ar(o.grad, o.count * 4, true); break;
+    case OP_LOSS_GATHER: ar(o.dev, (uint64_t)p.N * o.count * 8, true); break;
+    case OP_LOSS_OUT: ar(o.dev, o.bytes, false); break;
+    default: break;
+  }
+  return v;
+}
+
+int validate_program(const Plan& p, std::string* first) {
+  const size_t n = p.ops.size();
+  std::vector<std::array<int, S_NUM>> vc(n);
+  std::vector<int> pos(n);
+  std::array<int, S_NUM> cnt{};
+  std::array<int, S_NUM> last{};
+  last.fill(-1);
+  for (size_t i = 0; i < n; ++i) {
+    const Op& o = p.ops[i];
+    std::array<int, S_NUM> c;
+    c.fill(-1);
+    if (last[o.stream] >= 0) c = vc[last[o.stream]];
+    for (int w : o.waits)
+      for (int s = 0; s < S_NUM; ++s) c[s] = std::max(c[s], vc[w][s]);
+    pos[i] = cnt[o.stream]++;
+    c[o.stream] = pos[i];
+    vc[i] = c;
+    last[o.stream] = (int)i;
+  }
+  auto hb = [&](size_t a, size_t b) { return vc[b][p.ops[a].stream] >= pos[a]; };
+  std::vector<std::vector<Acc>> acc(n);
+  for (size_t i = 0; i < n; ++i) acc[i] = accesses(p, p.ops[i]);
+  int hazards = 0;
+  for (size_t j = 0; j < n; ++j)
+    for (size_t i = 0; i < j; ++i) {
+      if (p.ops[i].stream == p.ops[j].stream || hb(i, j)) continue;
+      for (const Acc& a : acc[i])
+        for (const Acc& b : acc[j])
+          if ((a.write || b.write) && a.space == b.space && a.idx == b.idx && a.lo < b.hi && b.lo < a.hi) {
+            if (hazards == 0 && first)
+              *first = "ops " + std::to_string(i) + " and " + std::to_string(j) + " race on space " +
+                       std::to_string(a.space) + "[" + std::to_string(a.idx) + "]";
+            ++hazards;
+            goto next_pair;
+          }
+    next_pair:;
+    }
+  return hazards;
+}
+
+// ------------------------------------------------------------------------------------ make_plan
+Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs) {
+  validate_config(cfg);
+  validate_layers(cfg, n_layers, descs);
+  Plan p;
+  p.N = cfg.world_size;
+  p.rank = cfg.rank;
+  p.m = cfg.microbatches;
+  p.b = cfg.microbatch_size;
+  p.dtype = cfg.precision == HARMONY_BF16_FP32MASTER ? 1 : 0;
+  p.stash_policy = cfg.stash_policy;
+  p.schedule = cfg.schedule;
+  p.retain_grads = cfg.retain_grads;
+  p.cap = cfg.hbm_cap_bytes;
+  p.upd_lag = (p.N > 1 && p.schedule == HARMONY_SCHED_HARMONY_DP) ? 1 : 0;
+  const int L = n_layers, m = p.m, N = p.N, r = p.rank;
+  const uint64_t ts = p.dtype ? 2 : 4;
+
+  p.layers.resize(L);
+  int dmax = 0;
+  uint64_t ws_need = 256, maxP = 0, max_shard = 0;
+  for (int l = 0; l < L; ++l) {
+    LayerPlan& lp = p.layers[l];
+    lp.g = make_geom(descs[l], p.b, p.dtype, p.stash_policy);
+    lp.P = lp.g.n_params;
+    lp.Ppad = (int64_t)align_up((uint64_t)lp.P, (uint64_t)N * 1024);
+    lp.shard = lp.Ppad / N;
+    lp.wc_bytes = (uint64_t)lp.Ppad * ts;
+    lp.state_bytes = 3 * (uint64_t)lp.shard * 4;
+    lp.stash_res.assign(m, -1);
+    dmax = std::max({dmax, descs[l].d_in, descs[l].d_out});
+    ws_need = std::max({ws_need, lp.g.ws_fwd, lp.g.ws_bwd});
+    maxP = std::max<uint64_t>(maxP, (uint64_t)lp.Ppad);
+    max_shard = std::max<uint64_t>(max_shard, (uint64_t)lp.shard);
+    p.n_params += lp.P;
+  }
+  const int64_t rows = p.layers[0].g.rows;
+  p.d_in0 = descs[0].d_in;
+  p.d_out_last = descs[L - 1].d_out;
+  p.in_elems_per_mb = rows * descs[0].d_in;
+  p.out_elems_per_mb = rows * descs[L - 1].d_out;
+
+  // ---------------------------------------------------------------- fixed working set
+  const uint64_t bnd_stride = align_up((uint64_t)rows * dmax * 4, ALIGN);
+  const uint64_t tgt_stride = align_up((uint64_t)p.out_elems_per_mb * 4, ALIGN);
+  const int nDW = N > 1 ? 2 : 1;
+  auto fixed_bytes = [&]() {
+    uint64_t f = 0;
+    f += 2 * bnd_stride * m;                          // activation / gradient ping-pong
+    f += tgt_stride * m;                              // targets
+    f += align_up(ws_need, ALIGN);                    // one task's transients
+    f += nDW * align_up(maxP * 4, ALIGN);             // fp32 dW accumulators
+    if (N > 1) f += 2 * align_up(max_shard * 4, ALIGN);  // reduced-gradient shards
+    f += align_up((uint64_t)N * m * 8, ALIGN) + align_up(mse_scratch_bytes(), ALIGN);
+    return f;
+  };
+  const uint64_t fixed = fixed_bytes();
+
+  // ---------------------------------------------------------------- residency (late binding of memory)
+  const bool uncapped = p.cap == 0;
+  const bool baseline = p.schedule == HARMONY_SCHED_PER_GPU_VIRT;
+  uint64_t all_res = fixed;
+  for (auto& lp : p.layers) all_res += align_up(lp.wc_bytes, ALIGN) + align_up(lp.state_bytes, ALIGN) +
+                                       (uint64_t)m * align_up(lp.g.st.total, ALIGN);
+  int nW = 0, nS = 0, nG = 0;
+  {
+    uint64_t mw = 0, ms = 0, mst = 0;
+    for (auto& lp : p.layers) {
+      mw = std::max(mw, align_up(lp.wc_bytes, ALIGN));
+      ms = std::max(ms, align_up(lp.state_bytes, ALIGN));
+      mst = std::max(mst, align_up(lp.g.st.total, ALIGN));
+    }
+    p.min_ws_bytes = std::min(all_res, fixed + mw + ms + mst);
+  }
+  if (uncapped || (!baseline && all_res <= p.cap)) {
+    for (auto& lp : p.layers) {
+      lp.wc_res = 0; lp.state_res = 0;
+      for (int i = 0; i < m; ++i) lp.stash_res[i] = 0;
+    }
+  } else {
+    uint64_t maxw = 0, maxs = 0, maxst = 0;
+    for (auto& lp : p.layers) {
+      maxw = std::max(maxw, align_up(lp.wc_bytes, ALIGN));
+      maxs = std::max(maxs, align_up(lp.state_bytes, ALIGN));
+      maxst = std::max(maxst, align_up(lp.g.st.total, ALIGN));
+    }
+    HM_CHECK(p.min_ws_bytes <= p.cap, HARMONY_E_CAP_TOO_SMALL,
+             "hbm_cap_bytes " + std::to_string(p.cap) + " < minimum working set " + std::to_string(p.min_ws_bytes));
+    // slot counts in order of preference (double buffering needs memory)
+    const int pref[][3] = {{2, 2, 2}, {2, 1, 2}, {2, 1, 1}, {1, 1, 2}, {1, 1, 1}};
+    for (auto& c : pref) {
+      if (fixed + c[0] * maxw + c[1] * maxs + c[2] * maxst <= p.cap) { nW = c[0]; nS = c[1]; nG = c[2]; break; }
+    }
+    // fill residency, then reclaim slots of classes that became fully resident; iterate
+    for (int pass = 0; pass < 4; ++pass) {
+      for (auto& lp : p.layers) {
+        lp.wc_res = -1; lp.state_res = -1;
+        std::fill(lp.stash_res.begin(), lp.stash_res.end(), -1);
+      }
+      uint64_t used = fixed + nW * maxw + nS * maxs + nG * maxst;
+      uint64_t room = p.cap > used ? p.cap - used : 0;
+      if (!baseline) {
+        // compute weights: 3 B of transfer saved per resident byte; backward order
+        for (int l = L - 1; l >= 0; --l) {
+          uint64_t sz = align_up(p.layers[l].wc_bytes, ALIGN);
+          if (sz <= room) { p.layers[l].wc_res = 0; room -= sz; }
+        }
+        for (int l = L - 1; l >= 0; --l) {  // master/m/v: 2 B saved per byte
+          uint64_t sz = align_up(p.layers[l].state_bytes, ALIGN);
+          if (sz <= room) { p.layers[l].state_res = 0; room -= sz; }
+        }
+      }
+      for (int l = L - 1; l >= 0; --l)  // stash: LIFO (consumed first in the backward)
+        for (int i = 0; i < m; ++i) {
+          uint64_t sz = align_up(p.layers[l].g.st.total, ALIGN);
+          if (sz <= room) { p.layers[l].stash_res[i] = 0; room -= sz; }
+        }
+      // recompute the slot sizes from what is still streamed
+      uint64_t nmaxw = 0, nmaxs = 0, nmaxst = 0;
+      for (auto& lp : p.layers) {
+        if (lp.wc_res < 0) nmaxw = std::max(nmaxw, align_up(lp.wc_bytes, ALIGN));
+        if (lp.state_res < 0) nmaxs = std::max(nmaxs, align_up(lp.state_bytes, ALIGN));
+        for (int i = 0; i < m; ++i)
+          if (lp.stash_res[i] < 0) nmaxst = std::max(nmaxst, align_up(lp.g.st.total, ALIGN));
+      }
+      bool changed = nmaxw != maxw || nmaxs != maxs || nmaxst != maxst;
+      maxw = nmaxw; maxs = nmaxs; maxst = nmaxst;
+      if (maxw == 0) nW = 0;
+      if (maxs == 0) nS = 0;
+      if (maxst == 0) nG = 0;
+      if (!changed) break;
+      // slots shrank: retry preferences with the new sizes (never below one slot per streamed class)
+      for (auto& c : pref) {
+        int w = maxw ? c[0] : 0, s = maxs ? c[1] : 0, g2 = maxst ? c[2] : 0;
+        if (fixed + w * maxw + s * maxs + g2 * maxst <= p.cap) { nW = w; nS = s; nG = g2; break; }
+      }
+    }
+    p.wslot_bytes = maxw; p.sslot_bytes = maxs; p.stage_bytes = maxst;
+  }
+  // A lagged update (N > 1) writes the compute copy back into the slot its backward used;
+  // with a single weight slot that slot already holds the next layer, so update immediately.
+  if (nW == 1) p.upd_lag = 0;
+
+  // ---------------------------------------------------------------- arena layout
+  Arena a;
+  p.bnd_row_stride = bnd_stride;
+  p.tgt_row_stride = tgt_stride;
+  p.bnd_bytes = bnd_stride * m;
+  p.bnd[0] = a.take(p.bnd_bytes);
+  p.bnd[1] = a.take(p.bnd_bytes);
+  p.tgt = a.take(tgt_stride * m);
+  p.ws_bytes = ws_need;
+  p.ws = a.take(ws_need);
+  for (int j = 0; j < nDW; ++j) p.dw[j] = a.take(maxP * 4);
+  if (N > 1) for (int j = 0; j < 2; ++j) p.gsh[j] = a.take(max_shard * 4);
+  p.loss = a.take((uint64_t)N * m * 8);
+  p.loss_scratch = a.take(mse_scratch_bytes());
+  for (int j = 0; j < nW; ++j) p.wslot.push_back(a.take(p.wslot_bytes));
+  for (int j = 0; j < nS; ++j) p.sslot.push_back(a.take(p.sslot_bytes));
+  for (int j = 0; j < nG; ++j) p.stage.push_back(a.take(p.stage_bytes));
+  for (auto& lp : p.layers) {
+    if (lp.wc_res >= 0) lp.wc_res = (int64_t)a.take(lp.wc_bytes);
+    if (lp.state_res >= 0) lp.state_res = (int64_t)a.take(lp.state_bytes);
+  }
+  for (int l = L - 1; l >= 0; --l)
+    for (int i = 0; i < m; ++i)
+      if (p.layers[l].stash_res[i] >= 0) p.layers[l].stash_res[i] = (int64_t)a.take(p.layers[l].g.st.total);
+  p.arena_bytes = a.cur;
+  HM_CHECK(uncapped || p.arena_bytes <= p.cap, HARMONY_E_CAP_TOO_SMALL, "internal: arena layout exceeds the cap");
+
+  // ---------------------------------------------------------------- program
+  Tracker tr;
+  tr.ops = &p.ops;
+  auto bnd_row = [&](int buf, int i) { return p.bnd[buf] + (uint64_t)i * bnd_stride; };
+
+  // Input items (prefetchable swap-ins) and their slot occupancies.
+  struct Item {
+    int need = 0;                 // task index that needs it
+    int release = -1;             // task after which the slot is free
+    std::vector<std::pair<Op, std::pair<std::vector<uint64_t>, std::vector<uint64_t>>>> ops;
+  };
+  struct Task {
+    Op op;
+    std::vector<uint64_t> rd, wr;
+    std::vector<std::pair<Op, std::pair<std::vector<uint64_t>, std::vector<uint64_t>>>> post;
+  };
+  std::vector<Task> tasks;
+  std::vector<Item> items;
+
+  // slot bookkeeping: last task index using each slot
+  std::vector<int> wslot_last(nW, -1), sslot_last(nS, -1), stage_last(nG, -1);
+  int wnext = 0, snext = 0, gnext = 0;
+
+  // weight location for each layer use (fwd / bwd)
+  auto weight_use = [&](int l, int need_task, int& slot) -> uint64_t {
+    LayerPlan& lp = p.layers[l];
+    if (lp.wc_res >= 0) { slot = -1; return (uint64_t)lp.wc_res; }
+    slot = wnext;
+    wnext = (wnext + 1) % nW;
+    Item it;
+    it.need = need_task;
+    it.release = wslot_last[slot];
+    const uint64_t dst = p.wslot[slot];
+    const uint64_t sh_bytes = (uint64_t)lp.shard * ts;
+    Op h;
+    h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_WEIGHT; h.layer = l;
+    h.hbuf = HB_WC; h.hidx = l; h.hoff = 0; h.dev = dst + (uint64_t)r * sh_bytes; h.bytes = sh_bytes;
+    it.ops.push_back({h, {{key(H_WC, l)}, {key(R_WSLOT, slot)}}});
+    if (N > 1) {
+      Op g;
+      g.kind = OP_ALLGATHER; g.stream = S_COMM; g.cat = CAT_WEIGHT; g.layer = l;
+      g.dev = dst; g.count = (uint64_t)lp.shard; g.bytes = sh_bytes * (N - 1);
+      it.ops.push_back({g, {{key(R_WSLOT, slot)}, {key(R_WSLOT, slot)}}});
+    }
+    items.push_back(it);
+    return dst;
+  };
+  auto wkey = [&](int l, int slot) { return slot >= 0 ? key(R_WSLOT, slot) : key(R_WRES, l); };
+
+  // ---- forward
+  std::vector<int> fwd_wslot(L, -1);
+  {
+    Task t;  // inputs are issued as the first ops (not prefetch items)
+    (void)t;
+  }
+  for (int l = 0; l < L; ++l) {
+    LayerPlan& lp = p.layers[l];
+    const int in_buf = l % 2, out_buf = (l + 1) % 2;
+    for (int i = 0; i < m; ++i) {
+      int slot = -1;
+      uint64_t wdev;
+      if (baseline || i == 0) wdev = weight_use(l, (int)tasks.size(), slot);  // grouping: one swap-in per layer
+      else { slot = fwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
+      fwd_wslot[l] = slot;
+      Task t;
+      t.op.kind = OP_FWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i;
+      t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws;
+      t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
+      t.wr = {key(R_BND, out_buf, i)};
+      if (lp.stash_res[i] >= 0) {
+        t.op.stash = (uint64_t)lp.stash_res[i];
+        t.wr.push_back(key(R_STASHRES, l, i));
+      } else {
+        int g = gnext;
+        gnext = (gnext + 1) % nG;
+        t.op.stash = p.stage[g];
+        t.wr.push_back(key(R_STAGE, g));
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = l; d.mb = i;
+        d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + i; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
+        t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, i)}}});
+        stage_last[g] = (int)tasks.size();
+      }
+      if (slot >= 0) wslot_last[slot] = (int)tasks.size();
+      tasks.push_back(t);
+    }
+  }
+  // ---- loss
+  const int Lb = L % 2, dYb = (L + 1) % 2;
+  for (int i = 0; i < m; ++i) {
+    Task t;
+    t.op.kind = OP_LOSS; t.op.stream = S_COMPUTE; t.op.mb = i;
+    t.op.in = bnd_row(Lb, i); t.op.tgt = p.tgt + (uint64_t)i * tgt_stride; t.op.out = bnd_row(dYb, i);
+    t.op.loss = p.loss + (uint64_t)(r * m + i) * 8;
+    t.rd = {key(R_BND, Lb, i), key(R_TGT, i)};
+    t.wr = {key(R_BND, dYb, i), key(R_LOSS, i)};
+    if (i == m - 1) {
+      Op o;
+      if (N > 1) {
+        o.kind = OP_LOSS_GATHER; o.stream = S_COMM; o.dev = p.loss; o.count = (uint64_t)m; o.bytes = (uint64_t)m * 8 * (N - 1);
+        std::vector<uint64_t> rds;
+        for (int j = 0; j < m; ++j) rds.push_back(key(R_LOSS, j));
+        t.post.push_back({o, {rds, {key(R_LOSSALL, 0)}}});
+        Op d;
+        d.kind = OP_LOSS_OUT; d.stream = S_D2H; d.cat = CAT_OUTPUT; d.dev = p.loss; d.bytes = (uint64_t)N * m * 8;
+        t.post.push_back({d, {{key(R_LOSSALL, 0)}, {}}});
+      } else {
+        o.kind = OP_LOSS_OUT; o.stream = S_D2H; o.cat = CAT_OUTPUT; o.dev = p.loss; o.bytes = (uint64_t)m * 8;
+        std::vector<uint64_t> rds;
+        for (int j = 0; j < m; ++j) rds.push_back(key(R_LOSS, j));
+        t.post.push_back({o, {rds, {}}});
+      }
+    }
+    tasks.push_back(t);
+  }
+  // ---- backward + JIT update
+  std::vector<int> bwd_wslot(L, -1);
+  std::vector<int> pending_upd;
+  auto emit_upd = [&](int l) {
+    LayerPlan& lp = p.layers[l];
+    Task t;
+    t.op.kind = OP_UPD; t.op.stream = S_COMPUTE; t.op.layer = l;
+    const int j = l % nDW;
+    uint64_t gkey = key(R_DW, j);
+    if (N > 1) { t.op.grad = p.gsh[l % 2]; gkey = key(R_GSH, l % 2); }
+    else t.op.grad = p.dw[j];
+    t.rd = {gkey};
+    int sslot = -1;
+    if (lp.state_res >= 0) {
+      t.op.state = (uint64_t)lp.state_res;
+      t.rd.push_back(key(R_SRES, l));
+      t.wr.push_back(key(R_SRES, l));
+    } else {
+      sslot = snext;
+      snext = (snext + 1) % nS;
+      Item it;
+      it.need = (int)tasks.size();
+      it.release = sslot_last[sslot];
+      Op h;
+      h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STATE; h.layer = l;
+      h.hbuf = HB_STATE; h.hidx = l; h.dev = p.sslot[sslot]; h.bytes = lp.state_bytes;
+      it.ops.push_back({h, {{key(H_STATE, l)}, {key(R_SSLOT, sslot)}}});
+      items.push_back(it);
+      t.op.state = p.sslot[sslot];
+      t.rd.push_back(key(R_SSLOT, sslot));
+      t.wr.push_back(key(R_SSLOT, sslot));
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STATE; d.layer = l;
+      d.hbuf = HB_STATE; d.hidx = l; d.dev = p.sslot[sslot]; d.bytes = lp.state_bytes;
+      t.post.push_back({d, {{key(R_SSLOT, sslot)}, {key(H_STATE, l)}}});
+      sslot_last[sslot] = (int)tasks.size();
+    }
+    // the compute copy this rank's shard is written into
+    const int wsl = bwd_wslot[l];
+    const uint64_t sh_bytes = (uint64_t)lp.shard * ts;
+    if (lp.wc_res >= 0) {
+      t.op.w = (uint64_t)lp.wc_res;
+      t.wr.push_back(key(R_WRES, l));
+      if (N > 1) {
+        Op g;
+        g.kind = OP_ALLGATHER; g.stream = S_COMM; g.cat = CAT_WEIGHT; g.layer = l;
+        g.dev = (uint64_t)lp.wc_res; g.count = (uint64_t)lp.shard; g.bytes = sh_bytes * (N - 1);
+        t.post.push_back({g, {{key(R_WRES, l)}, {key(R_WRES, l)}}});
+      }
+    } else {
+      t.op.w = p.wslot[wsl];
+      t.wr.push_back(key(R_WSLOT, wsl));
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l;
+      d.hbuf = HB_WC; d.hidx = l; d.dev = p.wslot[wsl] + (uint64_t)r * sh_bytes; d.bytes = sh_bytes;
+      t.post.push_back({d, {{key(R_WSLOT, wsl)}, {key(H_WC, l)}}});
+      wslot_last[wsl] = (int)tasks.size();
+    }
+    if (p.retain_grads) {
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_GRAD; d.layer = l;
+      d.hbuf = HB_GRAD; d.hidx = l; d.dev = t.op.grad; d.bytes = (uint64_t)lp.shard * 4;
+      t.post.push_back({d, {{gkey}, {key(H_GRAD, l)}}});
+    }
+    tasks.push_back(t);
+  };
+
+  for (int l = L - 1; l >= 0; --l) {
+    LayerPlan& lp = p.layers[l];
+    const int in_buf = l % 2, out_buf = (l + 1) % 2;
+    const int j = l % nDW;
+    for (int i = 0; i < m; ++i) {
+      int slot = -1;
+      uint64_t wdev;
+      if (baseline || i == 0) wdev = weight_use(l, (int)tasks.size(), slot);
+      else { slot = bwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
+      bwd_wslot[l] = slot;
+      Task t;
+      t.op.kind = OP_BWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i; t.op.first = i == 0;
+      t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws; t.op.dw = p.dw[j];
+      t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
+      t.wr = {key(R_BND, out_buf, i), key(R_DW, j)};
+      if (i > 0) t.rd.push_back(key(R_DW, j));
+      if (lp.stash_res[i] >= 0) {
+        t.op.stash = (uint64_t)lp.stash_res[i];
+        t.rd.push_back(key(R_STASHRES, l, i));
+      } else {
+        int g = gnext;
+        gnext = (gnext + 1) % nG;
+        Item it;
+        it.need = (int)tasks.size();
+        it.release = stage_last[g];
+        Op h;
+        h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STASH; h.layer = l; h.mb = i;
+        h.hbuf = HB_STASH; h.hidx = (int64_t)l * m + i; h.dev = p.stage[g]; h.bytes = lp.g.st.total;
+        it.ops.push_back({h, {{key(H_STASH, l, i)}, {key(R_STAGE, g)}}});
+        items.push_back(it);
+        t.op.stash = p.stage[g];
+        t.rd.push_back(key(R_STAGE, g));
+        stage_last[g] = (int)tasks.size();
+      }
+      if (slot >= 0) wslot_last[slot] = (int)tasks.size();
+      if (i == m - 1 && N > 1) {
+        Op rs;
+        rs.kind = OP_REDUCESCATTER; rs.stream = S_COMM; rs.cat = CAT_GRAD; rs.layer = l;
+        rs.dev = p.dw[j]; rs.grad = p.gsh[l % 2]; rs.count = (uint64_t)lp.shard;
+        rs.bytes = (uint64_t)lp.shard * 4 * (N - 1);
+        t.post.push_back({rs, {{key(R_DW, j)}, {key(R_GSH, l % 2)}}});
+      }
+      tasks.push_back(t);
+    }
+    if (!baseline) {
+      pending_upd.push_back(l);
+      while ((int)pending_upd.size() > p.upd_lag) {
+        emit_upd(pending_upd.front());
+        pending_upd.erase(pending_upd.begin());
+      }
+    } else {
+      pending_upd.push_back(l);  // baseline: every update after the whole backward
+    }
+  }
+  for (int l : pending_upd) emit_upd(l);
+
+  // ---- merge tasks and prefetch items into one program
+  {
+    // inputs first (user X into the layer-0 activation rows, targets)
+    Op x;
+    x.kind = OP_INPUT; x.stream = S_H2D; x.cat = CAT_INPUT; x.hbuf = HB_USER_X; x.dev = p.bnd[0];
+    x.bytes = (uint64_t)p.in_elems_per_mb * 4;
+    for (int i = 0; i < m; ++i) {
+      Op xi = x;
+      xi.mb = i; xi.dev = bnd_row(0, i); xi.hoff = (uint64_t)i * p.in_elems_per_mb * 4;
+      tr.add(xi, {}, {key(R_BND, 0, i)});
+    }
+    for (int i = 0; i < m; ++i) {
+      Op ti = x;
+      ti.hbuf = HB_USER_T; ti.mb = i; ti.dev = p.tgt + (uint64_t)i * tgt_stride;
+      ti.hoff = (uint64_t)i * p.out_elems_per_mb * 4; ti.bytes = (uint64_t)p.out_elems_per_mb * 4;
+      tr.add(ti, {}, {key(R_TGT, i)});
+    }
+    // items are created in need order per class; merge them by need
+    std::stable_sort(items.begin(), items.end(), [](const Item& a2, const Item& b2) { return a2.need < b2.need; });
+    size_t next = 0;
+    auto emit_item = [&](Item& it) {
+      for (auto& o : it.ops) tr.add(o.first, o.second.first, o.second.second);
+    };
+    for (int k = 0; k < (int)tasks.size(); ++k) {
+      while (next < items.size() && items[next].need <= k) emit_item(items[next++]);
+      Task& t = tasks[k];
+      tr.add(t.op, t.rd, t.wr);
+      for (auto& o : t.post) tr.add(o.first, o.second.first, o.second.second);
+      while (next < items.size() && items[next].release <= k) emit_item(items[next++]);
+    }
+    while (next < items.size()) emit_item(items[next++]);
+  }
+  // events: one per op that another stream waits on
+  {
+    std::vector<int> ev(p.ops.size(), -1);
+    int ne = 0;
+    for (auto& o : p.ops)
+      for (int w : o.waits)
+        if (ev[w] < 0) ev[w] = ne++;
+    for (size_t i = 0; i < p.ops.size(); ++i) p.ops[i].event = ev[i];
+    p.n_events = ne;
+  }
+
+  // ---------------------------------------------------------------- summary
+  harmony_plan_summary& s = p.summary;
+  s.arena_bytes = p.arena_bytes;
+  s.min_working_set_bytes = p.min_ws_bytes;
+  s.n_params = p.n_params;
+  s.weight_slots = nW; s.state_slots = nS; s.stash_slots = nG;
+  double fl = 0;
+  for (auto& lp : p.layers) {
+    s.total_weight_bytes += lp.wc_bytes;
+    s.total_state_bytes += lp.state_bytes;
+    s.total_stash_bytes += (uint64_t)m * lp.g.st.total;
+    if (lp.wc_res >= 0) s.resident_weight_bytes += lp.wc_bytes;
+    if (lp.state_res >= 0) s.resident_state_bytes += lp.state_bytes;
+    for (int i = 0; i < m; ++i)
+      if (lp.stash_res[i] >= 0) s.resident_stash_bytes += lp.g.st.total;
+    fl += 3.0 * lp.g.flops_fwd * m;
+  }
+  s.flops_per_step = (uint64_t)fl;
+  for (auto& o : p.ops) {
+    const bool copy_in = o.kind == OP_H2D || o.kind == OP_INPUT;
+    const bool copy_out = o.kind == OP_D2H || o.kind == OP_LOSS_OUT;
+    if (copy_in) s.pred_h2d_bytes += o.bytes;
+    if (copy_out) s.pred_d2h_bytes += o.bytes;
+    if (copy_in && o.cat == CAT_WEIGHT) s.pred_h2d_weight_bytes += o.bytes;
+    if (copy_out && o.cat == CAT_WEIGHT) s.pred_d2h_weight_bytes += o.bytes;
+    if (o.stream == S_COMPUTE) s.n_compute_ops++;
+    else if (o.stream == S_COMM) s.n_comm_ops++;
+    else s.n_copy_ops++;
+  }
+  s.n_ops = (int32_t)p.ops.size();
+  std::string why;
+  s.hazards = validate_program(p, &why);
+  p.hazard_msg = why;
+  return p;
+}
+
+std::string dump_plan(const Plan& p) {
+  static const char* kn[] = {"INPUT", "H2D", "D2H", "FWD", "LOSS", "BWD", "UPD", "ALLGATHER", "REDUCESCATTER",
+                             "LOSS_GATHER", "LOSS_OUT"};
+  static const char* sn[] = {"compute", "h2d", "d2h", "comm"};
+  static const char* cn[] = {"weight", "state", "stash", "input", "output", "grad", "-"};
+  std::ostringstream os;
+  os << "# plan N=" << p.N << " rank=" << p.rank << " m=" << p.m << " b=" << p.b << " dtype=" << p.dtype
+     << " cap=" << p.cap << " arena=" << p.arena_bytes << " wslots=" << p.wslot.size() << " sslots=" << p.sslot.size()
+     << " stage=" << p.stage.size() << " ops=" << p.ops.size() << " events=" << p.n_events << "\n";
+  for (size_t i = 0; i < p.ops.size(); ++i) {
+    const Op& o = p.ops[i];
+    os << i << " " << kn[o.kind] << " " << sn[o.stream] << " cat=" << cn[o.cat] << " l=" << o.layer << " i=" << o.mb
+       << " bytes=" << o.bytes;
+    if (o.kind == OP_BWD) os << " first=" << o.first;
+    os << " waits=";
+    for (size_t k = 0; k < o.waits.size(); ++k) os << (k ? "," : "") << o.waits[k];
+    os << "\n";
+  }
+  return os.str();
+}
+
+}  // namespace hm

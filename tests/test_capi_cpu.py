@@ -1,0 +1,204 @@
+"""The C-ABI library on a host without a GPU: it loads, exports every declared symbol, its
+ABI structs match the binding, and the host-only planner (harmony_plan_dry) builds programs
+with the paper's scheduling properties (grouping, JIT update, swap volumes, Fig. 5(a) swap
+sets) and no data races (independent byte-range validator)."""
+import ctypes as C
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from paper_conf_hotos_lipmk21_b200 import harmony as H
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    names = set()
+    for h in ("harmony.h", "harmony_kernels.h"):
+        src = open(os.path.join(ROOT, "include", h)).read()
+        src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+        for m in re.finditer(r"^\s*(?:const\s+)?[A-Za-z_][A-Za-z0-9_]*\s*\**\s+\**\s*((?:harmony|hk)_[a-z0-9_]+)\s*\(",
+                             src, flags=re.M):
+            names.add(m.group(1))
+    return sorted(names)
+
+
+def test_library_loads_and_exports_every_declared_symbol():
+    L = H.lib()
+    names = declared_functions()
+    assert len(names) >= 20, names
+    for n in names:
+        assert hasattr(L, n), f"libharmony.so does not export {n}"
+    assert L.harmony_abi_version() == 1
+
+
+def test_abi_struct_sizes_match_binding():
+    out = (C.c_uint64 * 5)()
+    H.lib().harmony_abi_sizes(out)
+    assert list(out) == [C.sizeof(H.harmony_config), C.sizeof(H.harmony_layer_desc),
+                         C.sizeof(H.harmony_step_stats), C.sizeof(H.harmony_plan_summary), C.sizeof(H.hk_gemm_args)]
+
+
+def test_library_is_built_for_sm100a():
+    import subprocess
+    out = subprocess.run(["cuobjdump", "-lelf", H.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run(["cuobjdump", "-sass", H.LIB_PATH], capture_output=True, text=True).stdout
+    assert "UTCHMMA" in sass and "UTMALDG" in sass and "LDTM" in sass  # tcgen05.mma, TMA, tcgen05.ld
+
+
+def plan(descs, **kw):
+    cfg = H.make_config(**kw)
+    s, txt = H.harmony_plan_dry(cfg, descs)
+    ops = []
+    for line in txt.splitlines()[1:]:
+        f = line.split()
+        d = dict(kv.split("=", 1) for kv in f[3:])
+        ops.append(dict(idx=int(f[0]), kind=f[1], stream=f[2], cat=d["cat"], l=int(d["l"]), i=int(d["i"]),
+                        bytes=int(d["bytes"]), waits=[int(w) for w in d["waits"].split(",") if w]))
+    return s, ops
+
+
+MLP = synth.mlp_stack(4, 256)
+CFG1 = dict(microbatches=4, microbatch_size=8, hbm_cap_bytes=synth.CONFIGS["cfg1"]["cap"])
+
+
+def min_cap(descs, **kw):
+    s, _ = plan(descs, **dict(kw, hbm_cap_bytes=1 << 40))
+    return s.min_working_set_bytes
+
+
+@pytest.mark.parametrize("kw", [CFG1, dict(CFG1, hbm_cap_bytes=0), dict(CFG1, microbatches=1, microbatch_size=32),
+                                dict(CFG1, hbm_cap_bytes=3_000_000), dict(CFG1, retain_grads=1)])
+def test_plans_are_hazard_free(kw):
+    s, ops = plan(MLP, **kw)
+    assert s.hazards == 0
+    assert s.arena_bytes <= (kw["hbm_cap_bytes"] or 1 << 62)
+
+
+def test_transformer_plans_hazard_free_over_caps():
+    descs = synth.transformer_stack(6, 64, 4, 16, True)
+    base = min_cap(descs, microbatches=3, microbatch_size=2, precision=1)
+    for f in (1.0, 1.3, 2.0, 3.0, 6.0):
+        s, _ = plan(descs, microbatches=3, microbatch_size=2, precision=1, hbm_cap_bytes=int(base * f))
+        assert s.hazards == 0
+
+
+def test_cap_too_small_is_reported():
+    cap = min_cap(MLP, **dict(CFG1))
+    with pytest.raises(H.HarmonyError) as e:
+        plan(MLP, **dict(CFG1, hbm_cap_bytes=cap - 1))
+    assert e.value.code == H.HARMONY_E_CAP_TOO_SMALL
+    s, _ = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap))
+    assert s.hazards == 0
+
+
+def test_harmony_dp_weight_swap_volume_is_3W():
+    """Harmony-DP swaps W in once for the forward and once for the backward (grouping)
+    and out once after the update (JIT): 3N|W| per iteration; here N = 1 and nothing resident."""
+    cap = min_cap(MLP, **CFG1)
+    s, ops = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap))
+    assert s.resident_weight_bytes == 0
+    Wb = s.total_weight_bytes
+    assert s.pred_h2d_weight_bytes + s.pred_d2h_weight_bytes == oracle.weight_swap_harmony_dp(Wb, 4, 1)
+    assert s.pred_h2d_weight_bytes == 2 * Wb and s.pred_d2h_weight_bytes == Wb
+    assert s.pred_h2d_weight_bytes + s.pred_d2h_weight_bytes < oracle.weight_swap_baseline_dp(Wb, 4, 1)
+
+
+@pytest.mark.parametrize("m", [1, 2, 4, 8])
+def test_grouping_weight_traffic_independent_of_m(m):
+    """a task runs over its group of m microbatches back to back, so W is swapped once."""
+    cap = min_cap(MLP, microbatches=8, microbatch_size=4)
+    s, ops = plan(MLP, microbatches=m, microbatch_size=4, hbm_cap_bytes=cap)
+    assert s.pred_h2d_weight_bytes == 2 * s.total_weight_bytes - 2 * s.resident_weight_bytes
+    n_w_in = sum(1 for o in ops if o["kind"] == "H2D" and o["cat"] == "weight")
+    streamed_layers = 4 - s.resident_weight_bytes // (s.total_weight_bytes // 4)
+    assert n_w_in == 2 * streamed_layers  # one swap-in per layer per pass, whatever m is
+
+
+def test_jit_update_right_after_backward():
+    """UPD(l) is scheduled right after BWD(l, m) — before any BWD of layer l-1."""
+    s, ops = plan(MLP, **CFG1)
+    comp = [o for o in ops if o["stream"] == "compute"]
+    seq = [(o["kind"], o["l"], o["i"]) for o in comp]
+    for l in range(4):
+        u = seq.index(("UPD", l, -1))
+        last_b = max(k for k, t in enumerate(seq) if t[0] == "BWD" and t[1] == l)
+        assert u == last_b + 1
+        if l > 0:
+            assert u < min(k for k, t in enumerate(seq) if t[0] == "BWD" and t[1] == l - 1)
+
+
+def test_no_gradient_bytes_cross_pcie_and_swap_sets_follow_fig5a():
+    """Fig. 5(a) / readings c5, c6: dW stays resident across the group (0 bytes), reset on device;
+    forward swaps in W, swaps out stash; backward swaps in W and stash; update swaps K in and W', K' out."""
+    cap = min_cap(MLP, **CFG1)
+    s, ops = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap))
+    assert not any(o["cat"] == "grad" and o["kind"] in ("H2D", "D2H") for o in ops)
+    compute = {o["idx"]: o for o in ops if o["stream"] == "compute"}
+    for o in ops:
+        if o["kind"] == "D2H":
+            assert o["cat"] in ("stash", "state", "weight")
+            src = [compute[w] for w in o["waits"] if w in compute]
+            assert src, o
+            task = src[-1]["kind"]
+            assert (o["cat"], task) in {("stash", "FWD"), ("state", "UPD"), ("weight", "UPD")}, (o, task)
+        if o["kind"] == "H2D":
+            assert o["cat"] in ("stash", "state", "weight")
+
+
+def test_uncapped_moves_only_inputs_and_loss():
+    s, ops = plan(MLP, **dict(CFG1, hbm_cap_bytes=0))
+    assert {o["kind"] for o in ops if o["stream"] in ("h2d", "d2h")} == {"INPUT", "LOSS_OUT"}
+    assert s.pred_h2d_bytes == 2 * 32 * 256 * 4 and s.pred_d2h_bytes == 4 * 8
+
+
+def test_stash_residency_is_lifo():
+    """The last layers' stash (consumed first by the backward) is the one kept resident."""
+    descs = synth.transformer_stack(8, 64, 4, 16, False)
+    base = min_cap(descs, microbatches=2, microbatch_size=2, precision=1)
+    s, ops = plan(descs, microbatches=2, microbatch_size=2, precision=1, hbm_cap_bytes=int(base * 8))
+    spilled = {(o["l"], o["i"]) for o in ops if o["kind"] == "D2H" and o["cat"] == "stash"}
+    if spilled and s.resident_stash_bytes:
+        assert max(l for l, _ in spilled) < 7
+
+
+def test_config_validation_errors():
+    with pytest.raises(H.HarmonyError) as e:
+        plan([synth.LayerDesc(1, 64, 64, n_heads=5, seq_len=8)], microbatches=1, microbatch_size=1)
+    assert e.value.code == H.HARMONY_E_INVALID_ARG  # d % h != 0
+    with pytest.raises(H.HarmonyError) as e:
+        plan([synth.LayerDesc(0, 12, 12)], microbatches=1, microbatch_size=1, precision=1)
+    assert e.value.code == H.HARMONY_E_UNSUPPORTED  # bf16 needs widths % 8
+    with pytest.raises(H.HarmonyError) as e:
+        plan(MLP, microbatches=1, microbatch_size=1, weight_decay=0.1)
+    assert e.value.code == H.HARMONY_E_UNSUPPORTED
+    with pytest.raises(H.HarmonyError) as e:
+        plan([synth.LayerDesc(0, 8, 16), synth.LayerDesc(0, 8, 8)], microbatches=1, microbatch_size=1)
+    assert e.value.code == H.HARMONY_E_INVALID_ARG  # widths do not chain
+
+
+def test_init_without_gpu_fails_cleanly():
+    cfg = H.make_config(microbatches=1, microbatch_size=1)
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("GPU present")
+    except Exception:
+        pass
+    with pytest.raises(H.HarmonyError) as e:
+        H.harmony_init(cfg)
+    assert e.value.code in (H.HARMONY_E_CUDA, H.HARMONY_E_INVALID_ARG)
+
+
+def test_plan_scales_to_paper_configs():
+    for name in ("cfg2", "cfg3"):
+        c = synth.CONFIGS[name]
+        s, _ = plan(c["descs"](), microbatches=c["m"], microbatch_size=c["batch"] // c["m"], precision=1,
+                    hbm_cap_bytes=c["cap"])
+        assert s.hazards == 0 and s.arena_bytes <= c["cap"]
+        assert s.pred_h2d_bytes > 30e9  # host-link bound

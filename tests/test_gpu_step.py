@@ -1,0 +1,201 @@
+"""End-to-end parity of the swapped, microbatched, JIT-updated step (the C ABI) with the plain
+full-batch fp64 oracle, on a B200.
+
+Tolerances (BASELINE.json north_star, reading c16): relative L2 per tensor <= 1e-5 on the fp32
+path, <= 2e-2 on the bf16 tensor-core path, for the loss, every gradient, W, m and sqrt(v) after
+each of 3 steps.  Capped (swapping) and uncapped runs must be bit-identical (reading c21)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from synth import LayerDesc, LAYER_MLP, ACT_RELU, ACT_NONE, pack, unpack
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+from paper_conf_hotos_lipmk21_b200 import harmony as H  # noqa: E402
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64); b = np.asarray(b, np.float64)
+    nb = np.linalg.norm(b)
+    return np.linalg.norm(a - b) / (nb if nb > 1e-30 else 1.0)
+
+
+def run_gpu(descs, params, batches, **cfg):
+    """Run len(batches) steps; returns per-step (loss, grads, W, m, v, stats)."""
+    out = []
+    with H.Harmony(descs, params, retain_grads=1, **cfg) as h:
+        for X, T in batches:
+            loss, st = h.step(np.ascontiguousarray(X), np.ascontiguousarray(T))
+            out.append(dict(loss=loss, stats=st.as_dict(),
+                            g=[h.read(l, H.HARMONY_GRAD) for l in range(len(descs))],
+                            W=[h.read(l, H.HARMONY_PARAM) for l in range(len(descs))],
+                            m=[h.read(l, H.HARMONY_ADAM_M) for l in range(len(descs))],
+                            v=[h.read(l, H.HARMONY_ADAM_V) for l in range(len(descs))]))
+        plan = h.plan().as_dict()
+    return out, plan
+
+
+def run_oracle(descs, params, batches, lr=1e-3):
+    P = [p.astype(np.float64) for p in params]
+    st = oracle.AdamState.zeros(P)
+    out = []
+    for X, T in batches:
+        loss, grads, P, st = oracle.train_step(descs, P, st, X.astype(np.float64), T.astype(np.float64), lr=lr)
+        out.append(dict(loss=loss, g=grads, W=P, m=st.m, v=st.v))
+    return out
+
+
+def compare(gpu, ref, tol):
+    worst = {}
+    for s, (a, b) in enumerate(zip(gpu, ref)):
+        worst["loss"] = max(worst.get("loss", 0), abs(a["loss"] - b["loss"]) / abs(b["loss"]))
+        for key in ("g", "W", "m"):
+            for x, y in zip(a[key], b[key]):
+                worst[key] = max(worst.get(key, 0), rel(x, y))
+        for x, y in zip(a["v"], b["v"]):
+            worst["sqrt_v"] = max(worst.get("sqrt_v", 0), rel(np.sqrt(np.maximum(x, 0)), np.sqrt(y)))
+    for k, v in worst.items():
+        assert v <= tol, (k, v, worst)
+    return worst
+
+
+def batches_for(descs, B, steps, precision):
+    return [synth.gen_batch(descs, B, t, precision) for t in range(1, steps + 1)]
+
+
+def bitwise_equal(a, b):
+    for s1, s2 in zip(a, b):
+        assert s1["loss"] == s2["loss"]
+        for key in ("g", "W", "m", "v"):
+            for x, y in zip(s1[key], s2[key]):
+                assert np.array_equal(x.view(np.uint32), y.view(np.uint32)), key
+
+
+# --------------------------------------------------------------------------------------- Appendix A
+def test_appendix_a_bitwise_on_gpu():
+    """the fp32 GPU path reproduces the hand-computed loss and gradients
+    bit for bit (every intermediate is a short dyadic rational), W' within 1e-7."""
+    g = json.load(open(os.path.join(GOLD, "appendix_a_mlp_step.json")))
+    descs = [LayerDesc(LAYER_MLP, 2, 2, act=ACT_RELU), LayerDesc(LAYER_MLP, 2, 2, act=ACT_NONE)]
+    params = [pack(descs[0], {"w": g["W1"], "b": g["b1"]}, np.float32),
+              pack(descs[1], {"w": g["W2"], "b": g["b2"]}, np.float32)]
+    X = np.array(g["x"], np.float32); T = np.array(g["t"], np.float32)
+    (res,), _ = run_gpu(descs, params, [(X, T)], microbatches=2, microbatch_size=1)
+    assert res["loss"] == g["loss_num"] / g["loss_den"]
+    g1 = unpack(descs[0], res["g"][0]); g2 = unpack(descs[1], res["g"][1])
+    assert np.array_equal(g1["w"], np.array(g["dW1"], np.float32)) and np.array_equal(g1["b"], np.array(g["db1"], np.float32))
+    assert np.array_equal(g2["w"], np.array(g["dW2"], np.float32)) and np.array_equal(g2["b"], np.array(g["db2"], np.float32))
+    W1 = unpack(descs[0], res["W"][0])
+    assert np.max(np.abs(W1["w"] - np.array(g["W1_new"])) / np.abs(np.array(g["W1_new"]))) < 1e-7
+
+
+# --------------------------------------------------------------------------------------- cfg1 (fp32, capped)
+CFG1 = synth.CONFIGS["cfg1"]
+
+
+def test_cfg1_mlp_fp32_matches_oracle_and_capped_equals_uncapped():
+    descs = CFG1["descs"]()
+    params = synth.gen_params(descs)
+    batches = batches_for(descs, CFG1["batch"], 3, 0)
+    kw = dict(microbatches=CFG1["m"], microbatch_size=CFG1["batch"] // CFG1["m"])
+    capped, plan = run_gpu(descs, params, batches, hbm_cap_bytes=CFG1["cap"], **kw)
+    assert plan["arena_bytes"] <= CFG1["cap"]
+    st = capped[0]["stats"]
+    assert st["h2d_weight_bytes"] + st["h2d_state_bytes"] + st["h2d_stash_bytes"] > 0  # it really swaps
+    assert st["h2d_grad_bytes"] == 0
+    ref = run_oracle(descs, params, batches)
+    compare(capped, ref, 1e-5)
+    uncapped, _ = run_gpu(descs, params, batches, hbm_cap_bytes=0, **kw)
+    bitwise_equal(capped, uncapped)
+    # ledger == plan
+    assert st["h2d_bytes"] == plan["pred_h2d_bytes"] and st["d2h_bytes"] == plan["pred_d2h_bytes"]
+
+
+def test_rerun_is_deterministic():
+    descs = CFG1["descs"]()
+    params = synth.gen_params(descs)
+    batches = batches_for(descs, 32, 2, 0)
+    a, _ = run_gpu(descs, params, batches, microbatches=4, microbatch_size=8, hbm_cap_bytes=CFG1["cap"])
+    b, _ = run_gpu(descs, params, batches, microbatches=4, microbatch_size=8, hbm_cap_bytes=CFG1["cap"])
+    bitwise_equal(a, b)
+
+
+# --------------------------------------------------------------------------------------- transformer
+def tiny_transformer(causal, precision, L=2, d=64, h=4, S=32, B=4, m=2):
+    descs = synth.transformer_stack(L, d, h, S, causal)
+    params = synth.gen_params(descs, precision)
+    if precision == 0:  # larger weights so attention is non-trivial at fp32 parity
+        params = [p * 1.0 for p in params]
+    batches = batches_for(descs, B, 3, precision)
+    return descs, params, batches, dict(microbatches=m, microbatch_size=B // m, precision=precision)
+
+
+@pytest.mark.parametrize("causal", [False, True])
+def test_transformer_fp32_matches_oracle(causal):
+    descs, params, batches, kw = tiny_transformer(causal, 0)
+    gpu, _ = run_gpu(descs, params, batches, **kw)
+    ref = run_oracle(descs, params, batches)
+    compare(gpu, ref, 1e-5)
+
+
+@pytest.mark.parametrize("causal", [False, True])
+def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal):
+    descs, params, batches, kw = tiny_transformer(causal, 1, L=3, d=128, h=2, S=136, B=4, m=2)
+    uncapped, plan = run_gpu(descs, params, batches, **kw)
+    ref = run_oracle(descs, params, batches)
+    w = compare(uncapped, ref, 2e-2)
+    print("bf16 worst rel", w)
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, **kw), descs, text_len=0)
+    cap = int(s.min_working_set_bytes * 1.5)
+    capped, plan_c = run_gpu(descs, params, batches, hbm_cap_bytes=cap, **kw)
+    assert plan_c["arena_bytes"] <= cap
+    assert capped[0]["stats"]["h2d_stash_bytes"] > 0 or capped[0]["stats"]["h2d_weight_bytes"] > 0
+    bitwise_equal(capped, uncapped)
+
+
+def test_transformer_bf16_recompute_policy_matches():
+    """stash_policy = 1 recomputes LN outputs and GeLU in the backward: same math, fewer swap bytes."""
+    descs, params, batches, kw = tiny_transformer(True, 1, L=2, d=64, h=2, S=64, B=4, m=2)
+    a, pa = run_gpu(descs, params, batches, **kw)
+    b, pb = run_gpu(descs, params, batches, stash_policy=1, **kw)
+    ref = run_oracle(descs, params, batches)
+    compare(b, ref, 2e-2)
+    assert pb["total_stash_bytes"] < pa["total_stash_bytes"]
+
+
+def test_device_pointer_inputs_match_host_inputs():
+    descs = CFG1["descs"]()
+    params = synth.gen_params(descs)
+    X, T = synth.gen_batch(descs, 32, 1)
+    with H.Harmony(descs, params, microbatches=4, microbatch_size=8, hbm_cap_bytes=CFG1["cap"]) as h:
+        l1, s1 = h.step(torch.tensor(X, device="cuda"), torch.tensor(T, device="cuda"))
+        assert s1.h2d_input_bytes == 0
+    with H.Harmony(descs, params, microbatches=4, microbatch_size=8, hbm_cap_bytes=CFG1["cap"]) as h:
+        l2, s2 = h.step(X, T)
+        assert s2.h2d_input_bytes == 2 * X.nbytes
+    assert l1 == l2
+
+
+def test_step_errors():
+    descs = CFG1["descs"]()
+    params = synth.gen_params(descs)
+    with H.Harmony(descs, params, microbatches=4, microbatch_size=8) as h:
+        X, T = synth.gen_batch(descs, 32, 1)
+        with pytest.raises(H.HarmonyError) as e:
+            H.harmony_step(h.ctx, X, T, 31)
+        assert e.value.code == H.HARMONY_E_INVALID_ARG
+        with pytest.raises(H.HarmonyError) as e:
+            H.harmony_read_state(h.ctx, 0, H.HARMONY_GRAD, params[0].size)
+        assert e.value.code == H.HARMONY_E_BAD_STATE
+    ctx = H.harmony_init(H.make_config(microbatches=1, microbatch_size=1))
+    with pytest.raises(H.HarmonyError) as e:
+        H.harmony_step(ctx, X, T, 1)
+    assert e.value.code == H.HARMONY_E_BAD_STATE
+    H.harmony_finalize(ctx)
