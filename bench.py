@@ -1,0 +1,342 @@
+"""Benchmark of the Harmony-DP step (BASELINE.json metric: samples/sec/step under an HBM cap,
+swap GB/s and % of roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload cfg2] [--impl ours|reference]
+
+N=1: the workload BASELINE.json's metric is quoted on that fits one GPU — configs[1], BERT-Large
+(24 pre-LN blocks, d=1024, h=16, S=512), 64 sequences per GPU as 8 microbatches, bf16 tensor-core
+compute with fp32 master weights + Adam, per-GPU HBM cap 8 GiB.  N>1 (torchrun, one process per
+GPU): the same per-GPU work on every rank (weak scaling), data-parallel with NCCL reduce-scatter
+of gradients and all-gather of weight shards inside the library.
+
+`value` = samples / device time of the K timed steps (CUDA events on the library's streams,
+inputs resident in HBM, max over ranks).  `e2e` = the same through the C ABI with pinned HOST
+inputs (the H2D of X and T and the D2H of the loss inside the timed region), host wall clock.
+`--impl reference` times the CPU oracle (fp64 NumPy) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+WORKLOADS = {
+    "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=8 x b=8), bf16/fp32-master Adam, "
+                      "HBM cap 8 GiB/GPU", model="bert-large-like-preLN", descs=lambda: synth.transformer_stack(24, 1024, 16, 512, False),
+                 per_gpu_batch=64, m=8, cap=8 << 30, S=512),
+    "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=4 x b=2), bf16/fp32-master Adam, "
+                      "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
+                 per_gpu_batch=8, m=4, cap=16 << 30, S=1024),
+    "cfg1": dict(name="cfg1: 4-layer MLP d256, batch 32 as 4 microbatches, fp32, cap = 2 layers' state",
+                 model="mlp4-d256", descs=lambda: synth.mlp_stack(4, 256), per_gpu_batch=32, m=4,
+                 cap=2 * 16 * (256 * 256 + 256), S=1, precision=0),
+}
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_FILE) as f:
+            p = json.load(f)
+        return p, "measured"
+    except Exception:
+        return FALLBACK, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def start(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 8:
+                self.samples.append(f)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[4 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def host_link_bandwidth(torch, device):
+    """Pinned H2D, D2H and concurrent duplex GB/s (1 GiB in 128 MiB chunks, best of 3)."""
+    GiB, chunk = 1 << 30, 128 << 20
+    hs = torch.empty(GiB, dtype=torch.uint8).pin_memory()
+    hd = torch.empty(GiB, dtype=torch.uint8).pin_memory()
+    d1 = torch.empty(GiB, dtype=torch.uint8, device=device)
+    d2 = torch.empty(GiB, dtype=torch.uint8, device=device)
+    s1, s2 = torch.cuda.Stream(device), torch.cuda.Stream(device)
+    out = {}
+    for mode in ("h2d", "d2h", "duplex"):
+        best = 0.0
+        for _ in range(3):
+            torch.cuda.synchronize(device)
+            t0 = time.perf_counter()
+            n = 0
+            for off in range(0, GiB, chunk):
+                if mode in ("h2d", "duplex"):
+                    with torch.cuda.stream(s1):
+                        d1[off:off + chunk].copy_(hs[off:off + chunk], non_blocking=True)
+                    n += chunk
+                if mode in ("d2h", "duplex"):
+                    with torch.cuda.stream(s2):
+                        hd[off:off + chunk].copy_(d2[off:off + chunk], non_blocking=True)
+                    n += chunk
+            torch.cuda.synchronize(device)
+            best = max(best, n / (time.perf_counter() - t0) / 1e9)
+        out[mode] = best
+    del hs, hd, d1, d2
+    return out
+
+
+def cpu_oracle_sample(wl, budget_s=20.0):
+    """Time the fp64 oracle (as it stands) on a bounded sample of the workload: forward+backward
+    of ONE sample through `ls` of the L layers, plus Adam on those layers' parameters; scale to the
+    full step (per-sample cost x batch + Adam) x L/ls.  Returns (samples/s, description, cores)."""
+    import oracle
+    descs = wl["descs"]()
+    L = len(descs)
+    ls = 1 if descs[0].kind == synth.LAYER_TRANSFORMER else L
+    sub = descs[:ls]
+    params = [p.astype(np.float64) for p in synth.gen_params(sub, wl.get("precision", 1))]
+    X, T = synth.gen_batch(sub, 1, 1, wl.get("precision", 1))
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        _, grads, _ = oracle.stack_loss_and_grads(sub, params, X.astype(np.float64), T.astype(np.float64))
+        reps += 1
+        if time.perf_counter() - t0 > budget_s * 0.6 or reps >= 50:
+            break
+    t_fb = (time.perf_counter() - t0) / reps
+    st = oracle.AdamState.zeros(params)
+    t1 = time.perf_counter()
+    for W, g, m, v in zip(params, grads, st.m, st.v):
+        oracle.adam_update(W, g, m, v, 1, 1e-3, 0.9, 0.999, 1e-8)
+    t_adam = time.perf_counter() - t1
+    B = wl["per_gpu_batch"]
+    step = (B * t_fb + t_adam) * (L / ls)
+    desc = (f"fp64 NumPy oracle: fwd+bwd of 1 sample through {ls} of {L} layers ({reps} reps, {t_fb:.3f} s each) "
+            f"+ Adam on those layers ({t_adam:.3f} s); scaled x{B} samples x{L // ls} layers = {step:.1f} s/step")
+    return B / step, desc, (len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count())
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="cfg2", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--stash-policy", type=int, default=1)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    wl = WORKLOADS[args.workload]
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    metric = "samples/sec/step under HBM cap"
+    unit = "samples/s"
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        vals = []
+        desc = cores = None
+        for _ in range(args.warmup):
+            cpu_oracle_sample(wl, budget_s=2.0)
+        for _ in range(args.steps):
+            v, desc, cores = cpu_oracle_sample(wl, budget_s=8.0)
+            vals.append(v)
+        value = statistics.median(vals)
+        line = {"impl": "reference", "metric": metric, "value": value, "unit": unit, "n_gpus": args.gpus,
+                "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": wl["name"], "global_batch": wl["per_gpu_batch"] * max(args.gpus, 1),
+                           "seq_len": wl["S"], "parallelism": f"dp{args.gpus}"},
+                "cpu_baseline": {"value": value, "unit": unit, "cores": cores, "kind": "oracle", "sample": desc},
+                "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line))
+        return
+
+    import torch
+    from paper_conf_hotos_lipmk21_b200 import harmony as H
+
+    torch.cuda.set_device(local)
+    device = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo", init_method="env://")
+    precision = wl.get("precision", 1)
+    descs = wl["descs"]()
+    B = wl["per_gpu_batch"]
+    m = wl["m"]
+    nccl_id = None
+    if world > 1:
+        obj = [H.harmony_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    t_setup = time.perf_counter()
+    params = synth.gen_params(descs, precision)
+    cfg = dict(rank=rank, world_size=world, device=local, hbm_cap_bytes=wl["cap"], microbatches=m,
+               microbatch_size=B // m, precision=precision, stash_policy=args.stash_policy if precision else 0,
+               lr=1e-4, nccl_id=nccl_id)
+    h = H.Harmony(descs, params, **cfg)
+    del params
+    plan = h.plan().as_dict()
+    setup_s = time.perf_counter() - t_setup
+    # this rank's rows of the global batch (reading c14); resident inputs for `value`
+    X, T = synth.gen_batch(descs, B * world, 1, precision)
+    X = X[rank * B:(rank + 1) * B]
+    T = T[rank * B:(rank + 1) * B]
+    Xd, Td = torch.tensor(X, device=device), torch.tensor(T, device=device)
+    Xh, Th = torch.tensor(X).pin_memory(), torch.tensor(T).pin_memory()
+
+    def barrier():
+        torch.cuda.synchronize(device)
+        if dist is not None:
+            dist.barrier()
+
+    bw = host_link_bandwidth(torch, device) if rank == 0 else None
+    for _ in range(args.warmup):
+        h.step(Xd, Td)
+    # ---- timed region: device-resident inputs
+    H.harmony_set_profiling(h.ctx, 1)
+    clocks = ClockSampler(local)
+    clocks.start()
+    barrier()
+    dev_s, losses, stats = 0.0, [], []
+    wall0 = time.perf_counter()
+    for _ in range(args.steps):
+        loss, st = h.step(Xd, Td)
+        dev_s += st.step_seconds
+        losses.append(loss)
+        stats.append(st.as_dict())
+    barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    prof = H.harmony_read_profile(h.ctx).as_dict()
+    H.harmony_set_profiling(h.ctx, 0)
+    # ---- e2e: pinned host inputs through the C ABI, host wall clock
+    barrier()
+    e0 = time.perf_counter()
+    e2e_stats = []
+    for _ in range(args.steps):
+        loss, st = h.step(Xh, Th)
+        e2e_stats.append(st.as_dict())
+    barrier()
+    e2e_wall = time.perf_counter() - e0
+    if dist is not None:
+        t = torch.tensor([dev_s, wall, e2e_wall], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev_s, wall, e2e_wall = t.tolist()
+    h.close()
+    if rank != 0:
+        return
+
+    peaks, peak_src = load_peaks()
+    samples = B * world * args.steps
+    value = samples / dev_s
+    ms = dev_s / args.steps * 1e3
+    s0 = stats[-1]
+    h2d = s0["h2d_bytes"]; d2h = s0["d2h_bytes"]
+    # step roofline (north_star): slower of GEMM FLOPs at tensor peak and swap bytes at host-link BW
+    F = plan["flops_per_step"]
+    t_gemm = F / (peaks["bf16_tflops"] * 1e12)
+    t_strict = max(h2d / (bw["h2d"] * 1e9), d2h / (bw["d2h"] * 1e9), (h2d + d2h) / (bw["duplex"] * 1e9))
+    t_lenient = (h2d + d2h) / (max(bw["h2d"], bw["d2h"]) * 1e9)
+    t_roof = max(t_gemm, t_strict)
+    g = prof["gemm"]
+    gemm_tflops = g["work"] / g["seconds"] / 1e12 if g["seconds"] else 0.0
+    gemm_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    adam = prof["adam"]
+    line = {
+        "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "bf16" if precision else "f32", "data": "synthetic (seeded, paper-shaped)",
+        "config": {"workload": wl["name"], "global_batch": B * world, "seq_len": wl["S"],
+                   "parallelism": f"dp{world}", "hbm_cap_bytes_per_gpu": wl["cap"],
+                   "arena_bytes": plan["arena_bytes"], "stash_policy": cfg["stash_policy"],
+                   "l2": "inputs and per-step swap traffic (tens of GB) far larger than the 126 MB L2; no flush"},
+        "roofline": {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05, all GEMM launches of the step)",
+                     "achieved": gemm_tflops, "peak": gemm_peak, "unit": "TFLOP/s",
+                     "frac": gemm_tflops / gemm_peak if gemm_peak else None, "traffic": None,
+                     "peak_source": f"{peak_src} bf16_tflops_sustained (kernel timed inside a long step)",
+                     "launches_per_step": g["launches"] / args.steps,
+                     "flops_per_step": g["work"] / args.steps},
+        "step_roofline": {"bound": "host_link" if t_strict > t_gemm else "tensor", "t_roof_ms": t_roof * 1e3,
+                          "t_gemm_ms": t_gemm * 1e3, "t_swap_strict_ms": t_strict * 1e3,
+                          "t_swap_lenient_ms": t_lenient * 1e3, "frac_strict": t_roof / (dev_s / args.steps),
+                          "frac_lenient": max(t_gemm, t_lenient) / (dev_s / args.steps),
+                          "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                          "swap_gbs": (h2d + d2h) / (dev_s / args.steps) / 1e9,
+                          "host_link_gbs_measured": bw, "flops_per_step": F},
+        "kernels": {k: dict(v, per_launch_us=(v["seconds"] / v["launches"] * 1e6 if v["launches"] else None))
+                    for k, v in prof.items()},
+        "adam_hbm": {"achieved_gbs": adam["work"] / adam["seconds"] / 1e9 if adam["seconds"] else None,
+                     "peak_gbs": peaks["hbm_gbs"]},
+        "e2e": {"value": samples / e2e_wall, "unit": unit, "h2d_bytes_per_step": e2e_stats[-1]["h2d_input_bytes"],
+                "d2h_bytes_per_step": e2e_stats[-1]["d2h_output_bytes"], "timing": "host wall clock around harmony_step"},
+        "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
+        "clocks": clk,
+        "loss": losses[-1],
+        "wall_s": wall, "setup_s": setup_s,
+        "plan": {k: plan[k] for k in ("arena_bytes", "resident_weight_bytes", "resident_state_bytes",
+                                      "resident_stash_bytes", "total_stash_bytes", "pred_h2d_bytes",
+                                      "pred_d2h_bytes", "n_ops", "hazards")},
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        v, desc, cores = cpu_oracle_sample(wl)
+        line["cpu_baseline"] = {"value": v, "unit": unit, "cores": cores, "kind": "oracle", "sample": desc}
+    txt = json.dumps(line)
+    print(txt)
+    if args.out:
+        with open(args.out, "w") as f:
+            f.write(txt + "\n")
+
+
+if __name__ == "__main__":
+    main()

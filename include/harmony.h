@@ -97,7 +97,8 @@ typedef struct {
   int32_t stash_policy;      /* 0 = stash every op input (36d+2hS+16 B/token/block);
                                 1 = recompute elementwise outputs (LN outputs, GeLU) in the
                                 backward (24d+2hS+16 B/token/block)                          */
-  float lr, beta1, beta2, eps, weight_decay; /* Adam; weight_decay must be 0 (reading c3)    */
+  double lr, beta1, beta2, eps, weight_decay; /* Adam; weight_decay must be 0 (reading c3).  Doubles:
+                                the kernel uses fp32 b and (1-b) each rounded once from these */
   uint8_t nccl_id[128];      /* ncclUniqueId from harmony_get_unique_id() on rank 0, broadcast
                                 to all ranks by the caller (ignored when world_size == 1)    */
 } harmony_config;
@@ -146,8 +147,22 @@ typedef struct {
 } harmony_plan_summary;
 
 /* sizeof of the ABI structs as the library was compiled: harmony_config, harmony_layer_desc,
- * harmony_step_stats, harmony_plan_summary, hk_gemm_args (bindings check their mirrors). */
-void harmony_abi_sizes(uint64_t out[5]);
+ * harmony_step_stats, harmony_plan_summary, hk_gemm_args, harmony_kernel_profile (bindings
+ * check their mirrors). */
+void harmony_abi_sizes(uint64_t out[6]);
+
+/* Per-kernel-class timing (CUDA events recorded on the launching stream around every launch
+ * while profiling is on).  Classes: 0 GEMM (work = algorithmic FLOPs 2MNK), 1 Adam (work =
+ * algorithmic HBM bytes, 30 B/param bf16 / 32 fp32), 2 LayerNorm fwd+bwd (bytes), 3 softmax
+ * fwd+bwd (bytes), 4 other.  Totals accumulate over steps since harmony_set_profiling(ctx, 1). */
+typedef struct {
+  uint64_t launches[5];
+  double seconds[5];
+  double work[5];
+} harmony_kernel_profile;
+
+harmony_status harmony_set_profiling(harmony_ctx* ctx, int32_t on);
+harmony_status harmony_read_profile(const harmony_ctx* ctx, harmony_kernel_profile* out);
 
 /* Writes an ncclUniqueId (128 bytes) into out.  Call on rank 0 only, then broadcast. */
 harmony_status harmony_get_unique_id(uint8_t out[128]);

@@ -85,8 +85,8 @@ harmony_status hk_colsum(int32_t in_dtype, int64_t rows, int32_t n, const void* 
 
 /* Fused Adam on n elements (reading c3): m = b1 m + (1-b1) g; v = b2 v + (1-b2) g^2;
  * W -= lr * (m/bc1) / (sqrt(v/bc2) + eps); Wc(T) = round(W).  bc1 = 1-b1^t, bc2 = 1-b2^t. */
-harmony_status hk_adam(int32_t dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr,
-                       float beta1, float beta2, float eps, int32_t t, void* stream);
+harmony_status hk_adam(int32_t dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr,
+                       double beta1, double beta2, double eps, int32_t t, void* stream);
 
 /* MSE (reading c2): dY = (Y - T) * inv_batch; loss_out[0] (double) = 0.5*inv_batch*sum (Y-T)^2,
  * reduced in a fixed order.  Y, T, dY fp32 [n]. */

@@ -7,6 +7,7 @@
 #include <stdio.h>
 #include <cmath>
 #include <string>
+#include <vector>
 
 #include "harmony.h"
 
@@ -37,6 +38,33 @@ struct Error {
 
 // Kernel launch accounting (the ledger counts the kernels a step launches).
 extern thread_local uint64_t g_kernel_launches;
+
+// Optional per-launch timing (harmony_set_profiling): CUDA events recorded on the launching
+// stream around each kernel of a class, with the launch's algorithmic work (FLOPs or bytes).
+enum ProfCat { PROF_GEMM = 0, PROF_ADAM = 1, PROF_LN = 2, PROF_SOFTMAX = 3, PROF_OTHER = 4, PROF_NUM = 5 };
+struct KProf {
+  bool on = false;
+  std::vector<cudaEvent_t> pool;
+  size_t used = 0;
+  struct Rec { int cat, e0, e1; double work; };
+  std::vector<Rec> recs;
+  int begin(cudaStream_t st) {
+    if (!on) return -1;
+    if (used == pool.size()) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) != cudaSuccess) return -1;
+      pool.push_back(e);
+    }
+    cudaEventRecord(pool[used], st);
+    return (int)used++;
+  }
+  void end(int cat, int e0, cudaStream_t st, double work) {
+    if (e0 < 0) return;
+    int e1 = begin(st);
+    if (e1 >= 0) recs.push_back({cat, e0, e1, work});
+  }
+};
+extern thread_local KProf g_prof;
 inline void count_launch() { ++g_kernel_launches; }
 
 inline void check_launch(const char* what) {

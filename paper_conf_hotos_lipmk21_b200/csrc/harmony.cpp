@@ -24,6 +24,7 @@
 
 namespace hm {
 thread_local uint64_t g_kernel_launches = 0;
+thread_local KProf g_prof;
 static thread_local std::string g_err;
 void set_global_error(const std::string& msg) { g_err = msg; }
 const char* global_error() { return g_err.c_str(); }
@@ -57,6 +58,8 @@ struct harmony_ctx {
   double* h_loss = nullptr;
   int t = 0;
   harmony_step_stats last{};
+  bool profiling = false;
+  harmony_kernel_profile prof{};
 };
 
 namespace {
@@ -137,6 +140,9 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
   s.n_ops = p.ops.size();
   s.peak_arena_bytes = p.arena_bytes;
   g_kernel_launches = 0;
+  g_prof.on = c->profiling;
+  g_prof.used = 0;
+  g_prof.recs.clear();
   c->t += 1;
   const bool x_dev = is_device_ptr(x), t_dev = is_device_ptr(tg);
   const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
@@ -255,6 +261,16 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     ms = std::max(ms, e);
   }
   HM_CUDA(cudaGetLastError());
+  if (g_prof.on) {
+    for (auto& rc : g_prof.recs) {
+      float e = 0.f;
+      HM_CUDA(cudaEventElapsedTime(&e, g_prof.pool[rc.e0], g_prof.pool[rc.e1]));
+      c->prof.launches[rc.cat] += 1;
+      c->prof.seconds[rc.cat] += e * 1e-3;
+      c->prof.work[rc.cat] += rc.work;
+    }
+    g_prof.on = false;
+  }
   double loss = 0.0;  // rank partials summed in rank order, microbatches in order (reading c22)
   for (int r = 0; r < p.N; ++r)
     for (int i = 0; i < p.m; ++i) loss += c->h_loss[r * p.m + i];
@@ -278,6 +294,7 @@ void harmony_abi_sizes(uint64_t out[5]) {
   out[2] = sizeof(harmony_step_stats);
   out[3] = sizeof(harmony_plan_summary);
   out[4] = sizeof(hk_gemm_args);
+  out[5] = sizeof(harmony_kernel_profile);
 }
 
 const char* harmony_last_error(const harmony_ctx* ctx) { return ctx ? ctx->err.c_str() : global_error(); }
@@ -484,6 +501,19 @@ harmony_status harmony_plan_info(const harmony_ctx* c, harmony_plan_summary* out
   if (!c || !out) return HARMONY_E_INVALID_ARG;
   if (!c->registered) return HARMONY_E_BAD_STATE;
   *out = c->plan.summary;
+  return HARMONY_OK;
+}
+
+harmony_status harmony_set_profiling(harmony_ctx* c, int32_t on) {
+  if (!c) return HARMONY_E_INVALID_ARG;
+  c->profiling = on != 0;
+  c->prof = harmony_kernel_profile{};
+  return HARMONY_OK;
+}
+
+harmony_status harmony_read_profile(const harmony_ctx* c, harmony_kernel_profile* out) {
+  if (!c || !out) return HARMONY_E_INVALID_ARG;
+  *out = c->prof;
   return HARMONY_OK;
 }
 

@@ -90,8 +90,8 @@ harmony_status hk_colsum(int32_t in_dtype, int64_t rows, int32_t n, const void* 
   K_END
 }
 
-harmony_status hk_adam(int32_t dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr,
-                       float beta1, float beta2, float eps, int32_t t, void* stream) {
+harmony_status hk_adam(int32_t dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr,
+                       double beta1, double beta2, double eps, int32_t t, void* stream) {
   K_BEGIN
   HM_CHECK(t >= 1, HARMONY_E_INVALID_ARG, "Adam step t starts at 1");
   adam(dtype, n, W, m, v, g, Wc, lr, beta1, beta2, eps, t, static_cast<cudaStream_t>(stream));

@@ -368,6 +368,8 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
   e.C = a.C; e.ldc = a.ldc; e.c_sz0 = a.c_sz0; e.c_sz1 = a.c_sz1;
   e.epi = a.epilogue; e.act = a.act; e.accumulate = a.accumulate; e.alpha = a.alpha;
   e.bias = a.bias; e.aux = a.aux; e.aux_out = a.aux_out; e.M = a.M; e.N = a.N;
+  const int e0 = g_prof.begin(st);
+  const double flops = 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1;
   if (a.dtype == 0) {
     SimtParams p;
     p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0;
@@ -377,6 +379,7 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
     dim3 grid((unsigned)ceil_div(a.N, SBN), (unsigned)ceil_div(a.M, SBM), (unsigned)(a.nz0 * a.nz1));
     gemm_simt_kernel<<<grid, 256, 0, st>>>(p);
     check_launch("gemm_simt_kernel");
+    g_prof.end(PROF_GEMM, e0, st, flops);
     return;
   }
   // Tile width from the shape only (never from the memory cap): bit-exact capped == uncapped.
@@ -386,6 +389,7 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
     tc::launch_tc<128, 6>(a, e, st);
   else
     tc::launch_tc<256, 4>(a, e, st);
+  g_prof.end(PROF_GEMM, e0, st, flops);
 }
 
 }  // namespace hm

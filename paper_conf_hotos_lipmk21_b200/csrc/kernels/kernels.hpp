@@ -22,8 +22,8 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st);
 void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
                  cudaStream_t st);
-void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr, float b1, float b2,
-          float eps, int t, cudaStream_t st);
+void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr, double b1, double b2,
+          double eps, int t, cudaStream_t st);
 size_t mse_scratch_bytes();
 void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY, double* loss_out, double* scratch,
          cudaStream_t st);

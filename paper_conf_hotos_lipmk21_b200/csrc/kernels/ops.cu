@@ -168,8 +168,8 @@ __global__ void __launch_bounds__(256) softmax_bwd_kernel(int64_t rows, int S, f
 // Kingma & Ba [30], Algorithm 1 with bias correction; fp32 master state (reading c3).
 template <typename T>
 __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict__ m, float* __restrict__ v,
-                            const float* __restrict__ g, T* __restrict__ Wc, float lr, float b1, float b2, float eps,
-                            float inv_bc1, float inv_bc2) {
+                            const float* __restrict__ g, T* __restrict__ Wc, float lr, float b1, float omb1, float b2,
+                            float omb2, float eps, float inv_bc1, float inv_bc2) {
   const int64_t n4 = n / 4;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
@@ -181,8 +181,8 @@ __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict_
     float out[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      mp[j] = b1 * mp[j] + (1.f - b1) * gp[j];
-      vp[j] = b2 * vp[j] + (1.f - b2) * gp[j] * gp[j];
+      mp[j] = b1 * mp[j] + omb1 * gp[j];
+      vp[j] = b2 * vp[j] + omb2 * gp[j] * gp[j];
       wp[j] = wp[j] - lr * (mp[j] * inv_bc1) / (sqrtf(vp[j] * inv_bc2) + eps);
       out[j] = wp[j];
     }
@@ -201,8 +201,8 @@ __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict_
     }
   }
   for (int64_t i = n4 * 4 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-    float mi = b1 * m[i] + (1.f - b1) * g[i];
-    float vi = b2 * v[i] + (1.f - b2) * g[i] * g[i];
+    float mi = b1 * m[i] + omb1 * g[i];
+    float vi = b2 * v[i] + omb2 * g[i] * g[i];
     float wi = W[i] - lr * (mi * inv_bc1) / (sqrtf(vi * inv_bc2) + eps);
     m[i] = mi; v[i] = vi; W[i] = wi;
     Wc[i] = from_f32<T>(wi);
@@ -277,9 +277,11 @@ __global__ void copy_rows_kernel(int64_t n4, const float4* __restrict__ src, flo
 void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
                    float* rstd, cudaStream_t st) {
   if (rows == 0) return;
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (layernorm_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(
                            rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)));
   check_launch("layernorm_fwd");
+  g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 + (dtype ? 2 : 4)) + rows * 8.0);
 }
 
 size_t layernorm_bwd_scratch_bytes(int64_t rows, int d) {
@@ -293,6 +295,7 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
     return;
   }
   int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (layernorm_bwd_kernel<T><<<nblk, 256, 0, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres,
                                                                       dX, scratch)));
   check_launch("layernorm_bwd");
@@ -300,6 +303,7 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
   check_launch("colreduce(dgamma)");
   colreduce_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
   check_launch("colreduce(dbeta)");
+  g_prof.end(PROF_LN, e0, st, (double)rows * d * 4 * (dres ? 4 : 3) + rows * 8.0);
 }
 
 size_t colsum_scratch_bytes(int64_t rows, int n) { return (size_t)ceil_div(rows, CS_ROWS) * n * sizeof(float); }
@@ -320,29 +324,36 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
 
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st) {
   if (rows == 0) return;
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (softmax_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, causal, scale, Z,
                                                                                           (T*)P)));
   check_launch("softmax_fwd");
+  g_prof.end(PROF_SOFTMAX, e0, st, (double)rows * S * (4 + (dtype ? 2 : 4)));
 }
 
 void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
                  cudaStream_t st) {
   if (rows == 0) return;
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (softmax_bwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, alpha, dP,
                                                                                           (const T*)P, (T*)dZ)));
   check_launch("softmax_bwd");
+  g_prof.end(PROF_SOFTMAX, e0, st, (double)rows * S * (4 + 2 * (dtype ? 2 : 4)));
 }
 
-void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, float lr, float b1, float b2,
-          float eps, int t, cudaStream_t st) {
+void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr, double b1, double b2,
+          double eps, int t, cudaStream_t st) {
   if (n == 0) return;
   // bias corrections computed in double on the host, applied as fp32 reciprocals
-  double bc1 = 1.0 - std::pow((double)b1, (double)t), bc2 = 1.0 - std::pow((double)b2, (double)t);
+  double bc1 = 1.0 - std::pow(b1, (double)t), bc2 = 1.0 - std::pow(b2, (double)t);
   HM_CHECK(((uintptr_t)W | (uintptr_t)m | (uintptr_t)v | (uintptr_t)g) % 16 == 0, HARMONY_E_INVALID_ARG,
            "adam: fp32 state must be 16-byte aligned");
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (adam_kernel<T><<<grid_for(ceil_div(n, 4), 256), 256, 0, st>>>(
-                           n, W, m, v, g, (T*)Wc, lr, b1, b2, eps, (float)(1.0 / bc1), (float)(1.0 / bc2))));
+                           n, W, m, v, g, (T*)Wc, (float)lr, (float)b1, (float)(1.0 - b1), (float)b2, (float)(1.0 - b2), (float)eps,
+                           (float)(1.0 / bc1), (float)(1.0 / bc2))));
   check_launch("adam");
+  g_prof.end(PROF_ADAM, e0, st, (double)n * (16 + 12 + (dtype ? 2 : 4)));  // read W,m,v,g; write W,m,v,Wc
 }
 
 size_t mse_scratch_bytes() { return 1024 * sizeof(double); }

@@ -28,8 +28,8 @@ void validate_config(const harmony_config& c) {
   HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
            "the per-GPU-virtualization baseline schedule is not built yet (SURVEY NEXT-3)");
   HM_CHECK(c.stash_policy == 0 || c.stash_policy == 1, HARMONY_E_INVALID_ARG, "stash_policy must be 0 or 1");
-  HM_CHECK(c.weight_decay == 0.f, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
-  HM_CHECK(c.lr > 0.f && c.beta1 >= 0.f && c.beta1 < 1.f && c.beta2 >= 0.f && c.beta2 < 1.f && c.eps > 0.f,
+  HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
+  HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
 }
 

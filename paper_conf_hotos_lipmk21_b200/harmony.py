@@ -30,8 +30,8 @@ class harmony_config(C.Structure):
     _fields_ = [("struct_size", C.c_uint32), ("rank", C.c_int32), ("world_size", C.c_int32), ("device", C.c_int32),
                 ("hbm_cap_bytes", C.c_uint64), ("arena", C.c_void_p), ("microbatches", C.c_int32),
                 ("microbatch_size", C.c_int32), ("precision", C.c_int32), ("schedule", C.c_int32),
-                ("retain_grads", C.c_int32), ("stash_policy", C.c_int32), ("lr", C.c_float), ("beta1", C.c_float),
-                ("beta2", C.c_float), ("eps", C.c_float), ("weight_decay", C.c_float), ("nccl_id", C.c_uint8 * 128)]
+                ("retain_grads", C.c_int32), ("stash_policy", C.c_int32), ("lr", C.c_double), ("beta1", C.c_double),
+                ("beta2", C.c_double), ("eps", C.c_double), ("weight_decay", C.c_double), ("nccl_id", C.c_uint8 * 128)]
 
 
 class harmony_layer_desc(C.Structure):
@@ -61,6 +61,15 @@ class harmony_plan_summary(C.Structure):
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+class harmony_kernel_profile(C.Structure):
+    _fields_ = [("launches", C.c_uint64 * 5), ("seconds", C.c_double * 5), ("work", C.c_double * 5)]
+    CLASSES = ("gemm", "adam", "layernorm", "softmax", "other")
+
+    def as_dict(self):
+        return {c: dict(launches=self.launches[i], seconds=self.seconds[i], work=self.work[i])
+                for i, c in enumerate(self.CLASSES)}
 
 
 class hk_gemm_args(C.Structure):
@@ -120,13 +129,15 @@ def lib() -> C.CDLL:
         "hk_softmax_fwd": (st, [C.c_int32, C.c_int64, C.c_int32, C.c_int32, C.c_float, P, P, P]),
         "hk_softmax_bwd": (st, [C.c_int32, C.c_int64, C.c_int32, C.c_float, P, P, P, P]),
         "hk_colsum": (st, [C.c_int32, C.c_int64, C.c_int32, P, C.c_int64, P, C.c_int32, P]),
-        "hk_adam": (st, [C.c_int32, C.c_int64, P, P, P, P, P, C.c_float, C.c_float, C.c_float, C.c_float, C.c_int32,
-                         P]),
+        "hk_adam": (st, [C.c_int32, C.c_int64, P, P, P, P, P, C.c_double, C.c_double, C.c_double, C.c_double,
+                         C.c_int32, P]),
         "hk_mse": (st, [C.c_int64, P, P, C.c_float, P, P, P]),
         "hk_cast": (st, [C.c_int32, C.c_int64, P, P, P]),
         "hk_act_bwd": (st, [C.c_int32, C.c_int32, C.c_int64, P, P, P, P]),
         "hk_sync": (st, []),
         "harmony_abi_sizes": (None, [P]),
+        "harmony_set_profiling": (st, [P, C.c_int32]),
+        "harmony_read_profile": (st, [P, C.POINTER(harmony_kernel_profile)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -233,6 +244,16 @@ def harmony_plan_dry(cfg, descs, text_len=1 << 22):
     buf = C.create_string_buffer(text_len) if text_len else None
     _check(lib().harmony_plan_dry(C.byref(cfg), len(descs), make_descs(descs), C.byref(s), buf, text_len))
     return s, (buf.value.decode() if buf is not None else "")
+
+
+def harmony_set_profiling(ctx, on):
+    _check(lib().harmony_set_profiling(ctx, int(on)), ctx)
+
+
+def harmony_read_profile(ctx):
+    p = harmony_kernel_profile()
+    _check(lib().harmony_read_profile(ctx, C.byref(p)), ctx)
+    return p
 
 
 def harmony_finalize(ctx):

@@ -37,10 +37,11 @@ def test_library_loads_and_exports_every_declared_symbol():
 
 
 def test_abi_struct_sizes_match_binding():
-    out = (C.c_uint64 * 5)()
+    out = (C.c_uint64 * 6)()
     H.lib().harmony_abi_sizes(out)
     assert list(out) == [C.sizeof(H.harmony_config), C.sizeof(H.harmony_layer_desc),
-                         C.sizeof(H.harmony_step_stats), C.sizeof(H.harmony_plan_summary), C.sizeof(H.hk_gemm_args)]
+                         C.sizeof(H.harmony_step_stats), C.sizeof(H.harmony_plan_summary), C.sizeof(H.hk_gemm_args),
+                         C.sizeof(H.harmony_kernel_profile)]
 
 
 def test_library_is_built_for_sm100a():

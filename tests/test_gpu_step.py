@@ -137,12 +137,36 @@ def tiny_transformer(causal, precision, L=2, d=64, h=4, S=32, B=4, m=2):
     return descs, params, batches, dict(microbatches=m, microbatch_size=B // m, precision=precision)
 
 
+def teacher_forced(descs, params, batches, gpu, tol, lr=1e-3):
+    """DESIGN.md reading c16a: per step, (i) the GPU gradient vs the oracle's full-batch gradient at
+    the GPU's own pre-step weights, (ii) the GPU's W, m, sqrt(v) vs the oracle's Adam (fp64) applied
+    to the GPU's pre-step state and its own gradient, (iii) the loss trajectory.  Adam's step
+    lr*g/(|g|+eps) is ill-conditioned where g is a structural zero (e.g. the key bias: softmax is
+    shift invariant), so the untouched trajectory would compare floating-point noise there."""
+    W = [p.astype(np.float64) for p in params]
+    m = [np.zeros_like(w) for w in W]; v = [np.zeros_like(w) for w in W]
+    worst = dict(loss=0.0, g=0.0, W=0.0, m=0.0, sqrt_v=0.0)
+    for t, ((X, T), st) in enumerate(zip(batches, gpu), start=1):
+        loss, g_ref, _ = oracle.stack_loss_and_grads(descs, W, X.astype(np.float64), T.astype(np.float64))
+        worst["loss"] = max(worst["loss"], abs(st["loss"] - loss) / abs(loss))
+        for l in range(len(descs)):
+            worst["g"] = max(worst["g"], rel(st["g"][l], g_ref[l]))
+            W2, m2, v2 = oracle.adam_update(W[l], st["g"][l].astype(np.float64), m[l], v[l], t, lr, 0.9, 0.999, 1e-8)
+            worst["W"] = max(worst["W"], rel(st["W"][l], W2))
+            worst["m"] = max(worst["m"], rel(st["m"][l], m2))
+            worst["sqrt_v"] = max(worst["sqrt_v"], rel(np.sqrt(st["v"][l]), np.sqrt(v2)))
+        W = [w.astype(np.float64) for w in st["W"]]
+        m = [x.astype(np.float64) for x in st["m"]]; v = [x.astype(np.float64) for x in st["v"]]
+    for k, x in worst.items():
+        assert x <= tol, (k, x, worst)
+    return worst
+
+
 @pytest.mark.parametrize("causal", [False, True])
 def test_transformer_fp32_matches_oracle(causal):
     descs, params, batches, kw = tiny_transformer(causal, 0)
     gpu, _ = run_gpu(descs, params, batches, **kw)
-    ref = run_oracle(descs, params, batches)
-    compare(gpu, ref, 1e-5)
+    print("fp32 transformer teacher-forced worst rel", teacher_forced(descs, params, batches, gpu, 1e-5))
 
 
 @pytest.mark.parametrize("causal", [False, True])
