@@ -96,7 +96,10 @@ typedef struct {
   int32_t retain_grads;      /* 1 = keep the last reduced gradients readable (HARMONY_GRAD)  */
   int32_t stash_policy;      /* 0 = stash every op input (36d+2hS+16 B/token/block);
                                 1 = recompute elementwise outputs (LN outputs, GeLU) in the
-                                backward (24d+2hS+16 B/token/block)                          */
+                                backward (24d+2hS+16 B/token/block);
+                                2 = block recompute: stash only the fp32 block
+                                input (4d B/token/block), the backward re-runs the block's
+                                forward first (4/3 of the GEMM FLOPs, far fewer swap bytes)  */
   double lr, beta1, beta2, eps, weight_decay; /* Adam; weight_decay must be 0 (reading c3).  Doubles:
                                 the kernel uses fp32 b and (1-b) each rounded once from these */
   uint8_t nccl_id[128];      /* ncclUniqueId from harmony_get_unique_id() on rank 0, broadcast
@@ -127,6 +130,9 @@ typedef struct {
   uint64_t kernel_launches;                     /* kernels launched in the step        */
   uint64_t n_ops;                               /* ops in the static program           */
   double step_seconds;                          /* device time of the step (CUDA events)*/
+  uint64_t graph;                               /* 1 = the step replayed its captured CUDA graph
+                                                   (pinned/device inputs, profiling off; disable
+                                                   with HARMONY_NO_GRAPH=1)                  */
 } harmony_step_stats;
 
 /* Static plan summary (host-only; also available without a GPU via harmony_plan_dry). */

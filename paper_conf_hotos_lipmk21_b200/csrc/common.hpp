@@ -44,6 +44,7 @@ extern thread_local uint64_t g_kernel_launches;
 enum ProfCat { PROF_GEMM = 0, PROF_ADAM = 1, PROF_LN = 2, PROF_SOFTMAX = 3, PROF_OTHER = 4, PROF_NUM = 5 };
 struct KProf {
   bool on = false;
+  bool external = false;  // inside a stream capture: record event nodes into the graph
   std::vector<cudaEvent_t> pool;
   size_t used = 0;
   struct Rec { int cat, e0, e1; double work; };
@@ -55,7 +56,8 @@ struct KProf {
       if (cudaEventCreate(&e) != cudaSuccess) return -1;
       pool.push_back(e);
     }
-    cudaEventRecord(pool[used], st);
+    if (external) cudaEventRecordWithFlags(pool[used], st, cudaEventRecordExternal);
+    else cudaEventRecord(pool[used], st);
     return (int)used++;
   }
   void end(int cat, int e0, cudaStream_t st, double work) {

@@ -39,6 +39,18 @@ static inline uint16_t f32_to_bf16_rne(float f) {
 
 using namespace hm;
 
+// One captured instance of the step program.
+struct StepGraph {
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  int sig = -1;                           // (x on device) | (target on device) << 1 at capture
+  std::vector<cudaGraphNode_t> in_nodes;  // input copies, re-pointed every step
+  std::vector<int> in_ops;
+  harmony_step_stats stats{};
+  uint64_t launches = 0;
+  std::vector<KProf::Rec> recs;           // profiled graph: timing-event pairs of its kernels
+};
+
 struct harmony_ctx {
   harmony_config cfg{};
   std::string err;
@@ -60,6 +72,10 @@ struct harmony_ctx {
   harmony_step_stats last{};
   bool profiling = false;
   harmony_kernel_profile prof{};
+  int* h_step = nullptr;  // pinned: Adam's t, copied to the device at the start of every step
+  bool use_graph = true;
+  StepGraph g_plain, g_prof;  // the step as CUDA graphs: plain, and with per-kernel timing events
+  cudaEvent_t ev_fork = nullptr, ev_join[S_NUM] = {};
 };
 
 namespace {
@@ -101,11 +117,19 @@ harmony_status fail(harmony_ctx* ctx, const Error& e) {
   }                                                                   \
   return HARMONY_OK;
 
+void drop_graph(StepGraph& g);
+
 void destroy(harmony_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->cfg.device);
   for (int s = 0; s < S_NUM; ++s)
     if (c->st[s]) cudaStreamSynchronize(c->st[s]);
+  drop_graph(c->g_plain);
+  drop_graph(c->g_prof);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  for (int s = 0; s < S_NUM; ++s)
+    if (c->ev_join[s]) cudaEventDestroy(c->ev_join[s]);
+  free_host(c->h_step);
   for (auto e : c->events) cudaEventDestroy(e);
   if (c->ev_begin) cudaEventDestroy(c->ev_begin);
   for (int s = 0; s < S_NUM; ++s) {
@@ -132,24 +156,26 @@ bool is_device_ptr(const void* p) {
 }
 
 // ---------------------------------------------------------------------------------------- executor
-void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out, harmony_step_stats* out) {
+enum PtrKind { PTR_PAGEABLE = 0, PTR_PINNED = 1, PTR_DEVICE = 2 };
+PtrKind ptr_kind(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return PTR_PAGEABLE;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return PTR_DEVICE;
+  if (a.type == cudaMemoryTypeHost) return PTR_PINNED;
+  return PTR_PAGEABLE;
+}
+
+// Issue the static program once on the four streams (eagerly, or inside a stream capture).
+void issue_program(harmony_ctx* c, const float* x, const float* tg, bool x_dev, bool t_dev, harmony_step_stats& s) {
   Plan& p = c->plan;
   uint8_t* A = c->arena;
   const int dt = p.dtype;
-  harmony_step_stats s{};
-  s.n_ops = p.ops.size();
-  s.peak_arena_bytes = p.arena_bytes;
-  g_kernel_launches = 0;
-  g_prof.on = c->profiling;
-  g_prof.used = 0;
-  g_prof.recs.clear();
-  c->t += 1;
-  const bool x_dev = is_device_ptr(x), t_dev = is_device_ptr(tg);
   const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
-
-  HM_CUDA(cudaEventRecord(c->ev_begin, c->st[S_COMPUTE]));
-  for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_begin, 0));
-
+  // Adam's step t lives in device memory (read by the update kernels at execution time)
+  HM_CUDA(cudaMemcpyAsync(A + p.tstep, c->h_step, sizeof(int), cudaMemcpyHostToDevice, c->st[S_COMPUTE]));
   for (size_t oi = 0; oi < p.ops.size(); ++oi) {
     const Op& o = p.ops[oi];
     cudaStream_t st = c->st[o.stream];
@@ -214,7 +240,7 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
         const uint64_t sh = (uint64_t)lp.shard;
         uint8_t* wc = A + o.w + (uint64_t)p.rank * sh * (dt ? 2 : 4);
         adam(dt, (int64_t)sh, state, state + sh, state + 2 * sh, reinterpret_cast<const float*>(A + o.grad), wc,
-             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->t, st);
+             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->t, reinterpret_cast<const int*>(A + p.tstep), st);
         break;
       }
       case OP_ALLGATHER: {
@@ -240,8 +266,8 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
         break;
       }
       case OP_LOSS_OUT: {
-        uint8_t* dst = reinterpret_cast<uint8_t*>(c->h_loss) + (p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8);
-        HM_CUDA(cudaMemcpyAsync(dst, A + o.dev + (p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8), o.bytes,
+        const uint64_t off = p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8;
+        HM_CUDA(cudaMemcpyAsync(reinterpret_cast<uint8_t*>(c->h_loss) + off, A + o.dev + off, o.bytes,
                                 cudaMemcpyDeviceToHost, st));
         s.d2h_bytes += o.bytes;
         s.d2h_output_bytes += o.bytes;
@@ -252,17 +278,132 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     }
     if (o.event >= 0) HM_CUDA(cudaEventRecord(c->events[o.event], st));
   }
-  for (int k = 0; k < S_NUM; ++k) HM_CUDA(cudaEventRecord(c->ev_end[k], c->st[k]));
-  float ms = 0.f;
-  for (int k = 0; k < S_NUM; ++k) {
-    HM_CUDA(cudaEventSynchronize(c->ev_end[k]));
-    float e = 0.f;
-    HM_CUDA(cudaEventElapsedTime(&e, c->ev_begin, c->ev_end[k]));
-    ms = std::max(ms, e);
+}
+
+void drop_graph(StepGraph& g) {
+  if (g.exec) cudaGraphExecDestroy(g.exec);
+  if (g.graph) cudaGraphDestroy(g.graph);
+  g.exec = nullptr;
+  g.graph = nullptr;
+  g.in_nodes.clear();
+  g.recs.clear();
+  g.sig = -1;
+}
+
+// Capture the whole step (all four streams, NCCL included) as one CUDA graph; later steps only
+// patch the source pointers of the input copies and replay it (one launch per step).  With
+// `profiled`, every kernel of the step is bracketed by external event-record nodes, so the
+// per-kernel durations come from the real step without host-issue gaps.
+void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg, bool x_dev, bool t_dev, bool profiled) {
+  drop_graph(G);
+  Plan& p = c->plan;
+  cudaStream_t cs = c->st[S_COMPUTE];
+  harmony_step_stats s{};
+  g_kernel_launches = 0;
+  g_prof.on = profiled;
+  g_prof.external = profiled;
+  g_prof.used = 0;
+  g_prof.recs.clear();
+  HM_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+  try {
+    HM_CUDA(cudaEventRecord(c->ev_fork, cs));
+    for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_fork, 0));
+    issue_program(c, x, tg, x_dev, t_dev, s);
+    for (int k = 1; k < S_NUM; ++k) {
+      HM_CUDA(cudaEventRecord(c->ev_join[k], c->st[k]));
+      HM_CUDA(cudaStreamWaitEvent(cs, c->ev_join[k], 0));
+    }
+  } catch (...) {
+    cudaGraph_t g = nullptr;
+    cudaStreamEndCapture(cs, &g);
+    if (g) cudaGraphDestroy(g);
+    cudaGetLastError();
+    g_prof.on = g_prof.external = false;
+    throw;
+  }
+  g_prof.on = g_prof.external = false;
+  HM_CUDA(cudaStreamEndCapture(cs, &G.graph));
+  HM_CUDA(cudaGraphInstantiate(&G.exec, G.graph, 0));
+  G.stats = s;
+  G.launches = g_kernel_launches;
+  G.recs = g_prof.recs;
+  // find the input memcpy nodes by their destinations
+  size_t n = 0;
+  HM_CUDA(cudaGraphGetNodes(G.graph, nullptr, &n));
+  std::vector<cudaGraphNode_t> nodes(n);
+  HM_CUDA(cudaGraphGetNodes(G.graph, nodes.data(), &n));
+  G.in_ops.clear();
+  for (size_t i = 0; i < p.ops.size(); ++i)
+    if (p.ops[i].kind == OP_INPUT) G.in_ops.push_back((int)i);
+  G.in_nodes.assign(G.in_ops.size(), nullptr);
+  for (auto nd : nodes) {
+    cudaGraphNodeType ty;
+    HM_CUDA(cudaGraphNodeGetType(nd, &ty));
+    if (ty != cudaGraphNodeTypeMemcpy) continue;
+    cudaMemcpy3DParms mp;
+    HM_CUDA(cudaGraphMemcpyNodeGetParams(nd, &mp));
+    const uint8_t* dst = static_cast<const uint8_t*>(mp.dstPtr.ptr);
+    for (size_t j = 0; j < G.in_ops.size(); ++j)
+      if (dst == c->arena + p.ops[G.in_ops[j]].dev) G.in_nodes[j] = nd;
+  }
+  for (auto nd : G.in_nodes) HM_CHECK(nd != nullptr, HARMONY_E_CUDA, "graph capture: input copy node not found");
+  G.sig = (x_dev ? 1 : 0) | (t_dev ? 2 : 0);
+}
+
+void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out, harmony_step_stats* out) {
+  Plan& p = c->plan;
+  c->t += 1;
+  *c->h_step = c->t;
+  const PtrKind xk = ptr_kind(x), tk = ptr_kind(tg);
+  const bool x_dev = xk == PTR_DEVICE, t_dev = tk == PTR_DEVICE;
+  // graphs need pinned or device inputs (a pageable copy cannot be captured)
+  const bool use_graph = c->use_graph && xk != PTR_PAGEABLE && tk != PTR_PAGEABLE;
+  harmony_step_stats s{};
+  g_kernel_launches = 0;
+  g_prof.on = c->profiling;
+  g_prof.external = false;
+  g_prof.used = 0;
+  g_prof.recs.clear();
+  cudaStream_t cs = c->st[S_COMPUTE];
+  std::vector<KProf::Rec>* recs = &g_prof.recs;
+  if (use_graph) {
+    StepGraph& G = c->profiling ? c->g_prof : c->g_plain;
+    const int sig = (x_dev ? 1 : 0) | (t_dev ? 2 : 0);
+    if (!G.exec || G.sig != sig) capture_graph(c, G, x, tg, x_dev, t_dev, c->profiling);
+    for (size_t j = 0; j < G.in_nodes.size(); ++j) {
+      const Op& o = p.ops[G.in_ops[j]];
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)x : (const void*)tg);
+      HM_CUDA(cudaGraphExecMemcpyNodeSetParams1D(G.exec, G.in_nodes[j], c->arena + o.dev, src + o.hoff, o.bytes,
+                                                 cudaMemcpyDefault));
+    }
+    HM_CUDA(cudaEventRecord(c->ev_begin, cs));
+    HM_CUDA(cudaGraphLaunch(G.exec, cs));
+    HM_CUDA(cudaEventRecord(c->ev_end[0], cs));
+    HM_CUDA(cudaEventSynchronize(c->ev_end[0]));
+    float ms = 0.f;
+    HM_CUDA(cudaEventElapsedTime(&ms, c->ev_begin, c->ev_end[0]));
+    s = G.stats;
+    s.kernel_launches = G.launches;
+    s.step_seconds = ms * 1e-3;
+    recs = &G.recs;
+  } else {
+    HM_CUDA(cudaEventRecord(c->ev_begin, cs));
+    for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_begin, 0));
+    issue_program(c, x, tg, x_dev, t_dev, s);
+    for (int k = 0; k < S_NUM; ++k) HM_CUDA(cudaEventRecord(c->ev_end[k], c->st[k]));
+    float ms = 0.f;
+    for (int k = 0; k < S_NUM; ++k) {
+      HM_CUDA(cudaEventSynchronize(c->ev_end[k]));
+      float e = 0.f;
+      HM_CUDA(cudaEventElapsedTime(&e, c->ev_begin, c->ev_end[k]));
+      ms = std::max(ms, e);
+    }
+    s.step_seconds = ms * 1e-3;
+    s.kernel_launches = g_kernel_launches;
   }
   HM_CUDA(cudaGetLastError());
-  if (g_prof.on) {
-    for (auto& rc : g_prof.recs) {
+  if (c->profiling) {
+    for (auto& rc : *recs) {
       float e = 0.f;
       HM_CUDA(cudaEventElapsedTime(&e, g_prof.pool[rc.e0], g_prof.pool[rc.e1]));
       c->prof.launches[rc.cat] += 1;
@@ -275,8 +416,9 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
   for (int r = 0; r < p.N; ++r)
     for (int i = 0; i < p.m; ++i) loss += c->h_loss[r * p.m + i];
   if (loss_out) *loss_out = loss;
-  s.step_seconds = ms * 1e-3;
-  s.kernel_launches = g_kernel_launches;
+  s.n_ops = p.ops.size();
+  s.peak_arena_bytes = p.arena_bytes;
+  s.graph = use_graph ? 1 : 0;
   c->last = s;
   if (out) *out = s;
 }
@@ -288,7 +430,7 @@ extern "C" {
 
 int32_t harmony_abi_version(void) { return HARMONY_ABI_VERSION; }
 
-void harmony_abi_sizes(uint64_t out[5]) {
+void harmony_abi_sizes(uint64_t out[6]) {
   out[0] = sizeof(harmony_config);
   out[1] = sizeof(harmony_layer_desc);
   out[2] = sizeof(harmony_step_stats);
@@ -346,6 +488,13 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
     HM_CUDA(cudaEventCreate(&c->ev_end[s]));
   }
   HM_CUDA(cudaEventCreate(&c->ev_begin));
+  HM_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+  for (int s = 0; s < S_NUM; ++s) HM_CUDA(cudaEventCreateWithFlags(&c->ev_join[s], cudaEventDisableTiming));
+  c->h_step = static_cast<int*>(alloc_host(sizeof(int)));
+  {
+    const char* e = getenv("HARMONY_NO_GRAPH");
+    c->use_graph = !(e && *e && *e != '0');
+  }
   if (cfg->arena) {
     HM_CHECK(cfg->hbm_cap_bytes > 0, HARMONY_E_INVALID_ARG, "an adopted arena needs hbm_cap_bytes");
     HM_CHECK(is_device_ptr(cfg->arena), HARMONY_E_INVALID_ARG, "cfg.arena is not a device pointer");

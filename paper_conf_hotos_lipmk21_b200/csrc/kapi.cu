@@ -94,7 +94,7 @@ harmony_status hk_adam(int32_t dtype, int64_t n, float* W, float* m, float* v, c
                        double beta1, double beta2, double eps, int32_t t, void* stream) {
   K_BEGIN
   HM_CHECK(t >= 1, HARMONY_E_INVALID_ARG, "Adam step t starts at 1");
-  adam(dtype, n, W, m, v, g, Wc, lr, beta1, beta2, eps, t, static_cast<cudaStream_t>(stream));
+  adam(dtype, n, W, m, v, g, Wc, lr, beta1, beta2, eps, t, nullptr, static_cast<cudaStream_t>(stream));
   K_END
 }
 

@@ -38,9 +38,11 @@ __device__ __forceinline__ void epi_scalar(const EpiParams& e, int64_t off, int 
       break;
     }
     case HK_EPI_BIAS_ACT: {
-      float z = acc + b;
-      reinterpret_cast<T*>(e.C)[off] = from_f32<T>(z);
-      reinterpret_cast<T*>(e.aux_out)[off] = from_f32<T>(act_f(e.act, z));
+      // act is applied to the STORED pre-activation, so a backward that recomputes act(H) from
+      // the stashed H (stash policies 1, 2) reproduces G bit for bit
+      const T zt = from_f32<T>(acc + b);
+      reinterpret_cast<T*>(e.C)[off] = zt;
+      reinterpret_cast<T*>(e.aux_out)[off] = from_f32<T>(act_f(e.act, to_f32(zt)));
       break;
     }
     case HK_EPI_ACT_BWD: {
@@ -113,7 +115,10 @@ __device__ __forceinline__ void epi_row16(const EpiParams& e, int64_t row_off, i
       cp[1] = o[1];
       if (e.epi == HK_EPI_BIAS_ACT) {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) op[j] = __floats2bfloat162_rn(act_f(e.act, v[2 * j]), act_f(e.act, v[2 * j + 1]));
+        for (int j = 0; j < 8; ++j) {
+          const float2 zr = __bfloat1622float2(op[j]);  // the stored (rounded) pre-activation
+          op[j] = __floats2bfloat162_rn(act_f(e.act, zr.x), act_f(e.act, zr.y));
+        }
         uint4* gp = reinterpret_cast<uint4*>(reinterpret_cast<T*>(e.aux_out) + off);
         gp[0] = o[0];
         gp[1] = o[1];

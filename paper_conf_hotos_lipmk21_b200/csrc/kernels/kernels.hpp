@@ -13,6 +13,13 @@ void gemm(const hk_gemm_args& a, cudaStream_t st);
 void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
                    float* rstd, cudaStream_t st);
 size_t layernorm_bwd_scratch_bytes(int64_t rows, int d);
+// register-resident variants (d % 4 == 0, d <= 2048); return false when not applicable
+bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U,
+                       float* mean, float* rstd, cudaStream_t st);
+size_t layernorm_bwd_vec_scratch_bytes(int64_t rows, int d);
+bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                       const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
+                       int accumulate, float* scratch, cudaStream_t st);
 void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                    const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
                    float* scratch, cudaStream_t st);
@@ -22,8 +29,9 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st);
 void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
                  cudaStream_t st);
+// t_dev (nullable): device int holding the step t (read at execution time; CUDA-graph friendly)
 void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr, double b1, double b2,
-          double eps, int t, cudaStream_t st);
+          double eps, int t, const int* t_dev, cudaStream_t st);
 size_t mse_scratch_bytes();
 void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY, double* loss_out, double* scratch,
          cudaStream_t st);

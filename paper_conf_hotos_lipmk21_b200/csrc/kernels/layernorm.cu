@@ -1,0 +1,251 @@
+// layernorm.cu — register-resident LayerNorm forward/backward (K8).
+//
+// One warp per row; the row is read ONCE with float4 loads and kept in registers (VPT float4 per
+// lane, d <= 128*VPT), so the kernel moves the algorithmic bytes only: fwd reads X (4d) and
+// writes U (ts*d) + 8 B of statistics per row; bwd reads dU, X, dres (12d) and writes dX (4d).
+// Statistics are two-pass on the registers (mean, then centred sum of squares; reading c10).
+// The backward also accumulates this warp's dgamma/dbeta column partials in registers (each lane
+// owns fixed columns), the 8 warps of a block are combined in warp order through shared memory
+// and the block partial is written for the fixed-order column reduction — no atomics.
+#include "../common.hpp"
+#include "kernels.hpp"
+
+namespace hm {
+
+constexpr int LNV_ROWS = 16;  // rows per block in the backward (2 per warp)
+
+__device__ __forceinline__ float wsum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+template <typename T>
+__device__ __forceinline__ float4 ld4(const T* p);
+template <>
+__device__ __forceinline__ float4 ld4<float>(const float* p) { return *reinterpret_cast<const float4*>(p); }
+template <>
+__device__ __forceinline__ float4 ld4<__nv_bfloat16>(const __nv_bfloat16* p) {
+  uint2 u = *reinterpret_cast<const uint2*>(p);
+  __nv_bfloat162 a = *reinterpret_cast<__nv_bfloat162*>(&u.x), b = *reinterpret_cast<__nv_bfloat162*>(&u.y);
+  float2 fa = __bfloat1622float2(a), fb = __bfloat1622float2(b);
+  return make_float4(fa.x, fa.y, fb.x, fb.y);
+}
+template <typename T>
+__device__ __forceinline__ void st4(T* p, float4 v);
+template <>
+__device__ __forceinline__ void st4<float>(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+template <>
+__device__ __forceinline__ void st4<__nv_bfloat16>(__nv_bfloat16* p, float4 v) {
+  __nv_bfloat162 a = __floats2bfloat162_rn(v.x, v.y), b = __floats2bfloat162_rn(v.z, v.w);
+  uint2 u;
+  u.x = *reinterpret_cast<uint32_t*>(&a);
+  u.y = *reinterpret_cast<uint32_t*>(&b);
+  *reinterpret_cast<uint2*>(p) = u;
+}
+
+template <typename T, int VPT>
+__global__ void __launch_bounds__(256) ln_fwd_v(int64_t rows, int d, const float* __restrict__ X,
+                                               const T* __restrict__ g, const T* __restrict__ b, T* __restrict__ U,
+                                               float* __restrict__ mean, float* __restrict__ rstd) {
+  const int lane = threadIdx.x & 31;
+  const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (row >= rows) return;
+  const float* x = X + row * d;
+  float4 v[VPT];
+  float s = 0.f;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    const int c = (j * 32 + lane) * 4;
+    v[j] = c < d ? *reinterpret_cast<const float4*>(x + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+    s += (v[j].x + v[j].y) + (v[j].z + v[j].w);
+  }
+  const float mu = wsum(s) / (float)d;
+  float q = 0.f;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    const int c = (j * 32 + lane) * 4;
+    if (c < d) {
+      float a0 = v[j].x - mu, a1 = v[j].y - mu, a2 = v[j].z - mu, a3 = v[j].w - mu;
+      q += (a0 * a0 + a1 * a1) + (a2 * a2 + a3 * a3);
+    }
+  }
+  const float rs = rsqrtf(wsum(q) / (float)d + 1e-5f);
+  T* u = U + row * d;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    const int c = (j * 32 + lane) * 4;
+    if (c < d) {
+      float4 gg = ld4<T>(g + c), bb = ld4<T>(b + c);
+      st4<T>(u + c, make_float4((v[j].x - mu) * rs * gg.x + bb.x, (v[j].y - mu) * rs * gg.y + bb.y,
+                                (v[j].z - mu) * rs * gg.z + bb.z, (v[j].w - mu) * rs * gg.w + bb.w));
+    }
+  }
+  if (lane == 0) { mean[row] = mu; rstd[row] = rs; }
+}
+
+template <typename T, int VPT>
+__global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float* __restrict__ dU,
+                                               const float* __restrict__ X, const float* __restrict__ mean,
+                                               const float* __restrict__ rstd, const T* __restrict__ g,
+                                               const float* __restrict__ dres, float* __restrict__ dX,
+                                               float* __restrict__ partial) {
+  extern __shared__ float sred[];  // [2d]: block column partials, combined in warp order
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t r0 = (int64_t)blockIdx.x * LNV_ROWS;
+  float4 ag[VPT], ab[VPT];
+  float4 gv[VPT];
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    ag[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+    ab[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+    const int c = (j * 32 + lane) * 4;
+    gv[j] = c < d ? ld4<T>(g + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  for (int i = warp; i < LNV_ROWS; i += 8) {
+    const int64_t row = r0 + i;
+    if (row >= rows) break;
+    const float mu = mean[row], rs = rstd[row];
+    const float* x = X + row * d;
+    const float* du = dU + row * d;
+    float4 xh[VPT], dv[VPT];
+    float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int c = (j * 32 + lane) * 4;
+      if (c < d) {
+        float4 xv = *reinterpret_cast<const float4*>(x + c);
+        dv[j] = *reinterpret_cast<const float4*>(du + c);
+        xh[j] = make_float4((xv.x - mu) * rs, (xv.y - mu) * rs, (xv.z - mu) * rs, (xv.w - mu) * rs);
+        float4 dx = make_float4(dv[j].x * gv[j].x, dv[j].y * gv[j].y, dv[j].z * gv[j].z, dv[j].w * gv[j].w);
+        s1 += (dx.x + dx.y) + (dx.z + dx.w);
+        s2 += (dx.x * xh[j].x + dx.y * xh[j].y) + (dx.z * xh[j].z + dx.w * xh[j].w);
+        ag[j].x += dv[j].x * xh[j].x; ag[j].y += dv[j].y * xh[j].y; ag[j].z += dv[j].z * xh[j].z; ag[j].w += dv[j].w * xh[j].w;
+        ab[j].x += dv[j].x; ab[j].y += dv[j].y; ab[j].z += dv[j].z; ab[j].w += dv[j].w;
+      }
+    }
+    s1 = wsum(s1) / (float)d;
+    s2 = wsum(s2) / (float)d;
+    float* dx = dX + row * d;
+    const float* dr = dres ? dres + row * d : nullptr;
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int c = (j * 32 + lane) * 4;
+      if (c < d) {
+        float4 o = make_float4(rs * (dv[j].x * gv[j].x - s1 - xh[j].x * s2), rs * (dv[j].y * gv[j].y - s1 - xh[j].y * s2),
+                               rs * (dv[j].z * gv[j].z - s1 - xh[j].z * s2), rs * (dv[j].w * gv[j].w - s1 - xh[j].w * s2));
+        if (dr) {
+          float4 rr = *reinterpret_cast<const float4*>(dr + c);
+          o.x = rr.x + o.x; o.y = rr.y + o.y; o.z = rr.z + o.z; o.w = rr.w + o.w;
+        }
+        *reinterpret_cast<float4*>(dx + c) = o;
+      }
+    }
+  }
+  // combine the 8 warps' column partials in warp order (deterministic)
+  for (int w = 0; w < 8; ++w) {
+    if (warp == w) {
+#pragma unroll
+      for (int j = 0; j < VPT; ++j) {
+        const int c = (j * 32 + lane) * 4;
+        if (c < d) {
+          float4* sg = reinterpret_cast<float4*>(sred + c);
+          float4* sb = reinterpret_cast<float4*>(sred + d + c);
+          if (w == 0) {
+            *sg = ag[j];
+            *sb = ab[j];
+          } else {
+            float4 a = *sg, bq = *sb;
+            *sg = make_float4(a.x + ag[j].x, a.y + ag[j].y, a.z + ag[j].z, a.w + ag[j].w);
+            *sb = make_float4(bq.x + ab[j].x, bq.y + ab[j].y, bq.z + ab[j].z, bq.w + ab[j].w);
+          }
+        }
+      }
+    }
+    __syncthreads();
+  }
+  float* pg = partial + (int64_t)blockIdx.x * 2 * d;
+  for (int c = threadIdx.x; c < 2 * d; c += 256) pg[c] = sred[c];
+}
+
+__global__ void colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial, int64_t stride,
+                                  float* __restrict__ out, int accumulate) {
+  int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  float s = 0.f;
+  for (int j = 0; j < nchunks; ++j) s += partial[(int64_t)j * stride + c];
+  out[c] = accumulate ? out[c] + s : s;
+}
+
+static int ln_vpt(int d) {
+  if (d % 4) return 0;
+  int v = (int)ceil_div(d, 128);
+  if (v <= 1) return 1;
+  if (v <= 2) return 2;
+  if (v <= 4) return 4;
+  if (v <= 8) return 8;
+  if (v <= 13) return 13;
+  if (v <= 16) return 16;
+  return 0;  // wider rows: the streaming kernels in ops.cu
+}
+
+bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U,
+                       float* mean, float* rstd, cudaStream_t st) {
+  const int v = ln_vpt(d);
+  if (!v) return false;
+  const unsigned grid = (unsigned)ceil_div(rows, 8);
+#define HM_LNF(T, V) ln_fwd_v<T, V><<<grid, 256, 0, st>>>(rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)
+#define HM_LNF_ALL(T)                   \
+  switch (v) {                          \
+    case 1: HM_LNF(T, 1); break;        \
+    case 2: HM_LNF(T, 2); break;        \
+    case 4: HM_LNF(T, 4); break;        \
+    case 8: HM_LNF(T, 8); break;        \
+    case 13: HM_LNF(T, 13); break;      \
+    default: HM_LNF(T, 16); break;      \
+  }
+  if (dtype == 1) { HM_LNF_ALL(__nv_bfloat16) } else { HM_LNF_ALL(float) }
+#undef HM_LNF_ALL
+#undef HM_LNF
+  check_launch("layernorm_fwd_vec");
+  return true;
+}
+
+size_t layernorm_bwd_vec_scratch_bytes(int64_t rows, int d) {
+  return (size_t)ceil_div(rows, LNV_ROWS) * 2 * d * sizeof(float);
+}
+
+bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                       const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
+                       int accumulate, float* scratch, cudaStream_t st) {
+  const int v = ln_vpt(d);
+  if (!v) return false;
+  const int nblk = (int)ceil_div(rows, LNV_ROWS);
+  const size_t smem = 2 * (size_t)d * sizeof(float);
+#define HM_LNB(T, V)                                                                                   \
+  do {                                                                                                 \
+    if (smem > 48 * 1024)                                                                              \
+      HM_CUDA(cudaFuncSetAttribute(ln_bwd_v<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
+    ln_bwd_v<T, V><<<nblk, 256, smem, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres, dX, scratch); \
+  } while (0)
+#define HM_LNB_ALL(T)                   \
+  switch (v) {                          \
+    case 1: HM_LNB(T, 1); break;        \
+    case 2: HM_LNB(T, 2); break;        \
+    case 4: HM_LNB(T, 4); break;        \
+    case 8: HM_LNB(T, 8); break;        \
+    case 13: HM_LNB(T, 13); break;      \
+    default: HM_LNB(T, 16); break;      \
+  }
+  if (dtype == 1) { HM_LNB_ALL(__nv_bfloat16) } else { HM_LNB_ALL(float) }
+#undef HM_LNB_ALL
+#undef HM_LNB
+  check_launch("layernorm_bwd_vec");
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
+  check_launch("colreduce(dgamma)");
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
+  check_launch("colreduce(dbeta)");
+  return true;
+}
+
+}  // namespace hm

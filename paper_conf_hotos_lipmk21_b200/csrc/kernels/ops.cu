@@ -169,7 +169,17 @@ __global__ void __launch_bounds__(256) softmax_bwd_kernel(int64_t rows, int S, f
 template <typename T>
 __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict__ m, float* __restrict__ v,
                             const float* __restrict__ g, T* __restrict__ Wc, float lr, float b1, float omb1, float b2,
-                            float omb2, float eps, float inv_bc1, float inv_bc2) {
+                            float omb2, float eps, double b1d, double b2d, const int* __restrict__ t_dev, int t_host) {
+  // bias corrections 1/(1-b^t) in double, once per block; t from device memory when given
+  // (a CUDA-graph replay updates it without re-launching)
+  __shared__ float s_bc[2];
+  if (threadIdx.x == 0) {
+    const double t = (double)(t_dev ? *t_dev : t_host);
+    s_bc[0] = (float)(1.0 / (1.0 - pow(b1d, t)));
+    s_bc[1] = (float)(1.0 / (1.0 - pow(b2d, t)));
+  }
+  __syncthreads();
+  const float inv_bc1 = s_bc[0], inv_bc2 = s_bc[1];
   const int64_t n4 = n / 4;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
@@ -278,6 +288,10 @@ void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g
                    float* rstd, cudaStream_t st) {
   if (rows == 0) return;
   const int e0 = g_prof.begin(st);
+  if (layernorm_fwd_vec(dtype, rows, d, X, g, b, U, mean, rstd, st)) {
+    g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 + (dtype ? 2 : 4)) + rows * 8.0);
+    return;
+  }
   HM_DISPATCH_T(dtype, (layernorm_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(
                            rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)));
   check_launch("layernorm_fwd");
@@ -285,7 +299,8 @@ void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g
 }
 
 size_t layernorm_bwd_scratch_bytes(int64_t rows, int d) {
-  return (size_t)ceil_div(rows, LN_ROWS_PER_BLOCK) * 2 * d * sizeof(float);
+  return std::max((size_t)ceil_div(rows, LN_ROWS_PER_BLOCK) * 2 * d * sizeof(float),
+                  layernorm_bwd_vec_scratch_bytes(rows, d));
 }
 
 void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
@@ -294,8 +309,12 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
   if (rows == 0) {
     return;
   }
-  int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
   const int e0 = g_prof.begin(st);
+  if (layernorm_bwd_vec(dtype, rows, d, dU, X, mean, rstd, g, dres, dX, dg, db, accumulate, scratch, st)) {
+    g_prof.end(PROF_LN, e0, st, (double)rows * d * 4 * (dres ? 4 : 3) + rows * 8.0);
+    return;
+  }
+  int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
   HM_DISPATCH_T(dtype, (layernorm_bwd_kernel<T><<<nblk, 256, 0, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres,
                                                                       dX, scratch)));
   check_launch("layernorm_bwd");
@@ -316,10 +335,12 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
     return;
   }
   dim3 grid((unsigned)ceil_div(n, 128), (unsigned)nch);
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
   check_launch("colsum_partial");
   colreduce_kernel<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(nch, n, scratch, n, out, accumulate);
   check_launch("colsum_reduce");
+  g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (in_dtype ? 2 : 4));
 }
 
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st) {
@@ -342,16 +363,14 @@ void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, c
 }
 
 void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, void* Wc, double lr, double b1, double b2,
-          double eps, int t, cudaStream_t st) {
+          double eps, int t, const int* t_dev, cudaStream_t st) {
   if (n == 0) return;
-  // bias corrections computed in double on the host, applied as fp32 reciprocals
-  double bc1 = 1.0 - std::pow(b1, (double)t), bc2 = 1.0 - std::pow(b2, (double)t);
   HM_CHECK(((uintptr_t)W | (uintptr_t)m | (uintptr_t)v | (uintptr_t)g) % 16 == 0, HARMONY_E_INVALID_ARG,
            "adam: fp32 state must be 16-byte aligned");
   const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (adam_kernel<T><<<grid_for(ceil_div(n, 4), 256), 256, 0, st>>>(
                            n, W, m, v, g, (T*)Wc, (float)lr, (float)b1, (float)(1.0 - b1), (float)b2, (float)(1.0 - b2), (float)eps,
-                           (float)(1.0 / bc1), (float)(1.0 / bc2))));
+                           b1, b2, t_dev, t)));
   check_launch("adam");
   g_prof.end(PROF_ADAM, e0, st, (double)n * (16 + 12 + (dtype ? 2 : 4)));  // read W,m,v,g; write W,m,v,Wc
 }
@@ -369,14 +388,18 @@ void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY,
 
 void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st) {
   if (n == 0) return;
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (cast_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(n, in, (T*)out)));
   check_launch("cast");
+  g_prof.end(PROF_OTHER, e0, st, (double)n * (4 + (dtype ? 2 : 4)));
 }
 
 void act_bwd(int dtype, int act, int64_t n, const float* dY, const void* Z, void* dZ, cudaStream_t st) {
   if (n == 0) return;
+  const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(dtype, (act_bwd_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(act, n, dY, (const T*)Z, (T*)dZ)));
   check_launch("act_bwd");
+  g_prof.end(PROF_OTHER, e0, st, (double)n * (4 + 2 * (dtype ? 2 : 4)));
 }
 
 void act_fwd_T(int dtype, int act, int64_t n, const void* Z, void* out, cudaStream_t st) {
@@ -388,8 +411,10 @@ void act_fwd_T(int dtype, int act, int64_t n, const void* Z, void* out, cudaStre
 void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st) {
   if (n == 0) return;
   if (n % 4 == 0 && ((uintptr_t)src | (uintptr_t)dst) % 16 == 0) {
+    const int e0 = g_prof.begin(st);
     copy_rows_kernel<<<grid_for(n / 4, 256), 256, 0, st>>>(n / 4, (const float4*)src, (float4*)dst);
     check_launch("copy_f32");
+    g_prof.end(PROF_OTHER, e0, st, (double)n * 8);
   } else {
     HM_CUDA(cudaMemcpyAsync(dst, src, n * sizeof(float), cudaMemcpyDeviceToDevice, st));
   }

@@ -30,6 +30,26 @@ static uint64_t bump(uint64_t& cur, uint64_t bytes) {
 }
 
 LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_policy) {
+  if (stash_policy == 2 && desc.kind == HARMONY_LAYER_TRANSFORMER) {
+    // Block recompute ([7] P:881): the stash is the block input X; the forward and the
+    // backward both run the policy-0 block on a workspace-resident copy of the full stash.
+    LayerGeom core = make_geom(desc, b, dtype, 0);
+    LayerGeom g = core;
+    g.stash_policy = 2;
+    g.core_st = core.st;
+    g.core_ws_fwd = core.ws_fwd;
+    g.core_ws_bwd = core.ws_bwd;
+    g.st = StashLayout{};
+    uint64_t c = 0;
+    g.st.X = bump(c, (uint64_t)core.rows * core.d * 4);
+    g.st.total = c;
+    const uint64_t full = align_up(core.st.total, 256);
+    g.core_off = 0;
+    g.ws_fwd = full + core.ws_fwd;
+    g.ws_bwd = full + std::max(core.ws_fwd, core.ws_bwd) + align_up((uint64_t)core.rows * core.d * 4, 256);
+    return g;
+  }
+  if (stash_policy == 2) stash_policy = 0;  // MLP: the op-input stash is already minimal
   LayerGeom g;
   g.desc = desc;
   g.dtype = dtype;
@@ -137,7 +157,8 @@ static hk_gemm_args lin_wgrad(const LayerGeom& g, int64_t rows, int n, int k, co
 }
 
 // ------------------------------------------------------------------------------------------------ forward
-void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* stv) {
+static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws,
+                     void* stv) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   if (d.kind == HARMONY_LAYER_MLP) {
@@ -226,8 +247,8 @@ void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint
 }
 
 // ------------------------------------------------------------------------------------------------ backward
-void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
-               int first, uint8_t* ws, void* stv) {
+static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
+                     int first, uint8_t* ws, void* stv) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   const int acc = first ? 0 : 1;
@@ -374,6 +395,37 @@ void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const fl
   // ---- LN1 backward: dX = dX2 + LN1'(dU)
   layernorm_bwd(dt, R, D, dUf, Xs, mean1, rstd1, wseg(g, W, P_LN1_G), dX2, dX, gseg(g, dW, P_LN1_G),
                 gseg(g, dW, P_LN1_B), acc, scratch, st);
+}
+
+// ------------------------------------------------------------------------------------------------ dispatch
+static LayerGeom core_geom(const LayerGeom& g) {
+  LayerGeom c = g;
+  c.stash_policy = 0;
+  c.st = g.core_st;
+  c.ws_fwd = g.core_ws_fwd;
+  c.ws_bwd = g.core_ws_bwd;
+  return c;
+}
+
+void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* st) {
+  if (g.stash_policy != 2) return fwd_core(g, W, X, Y, stash, ws, st);
+  const LayerGeom c = core_geom(g);
+  uint8_t* full = ws + g.core_off;
+  uint8_t* rest = ws + align_up(c.st.total, 256);
+  fwd_core(c, W, X, Y, full, rest, st);
+  copy_f32(g.rows * g.d, X, reinterpret_cast<float*>(stash + g.st.X), static_cast<cudaStream_t>(st));
+}
+
+void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
+               int first, uint8_t* ws, void* st) {
+  if (g.stash_policy != 2) return bwd_core(g, W, stash, dY, dX, dW, first, ws, st);
+  const LayerGeom c = core_geom(g);
+  uint8_t* full = ws + g.core_off;
+  uint8_t* rest = ws + align_up(c.st.total, 256);
+  float* yscratch = reinterpret_cast<float*>(rest + align_up(std::max(c.ws_fwd, c.ws_bwd), 256));
+  // recompute the block's forward from its stashed input: the same kernels, hence the same bits
+  fwd_core(c, W, reinterpret_cast<const float*>(stash + g.st.X), yscratch, full, rest, st);
+  bwd_core(c, W, full, dY, dX, dW, first, rest, st);
 }
 
 }  // namespace hm

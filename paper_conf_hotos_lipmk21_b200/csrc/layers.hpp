@@ -25,7 +25,9 @@ struct LayerGeom {
   harmony_layer_desc desc{};
   int dtype = 0;            // 0 = fp32 activations / SIMT GEMM, 1 = bf16 / tcgen05
   int ts = 4;               // bytes per activation element
-  int stash_policy = 0;     // 0 = all op inputs, 1 = recompute LN outputs and GeLU in the backward
+  int stash_policy = 0;     // 0 = all op inputs, 1 = recompute LN outputs and GeLU in the backward,
+                            // 2 = stash only the block input; the backward recomputes the block
+  int64_t core_off = 0;     // policy 2: offset of the full (policy-0) stash inside the workspace
   int b = 0;                // samples per microbatch
   int64_t rows = 0;         // tokens per microbatch (b*S; MLP: b)
   int d = 0, dh = 0, h = 0, S = 1;
@@ -34,6 +36,8 @@ struct LayerGeom {
   StashLayout st;
   uint64_t ws_fwd = 0, ws_bwd = 0;  // workspace bytes
   double flops_fwd = 0;             // algorithmic GEMM FLOPs of one forward task
+  StashLayout core_st;              // policy 2: the policy-0 layout the recompute materialises
+  uint64_t core_ws_fwd = 0, core_ws_bwd = 0;
 };
 
 enum { P_LN1_G = 0, P_LN1_B, P_WQKV, P_BQKV, P_WO, P_BO, P_LN2_G, P_LN2_B, P_WFC1, P_BFC1, P_WFC2, P_BFC2 };

@@ -27,7 +27,7 @@ void validate_config(const harmony_config& c) {
            "unknown schedule");
   HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
            "the per-GPU-virtualization baseline schedule is not built yet (SURVEY NEXT-3)");
-  HM_CHECK(c.stash_policy == 0 || c.stash_policy == 1, HARMONY_E_INVALID_ARG, "stash_policy must be 0 or 1");
+  HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 2, HARMONY_E_INVALID_ARG, "stash_policy must be 0, 1 or 2");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
@@ -283,7 +283,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     f += align_up(ws_need, ALIGN);                    // one task's transients
     f += nDW * align_up(maxP * 4, ALIGN);             // fp32 dW accumulators
     if (N > 1) f += 2 * align_up(max_shard * 4, ALIGN);  // reduced-gradient shards
-    f += align_up((uint64_t)N * m * 8, ALIGN) + align_up(mse_scratch_bytes(), ALIGN);
+    f += align_up((uint64_t)N * m * 8, ALIGN) + align_up(mse_scratch_bytes(), ALIGN) + ALIGN;
     return f;
   };
   const uint64_t fixed = fixed_bytes();
@@ -387,6 +387,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   if (N > 1) for (int j = 0; j < 2; ++j) p.gsh[j] = a.take(max_shard * 4);
   p.loss = a.take((uint64_t)N * m * 8);
   p.loss_scratch = a.take(mse_scratch_bytes());
+  p.tstep = a.take(256);
   for (int j = 0; j < nW; ++j) p.wslot.push_back(a.take(p.wslot_bytes));
   for (int j = 0; j < nS; ++j) p.sslot.push_back(a.take(p.sslot_bytes));
   for (int j = 0; j < nG; ++j) p.stage.push_back(a.take(p.stage_bytes));

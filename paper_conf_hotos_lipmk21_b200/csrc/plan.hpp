@@ -72,7 +72,7 @@ struct Plan {
   uint64_t ws = 0, ws_bytes = 0;
   uint64_t dw[2] = {0, 0};
   uint64_t gsh[2] = {0, 0};
-  uint64_t loss = 0, loss_scratch = 0;
+  uint64_t loss = 0, loss_scratch = 0, tstep = 0;  // tstep: device int holding Adam's t
   std::vector<uint64_t> wslot, sslot, stage;  // slot offsets
   uint64_t wslot_bytes = 0, sslot_bytes = 0, stage_bytes = 0;
   // program

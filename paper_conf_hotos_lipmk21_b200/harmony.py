@@ -44,7 +44,7 @@ class harmony_step_stats(C.Structure):
         "h2d_bytes", "d2h_bytes", "h2d_weight_bytes", "d2h_weight_bytes", "h2d_state_bytes", "d2h_state_bytes",
         "h2d_stash_bytes", "d2h_stash_bytes", "h2d_input_bytes", "d2h_output_bytes", "h2d_grad_bytes",
         "d2h_grad_bytes", "nvlink_bytes", "peak_arena_bytes", "kernel_launches", "n_ops")] + [
-        ("step_seconds", C.c_double)]
+        ("step_seconds", C.c_double), ("graph", C.c_uint64)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}

@@ -184,14 +184,20 @@ def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal):
     bitwise_equal(capped, uncapped)
 
 
-def test_transformer_bf16_recompute_policy_matches():
-    """stash_policy = 1 recomputes LN outputs and GeLU in the backward: same math, fewer swap bytes."""
-    descs, params, batches, kw = tiny_transformer(True, 1, L=2, d=64, h=2, S=64, B=4, m=2)
+@pytest.mark.parametrize("policy", [1, 2])
+def test_transformer_bf16_recompute_policies_are_bitwise_identical(policy):
+    """stash_policy 1 recomputes LN outputs and GeLU, 2 recomputes the whole block from its input, in
+    the backward: the same kernels recompute the same bits, so the step is bit-identical to policy 0
+    with fewer stash bytes; capped (swapping) runs included."""
+    descs, params, batches, kw = tiny_transformer(True, 1, L=3, d=64, h=2, S=64, B=4, m=2)
     a, pa = run_gpu(descs, params, batches, **kw)
-    b, pb = run_gpu(descs, params, batches, stash_policy=1, **kw)
-    ref = run_oracle(descs, params, batches)
-    compare(b, ref, 2e-2)
+    b, pb = run_gpu(descs, params, batches, stash_policy=policy, **kw)
+    bitwise_equal(a, b)
     assert pb["total_stash_bytes"] < pa["total_stash_bytes"]
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, stash_policy=policy, **kw), descs, text_len=0)
+    c, pc = run_gpu(descs, params, batches, stash_policy=policy, hbm_cap_bytes=int(s.min_working_set_bytes * 1.2), **kw)
+    bitwise_equal(a, c)
+    compare(b, run_oracle(descs, params, batches), 2e-2)
 
 
 def test_device_pointer_inputs_match_host_inputs():
@@ -223,3 +229,23 @@ def test_step_errors():
         H.harmony_step(ctx, X, T, 1)
     assert e.value.code == H.HARMONY_E_BAD_STATE
     H.harmony_finalize(ctx)
+
+
+def test_graph_replay_equals_eager_and_tracks_input_pointers():
+    """Pinned or device inputs replay the captured CUDA graph (input copy nodes re-pointed every
+    step); pageable inputs run the same program eagerly.  Both are bit-identical."""
+    descs, params, batches, kw = tiny_transformer(True, 1, L=2, d=64, h=2, S=64, B=4, m=2)
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, **kw), descs, text_len=0)
+    kw["hbm_cap_bytes"] = int(s.min_working_set_bytes * 1.3)
+    eager, _ = run_gpu(descs, params, batches, **kw)
+    pinned = [(torch.tensor(X).pin_memory(), torch.tensor(T).pin_memory()) for X, T in batches]
+    res = []
+    with H.Harmony(descs, params, retain_grads=1, **kw) as h:
+        for X, T in pinned:
+            loss, st = h.step(X, T)
+            assert st.graph == 1
+            res.append(dict(loss=loss, g=[h.read(l, H.HARMONY_GRAD) for l in range(len(descs))],
+                            W=[h.read(l) for l in range(len(descs))],
+                            m=[h.read(l, H.HARMONY_ADAM_M) for l in range(len(descs))],
+                            v=[h.read(l, H.HARMONY_ADAM_V) for l in range(len(descs))]))
+    bitwise_equal(eager, res)
