@@ -100,6 +100,19 @@ harmony_status hk_cast(int32_t dtype, int64_t n, const float* in, void* out, voi
 harmony_status hk_act_bwd(int32_t dtype, int32_t act, int64_t n, const float* dY, const void* Z, void* dZ,
                           void* stream);
 
+/* Fused multi-head attention forward (bf16, tcgen05; S % 128 == 0, dh in {64, 128}) on the packed
+ * QKV [b*S][3*H*dh] layout: C[b*S][H*dh] (bf16, heads interleaved) = softmax(scale Q K^T (+causal)) V
+ * per head, lse[b][H][S] = log-sum-exp of the scaled scores (natural log).  HARMONY_E_UNSUPPORTED
+ * when the shape does not qualify. */
+harmony_status hk_attention_fwd(int64_t b, int32_t S, int32_t H, int32_t dh, int32_t causal, const void* QKV, void* C,
+                                float* lse, void* stream);
+
+/* Fused attention backward: dQKV[b*S][3d] (bf16: dQ, dK, dV column blocks) from QKV, O = C of the
+ * forward, dO = dC (bf16 [b*S][d]) and lse; deterministic (dS^T materialised, dQ by GEMM).
+ * Synchronous.  Same shape conditions as hk_attention_fwd. */
+harmony_status hk_attention_bwd(int64_t b, int32_t S, int32_t H, int32_t dh, int32_t causal, const void* QKV,
+                                const void* O, const void* dO, const float* lse, void* dQKV, void* stream);
+
 /* Blocks until the device is idle; returns HARMONY_E_CUDA with the message on error. */
 harmony_status hk_sync(void);
 

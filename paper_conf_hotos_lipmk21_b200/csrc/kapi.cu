@@ -121,6 +121,25 @@ harmony_status hk_act_bwd(int32_t dtype, int32_t act, int64_t n, const float* dY
   K_END
 }
 
+harmony_status hk_attention_fwd(int64_t b, int32_t S, int32_t H, int32_t dh, int32_t causal, const void* QKV, void* C,
+                                float* lse, void* stream) {
+  K_BEGIN
+  HM_CHECK(attention_fwd_fused(b, S, H, dh, causal, QKV, C, lse, static_cast<cudaStream_t>(stream)),
+           HARMONY_E_UNSUPPORTED, "fused attention needs S % 128 == 0 and dh in {64, 128}");
+  K_END
+}
+
+harmony_status hk_attention_bwd(int64_t b, int32_t S, int32_t H, int32_t dh, int32_t causal, const void* QKV,
+                                const void* O, const void* dO, const float* lse, void* dQKV, void* stream) {
+  K_BEGIN
+  std::lock_guard<std::mutex> lk(scratch().mu);
+  void* sc = scratch().get(attention_bwd_scratch_bytes(b, S, H));
+  HM_CHECK(attention_bwd_fused(b, S, H, dh, causal, QKV, O, dO, lse, dQKV, sc, static_cast<cudaStream_t>(stream)),
+           HARMONY_E_UNSUPPORTED, "fused attention needs S % 128 == 0 and dh in {64, 128}");
+  HM_CUDA(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+  K_END
+}
+
 harmony_status hk_sync(void) {
   K_BEGIN
   HM_CUDA(cudaDeviceSynchronize());

@@ -1,0 +1,626 @@
+// attention.cu — fused multi-head attention forward on tcgen05 (SURVEY §8(a) rows a4/a5, K4 + K9).
+//
+// One CTA per (128-query tile, head, sequence).  The scores never touch HBM: S = Q K^T lands in
+// TMEM, four softmax warps (one query row per thread) read it with tcgen05.ld, and the
+// probabilities go to shared memory in the UMMA K-major 128B-swizzled layout where they are the A
+// operand of O += P V (accumulated in TMEM).  Softmax is exact and two-pass over the key tiles:
+// pass 1 computes each row's max and sum (online, scalars only), pass 2 recomputes S and
+// normalises P with the final statistics, so O needs no rescaling (1.5x the QK^T FLOPs of a
+// one-pass kernel, in exchange for no TMEM read-modify-write of O).  Outputs: C (bf16, heads
+// interleaved in [T, d]) and the row log-sum-exp (fp32 [b, h, S]) the backward needs.
+// Numerics match the unfused path's reading c11: P = softmax(scale * Q K^T) with causal rows
+// masked to exactly 0 above the diagonal.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include "../common.hpp"
+#include "kernels.hpp"
+#include "tc_common.cuh"
+
+namespace hm {
+namespace attn {
+
+using namespace tcx;
+
+constexpr int BQ = 128;   // query rows per CTA
+constexpr int BKV = 128;  // keys per tile
+constexpr int THREADS = 192;
+
+template <int DH>
+struct FwdCfg {
+  static constexpr int Q_BYTES = BQ * DH * 2;           // DH/64 K-atoms of 16 KB
+  static constexpr int K_BYTES = BKV * DH * 2;
+  static constexpr int V_BYTES = BKV * DH * 2;          // 2 key-atoms x DH/64 MN-chunks of 8 KB
+  static constexpr int P_BYTES = BQ * BKV * 2;          // 2 key-atoms of 16 KB
+  static constexpr int KST = 2, VST = 2, PST = 2;
+  static constexpr int SMEM = Q_BYTES + KST * K_BYTES + VST * V_BYTES + PST * P_BYTES + 1024 + 512;
+  static constexpr int S_COLS = BKV;                    // fp32 accumulator columns per S buffer
+  static constexpr int O_COL = 2 * BKV;                 // O after the two S buffers
+  static constexpr int TMEM_COLS = 512;
+};
+
+struct FwdParams {
+  int S, H, causal;
+  float scale_log2;  // scale * log2(e)
+  float scale;
+  __nv_bfloat16* C;  // [b*S, H*DH]
+  float* lse;        // [b, H, S]
+  int ldc;
+};
+
+template <int DH>
+__global__ void __launch_bounds__(THREADS, 1)
+    attn_fwd_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                    const __grid_constant__ CUtensorMap tmV, FwdParams p) {
+  using Cfg = FwdCfg<DH>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = sQ + Cfg::Q_BYTES;
+  uint8_t* sV = sK + Cfg::KST * Cfg::K_BYTES;
+  uint8_t* sP = sV + Cfg::VST * Cfg::V_BYTES;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + Cfg::PST * Cfg::P_BYTES);
+  uint64_t* q_full = bars;
+  uint64_t* k_full = bars + 1;   // [2]
+  uint64_t* k_empty = bars + 3;  // [2]
+  uint64_t* v_full = bars + 5;   // [2]
+  uint64_t* v_empty = bars + 7;  // [2]
+  uint64_t* s_full = bars + 9;   // [2]
+  uint64_t* s_empty = bars + 11; // [2]
+  uint64_t* p_full = bars + 13;  // [2]
+  uint64_t* p_empty = bars + 15; // [2]
+  uint64_t* o_full = bars + 17;
+  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 18);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int qt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
+  const int q0 = qt * BQ;
+  const int ntiles = p.causal ? qt + 1 : p.S / BKV;
+
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1);
+      mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 128);
+      mbar_init(&p_full[i], 128); mbar_init(&p_empty[i], 1);
+    }
+    mbar_init(o_full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_base_s)),
+                 "r"(Cfg::TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_base_s;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ===== TMA producer: Q once; K tiles for both passes; V tiles for pass 2 =====
+      mbar_expect_tx(q_full, Cfg::Q_BYTES);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) tma_load_4d(sQ + a * (BQ * 128), &tmQ, q_full, a * 64, q0, h, b);
+      int ks = 0; uint32_t kph = 0;
+      int vs = 0; uint32_t vph = 0;
+      for (int pass = 0; pass < 2; ++pass) {
+        for (int j = 0; j < ntiles; ++j) {
+          mbar_wait(&k_empty[ks], kph ^ 1);
+          mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
+#pragma unroll
+          for (int a = 0; a < DH / 64; ++a)
+            tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
+          if (++ks == 2) { ks = 0; kph ^= 1; }
+          if (pass == 1) {
+            mbar_wait(&v_empty[vs], vph ^ 1);
+            mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
+#pragma unroll
+            for (int ka = 0; ka < 2; ++ka)
+#pragma unroll
+              for (int c = 0; c < DH / 64; ++c)
+                tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
+                            j * BKV + ka * 64, h, b);
+            if (++vs == 2) { vs = 0; vph ^= 1; }
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ===== MMA issuer =====
+      // S = Q K^T: M=128, N=128 (keys), K=DH; both operands K-major.
+      const uint32_t idesc_s = make_idesc_f16(128, BKV, 0, 0);
+      // O += P V: M=128, N=DH, K=128 keys; P K-major (smem), V MN-major.
+      const uint32_t idesc_o = make_idesc_f16(128, DH, 0, 1);
+      mbar_wait(q_full, 0);
+      const uint32_t qa = smem_u32(sQ);
+      int ks = 0; uint32_t kph = 0;
+      int vs = 0; uint32_t vph = 0;
+      int it = 0;  // S-buffer use counter across both passes
+      auto issue_s = [&](int sb) {
+        mbar_wait(&k_full[ks], kph);
+        mbar_wait(&s_empty[sb], (((it >> 1) & 1) ^ 1));
+        tc_fence_after();
+        const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const int atom = kk / 4, sub = kk % 4;
+          uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
+          uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
+          mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
+        }
+        mma_commit(&k_empty[ks]);
+        mma_commit(&s_full[sb]);
+        if (++ks == 2) { ks = 0; kph ^= 1; }
+        ++it;
+      };
+      for (int j = 0; j < ntiles; ++j) issue_s(it & 1);  // pass 1
+      // pass 2: S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
+      issue_s(it & 1);
+      for (int j = 0; j < ntiles; ++j) {
+        if (j + 1 < ntiles) issue_s(it & 1);
+        const int pb = j & 1;
+        mbar_wait(&p_full[pb], (j >> 1) & 1);
+        mbar_wait(&v_full[vs], vph);
+        tc_fence_after();
+        const uint32_t pa = smem_u32(sP + pb * Cfg::P_BYTES);
+        const uint32_t va = smem_u32(sV + vs * Cfg::V_BYTES);
+#pragma unroll
+        for (int kk = 0; kk < BKV / 16; ++kk) {
+          const int atom = kk / 4, sub = kk % 4;
+          uint64_t ad = make_sdesc(pa + atom * (BQ * 128) + sub * 32, 16, 1024);
+          uint64_t bd = make_sdesc(va + atom * (DH / 64) * 8192 + sub * 2048, 8192, 1024);
+          mma_bf16(tmem + Cfg::O_COL, ad, bd, idesc_o, (j | kk) ? 1u : 0u);
+        }
+        mma_commit(&v_empty[vs]);
+        mma_commit(&p_empty[pb]);
+        if (++vs == 2) { vs = 0; vph ^= 1; }
+      }
+      mma_commit(o_full);
+    }
+    __syncwarp();
+  } else {
+    // ===== softmax warps: thread = query row =====
+    const int qd = warp & 3;
+    const int r = qd * 32 + lane;        // row within the tile
+    const int qrow = q0 + r;             // query index within the sequence
+    const uint32_t trow = (uint32_t)(qd * 32) << 16;
+    float m = -INFINITY, l = 0.f;
+    int it = 0;
+    // ---- pass 1: row max and sum of exp2((s - m) * scale*log2e)
+    for (int j = 0; j < ntiles; ++j, ++it) {
+      const int sb = it & 1;
+      mbar_wait(&s_full[sb], (it >> 1) & 1);
+      tc_fence_after();
+      const bool diag = p.causal && j == qt;
+#pragma unroll 1
+      for (int c = 0; c < BKV; c += 16) {
+        float v[16];
+        tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
+        float mx = m;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          if (diag && j * BKV + c + i > qrow) v[i] = -INFINITY;
+          mx = fmaxf(mx, v[i]);
+        }
+        float sum = 0.f;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) sum += exp2f((v[i] - mx) * p.scale_log2);
+        l = l * exp2f((m - mx) * p.scale_log2) + sum;
+        m = mx;
+      }
+      tc_fence_before();
+      mbar_arrive_local(&s_empty[sb]);
+    }
+    const float inv_l = 1.f / l;
+    // ---- pass 2: normalised P (bf16) into shared memory, swizzled K-major (A operand of P V)
+    for (int j = 0; j < ntiles; ++j, ++it) {
+      const int sb = it & 1, pb = j & 1;
+      mbar_wait(&s_full[sb], (it >> 1) & 1);
+      mbar_wait(&p_empty[pb], ((j >> 1) & 1) ^ 1);
+      tc_fence_after();
+      const bool diag = p.causal && j == qt;
+      uint8_t* prow = sP + pb * Cfg::P_BYTES + r * 128;
+#pragma unroll 1
+      for (int c = 0; c < BKV; c += 16) {
+        float v[16];
+        tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
+        uint32_t pk[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : exp2f((v[2 * i] - m) * p.scale_log2) * inv_l;
+          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : exp2f((v[2 * i + 1] - m) * p.scale_log2) * inv_l;
+          __nv_bfloat162 h2 = __floats2bfloat162_rn(a0, a1);
+          pk[i] = *reinterpret_cast<uint32_t*>(&h2);
+        }
+        // keys c..c+15 = two 16-byte chunks of key-atom (c / 64), chunk index (c % 64) / 8
+        const int atom = c / 64, ch = (c % 64) / 8;
+        uint8_t* base = prow + atom * (BQ * 128);
+        *reinterpret_cast<uint4*>(base + (((ch) ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        *reinterpret_cast<uint4*>(base + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async (UMMA) reads
+      tc_fence_before();
+      mbar_arrive_local(&s_empty[sb]);
+      mbar_arrive_local(&p_full[pb]);
+    }
+    // ---- epilogue: O row -> bf16 C, LSE
+    mbar_wait(o_full, 0);
+    tc_fence_after();
+    __nv_bfloat16* crow = p.C + ((int64_t)b * p.S + qrow) * p.ldc + h * DH;
+#pragma unroll 1
+    for (int c = 0; c < DH; c += 16) {
+      float v[16];
+      tmem_ld16(tmem + trow + Cfg::O_COL + c, v);
+      uint32_t pk[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+        pk[i] = *reinterpret_cast<uint32_t*>(&h2);
+      }
+      uint4* dst = reinterpret_cast<uint4*>(crow + c);
+      dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+      dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+    }
+    // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
+    p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS) : "memory");
+  }
+}
+
+
+// ============================================================================================ backward
+// One CTA per (128-key tile j, head, sequence), looping over the query tiles i that see it.  With
+// M = keys, the CTA keeps dK_j and dV_j in TMEM for the whole loop.  Per query tile:
+//   S^T = K_j Q_i^T,  dP^T = V_j dO_i^T                      (TMEM, fp32)
+//   P^T = exp(scale S^T - lse_i),  dS^T = scale P^T (dP^T - D_i)   (softmax warps, thread = key)
+//   dV_j += P^T dO_i,  dK_j += dS^T Q_i                       (P^T, dS^T from shared memory)
+// D_i = rowsum(dO_i . O_i) comes from attn_bwd_prep.  dS^T is also written to global memory so that
+// dQ = dS K is one deterministic batched GEMM afterwards (no atomics).  Q_i and dO_i are each
+// staged once: their K-major smem tiles double as the MN-major B operands of dK and dV.
+template <int DH>
+struct BwdCfg {
+  static constexpr int KV_BYTES = BKV * DH * 2;   // K_j or V_j
+  static constexpr int QT_BYTES = BQ * DH * 2;    // Q_i or dO_i
+  static constexpr int ST = DH == 64 ? 2 : 1;     // (Q, dO) stages
+  static constexpr int PS_BYTES = BKV * BQ * 2;   // P^T or dS^T
+  static constexpr int SMEM = 2 * KV_BYTES + ST * 2 * QT_BYTES + 2 * PS_BYTES + 1024 + 512;
+  static constexpr int ST_COL = 0, DP_COL = 128, DV_COL = 256, DK_COL = 256 + DH;
+  static constexpr int TMEM_COLS = 512;
+};
+
+struct BwdParams {
+  int S, H, causal;
+  float scale;
+  const float* lse;    // [b, H, S]
+  const float* D;      // [b, H, S]
+  __nv_bfloat16* dqkv; // [b*S, 3d]: dK, dV columns written here
+  __nv_bfloat16* dst;  // [b, H, S(keys), S(queries)]: scale * dS^T
+  int d;
+};
+
+template <int DH>
+__global__ void __launch_bounds__(THREADS, 1)
+    attn_bwd_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
+                    const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmdO, BwdParams p) {
+  using Cfg = BwdCfg<DH>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sK = smem;
+  uint8_t* sV = sK + Cfg::KV_BYTES;
+  uint8_t* sQ = sV + Cfg::KV_BYTES;                  // [ST] (Q_i, dO_i)
+  uint8_t* sP = sQ + Cfg::ST * 2 * Cfg::QT_BYTES;    // P^T
+  uint8_t* sdS = sP + Cfg::PS_BYTES;                 // dS^T
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sdS + Cfg::PS_BYTES);
+  uint64_t* kv_full = bars;
+  uint64_t* q_full = bars + 1;   // [2]
+  uint64_t* q_empty = bars + 3;  // [2]
+  uint64_t* s_full = bars + 5;
+  uint64_t* s_empty = bars + 6;
+  uint64_t* p_full = bars + 7;
+  uint64_t* p_empty = bars + 8;
+  uint64_t* kd_full = bars + 9;
+  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 10);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int kt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
+  const int k0 = kt * BKV;
+  const int nq = p.S / BQ;
+  const int i0 = p.causal ? kt : 0;
+  const int niter = nq - i0;
+
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO);
+    mbar_init(kv_full, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
+    mbar_init(s_full, 1); mbar_init(s_empty, 128);
+    mbar_init(p_full, 128); mbar_init(p_empty, 1);
+    mbar_init(kd_full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_base_s)),
+                 "r"(Cfg::TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_base_s;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      mbar_expect_tx(kv_full, 2 * Cfg::KV_BYTES);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_4d(sK + a * (BKV * 128), &tmK, kv_full, a * 64, k0, h, b);
+        tma_load_4d(sV + a * (BKV * 128), &tmV, kv_full, a * 64, k0, h, b);
+      }
+      int st = 0; uint32_t ph = 0;
+      for (int n = 0; n < niter; ++n) {
+        const int q0 = (i0 + n) * BQ;
+        mbar_wait(&q_empty[st], ph ^ 1);
+        mbar_expect_tx(&q_full[st], 2 * Cfg::QT_BYTES);
+        uint8_t* q = sQ + st * 2 * Cfg::QT_BYTES;
+        uint8_t* o = q + Cfg::QT_BYTES;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_4d(q + a * (BQ * 128), &tmQ, &q_full[st], a * 64, q0, h, b);
+          tma_load_4d(o + a * (BQ * 128), &tmdO, &q_full[st], a * 64, q0, h, b);
+        }
+        if (++st == Cfg::ST) { st = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      const uint32_t idesc_s = make_idesc_f16(128, BQ, 0, 0);   // S^T, dP^T: M=keys, N=queries, K=DH
+      const uint32_t idesc_g = make_idesc_f16(128, DH, 0, 1);   // dV, dK: M=keys, N=DH, K=queries
+      mbar_wait(kv_full, 0);
+      const uint32_t ka = smem_u32(sK), va = smem_u32(sV);
+      int st = 0; uint32_t ph = 0;
+      for (int n = 0; n < niter; ++n) {
+        mbar_wait(&q_full[st], ph);
+        mbar_wait(s_empty, (n & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t qa = smem_u32(sQ + st * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const int atom = kk / 4, sub = kk % 4;
+          const uint32_t off = atom * (128 * 128) + sub * 32;
+          mma_bf16(tmem + Cfg::ST_COL, make_sdesc(ka + off, 16, 1024), make_sdesc(qa + off, 16, 1024), idesc_s, kk ? 1u : 0u);
+          mma_bf16(tmem + Cfg::DP_COL, make_sdesc(va + off, 16, 1024), make_sdesc(oa + off, 16, 1024), idesc_s, kk ? 1u : 0u);
+        }
+        mma_commit(s_full);
+        mbar_wait(p_full, n & 1);
+        tc_fence_after();
+        const uint32_t pa = smem_u32(sP), da = smem_u32(sdS);
+#pragma unroll
+        for (int kk = 0; kk < BQ / 16; ++kk) {
+          const int atom = kk / 4, sub = kk % 4;
+          const uint32_t aoff = atom * (128 * 128) + sub * 32;  // P^T / dS^T: K-major (K = queries)
+          const uint32_t boff = kk * 2048;                      // dO / Q as MN-major B (k = query rows)
+          const uint32_t acc = (n | kk) ? 1u : 0u;
+          mma_bf16(tmem + Cfg::DV_COL, make_sdesc(pa + aoff, 16, 1024), make_sdesc(oa + boff, 128 * 128, 1024), idesc_g, acc);
+          mma_bf16(tmem + Cfg::DK_COL, make_sdesc(da + aoff, 16, 1024), make_sdesc(qa + boff, 128 * 128, 1024), idesc_g, acc);
+        }
+        mma_commit(p_empty);
+        mma_commit(&q_empty[st]);
+        if (++st == Cfg::ST) { st = 0; ph ^= 1; }
+      }
+      mma_commit(kd_full);
+    }
+    __syncwarp();
+  } else {
+    const int qd = warp & 3;
+    const int r = qd * 32 + lane;   // key row within the tile
+    const int key = k0 + r;
+    const uint32_t trow = (uint32_t)(qd * 32) << 16;
+    const float* lse = p.lse + ((int64_t)b * p.H + h) * p.S;
+    const float* Dv = p.D + ((int64_t)b * p.H + h) * p.S;
+    __nv_bfloat16* dst_row = p.dst + (((int64_t)b * p.H + h) * p.S + key) * p.S;
+    for (int n = 0; n < niter; ++n) {
+      const int q0 = (i0 + n) * BQ;
+      mbar_wait(s_full, n & 1);
+      mbar_wait(p_empty, (n & 1) ^ 1);
+      tc_fence_after();
+      const bool diag = p.causal && (i0 + n) == kt;
+      uint8_t* prow = sP + r * 128;
+      uint8_t* drow = sdS + r * 128;
+#pragma unroll 1
+      for (int c = 0; c < BQ; c += 16) {
+        float sv[16], dp[16];
+        tmem_ld16(tmem + trow + Cfg::ST_COL + c, sv);
+        tmem_ld16(tmem + trow + Cfg::DP_COL + c, dp);
+        uint32_t pk[8], dk[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          float pr[2], dr[2];
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const int q = q0 + c + 2 * i + u;
+            const bool masked = diag && key > q;
+            const float pv = masked ? 0.f : __expf(sv[2 * i + u] * p.scale - __ldg(lse + q));
+            pr[u] = pv;
+            dr[u] = p.scale * pv * (dp[2 * i + u] - __ldg(Dv + q));
+          }
+          __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
+          pk[i] = *reinterpret_cast<uint32_t*>(&a2);
+          dk[i] = *reinterpret_cast<uint32_t*>(&b2);
+        }
+        const int atom = c / 64, ch = (c % 64) / 8;
+        uint8_t* pb = prow + atom * (128 * 128);
+        uint8_t* db = drow + atom * (128 * 128);
+        *reinterpret_cast<uint4*>(pb + ((ch ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        *reinterpret_cast<uint4*>(pb + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        *reinterpret_cast<uint4*>(db + ((ch ^ (r & 7)) << 4)) = make_uint4(dk[0], dk[1], dk[2], dk[3]);
+        *reinterpret_cast<uint4*>(db + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(dk[4], dk[5], dk[6], dk[7]);
+        uint4* g = reinterpret_cast<uint4*>(dst_row + q0 + c);
+        g[0] = make_uint4(dk[0], dk[1], dk[2], dk[3]);
+        g[1] = make_uint4(dk[4], dk[5], dk[6], dk[7]);
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      tc_fence_before();
+      mbar_arrive_local(s_empty);
+      mbar_arrive_local(p_full);
+    }
+    // epilogue: dV_j, dK_j rows -> dQKV (bf16)
+    mbar_wait(kd_full, 0);
+    tc_fence_after();
+    __nv_bfloat16* base = p.dqkv + ((int64_t)b * p.S + key) * 3 * p.d + h * DH;
+#pragma unroll 1
+    for (int part = 0; part < 2; ++part) {
+      __nv_bfloat16* out = base + (part == 0 ? 2 * p.d : p.d);  // dV, then dK
+      const int col = part == 0 ? Cfg::DV_COL : Cfg::DK_COL;
+#pragma unroll 1
+      for (int c = 0; c < DH; c += 16) {
+        float v[16];
+        tmem_ld16(tmem + trow + col + c, v);
+        uint32_t pk[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+          pk[i] = *reinterpret_cast<uint32_t*>(&h2);
+        }
+        uint4* dst = reinterpret_cast<uint4*>(out + c);
+        dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS) : "memory");
+  }
+}
+
+// D[b, h, q] = sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e]   (one thread per (token, head))
+__global__ void attn_bwd_prep(int64_t ntok, int S, int H, int dh, const __nv_bfloat16* __restrict__ dO,
+                              const __nv_bfloat16* __restrict__ O, float* __restrict__ D) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= ntok * H) return;
+  const int64_t tok = t / H;
+  const int h = (int)(t % H);
+  const int d = H * dh;
+  const uint4* a = reinterpret_cast<const uint4*>(dO + tok * d + h * dh);
+  const uint4* o = reinterpret_cast<const uint4*>(O + tok * d + h * dh);
+  float s = 0.f;
+  for (int i = 0; i < dh / 8; ++i) {
+    uint4 x = a[i], y = o[i];
+    const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&x);
+    const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&y);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
+      s += fx.x * fy.x + fx.y * fy.y;
+    }
+  }
+  const int64_t bb = tok / S, q = tok % S;
+  D[(bb * H + h) * S + q] = s;
+}
+}  // namespace attn
+
+// Returns false when the fused path does not apply (then the caller uses GEMM + softmax + GEMM).
+bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, void* C, float* lse,
+                         cudaStream_t st) {
+  using namespace attn;
+  if (S % BQ != 0 || (dh != 64 && dh != 128)) return false;
+  const int d = H * dh;
+  CUtensorMap mq, mk, mv;
+  // Q, K: K-major operands (inner = dh, rows = S, z0 = head, z1 = sequence); V: MN-major (inner = dh)
+  tcx::make_map_4d(&mq, QKV, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BQ);
+  tcx::make_map_4d(&mk, static_cast<const __nv_bfloat16*>(QKV) + d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
+  tcx::make_map_4d(&mv, static_cast<const __nv_bfloat16*>(QKV) + 2 * d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64,
+                   64);
+  FwdParams p;
+  p.S = S; p.H = H; p.causal = causal;
+  p.scale = 1.0f / std::sqrt((float)dh);
+  p.scale_log2 = p.scale * 1.4426950408889634f;
+  p.C = static_cast<__nv_bfloat16*>(C);
+  p.lse = lse;
+  p.ldc = d;
+  dim3 grid((unsigned)(S / BQ), (unsigned)H, (unsigned)b);
+  const int e0 = g_prof.begin(st);
+  if (dh == 64) {
+    static bool set = false;
+    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<64>::SMEM)); set = true; }
+    attn_fwd_kernel<64><<<grid, THREADS, FwdCfg<64>::SMEM, st>>>(mq, mk, mv, p);
+  } else {
+    static bool set = false;
+    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<128>::SMEM)); set = true; }
+    attn_fwd_kernel<128><<<grid, THREADS, FwdCfg<128>::SMEM, st>>>(mq, mk, mv, p);
+  }
+  check_launch("attn_fwd_kernel");
+  // algorithmic FLOPs of the attention contractions (QK^T and PV, causal or not)
+  g_prof.end(PROF_GEMM, e0, st, 4.0 * b * H * (double)S * S * dh);
+  return true;
+}
+
+
+size_t attention_bwd_scratch_bytes(int64_t b, int S, int H) {
+  return align_up((uint64_t)b * H * S * S * 2, 256) + align_up((uint64_t)b * H * S * 4, 256);
+}
+
+// Fused attention backward: dQKV (bf16 [b*S, 3d]) from QKV, O (= C), dO (= dC), lse.
+bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, const void* O, const void* dO,
+                         const float* lse, void* dQKV, void* scratch, cudaStream_t st) {
+  using namespace attn;
+  if (S % BQ != 0 || (dh != 64 && dh != 128)) return false;
+  const int d = H * dh;
+  uint8_t* sc = static_cast<uint8_t*>(scratch);
+  __nv_bfloat16* dst = reinterpret_cast<__nv_bfloat16*>(sc);
+  float* D = reinterpret_cast<float*>(sc + align_up((uint64_t)b * H * S * S * 2, 256));
+  const int e0 = g_prof.begin(st);
+  const int64_t n = b * S * H;
+  attn_bwd_prep<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(b * S, S, H, dh, static_cast<const __nv_bfloat16*>(dO),
+                                                           static_cast<const __nv_bfloat16*>(O), D);
+  check_launch("attn_bwd_prep");
+  if (causal) HM_CUDA(cudaMemsetAsync(dst, 0, (size_t)b * H * S * S * 2, st));  // key tiles never visited by a query tile
+  CUtensorMap mq, mk, mv, mo;
+  const __nv_bfloat16* q = static_cast<const __nv_bfloat16*>(QKV);
+  tcx::make_map_4d(&mq, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BQ);
+  tcx::make_map_4d(&mk, q + d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
+  tcx::make_map_4d(&mv, q + 2 * d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
+  tcx::make_map_4d(&mo, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BQ);
+  BwdParams p;
+  p.S = S; p.H = H; p.causal = causal;
+  p.scale = 1.0f / std::sqrt((float)dh);
+  p.lse = lse; p.D = D;
+  p.dqkv = static_cast<__nv_bfloat16*>(dQKV);
+  p.dst = dst;
+  p.d = d;
+  dim3 grid((unsigned)(S / BKV), (unsigned)H, (unsigned)b);
+  if (dh == 64) {
+    static bool set = false;
+    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<64>::SMEM)); set = true; }
+    attn_bwd_kernel<64><<<grid, THREADS, BwdCfg<64>::SMEM, st>>>(mq, mk, mv, mo, p);
+  } else {
+    static bool set = false;
+    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }
+    attn_bwd_kernel<128><<<grid, THREADS, BwdCfg<128>::SMEM, st>>>(mq, mk, mv, mo, p);
+  }
+  check_launch("attn_bwd_kernel");
+  g_prof.end(PROF_GEMM, e0, st, 8.0 * b * H * (double)S * S * dh);  // S^T, dP^T, dV, dK contractions
+  // dQ = dS K: A(m=q, k=key) = dS^T[key][q] (MN-major), B(n=e, k=key) = K[key][e] (MN-major)
+  hk_gemm_args a = gemm_args(1, S, dh, S);
+  a.nz0 = H; a.nz1 = (int)b;
+  a.A = dst; a.a_mn_major = 1; a.lda = S; a.a_sz0 = (int64_t)S * S; a.a_sz1 = (int64_t)H * S * S;
+  a.B = q + d; a.b_mn_major = 1; a.ldb = 3 * d; a.b_sz0 = dh; a.b_sz1 = (int64_t)S * 3 * d;
+  a.C = dQKV; a.ldc = 3 * d; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * 3 * d;
+  a.epilogue = HK_EPI_STORE_T;
+  gemm(a, st);
+  return true;
+}
+
+}  // namespace hm

@@ -18,6 +18,7 @@
 #include <mutex>
 
 #include "epilogue.cuh"
+#include "tc_common.cuh"
 
 namespace hm {
 
@@ -90,78 +91,9 @@ constexpr int BK = 64;                 // 64 bf16 = 128 bytes = one 128B swizzle
 constexpr int EPI_WARPS = 8;           // two epilogue warps per TMEM lane quadrant (column halves)
 constexpr int NUM_THREADS = 64 + 32 * EPI_WARPS;  // warp 0: TMA, warp 1: MMA + TMEM alloc, warps 2..9: epilogue
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+using namespace tcx;
 
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ bool mbar_try_wait(uint32_t addr, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-      "selp.u32 %0, 1, 0, p;\n\t}"
-      : "=r"(ok)
-      : "r"(addr), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  uint32_t a = smem_u32(bar);
-  while (!mbar_try_wait(a, parity)) {
-  }
-}
-__device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
-                                            int c3) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(
-          smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
-      : "memory");
-}
-__device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
-  asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
-}
-// UMMA shared-memory descriptor (sm_100): start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
-// version 1 [46,48), base offset 0, layout type SWIZZLE_128B = 2 at [61,64).
-__device__ __forceinline__ uint64_t make_sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
-  return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
-         ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46) | (2ull << 61);
-}
-// Instruction descriptor, kind::f16: D=F32 [4,6)=1, A=BF16 [7,10)=1, B=BF16 [10,13)=1,
-// a_major bit 15, b_major bit 16 (1 = MN-major), N>>3 at [17,23), M>>4 at [24,29).
-__device__ __forceinline__ uint32_t make_idesc(int bn, int a_mn, int b_mn) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
-         ((uint32_t)(bn >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
-}
-__device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
-}
-__device__ __forceinline__ void mma_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-               : "memory");
-}
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
-  uint32_t r[16];
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
-        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-      : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
-}
+__device__ __forceinline__ uint32_t make_idesc(int bn, int a_mn, int b_mn) { return make_idesc_f16(BM, bn, a_mn, b_mn); }
 
 struct TcParams {
   int M, N, K, nz0, nz, a_mn, b_mn;
@@ -345,51 +277,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   }
 }
 
-// ----- host: tensor maps through the driver entry point (no link-time libcuda dependency)
-static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  static std::once_flag once;
-  std::call_once(once, [] {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-  });
-  return fn;
-}
-
 // Operand (rows r, K) as a 4-D bf16 map (inner, outer, z0, z1).  K-major: inner = K, box (64, box_r);
 // MN-major: inner = r, box (64, BK).
 static void make_operand_map(CUtensorMap* map, const void* ptr, int mn_major, int64_t rows, int64_t K, int64_t ld,
                              int64_t nz0, int64_t sz0, int64_t nz1, int64_t sz1, int box_r) {
-  auto enc = get_encode();
-  HM_CHECK(enc != nullptr, HARMONY_E_CUDA, "cuTensorMapEncodeTiled unavailable (driver too old?)");
-  HM_CHECK((reinterpret_cast<uintptr_t>(ptr) & 15) == 0, HARMONY_E_UNSUPPORTED, "bf16 GEMM operand not 16-byte aligned");
-  HM_CHECK(ld % 8 == 0, HARMONY_E_UNSUPPORTED, "bf16 GEMM leading dimension must be a multiple of 8");
-  cuuint64_t dims[4];
-  cuuint64_t strides[3];
-  cuuint32_t box[4];
-  cuuint32_t estr[4] = {1, 1, 1, 1};
-  int64_t inner = mn_major ? rows : K, outer = mn_major ? K : rows;
-  dims[0] = (cuuint64_t)inner;
-  dims[1] = (cuuint64_t)outer;
-  dims[2] = (cuuint64_t)nz0;
-  dims[3] = (cuuint64_t)nz1;
-  strides[0] = (cuuint64_t)ld * 2;
-  int64_t s1 = nz0 > 1 ? sz0 * 2 : (int64_t)align_up((uint64_t)(ld * outer * 2), 16);
-  int64_t s2 = nz1 > 1 ? sz1 * 2 : (int64_t)align_up((uint64_t)(s1 * nz0), 16);
-  HM_CHECK(s1 % 16 == 0 && s2 % 16 == 0, HARMONY_E_UNSUPPORTED, "bf16 GEMM batch strides must be multiples of 8");
-  strides[1] = (cuuint64_t)s1;
-  strides[2] = (cuuint64_t)s2;
-  box[0] = 64;
-  box[1] = mn_major ? BK : box_r;
-  box[2] = 1;
-  box[3] = 1;
-  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(ptr), dims, strides, box, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  HM_CHECK(r == CUDA_SUCCESS, HARMONY_E_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
+  const int64_t inner = mn_major ? rows : K, outer = mn_major ? K : rows;
+  make_map_4d(map, ptr, inner, outer, nz0, nz1, ld, sz0, sz1, 64, mn_major ? BK : box_r);
 }
 
 template <int BN, int STAGES>

@@ -38,6 +38,13 @@ void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY,
 void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st);
 void act_bwd(int dtype, int act, int64_t n, const float* dY, const void* Z, void* dZ, cudaStream_t st);
 void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st);
+// fused attention forward (attention.cu); false when the shape does not qualify
+bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, void* C, float* lse,
+                         cudaStream_t st);
+// fused attention backward: dQKV from QKV, O, dO, lse (scratch: attention_bwd_scratch_bytes)
+size_t attention_bwd_scratch_bytes(int64_t b, int S, int H);
+bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, const void* O, const void* dO,
+                         const float* lse, void* dQKV, void* scratch, cudaStream_t st);
 
 // Convenience: a GEMM descriptor with defaults (batch 1, alpha 1, no bias/aux).
 inline hk_gemm_args gemm_args(int dtype, int M, int N, int K) {

@@ -12,7 +12,7 @@
 
 namespace hm {
 
-constexpr int LNV_ROWS = 16;  // rows per block in the backward (2 per warp)
+constexpr int LNV_ROWS = 32;  // rows per block in the backward (4 per warp)
 
 __device__ __forceinline__ float wsum(float v) {
 #pragma unroll
@@ -168,13 +168,23 @@ __global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float
   for (int c = threadIdx.x; c < 2 * d; c += 256) pg[c] = sred[c];
 }
 
-__global__ void colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial, int64_t stride,
-                                  float* __restrict__ out, int accumulate) {
-  int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= n) return;
+// fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 8 warps per block
+__global__ void __launch_bounds__(256) colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial,
+                                                         int64_t stride, float* __restrict__ out, int accumulate) {
+  __shared__ float sh[8][33];
+  const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + cl;
   float s = 0.f;
-  for (int j = 0; j < nchunks; ++j) s += partial[(int64_t)j * stride + c];
-  out[c] = accumulate ? out[c] + s : s;
+  if (c < n)
+    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];
+  sh[g][cl] = s;
+  __syncthreads();
+  if (g == 0 && c < n) {
+    float t = sh[0][cl];
+#pragma unroll
+    for (int k = 1; k < 8; ++k) t += sh[k][cl];
+    out[c] = accumulate ? out[c] + t : t;
+  }
 }
 
 static int ln_vpt(int d) {
@@ -241,9 +251,9 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
 #undef HM_LNB_ALL
 #undef HM_LNB
   check_launch("layernorm_bwd_vec");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
   check_launch("colreduce(dgamma)");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
   check_launch("colreduce(dbeta)");
   return true;
 }

@@ -104,14 +104,30 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(int64_t rows, int d,
   }
 }
 
-// out[c] (+)= sum over chunks j in order of partial[j][c]  (partial row stride `stride`)
-__global__ void colreduce_kernel(int nchunks, int n, const float* __restrict__ partial, int64_t stride,
-                                 float* __restrict__ out, int accumulate) {
-  int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= n) return;
+// out[c] (+)= sum over chunks of partial[j][c] (row stride `stride`): 32 columns per block, 8 warps
+// each summing every 8th chunk, then the 8 warp sums in warp order — a fixed tree (deterministic),
+// coalesced along the columns and 8x more memory-level parallelism than one thread per column.
+__global__ void __launch_bounds__(256) colreduce_kernel(int nchunks, int n, const float* __restrict__ partial,
+                                                        int64_t stride, float* __restrict__ out, int accumulate) {
+  __shared__ float sh[8][33];
+  const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + cl;
   float s = 0.f;
-  for (int j = 0; j < nchunks; ++j) s += partial[(int64_t)j * stride + c];
-  out[c] = accumulate ? out[c] + s : s;
+  if (c < n)
+    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];
+  sh[g][cl] = s;
+  __syncthreads();
+  if (g == 0 && c < n) {
+    float t = sh[0][cl];
+#pragma unroll
+    for (int k = 1; k < 8; ++k) t += sh[k][cl];
+    out[c] = accumulate ? out[c] + t : t;
+  }
+}
+static void colreduce(int nchunks, int n, const float* partial, int64_t stride, float* out, int accumulate,
+                      cudaStream_t st) {
+  colreduce_kernel<<<(unsigned)ceil_div(n, 32), 256, 0, st>>>(nchunks, n, partial, stride, out, accumulate);
+  check_launch("colreduce");
 }
 
 // ------------------------------------------------------------------------------------- column sums
@@ -241,11 +257,19 @@ __global__ void mse_kernel(int64_t n, const float* __restrict__ Y, const float* 
     partial[blockIdx.x] = s;
   }
 }
-__global__ void mse_final_kernel(int nblk, const double* __restrict__ partial, double half_inv_batch,
-                                 double* __restrict__ out) {
+// fixed-order tree over the block partials: thread t sums t, t+256, ...; then a smem tree
+__global__ void __launch_bounds__(256) mse_final_kernel(int nblk, const double* __restrict__ partial,
+                                                        double half_inv_batch, double* __restrict__ out) {
+  __shared__ double sh[256];
   double s = 0.0;
-  for (int j = 0; j < nblk; ++j) s += partial[j];
-  *out = s * half_inv_batch;
+  for (int j = threadIdx.x; j < nblk; j += 256) s += partial[j];
+  sh[threadIdx.x] = s;
+  __syncthreads();
+  for (int w = 128; w > 0; w >>= 1) {
+    if (threadIdx.x < w) sh[threadIdx.x] += sh[threadIdx.x + w];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *out = sh[0] * half_inv_batch;
 }
 
 // ------------------------------------------------------------------------------------- elementwise
@@ -318,10 +342,8 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
   HM_DISPATCH_T(dtype, (layernorm_bwd_kernel<T><<<nblk, 256, 0, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres,
                                                                       dX, scratch)));
   check_launch("layernorm_bwd");
-  colreduce_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
-  check_launch("colreduce(dgamma)");
-  colreduce_kernel<<<(unsigned)ceil_div(d, 256), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
-  check_launch("colreduce(dbeta)");
+  colreduce(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate, st);
+  colreduce(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate, st);
   g_prof.end(PROF_LN, e0, st, (double)rows * d * 4 * (dres ? 4 : 3) + rows * 8.0);
 }
 
@@ -338,8 +360,7 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
   const int e0 = g_prof.begin(st);
   HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
   check_launch("colsum_partial");
-  colreduce_kernel<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(nch, n, scratch, n, out, accumulate);
-  check_launch("colsum_reduce");
+  colreduce(nch, n, scratch, n, out, accumulate, st);
   g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (in_dtype ? 2 : 4));
 }
 
@@ -382,7 +403,7 @@ void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY,
   int nblk = (int)std::min<int64_t>(1024, std::max<int64_t>(1, ceil_div(n, MSE_BLOCK * 8)));
   mse_kernel<<<nblk, MSE_BLOCK, 0, st>>>(n, Y, Tg, inv_batch, dY, scratch);
   check_launch("mse");
-  mse_final_kernel<<<1, 1, 0, st>>>(nblk, scratch, 0.5 * (double)inv_batch, loss_out);
+  mse_final_kernel<<<1, 256, 0, st>>>(nblk, scratch, 0.5 * (double)inv_batch, loss_out);
   check_launch("mse_final");
 }
 

@@ -86,13 +86,16 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   for (int i = 0; i < 12; ++i) { g.off[i] = o; o += seg[i]; }
   const uint64_t R = (uint64_t)g.rows, ts = (uint64_t)g.ts;
   const uint64_t SS = (uint64_t)b * g.h * g.S * g.S;
+  // fused tcgen05 attention (scores in TMEM, no S x S tensor in HBM) when the shape qualifies
+  g.fused_attn = dtype == 1 && g.S % 128 == 0 && (g.dh == 64 || g.dh == 128);
+  const uint64_t BHS = (uint64_t)b * g.h * g.S;
   uint64_t c = 0;
   g.st.X = bump(c, R * D * 4);
   g.st.mean1 = bump(c, R * 4);
   g.st.rstd1 = bump(c, R * 4);
   if (stash_policy == 0) g.st.U = bump(c, R * D * ts);
   g.st.QKV = bump(c, R * 3 * D * ts);
-  g.st.P = bump(c, SS * ts);
+  g.st.P = bump(c, g.fused_attn ? BHS * 4 : SS * ts);  // fused: row log-sum-exp instead of P
   g.st.C = bump(c, R * D * ts);
   g.st.X2 = bump(c, R * D * 4);
   g.st.mean2 = bump(c, R * 4);
@@ -103,7 +106,7 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   g.st.total = c;
   // forward workspace: scores Z (fp32) [+ recomputable U, U2, G under policy 1]
   uint64_t wf = 0;
-  bump(wf, SS * 4);
+  bump(wf, g.fused_attn ? 256 : SS * 4);
   if (stash_policy == 1) { bump(wf, R * D * ts); bump(wf, R * D * ts); bump(wf, R * 4 * D * ts); }
   g.ws_fwd = wf;
   // backward workspace (see layer_bwd for the aliasing)
@@ -113,8 +116,13 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   bump(wb, R * D * 4);           // dU2 / dU (fp32)
   bump(wb, R * D * 4);           // dX2 (fp32)
   bump(wb, R * D * ts);          // dC
-  bump(wb, SS * 4);              // dP (fp32)
-  bump(wb, SS * ts);             // dZ
+  if (g.fused_attn) {
+    bump(wb, attention_bwd_scratch_bytes(b, g.S, g.h));  // dS^T (bf16) + D
+    bump(wb, 256);
+  } else {
+    bump(wb, SS * 4);              // dP (fp32)
+    bump(wb, SS * ts);             // dZ
+  }
   bump(wb, bwd_scratch_bytes(g.rows, (int)D));
   if (stash_policy == 1) bump(wb, R * 4 * D * ts);  // recomputed G / U2 / U
   g.ws_bwd = wb;
@@ -185,7 +193,7 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   float* rstd2 = reinterpret_cast<float*>(stash + g.st.rstd2);
   uint8_t* Hh = stash + g.st.H;
   uint64_t wc = 0;
-  float* Z = reinterpret_cast<float*>(ws + bump(wc, (uint64_t)b * H * S * S * 4));
+  float* Z = reinterpret_cast<float*>(ws + bump(wc, g.fused_attn ? 256 : (uint64_t)b * H * S * S * 4));
   uint8_t *U, *U2, *G;
   if (g.stash_policy == 0) {
     U = stash + g.st.U; U2 = stash + g.st.U2; G = stash + g.st.G;
@@ -202,6 +210,11 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
     a.C = QKV; a.epilogue = HK_EPI_STORE_T; a.bias = wseg(g, W, P_BQKV);
     gemm(a, st);
   }
+  if (g.fused_attn) {
+    // C = softmax(Q K^T / sqrt(dh)) V per head, scores kept in TMEM; stash the row LSE
+    HM_CHECK(attention_fwd_fused(b, S, H, dh, d.causal, QKV, C, reinterpret_cast<float*>(P), st), HARMONY_E_INVALID_ARG,
+             "fused attention rejected a qualifying shape");
+  } else {
   // Z[b,h] = Q_h K_h^T (fp32), batched over heads (z0) and sequences (z1)
   {
     hk_gemm_args a = gemm_args(g.dtype, S, S, dh);
@@ -223,6 +236,7 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
     a.C = C; a.ldc = D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * D;
     a.epilogue = HK_EPI_STORE_T;
     gemm(a, st);
+  }
   }
   // X2 = X + C W_o + b_o   (fp32 residual stream)
   {
@@ -289,8 +303,16 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   float* dUf = reinterpret_cast<float*>(ws + bump(wc, R * D * 4));
   float* dX2 = reinterpret_cast<float*>(ws + bump(wc, R * D * 4));
   uint8_t* dC = ws + bump(wc, R * D * ts);
-  float* dP = reinterpret_cast<float*>(ws + bump(wc, SS * 4));
-  uint8_t* dZ = ws + bump(wc, SS * ts);
+  float* dP = nullptr;
+  uint8_t* dZ = nullptr;
+  uint8_t* attn_scratch = nullptr;
+  if (g.fused_attn) {
+    attn_scratch = ws + bump(wc, attention_bwd_scratch_bytes(b, S, H));
+    bump(wc, 256);
+  } else {
+    dP = reinterpret_cast<float*>(ws + bump(wc, SS * 4));
+    dZ = ws + bump(wc, SS * ts);
+  }
   float* scratch = reinterpret_cast<float*>(ws + bump(wc, bwd_scratch_bytes(R, D)));
   uint8_t* rec = g.stash_policy == 1 ? ws + bump(wc, R * 4 * D * ts) : nullptr;
 
@@ -339,6 +361,11 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   // ---- attention backward (batched over heads z0 and sequences z1)
   uint8_t* dQKV = dHb;
   const float scale = 1.0f / std::sqrt((float)dh);
+  if (g.fused_attn) {
+    HM_CHECK(attention_bwd_fused(b, S, H, dh, d.causal, QKV, C, dC, reinterpret_cast<const float*>(P), dQKV,
+                                 attn_scratch, st),
+             HARMONY_E_INVALID_ARG, "fused attention rejected a qualifying shape");
+  } else {
   {  // dP = dC_h V_h^T
     hk_gemm_args a = gemm_args(dt, S, S, dh);
     a.nz0 = H; a.nz1 = b;
@@ -376,6 +403,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     a.C = dQKV + (size_t)D * ts; a.ldc = 3 * D; a.c_sz0 = dh; a.c_sz1 = (int64_t)S * 3 * D;
     a.epilogue = HK_EPI_STORE_T;
     gemm(a, st);
+  }
   }
   // ---- QKV projection: dU = dQKV W_qkv^T; dW_qkv += U^T dQKV; db_qkv += sum dQKV
   {

@@ -31,6 +31,7 @@ struct LayerGeom {
   int b = 0;                // samples per microbatch
   int64_t rows = 0;         // tokens per microbatch (b*S; MLP: b)
   int d = 0, dh = 0, h = 0, S = 1;
+  bool fused_attn = false;  // tcgen05 fused attention (bf16, S % 128 == 0, dh in {64, 128})
   int64_t n_params = 0;     // canonical packing length
   int64_t off[12] = {};     // parameter segment offsets (elements): transformer order of harmony.h
   StashLayout st;

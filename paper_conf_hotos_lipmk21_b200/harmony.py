@@ -135,6 +135,8 @@ def lib() -> C.CDLL:
         "hk_cast": (st, [C.c_int32, C.c_int64, P, P, P]),
         "hk_act_bwd": (st, [C.c_int32, C.c_int32, C.c_int64, P, P, P, P]),
         "hk_sync": (st, []),
+        "hk_attention_fwd": (st, [C.c_int64, C.c_int32, C.c_int32, C.c_int32, C.c_int32, P, P, P, P]),
+        "hk_attention_bwd": (st, [C.c_int64, C.c_int32, C.c_int32, C.c_int32, C.c_int32, P, P, P, P, P, P]),
         "harmony_abi_sizes": (None, [P]),
         "harmony_set_profiling": (st, [P, C.c_int32]),
         "harmony_read_profile": (st, [P, C.POINTER(harmony_kernel_profile)]),

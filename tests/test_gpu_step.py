@@ -169,9 +169,10 @@ def test_transformer_fp32_matches_oracle(causal):
     print("fp32 transformer teacher-forced worst rel", teacher_forced(descs, params, batches, gpu, 1e-5))
 
 
+@pytest.mark.parametrize("S", [136, 256])  # 136: GEMM + softmax attention path; 256: fused tcgen05 attention
 @pytest.mark.parametrize("causal", [False, True])
-def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal):
-    descs, params, batches, kw = tiny_transformer(causal, 1, L=3, d=128, h=2, S=136, B=4, m=2)
+def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal, S):
+    descs, params, batches, kw = tiny_transformer(causal, 1, L=3, d=128, h=2, S=S, B=4, m=2)
     uncapped, plan = run_gpu(descs, params, batches, **kw)
     ref = run_oracle(descs, params, batches)
     w = compare(uncapped, ref, 2e-2)
@@ -184,12 +185,13 @@ def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal):
     bitwise_equal(capped, uncapped)
 
 
+@pytest.mark.parametrize("S", [64, 128])
 @pytest.mark.parametrize("policy", [1, 2])
-def test_transformer_bf16_recompute_policies_are_bitwise_identical(policy):
+def test_transformer_bf16_recompute_policies_are_bitwise_identical(policy, S):
     """stash_policy 1 recomputes LN outputs and GeLU, 2 recomputes the whole block from its input, in
     the backward: the same kernels recompute the same bits, so the step is bit-identical to policy 0
     with fewer stash bytes; capped (swapping) runs included."""
-    descs, params, batches, kw = tiny_transformer(True, 1, L=3, d=64, h=2, S=64, B=4, m=2)
+    descs, params, batches, kw = tiny_transformer(True, 1, L=3, d=128, h=2, S=S, B=4, m=2)
     a, pa = run_gpu(descs, params, batches, **kw)
     b, pb = run_gpu(descs, params, batches, stash_policy=policy, **kw)
     bitwise_equal(a, b)
