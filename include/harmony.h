@@ -212,6 +212,23 @@ harmony_status harmony_plan_info(const harmony_ctx* ctx, harmony_plan_summary* o
 harmony_status harmony_plan_dry(const harmony_config* cfg, int32_t n_layers, const harmony_layer_desc* descs,
                                 harmony_plan_summary* out, char* program_text, uint64_t text_len);
 
+/* ---- Operator decomposition of one GEMM fwd+bwd across the DP group.
+ * Y = X.W with X [M,K], W [K,N] (bf16, row-major), K split across the world_size ranks: rank r passes
+ * its K-slice X[:, r*K/N' .. ] as a [M][K/N'] array and W[r*K/N' .., :] as [K/N'][N] (N' = world).
+ * The forward runs as `chunks` row-chunk tile subtasks whose fp32 partials are reduce-scattered
+ * (NCCL) while the next chunk computes; rank r receives Y_shard = rows [r*M/N', (r+1)*M/N') of Y
+ * (fp32).  Backward: dY_shard (bf16, the same rows) is all-gathered, then dX_slice = dY.W_slice^T
+ * (bf16 [M][K/N']) and dW_slice = X_slice^T.dY (fp32 [K/N'][N]) are computed locally.  All pointers are
+ * DEVICE pointers owned by the caller; run() is synchronous and collective (every rank calls it).
+ * Requirements: K % (8*world) == 0, M % (world*chunks) == 0, M and N multiples of 8. */
+typedef struct harmony_split_gemm harmony_split_gemm;
+harmony_status harmony_split_gemm_init(const harmony_config* cfg, int64_t M, int64_t N, int64_t K, int32_t chunks,
+                                       harmony_split_gemm** out);
+harmony_status harmony_split_gemm_run(harmony_split_gemm* g, const void* X_slice, const void* W_slice,
+                                      const void* dY_shard, float* Y_shard, void* dX_slice, float* dW_slice,
+                                      double* seconds);
+harmony_status harmony_split_gemm_finalize(harmony_split_gemm* g);
+
 /* Frees every device and pinned allocation and the communicator; ctx is invalid after. */
 harmony_status harmony_finalize(harmony_ctx* ctx);
 

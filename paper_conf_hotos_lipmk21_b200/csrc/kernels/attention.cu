@@ -22,6 +22,13 @@ namespace attn {
 
 using namespace tcx;
 
+// 2^x on the SFU (ex2.approx.ftz: ~2 ulp, the same unit __expf uses)
+__device__ __forceinline__ float fast_exp2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
 constexpr int BQ = 128;   // query rows per CTA
 constexpr int BKV = 128;  // keys per tile
 constexpr int THREADS = 192;
@@ -209,8 +216,8 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
         float sum = 0.f;
 #pragma unroll
-        for (int i = 0; i < 16; ++i) sum += exp2f((v[i] - mx) * p.scale_log2);
-        l = l * exp2f((m - mx) * p.scale_log2) + sum;
+        for (int i = 0; i < 16; ++i) sum += fast_exp2((v[i] - mx) * p.scale_log2);
+        l = l * fast_exp2((m - mx) * p.scale_log2) + sum;
         m = mx;
       }
       tc_fence_before();
@@ -232,8 +239,8 @@ __global__ void __launch_bounds__(THREADS, 1)
         uint32_t pk[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : exp2f((v[2 * i] - m) * p.scale_log2) * inv_l;
-          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : exp2f((v[2 * i + 1] - m) * p.scale_log2) * inv_l;
+          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : fast_exp2((v[2 * i] - m) * p.scale_log2) * inv_l;
+          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : fast_exp2((v[2 * i + 1] - m) * p.scale_log2) * inv_l;
           __nv_bfloat162 h2 = __floats2bfloat162_rn(a0, a1);
           pk[i] = *reinterpret_cast<uint32_t*>(&h2);
         }

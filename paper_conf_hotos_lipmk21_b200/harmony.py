@@ -138,6 +138,10 @@ def lib() -> C.CDLL:
         "hk_attention_fwd": (st, [C.c_int64, C.c_int32, C.c_int32, C.c_int32, C.c_int32, P, P, P, P]),
         "hk_attention_bwd": (st, [C.c_int64, C.c_int32, C.c_int32, C.c_int32, C.c_int32, P, P, P, P, P, P]),
         "harmony_abi_sizes": (None, [P]),
+        "harmony_split_gemm_init": (st, [C.POINTER(harmony_config), C.c_int64, C.c_int64, C.c_int64, C.c_int32,
+                                         C.POINTER(P)]),
+        "harmony_split_gemm_run": (st, [P, P, P, P, P, P, P, C.POINTER(C.c_double)]),
+        "harmony_split_gemm_finalize": (st, [P]),
         "harmony_set_profiling": (st, [P, C.c_int32]),
         "harmony_read_profile": (st, [P, C.POINTER(harmony_kernel_profile)]),
     }
@@ -260,6 +264,32 @@ def harmony_read_profile(ctx):
 
 def harmony_finalize(ctx):
     _check(lib().harmony_finalize(ctx))
+
+
+class SplitGemm:
+    """Operator-split GEMM fwd+bwd (harmony_split_gemm_*): this rank's K-slice of X, W."""
+
+    def __init__(self, M, N, K, chunks=4, **cfg):
+        self.cfg = make_config(**cfg)
+        self.h = C.c_void_p()
+        _check(lib().harmony_split_gemm_init(C.byref(self.cfg), M, N, K, chunks, C.byref(self.h)))
+
+    def run(self, X_slice, W_slice, dY_shard, Y_shard, dX_slice, dW_slice):
+        sec = C.c_double()
+        _check(lib().harmony_split_gemm_run(self.h, _ptr(X_slice), _ptr(W_slice), _ptr(dY_shard), _ptr(Y_shard),
+                                            _ptr(dX_slice), _ptr(dW_slice), C.byref(sec)))
+        return sec.value
+
+    def close(self):
+        if self.h:
+            _check(lib().harmony_split_gemm_finalize(self.h))
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
 
 
 # ------------------------------------------------------------------------------- kernel ABI

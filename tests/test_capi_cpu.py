@@ -202,4 +202,4 @@ def test_plan_scales_to_paper_configs():
         s, _ = plan(c["descs"](), microbatches=c["m"], microbatch_size=c["batch"] // c["m"], precision=1,
                     hbm_cap_bytes=c["cap"])
         assert s.hazards == 0 and s.arena_bytes <= c["cap"]
-        assert s.pred_h2d_bytes > 30e9  # host-link bound
+        assert s.pred_h2d_bytes > 10e9  # op-input stash spills: host-link bound

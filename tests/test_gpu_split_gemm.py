@@ -1,0 +1,52 @@
+"""Operator split of one GEMM fwd+bwd (harmony_split_gemm_*; cfg5 =
+BASELINE.json configs[4]) against the fp64 oracle: a full check at 2048 x 2048 x 8192 and, at the
+full 16384 x 16384 x 65536 size, 4096 sampled entries of Y, dX and dW as fp64 dot products."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+from paper_conf_hotos_lipmk21_b200 import harmony as H  # noqa: E402
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64); b = np.asarray(b, np.float64)
+    return np.linalg.norm(a - b) / np.linalg.norm(b)
+
+
+def run(M, N, K, chunks, X, W, dY):
+    Xd = torch.tensor(X).to("cuda", torch.bfloat16); Wd = torch.tensor(W).to("cuda", torch.bfloat16)
+    dYd = torch.tensor(dY).to("cuda", torch.bfloat16)
+    Y = torch.empty(M, N, device="cuda"); dX = torch.empty(M, K, device="cuda", dtype=torch.bfloat16)
+    dW = torch.empty(K, N, device="cuda")
+    with H.SplitGemm(M, N, K, chunks=chunks) as g:
+        sec = g.run(Xd, Wd, dYd, Y, dX, dW)
+    return Y, dX, dW, sec
+
+
+def test_split_gemm_full_check():
+    M, N, K = 2048, 2048, 8192
+    X, W, dY = synth.gen_gemm_operands(M, N, K)
+    Y, dX, dW, _ = run(M, N, K, 4, X, W, dY)
+    rY, rdX, rdW = oracle.split_gemm_fwd_bwd(X, W, dY, n_k_splits=1, m_tiles=4)
+    assert rel(Y.cpu().numpy(), rY) < 1e-5
+    assert rel(dW.cpu().numpy(), rdW) < 1e-5
+    assert rel(dX.float().cpu().numpy(), rdX) < 4e-3
+
+
+@pytest.mark.slow
+def test_split_gemm_cfg5_full_size_sampled():
+    M, N, K = 16384, 16384, 65536
+    X, W, dY = synth.gen_gemm_operands(M, N, K)
+    Y, dX, dW, sec = run(M, N, K, 8, X, W, dY)
+    print(f"cfg5 fwd+bwd {sec * 1e3:.1f} ms = {3 * 2.0 * M * N * K / sec / 1e12:.0f} TFLOP/s")
+    rng = np.random.default_rng(5)
+    for which, out, (R, Cn) in (("Y", Y, (M, N)), ("dX", dX, (M, K)), ("dW", dW, (K, N))):
+        rows = rng.integers(0, R, 4096); cols = rng.integers(0, Cn, 4096)
+        ref = oracle.sampled_gemm_entries(X, W, dY, rows, cols, which)
+        got = out[torch.tensor(rows, device="cuda"), torch.tensor(cols, device="cuda")].float().cpu().numpy()
+        tol = 4e-3 if which == "dX" else 1e-5
+        assert rel(got, ref) < tol, which
