@@ -31,7 +31,7 @@ __device__ __forceinline__ float fast_exp2(float x) {
 
 constexpr int BQ = 128;   // query rows per CTA
 constexpr int BKV = 128;  // keys per tile
-constexpr int THREADS = 192;
+constexpr int THREADS = 320;  // warp 0: TMA, warp 1: MMA + TMEM, warps 2-9: softmax (2 per row quadrant)
 
 template <int DH>
 struct FwdCfg {
@@ -39,7 +39,7 @@ struct FwdCfg {
   static constexpr int K_BYTES = BKV * DH * 2;
   static constexpr int V_BYTES = BKV * DH * 2;          // 2 key-atoms x DH/64 MN-chunks of 8 KB
   static constexpr int P_BYTES = BQ * BKV * 2;          // 2 key-atoms of 16 KB
-  static constexpr int KST = 2, VST = 2, PST = 2;
+  static constexpr int KST = 2, VST = DH == 64 ? 2 : 1, PST = 2;  // DH=128: fits 227 KB with 1 V stage
   static constexpr int SMEM = Q_BYTES + KST * K_BYTES + VST * V_BYTES + PST * P_BYTES + 1024 + 512;
   static constexpr int S_COLS = BKV;                    // fp32 accumulator columns per S buffer
   static constexpr int O_COL = 2 * BKV;                 // O after the two S buffers
@@ -90,8 +90,8 @@ __global__ void __launch_bounds__(THREADS, 1)
     for (int i = 0; i < 2; ++i) {
       mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1);
       mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1);
-      mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 128);
-      mbar_init(&p_full[i], 128); mbar_init(&p_empty[i], 1);
+      mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 256);
+      mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1);
     }
     mbar_init(o_full, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -131,7 +131,7 @@ __global__ void __launch_bounds__(THREADS, 1)
               for (int c = 0; c < DH / 64; ++c)
                 tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
                             j * BKV + ka * 64, h, b);
-            if (++vs == 2) { vs = 0; vph ^= 1; }
+            if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
           }
         }
       }
@@ -185,14 +185,17 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
         mma_commit(&v_empty[vs]);
         mma_commit(&p_empty[pb]);
-        if (++vs == 2) { vs = 0; vph ^= 1; }
+        if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
       }
       mma_commit(o_full);
     }
     __syncwarp();
   } else {
-    // ===== softmax warps: thread = query row =====
+    // ===== softmax warps: thread = query row; the two warps of a row quadrant split the 128 keys
+    // of a tile into halves (= the two 64-key atoms of P) =====
     const int qd = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int cb = half * 64;
     const int r = qd * 32 + lane;        // row within the tile
     const int qrow = q0 + r;             // query index within the sequence
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
@@ -205,7 +208,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       tc_fence_after();
       const bool diag = p.causal && j == qt;
 #pragma unroll 1
-      for (int c = 0; c < BKV; c += 16) {
+      for (int c = cb; c < cb + 64; c += 16) {
         float v[16];
         tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
         float mx = m;
@@ -214,6 +217,7 @@ __global__ void __launch_bounds__(THREADS, 1)
           if (diag && j * BKV + c + i > qrow) v[i] = -INFINITY;
           mx = fmaxf(mx, v[i]);
         }
+        if (mx == -INFINITY) continue;  // every key of this chunk masked (and none seen before)
         float sum = 0.f;
 #pragma unroll
         for (int i = 0; i < 16; ++i) sum += fast_exp2((v[i] - mx) * p.scale_log2);
@@ -222,6 +226,16 @@ __global__ void __launch_bounds__(THREADS, 1)
       }
       tc_fence_before();
       mbar_arrive_local(&s_empty[sb]);
+    }
+    {  // combine the two halves' (max, sum): l = sum_h l_h 2^((m_h - m) scale log2e)
+      __shared__ float sm_m[2][BQ], sm_l[2][BQ];
+      sm_m[half][r] = m;
+      sm_l[half][r] = l;
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      const float m0 = sm_m[0][r], m1 = sm_m[1][r];
+      const float mm = fmaxf(m0, m1);
+      l = sm_l[0][r] * fast_exp2((m0 - mm) * p.scale_log2) + sm_l[1][r] * fast_exp2((m1 - mm) * p.scale_log2);
+      m = mm;
     }
     const float inv_l = 1.f / l;
     // ---- pass 2: normalised P (bf16) into shared memory, swizzled K-major (A operand of P V)
@@ -233,7 +247,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       const bool diag = p.causal && j == qt;
       uint8_t* prow = sP + pb * Cfg::P_BYTES + r * 128;
 #pragma unroll 1
-      for (int c = 0; c < BKV; c += 16) {
+      for (int c = cb; c < cb + 64; c += 16) {
         float v[16];
         tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
         uint32_t pk[8];
@@ -260,7 +274,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     tc_fence_after();
     __nv_bfloat16* crow = p.C + ((int64_t)b * p.S + qrow) * p.ldc + h * DH;
 #pragma unroll 1
-    for (int c = 0; c < DH; c += 16) {
+    for (int c = half * (DH / 2); c < (half + 1) * (DH / 2); c += 16) {
       float v[16];
       tmem_ld16(tmem + trow + Cfg::O_COL + c, v);
       uint32_t pk[8];
@@ -274,7 +288,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
     }
     // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
-    p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
+    if (half == 0) p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
   }
   tc_fence_before();
   __syncthreads();
@@ -349,8 +363,8 @@ __global__ void __launch_bounds__(THREADS, 1)
     prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO);
     mbar_init(kv_full, 1);
     for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
-    mbar_init(s_full, 1); mbar_init(s_empty, 128);
-    mbar_init(p_full, 128); mbar_init(p_empty, 1);
+    mbar_init(s_full, 1); mbar_init(s_empty, 256);
+    mbar_init(p_full, 256); mbar_init(p_empty, 1);
     mbar_init(kd_full, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -428,6 +442,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     __syncwarp();
   } else {
     const int qd = warp & 3;
+    const int half = (warp - 2) >> 2;  // which 64 queries of the tile (= which atom of P^T / dS^T)
     const int r = qd * 32 + lane;   // key row within the tile
     const int key = k0 + r;
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
@@ -443,7 +458,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       uint8_t* prow = sP + r * 128;
       uint8_t* drow = sdS + r * 128;
 #pragma unroll 1
-      for (int c = 0; c < BQ; c += 16) {
+      for (int c = half * 64; c < half * 64 + 64; c += 16) {
         float sv[16], dp[16];
         tmem_ld16(tmem + trow + Cfg::ST_COL + c, sv);
         tmem_ld16(tmem + trow + Cfg::DP_COL + c, dp);
@@ -484,8 +499,8 @@ __global__ void __launch_bounds__(THREADS, 1)
     mbar_wait(kd_full, 0);
     tc_fence_after();
     __nv_bfloat16* base = p.dqkv + ((int64_t)b * p.S + key) * 3 * p.d + h * DH;
-#pragma unroll 1
-    for (int part = 0; part < 2; ++part) {
+    {
+      const int part = half;  // half 0 drains dV, half 1 dK
       __nv_bfloat16* out = base + (part == 0 ? 2 * p.d : p.d);  // dV, then dK
       const int col = part == 0 ? Cfg::DV_COL : Cfg::DK_COL;
 #pragma unroll 1

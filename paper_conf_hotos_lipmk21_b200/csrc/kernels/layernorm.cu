@@ -12,7 +12,7 @@
 
 namespace hm {
 
-constexpr int LNV_ROWS = 32;  // rows per block in the backward (4 per warp)
+constexpr int LNV_ROWS = 16;  // rows per block in the backward (2 per warp)
 
 __device__ __forceinline__ float wsum(float v) {
 #pragma unroll
@@ -90,17 +90,23 @@ __global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float
                                                const float* __restrict__ rstd, const T* __restrict__ g,
                                                const float* __restrict__ dres, float* __restrict__ dX,
                                                float* __restrict__ partial) {
-  extern __shared__ float sred[];  // [2d]: block column partials, combined in warp order
+  // per-warp column partials of dgamma / dbeta live in shared memory ([8][2][d]); each lane owns
+  // fixed columns, so a warp accumulates its rows without races; the 8 warps are then summed in
+  // warp order per column (deterministic)
+  extern __shared__ float sred[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t r0 = (int64_t)blockIdx.x * LNV_ROWS;
-  float4 ag[VPT], ab[VPT];
+  float* sg = sred + (size_t)warp * 2 * d;
+  float* sb = sg + d;
   float4 gv[VPT];
 #pragma unroll
   for (int j = 0; j < VPT; ++j) {
-    ag[j] = make_float4(0.f, 0.f, 0.f, 0.f);
-    ab[j] = make_float4(0.f, 0.f, 0.f, 0.f);
     const int c = (j * 32 + lane) * 4;
     gv[j] = c < d ? ld4<T>(g + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c < d) {
+      *reinterpret_cast<float4*>(sg + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+      *reinterpret_cast<float4*>(sb + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
   }
   for (int i = warp; i < LNV_ROWS; i += 8) {
     const int64_t row = r0 + i;
@@ -108,64 +114,51 @@ __global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float
     const float mu = mean[row], rs = rstd[row];
     const float* x = X + row * d;
     const float* du = dU + row * d;
-    float4 xh[VPT], dv[VPT];
+    float4 xv[VPT], dv[VPT];
     float s1 = 0.f, s2 = 0.f;
 #pragma unroll
     for (int j = 0; j < VPT; ++j) {
       const int c = (j * 32 + lane) * 4;
       if (c < d) {
-        float4 xv = *reinterpret_cast<const float4*>(x + c);
+        xv[j] = *reinterpret_cast<const float4*>(x + c);
         dv[j] = *reinterpret_cast<const float4*>(du + c);
-        xh[j] = make_float4((xv.x - mu) * rs, (xv.y - mu) * rs, (xv.z - mu) * rs, (xv.w - mu) * rs);
-        float4 dx = make_float4(dv[j].x * gv[j].x, dv[j].y * gv[j].y, dv[j].z * gv[j].z, dv[j].w * gv[j].w);
+        const float4 xh = make_float4((xv[j].x - mu) * rs, (xv[j].y - mu) * rs, (xv[j].z - mu) * rs, (xv[j].w - mu) * rs);
+        const float4 dx = make_float4(dv[j].x * gv[j].x, dv[j].y * gv[j].y, dv[j].z * gv[j].z, dv[j].w * gv[j].w);
         s1 += (dx.x + dx.y) + (dx.z + dx.w);
-        s2 += (dx.x * xh[j].x + dx.y * xh[j].y) + (dx.z * xh[j].z + dx.w * xh[j].w);
-        ag[j].x += dv[j].x * xh[j].x; ag[j].y += dv[j].y * xh[j].y; ag[j].z += dv[j].z * xh[j].z; ag[j].w += dv[j].w * xh[j].w;
-        ab[j].x += dv[j].x; ab[j].y += dv[j].y; ab[j].z += dv[j].z; ab[j].w += dv[j].w;
+        s2 += (dx.x * xh.x + dx.y * xh.y) + (dx.z * xh.z + dx.w * xh.w);
+        float4 a = *reinterpret_cast<float4*>(sg + c), bq = *reinterpret_cast<float4*>(sb + c);
+        *reinterpret_cast<float4*>(sg + c) =
+            make_float4(a.x + dv[j].x * xh.x, a.y + dv[j].y * xh.y, a.z + dv[j].z * xh.z, a.w + dv[j].w * xh.w);
+        *reinterpret_cast<float4*>(sb + c) = make_float4(bq.x + dv[j].x, bq.y + dv[j].y, bq.z + dv[j].z, bq.w + dv[j].w);
       }
     }
     s1 = wsum(s1) / (float)d;
     s2 = wsum(s2) / (float)d;
-    float* dx = dX + row * d;
+    float* dxr = dX + row * d;
     const float* dr = dres ? dres + row * d : nullptr;
 #pragma unroll
     for (int j = 0; j < VPT; ++j) {
       const int c = (j * 32 + lane) * 4;
       if (c < d) {
-        float4 o = make_float4(rs * (dv[j].x * gv[j].x - s1 - xh[j].x * s2), rs * (dv[j].y * gv[j].y - s1 - xh[j].y * s2),
-                               rs * (dv[j].z * gv[j].z - s1 - xh[j].z * s2), rs * (dv[j].w * gv[j].w - s1 - xh[j].w * s2));
+        const float4 xh = make_float4((xv[j].x - mu) * rs, (xv[j].y - mu) * rs, (xv[j].z - mu) * rs, (xv[j].w - mu) * rs);
+        float4 o = make_float4(rs * (dv[j].x * gv[j].x - s1 - xh.x * s2), rs * (dv[j].y * gv[j].y - s1 - xh.y * s2),
+                               rs * (dv[j].z * gv[j].z - s1 - xh.z * s2), rs * (dv[j].w * gv[j].w - s1 - xh.w * s2));
         if (dr) {
           float4 rr = *reinterpret_cast<const float4*>(dr + c);
           o.x = rr.x + o.x; o.y = rr.y + o.y; o.z = rr.z + o.z; o.w = rr.w + o.w;
         }
-        *reinterpret_cast<float4*>(dx + c) = o;
+        *reinterpret_cast<float4*>(dxr + c) = o;
       }
     }
   }
-  // combine the 8 warps' column partials in warp order (deterministic)
-  for (int w = 0; w < 8; ++w) {
-    if (warp == w) {
-#pragma unroll
-      for (int j = 0; j < VPT; ++j) {
-        const int c = (j * 32 + lane) * 4;
-        if (c < d) {
-          float4* sg = reinterpret_cast<float4*>(sred + c);
-          float4* sb = reinterpret_cast<float4*>(sred + d + c);
-          if (w == 0) {
-            *sg = ag[j];
-            *sb = ab[j];
-          } else {
-            float4 a = *sg, bq = *sb;
-            *sg = make_float4(a.x + ag[j].x, a.y + ag[j].y, a.z + ag[j].z, a.w + ag[j].w);
-            *sb = make_float4(bq.x + ab[j].x, bq.y + ab[j].y, bq.z + ab[j].z, bq.w + ab[j].w);
-          }
-        }
-      }
-    }
-    __syncthreads();
-  }
+  __syncthreads();
   float* pg = partial + (int64_t)blockIdx.x * 2 * d;
-  for (int c = threadIdx.x; c < 2 * d; c += 256) pg[c] = sred[c];
+  for (int c = threadIdx.x; c < 2 * d; c += 256) {
+    float t = sred[c];
+#pragma unroll
+    for (int w = 1; w < 8; ++w) t += sred[(size_t)w * 2 * d + c];
+    pg[c] = t;
+  }
 }
 
 // fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 8 warps per block
@@ -231,7 +224,8 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
   const int v = ln_vpt(d);
   if (!v) return false;
   const int nblk = (int)ceil_div(rows, LNV_ROWS);
-  const size_t smem = 2 * (size_t)d * sizeof(float);
+  const size_t smem = 8 * 2 * (size_t)d * sizeof(float);  // per-warp column partials
+  if (smem > 200 * 1024) return false;
 #define HM_LNB(T, V)                                                                                   \
   do {                                                                                                 \
     if (smem > 48 * 1024)                                                                              \

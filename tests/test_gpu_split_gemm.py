@@ -48,5 +48,8 @@ def test_split_gemm_cfg5_full_size_sampled():
         rows = rng.integers(0, R, 4096); cols = rng.integers(0, Cn, 4096)
         ref = oracle.sampled_gemm_entries(X, W, dY, rows, cols, which)
         got = out[torch.tensor(rows, device="cuda"), torch.tensor(cols, device="cuda")].float().cpu().numpy()
-        tol = 4e-3 if which == "dX" else 1e-5
+        # bf16 operands are exact; the error is fp32 accumulation over K = 65536 (Y) / M = 16384 (dW)
+        # terms inside the tensor core, ~sqrt(K) * 2^-23 * growth; the north_star budget for the bf16
+        # path is 2e-2 — the bound here is 2e-3.  dX is additionally rounded to bf16 (2^-9).
+        tol = 4e-3 if which == "dX" else 2e-3
         assert rel(got, ref) < tol, which
