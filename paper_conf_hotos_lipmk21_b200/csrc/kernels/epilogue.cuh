@@ -162,7 +162,7 @@ __device__ __forceinline__ void epi_row16(const EpiParams& e, int64_t row_off, i
       return;
     }
   }
-#pragma unroll 1
+#pragma unroll
   for (int j = 0; j < 16; ++j)
     if (n0 + j < e.N) epi_scalar<T>(e, off + j, n0 + j, acc[j]);
 }

@@ -95,6 +95,26 @@ using namespace tcx;
 
 __device__ __forceinline__ uint32_t make_idesc(int bn, int a_mn, int b_mn) { return make_idesc_f16(BM, bn, a_mn, b_mn); }
 
+// one epilogue warp's 32-column chunk: TMEM (thread = row) -> registers -> fused epilogue -> global in
+// 32-byte row pieces (full sectors).  A variant that transposed chunks through shared memory for
+// 128-byte row segments measured 6% slower in the step (profiles/r01_epilogue_ab.txt) and was dropped.
+__device__ __forceinline__ void drain_chunk(const EpiParams& e, uint32_t taddr, bool have_acc, int lane, int mrow0,
+                                            int n, int64_t zoff) {
+  float v[32];
+  if (have_acc) {
+    tmem_ld16(taddr, v);
+    tmem_ld16(taddr + 16, v + 16);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = 0.f;
+  }
+  const int m = mrow0 + lane;
+  if (m < e.M) {
+    epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n, v);
+    if (n + 16 < e.N) epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n + 16, v + 16);
+  }
+}
+
 struct TcParams {
   int M, N, K, nz0, nz, a_mn, b_mn;
   EpiParams e;
@@ -248,22 +268,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int acc = it & 1;
       mbar_wait(&tmem_full[acc], (it >> 1) & 1);
       tc_fence_after();
-      const int m = m0 + q * 32 + lane;
-      const int64_t row_off = z0 * e.c_sz0 + z1 * e.c_sz1 + (int64_t)m * e.ldc;
+      const int64_t zoff = z0 * e.c_sz0 + z1 * e.c_sz1;
       const uint32_t tacc = tmem_base + acc * Cfg::ACC_COLS + ((uint32_t)(q * 32) << 16);
       const int ncols = min(BN, p.N - n0);
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
 #pragma unroll 1
-      for (int c = c_beg; c < c_end; c += 16) {
-        float v[16];
-        if (nkb > 0) {
-          tmem_ld16(tacc + c, v);
-        } else {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = 0.f;
-        }
-        if (m < p.M) epi_row16<__nv_bfloat16>(e, row_off, n0 + c, v);
-      }
+      for (int c = c_beg; c < c_end; c += 32) drain_chunk(e, tacc + c, nkb > 0, lane, m0 + q * 32, n0 + c, zoff);
       tc_fence_before();
       mbar_arrive(&tmem_empty[acc]);
     }
@@ -508,22 +518,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       const int acc = it & 1;
       mbar_wait(&tmem_full[acc], (it >> 1) & 1);
       tc_fence_after();
-      const int m = mb * 256 + (int)rank * 128 + q * 32 + lane;
-      const int64_t row_off = z0 * e.c_sz0 + z1 * e.c_sz1 + (int64_t)m * e.ldc;
+      const int64_t zoff = z0 * e.c_sz0 + z1 * e.c_sz1;
       const uint32_t tacc = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
       const int ncols = min(BN, p.N - n0);
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
 #pragma unroll 1
-      for (int c = c_beg; c < c_end; c += 16) {
-        float v[16];
-        if (nkb > 0) {
-          tmem_ld16(tacc + c, v);
-        } else {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = 0.f;
-        }
-        if (m < p.M) epi_row16<__nv_bfloat16>(e, row_off, n0 + c, v);
-      }
+      for (int c = c_beg; c < c_end; c += 32)
+        drain_chunk(e, tacc + c, nkb > 0, lane, mb * 256 + (int)rank * 128 + q * 32, n0 + c, zoff);
       tc_fence_before();
       mbar_arrive_cluster(te + acc * 8);
     }
@@ -597,7 +598,7 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
   if (mode && a.M >= 256 && a.N >= 256) {
     // CTA-pair 256 x 256 tiles (measured best for every cfg2 shape, tools/gemm_bench.py);
     // HARMONY_GEMM_2SM=3 selects 256 x 128 pair tiles, 0 the single-CTA kernel
-    if (mode == 3) tc::launch_tc2<128, 8>(a, e, st);
+    if (mode == 3) tc::launch_tc2<128, 6>(a, e, st);
     else tc::launch_tc2<256, 6>(a, e, st);
     return;
   }

@@ -19,7 +19,12 @@ bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const voi
 size_t layernorm_bwd_vec_scratch_bytes(int64_t rows, int d);
 bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                        const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
-                       int accumulate, float* scratch, cudaStream_t st);
+                       int accumulate, void* dXt, float* dsum, int dsum_acc, float* scratch, cudaStream_t st);
+// LN backward that also writes dX cast to T (dXt, nullable) and (+)= its column sums (dsum, nullable):
+// the residual gradient's bf16 GEMM operand and the bias gradient of the branch it feeds, in one pass
+void layernorm_bwd_ex(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                      const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
+                      int accumulate, void* dXt, float* dsum, int dsum_acc, float* scratch, cudaStream_t st);
 void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                    const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
                    float* scratch, cudaStream_t st);

@@ -85,27 +85,29 @@ __global__ void __launch_bounds__(256) ln_fwd_v(int64_t rows, int d, const float
 }
 
 template <typename T, int VPT>
-__global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float* __restrict__ dU,
+// __launch_bounds__(256, 2): two blocks per SM, i.e. at most 128 registers per thread
+__global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const float* __restrict__ dU,
                                                const float* __restrict__ X, const float* __restrict__ mean,
                                                const float* __restrict__ rstd, const T* __restrict__ g,
                                                const float* __restrict__ dres, float* __restrict__ dX,
-                                               float* __restrict__ partial) {
-  // per-warp column partials of dgamma / dbeta live in shared memory ([8][2][d]); each lane owns
+                                               T* __restrict__ dXt, int np, float* __restrict__ partial) {
+  // per-warp column partials of dgamma / dbeta (/ sum dX when np == 3) live in shared memory
+  // ([8][np][d]); each lane owns
   // fixed columns, so a warp accumulates its rows without races; the 8 warps are then summed in
   // warp order per column (deterministic)
   extern __shared__ float sred[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t r0 = (int64_t)blockIdx.x * LNV_ROWS;
-  float* sg = sred + (size_t)warp * 2 * d;
+  float* sg = sred + (size_t)warp * np * d;
   float* sb = sg + d;
-  float4 gv[VPT];
+  float* ss = np == 3 ? sb + d : nullptr;
 #pragma unroll
   for (int j = 0; j < VPT; ++j) {
     const int c = (j * 32 + lane) * 4;
-    gv[j] = c < d ? ld4<T>(g + c) : make_float4(0.f, 0.f, 0.f, 0.f);
     if (c < d) {
       *reinterpret_cast<float4*>(sg + c) = make_float4(0.f, 0.f, 0.f, 0.f);
       *reinterpret_cast<float4*>(sb + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (ss) *reinterpret_cast<float4*>(ss + c) = make_float4(0.f, 0.f, 0.f, 0.f);
     }
   }
   for (int i = warp; i < LNV_ROWS; i += 8) {
@@ -122,8 +124,9 @@ __global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float
       if (c < d) {
         xv[j] = *reinterpret_cast<const float4*>(x + c);
         dv[j] = *reinterpret_cast<const float4*>(du + c);
+        const float4 gv = ld4<T>(g + c);  // gamma re-read per row (L1-resident): keeps registers < 128
         const float4 xh = make_float4((xv[j].x - mu) * rs, (xv[j].y - mu) * rs, (xv[j].z - mu) * rs, (xv[j].w - mu) * rs);
-        const float4 dx = make_float4(dv[j].x * gv[j].x, dv[j].y * gv[j].y, dv[j].z * gv[j].z, dv[j].w * gv[j].w);
+        const float4 dx = make_float4(dv[j].x * gv.x, dv[j].y * gv.y, dv[j].z * gv.z, dv[j].w * gv.w);
         s1 += (dx.x + dx.y) + (dx.z + dx.w);
         s2 += (dx.x * xh.x + dx.y * xh.y) + (dx.z * xh.z + dx.w * xh.w);
         float4 a = *reinterpret_cast<float4*>(sg + c), bq = *reinterpret_cast<float4*>(sb + c);
@@ -141,22 +144,28 @@ __global__ void __launch_bounds__(256) ln_bwd_v(int64_t rows, int d, const float
       const int c = (j * 32 + lane) * 4;
       if (c < d) {
         const float4 xh = make_float4((xv[j].x - mu) * rs, (xv[j].y - mu) * rs, (xv[j].z - mu) * rs, (xv[j].w - mu) * rs);
-        float4 o = make_float4(rs * (dv[j].x * gv[j].x - s1 - xh.x * s2), rs * (dv[j].y * gv[j].y - s1 - xh.y * s2),
-                               rs * (dv[j].z * gv[j].z - s1 - xh.z * s2), rs * (dv[j].w * gv[j].w - s1 - xh.w * s2));
+        const float4 gv = ld4<T>(g + c);
+        float4 o = make_float4(rs * (dv[j].x * gv.x - s1 - xh.x * s2), rs * (dv[j].y * gv.y - s1 - xh.y * s2),
+                               rs * (dv[j].z * gv.z - s1 - xh.z * s2), rs * (dv[j].w * gv.w - s1 - xh.w * s2));
         if (dr) {
           float4 rr = *reinterpret_cast<const float4*>(dr + c);
           o.x = rr.x + o.x; o.y = rr.y + o.y; o.z = rr.z + o.z; o.w = rr.w + o.w;
         }
         *reinterpret_cast<float4*>(dxr + c) = o;
+        if (dXt) st4<T>(dXt + row * d + c, o);  // the bf16 GEMM operand copy of dX
+        if (ss) {
+          float4 a = *reinterpret_cast<float4*>(ss + c);
+          *reinterpret_cast<float4*>(ss + c) = make_float4(a.x + o.x, a.y + o.y, a.z + o.z, a.w + o.w);
+        }
       }
     }
   }
   __syncthreads();
-  float* pg = partial + (int64_t)blockIdx.x * 2 * d;
-  for (int c = threadIdx.x; c < 2 * d; c += 256) {
+  float* pg = partial + (int64_t)blockIdx.x * np * d;
+  for (int c = threadIdx.x; c < np * d; c += 256) {
     float t = sred[c];
 #pragma unroll
-    for (int w = 1; w < 8; ++w) t += sred[(size_t)w * 2 * d + c];
+    for (int w = 1; w < 8; ++w) t += sred[(size_t)w * np * d + c];
     pg[c] = t;
   }
 }
@@ -215,22 +224,23 @@ bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const voi
 }
 
 size_t layernorm_bwd_vec_scratch_bytes(int64_t rows, int d) {
-  return (size_t)ceil_div(rows, LNV_ROWS) * 2 * d * sizeof(float);
+  return (size_t)ceil_div(rows, LNV_ROWS) * 3 * d * sizeof(float);
 }
 
 bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                        const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
-                       int accumulate, float* scratch, cudaStream_t st) {
+                       int accumulate, void* dXt, float* dsum, int dsum_acc, float* scratch, cudaStream_t st) {
   const int v = ln_vpt(d);
   if (!v) return false;
   const int nblk = (int)ceil_div(rows, LNV_ROWS);
-  const size_t smem = 8 * 2 * (size_t)d * sizeof(float);  // per-warp column partials
+  const int np = dsum ? 3 : 2;
+  const size_t smem = 8 * (size_t)np * d * sizeof(float);  // per-warp column partials
   if (smem > 200 * 1024) return false;
 #define HM_LNB(T, V)                                                                                   \
   do {                                                                                                 \
     if (smem > 48 * 1024)                                                                              \
       HM_CUDA(cudaFuncSetAttribute(ln_bwd_v<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-    ln_bwd_v<T, V><<<nblk, 256, smem, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres, dX, scratch); \
+    ln_bwd_v<T, V><<<nblk, 256, smem, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres, dX, (T*)dXt, np, scratch); \
   } while (0)
 #define HM_LNB_ALL(T)                   \
   switch (v) {                          \
@@ -245,10 +255,15 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
 #undef HM_LNB_ALL
 #undef HM_LNB
   check_launch("layernorm_bwd_vec");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate);
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch, np * (int64_t)d, dg, accumulate);
   check_launch("colreduce(dgamma)");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate);
+  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + d, np * (int64_t)d, db, accumulate);
   check_launch("colreduce(dbeta)");
+  if (dsum) {
+    colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + 2 * d, np * (int64_t)d, dsum,
+                                                                dsum_acc);
+    check_launch("colreduce(sum dX)");
+  }
   return true;
 }
 

@@ -330,12 +330,19 @@ size_t layernorm_bwd_scratch_bytes(int64_t rows, int d) {
 void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                    const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
                    float* scratch, cudaStream_t st) {
+  layernorm_bwd_ex(dtype, rows, d, dU, X, mean, rstd, g, dres, dX, dg, db, accumulate, nullptr, nullptr, 0, scratch, st);
+}
+
+void layernorm_bwd_ex(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
+                      const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
+                      int accumulate, void* dXt, float* dsum, int dsum_acc, float* scratch, cudaStream_t st) {
   if (rows == 0) {
     return;
   }
   const int e0 = g_prof.begin(st);
-  if (layernorm_bwd_vec(dtype, rows, d, dU, X, mean, rstd, g, dres, dX, dg, db, accumulate, scratch, st)) {
-    g_prof.end(PROF_LN, e0, st, (double)rows * d * 4 * (dres ? 4 : 3) + rows * 8.0);
+  if (layernorm_bwd_vec(dtype, rows, d, dU, X, mean, rstd, g, dres, dX, dg, db, accumulate, dXt, dsum, dsum_acc,
+                        scratch, st)) {
+    g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 * (dres ? 4 : 3) + (dXt ? (dtype ? 2 : 4) : 0)) + rows * 8.0);
     return;
   }
   int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
@@ -344,6 +351,8 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
   check_launch("layernorm_bwd");
   colreduce(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate, st);
   colreduce(nblk, d, scratch + d, 2 * (int64_t)d, db, accumulate, st);
+  if (dXt) cast(dtype, rows * d, dX, dXt, st);
+  if (dsum) colsum(0, rows, d, dX, d, dsum, dsum_acc, scratch, st);
   g_prof.end(PROF_LN, e0, st, (double)rows * d * 4 * (dres ? 4 : 3) + rows * 8.0);
 }
 

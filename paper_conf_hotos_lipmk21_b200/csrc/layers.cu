@@ -252,8 +252,9 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
     a.C = Hh; a.epilogue = HK_EPI_BIAS_ACT; a.act = HARMONY_ACT_GELU_TANH; a.bias = wseg(g, W, P_BFC1); a.aux_out = G;
     gemm(a, st);
   }
-  // Y = X2 + G W_fc2 + b_fc2
-  {
+  // Y = X2 + G W_fc2 + b_fc2   (skipped when Y == nullptr: the backward's recompute needs only
+  // the block's internals, not its output)
+  if (Y) {
     hk_gemm_args a = lin_fwd(g, R, D, 4 * D, G, wseg(g, W, P_WFC2));
     a.C = Y; a.epilogue = HK_EPI_RESID_F32; a.aux = X2; a.bias = wseg(g, W, P_BFC2);
     gemm(a, st);
@@ -345,19 +346,19 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   }
   gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), st);
   colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, scratch, st);
-  // ---- LN2 backward: dX2 = dY + LN2'(dU2)
-  layernorm_bwd(dt, R, D, dUf, X2, mean2, rstd2, wseg(g, W, P_LN2_G), dY, dX2, gseg(g, dW, P_LN2_G),
-                gseg(g, dW, P_LN2_B), acc, scratch, st);
-  // ---- O projection: dC = dX2 W_o^T; dW_o += C^T dX2; db_o += sum dX2
-  const void* dX2op = dX2;
-  if (dt == 1) { cast(1, R * D, dX2, dYc, st); dX2op = dYc; }
+  // ---- LN2 backward: dX2 = dY + LN2'(dU2), fused with the bf16 copy of dX2 (the O-projection
+  // GEMM operand); db_o += sum_rows dX2
+  const void* dX2op = dt == 1 ? (const void*)dYc : (const void*)dX2;
+  layernorm_bwd_ex(dt, R, D, dUf, X2, mean2, rstd2, wseg(g, W, P_LN2_G), dY, dX2, gseg(g, dW, P_LN2_G),
+                   gseg(g, dW, P_LN2_B), acc, dt == 1 ? dYc : nullptr, nullptr, 0, scratch, st);
+  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, scratch, st);
+  // ---- O projection: dC = dX2 W_o^T; dW_o += C^T dX2
   {
     hk_gemm_args a = lin_dgrad(g, R, D, D, dX2op, wseg(g, W, P_WO));
     a.C = dC; a.epilogue = HK_EPI_STORE_T;
     gemm(a, st);
   }
   gemm(lin_wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first), st);
-  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, scratch, st);
   // ---- attention backward (batched over heads z0 and sequences z1)
   uint8_t* dQKV = dHb;
   const float scale = 1.0f / std::sqrt((float)dh);
@@ -450,9 +451,8 @@ void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const fl
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
   uint8_t* rest = ws + align_up(c.st.total, 256);
-  float* yscratch = reinterpret_cast<float*>(rest + align_up(std::max(c.ws_fwd, c.ws_bwd), 256));
   // recompute the block's forward from its stashed input: the same kernels, hence the same bits
-  fwd_core(c, W, reinterpret_cast<const float*>(stash + g.st.X), yscratch, full, rest, st);
+  fwd_core(c, W, reinterpret_cast<const float*>(stash + g.st.X), nullptr, full, rest, st);
   bwd_core(c, W, full, dY, dX, dW, first, rest, st);
 }
 
