@@ -6,7 +6,9 @@
 // operand of O += P V (accumulated in TMEM).  Softmax is exact and two-pass over the key tiles:
 // pass 1 computes each row's max and sum (online, scalars only), pass 2 recomputes S and
 // normalises P with the final statistics, so O needs no rescaling (1.5x the QK^T FLOPs of a
-// one-pass kernel, in exchange for no TMEM read-modify-write of O).  Outputs: C (bf16, heads
+// one-pass kernel, in exchange for no TMEM read-modify-write of O).  Pass 1 needs only the row max;
+// pass 2 forms P = exp(s - max) in (0, 1], accumulates the row sum beside it and O is divided by
+// the sum in the epilogue.  Outputs: C (bf16, heads
 // interleaved in [T, d]) and the row log-sum-exp (fp32 [b, h, S]) the backward needs.
 // Numerics match the unfused path's reading c11: P = softmax(scale * Q K^T) with causal rows
 // masked to exactly 0 above the diagonal.
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
     float m = -INFINITY, l = 0.f;
     int it = 0;
-    // ---- pass 1: row max and sum of exp2((s - m) * scale*log2e)
+    // ---- pass 1: row max only (no exponentials)
     for (int j = 0; j < ntiles; ++j, ++it) {
       const int sb = it & 1;
       mbar_wait(&s_full[sb], (it >> 1) & 1);
@@ -211,34 +213,19 @@ __global__ void __launch_bounds__(THREADS, 1)
       for (int c = cb; c < cb + 64; c += 16) {
         float v[16];
         tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
-        float mx = m;
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          if (diag && j * BKV + c + i > qrow) v[i] = -INFINITY;
-          mx = fmaxf(mx, v[i]);
-        }
-        if (mx == -INFINITY) continue;  // every key of this chunk masked (and none seen before)
-        float sum = 0.f;
-#pragma unroll
-        for (int i = 0; i < 16; ++i) sum += fast_exp2((v[i] - mx) * p.scale_log2);
-        l = l * fast_exp2((m - mx) * p.scale_log2) + sum;
-        m = mx;
+        for (int i = 0; i < 16; ++i)
+          if (!(diag && j * BKV + c + i > qrow)) m = fmaxf(m, v[i]);
       }
       tc_fence_before();
       mbar_arrive_local(&s_empty[sb]);
     }
-    {  // combine the two halves' (max, sum): l = sum_h l_h 2^((m_h - m) scale log2e)
-      __shared__ float sm_m[2][BQ], sm_l[2][BQ];
-      sm_m[half][r] = m;
-      sm_l[half][r] = l;
-      asm volatile("bar.sync 1, 256;" ::: "memory");
-      const float m0 = sm_m[0][r], m1 = sm_m[1][r];
-      const float mm = fmaxf(m0, m1);
-      l = sm_l[0][r] * fast_exp2((m0 - mm) * p.scale_log2) + sm_l[1][r] * fast_exp2((m1 - mm) * p.scale_log2);
-      m = mm;
-    }
-    const float inv_l = 1.f / l;
-    // ---- pass 2: normalised P (bf16) into shared memory, swizzled K-major (A operand of P V)
+    __shared__ float sm_x[2][BQ];
+    sm_x[half][r] = m;
+    asm volatile("bar.sync 1, 256;" ::: "memory");
+    m = fmaxf(sm_x[0][r], sm_x[1][r]);  // the row max over all keys (the diagonal key is always valid)
+    // ---- pass 2: P = 2^((s - m) scale log2e) in (0, 1] (bf16) into shared memory, swizzled K-major
+    // (A operand of O += P V); the row sum l accumulates alongside and O is divided by it at the end
     for (int j = 0; j < ntiles; ++j, ++it) {
       const int sb = it & 1, pb = j & 1;
       mbar_wait(&s_full[sb], (it >> 1) & 1);
@@ -253,8 +240,9 @@ __global__ void __launch_bounds__(THREADS, 1)
         uint32_t pk[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : fast_exp2((v[2 * i] - m) * p.scale_log2) * inv_l;
-          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : fast_exp2((v[2 * i + 1] - m) * p.scale_log2) * inv_l;
+          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : fast_exp2((v[2 * i] - m) * p.scale_log2);
+          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : fast_exp2((v[2 * i + 1] - m) * p.scale_log2);
+          l += a0 + a1;
           __nv_bfloat162 h2 = __floats2bfloat162_rn(a0, a1);
           pk[i] = *reinterpret_cast<uint32_t*>(&h2);
         }
@@ -269,6 +257,11 @@ __global__ void __launch_bounds__(THREADS, 1)
       mbar_arrive_local(&s_empty[sb]);
       mbar_arrive_local(&p_full[pb]);
     }
+    asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
+    sm_x[half][r] = l;
+    asm volatile("bar.sync 1, 256;" ::: "memory");
+    l = sm_x[0][r] + sm_x[1][r];
+    const float inv_l = 1.f / l;
     // ---- epilogue: O row -> bf16 C, LSE
     mbar_wait(o_full, 0);
     tc_fence_after();
@@ -280,7 +273,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       uint32_t pk[8];
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+        __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * i] * inv_l, v[2 * i + 1] * inv_l);
         pk[i] = *reinterpret_cast<uint32_t*>(&h2);
       }
       uint4* dst = reinterpret_cast<uint4*>(crow + c);
