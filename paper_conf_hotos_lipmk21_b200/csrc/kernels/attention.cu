@@ -306,8 +306,10 @@ struct BwdCfg {
   static constexpr int KV_BYTES = BKV * DH * 2;   // K_j or V_j
   static constexpr int QT_BYTES = BQ * DH * 2;    // Q_i or dO_i
   static constexpr int ST = DH == 64 ? 2 : 1;     // (Q, dO) stages
+  static constexpr int PB = DH == 64 ? 2 : 1;     // (P^T, dS^T) buffers: 2 lets the softmax of tile n+1
+                                                  // overlap the dV/dK MMAs of tile n
   static constexpr int PS_BYTES = BKV * BQ * 2;   // P^T or dS^T
-  static constexpr int SMEM = 2 * KV_BYTES + ST * 2 * QT_BYTES + 2 * PS_BYTES + 1024 + 512;
+  static constexpr int SMEM = 2 * KV_BYTES + ST * 2 * QT_BYTES + PB * 2 * PS_BYTES + 1024 + 512;
   static constexpr int ST_COL = 0, DP_COL = 128, DV_COL = 256, DK_COL = 256 + DH;
   static constexpr int TMEM_COLS = 512;
 };
@@ -332,18 +334,16 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint8_t* sK = smem;
   uint8_t* sV = sK + Cfg::KV_BYTES;
   uint8_t* sQ = sV + Cfg::KV_BYTES;                  // [ST] (Q_i, dO_i)
-  uint8_t* sP = sQ + Cfg::ST * 2 * Cfg::QT_BYTES;    // P^T
-  uint8_t* sdS = sP + Cfg::PS_BYTES;                 // dS^T
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sdS + Cfg::PS_BYTES);
+  uint8_t* sPS = sQ + Cfg::ST * 2 * Cfg::QT_BYTES;   // [PB] (P^T, dS^T)
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sPS + Cfg::PB * 2 * Cfg::PS_BYTES);
   uint64_t* kv_full = bars;
   uint64_t* q_full = bars + 1;   // [2]
   uint64_t* q_empty = bars + 3;  // [2]
   uint64_t* s_full = bars + 5;
-  uint64_t* s_empty = bars + 6;
-  uint64_t* p_full = bars + 7;
-  uint64_t* p_empty = bars + 8;
-  uint64_t* kd_full = bars + 9;
-  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 10);
+  uint64_t* p_full = bars + 6;   // [2]: softmax wrote P^T/dS^T buffer and finished reading S^T/dP^T
+  uint64_t* p_empty = bars + 8;  // [2]
+  uint64_t* kd_full = bars + 10;
+  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 11);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int kt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
@@ -356,8 +356,8 @@ __global__ void __launch_bounds__(THREADS, 1)
     prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO);
     mbar_init(kv_full, 1);
     for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
-    mbar_init(s_full, 1); mbar_init(s_empty, 256);
-    mbar_init(p_full, 256); mbar_init(p_empty, 1);
+    mbar_init(s_full, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1); }
     mbar_init(kd_full, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -400,10 +400,12 @@ __global__ void __launch_bounds__(THREADS, 1)
       const uint32_t idesc_g = make_idesc_f16(128, DH, 0, 1);   // dV, dK: M=keys, N=DH, K=queries
       mbar_wait(kv_full, 0);
       const uint32_t ka = smem_u32(sK), va = smem_u32(sV);
-      int st = 0; uint32_t ph = 0;
-      for (int n = 0; n < niter; ++n) {
-        mbar_wait(&q_full[st], ph);
-        mbar_wait(s_empty, (n & 1) ^ 1);
+      // order: S_0, dP_0 | for n: [wait P_n] S_{n+1}, dP_{n+1} | dV_n, dK_n — the tensor pipe computes the
+      // next scores while the softmax warps are still writing nothing (they wait), then the gradients
+      // of tile n run while the softmax warps turn S_{n+1} into P_{n+1} (PB = 2 buffers)
+      auto issue_s = [&](int n) {
+        const int st = n % Cfg::ST;
+        mbar_wait(&q_full[st], (n / Cfg::ST) & 1);
         tc_fence_after();
         const uint32_t qa = smem_u32(sQ + st * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
 #pragma unroll
@@ -414,9 +416,16 @@ __global__ void __launch_bounds__(THREADS, 1)
           mma_bf16(tmem + Cfg::DP_COL, make_sdesc(va + off, 16, 1024), make_sdesc(oa + off, 16, 1024), idesc_s, kk ? 1u : 0u);
         }
         mma_commit(s_full);
-        mbar_wait(p_full, n & 1);
+      };
+      issue_s(0);
+      for (int n = 0; n < niter; ++n) {
+        const int pb = n % Cfg::PB;
+        mbar_wait(&p_full[pb], (n / Cfg::PB) & 1);  // P^T/dS^T of tile n written, S/dP TMEM read
         tc_fence_after();
-        const uint32_t pa = smem_u32(sP), da = smem_u32(sdS);
+        if (n + 1 < niter && Cfg::PB == 2) issue_s(n + 1);
+        const int st = n % Cfg::ST;
+        const uint32_t qa = smem_u32(sQ + st * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
+        const uint32_t pa = smem_u32(sPS + pb * 2 * Cfg::PS_BYTES), da = pa + Cfg::PS_BYTES;
 #pragma unroll
         for (int kk = 0; kk < BQ / 16; ++kk) {
           const int atom = kk / 4, sub = kk % 4;
@@ -426,9 +435,9 @@ __global__ void __launch_bounds__(THREADS, 1)
           mma_bf16(tmem + Cfg::DV_COL, make_sdesc(pa + aoff, 16, 1024), make_sdesc(oa + boff, 128 * 128, 1024), idesc_g, acc);
           mma_bf16(tmem + Cfg::DK_COL, make_sdesc(da + aoff, 16, 1024), make_sdesc(qa + boff, 128 * 128, 1024), idesc_g, acc);
         }
-        mma_commit(p_empty);
+        mma_commit(&p_empty[pb]);
         mma_commit(&q_empty[st]);
-        if (++st == Cfg::ST) { st = 0; ph ^= 1; }
+        if (n + 1 < niter && Cfg::PB == 1) issue_s(n + 1);
       }
       mma_commit(kd_full);
     }
@@ -444,12 +453,13 @@ __global__ void __launch_bounds__(THREADS, 1)
     __nv_bfloat16* dst_row = p.dst + (((int64_t)b * p.H + h) * p.S + key) * p.S;
     for (int n = 0; n < niter; ++n) {
       const int q0 = (i0 + n) * BQ;
+      const int pb = n % Cfg::PB;
       mbar_wait(s_full, n & 1);
-      mbar_wait(p_empty, (n & 1) ^ 1);
+      mbar_wait(&p_empty[pb], ((n / Cfg::PB) & 1) ^ 1);
       tc_fence_after();
       const bool diag = p.causal && (i0 + n) == kt;
-      uint8_t* prow = sP + r * 128;
-      uint8_t* drow = sdS + r * 128;
+      uint8_t* prow = sPS + pb * 2 * Cfg::PS_BYTES + r * 128;
+      uint8_t* drow = prow + Cfg::PS_BYTES;
 #pragma unroll 1
       for (int c = half * 64; c < half * 64 + 64; c += 16) {
         float sv[16], dp[16];
@@ -485,8 +495,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       tc_fence_before();
-      mbar_arrive_local(s_empty);
-      mbar_arrive_local(p_full);
+      mbar_arrive_local(&p_full[pb]);
     }
     // epilogue: dV_j, dK_j rows -> dQKV (bf16)
     mbar_wait(kd_full, 0);
