@@ -76,6 +76,8 @@ struct harmony_ctx {
   bool use_graph = true;
   StepGraph g_plain, g_prof;  // the step as CUDA graphs: plain, and with per-kernel timing events
   cudaEvent_t ev_fork = nullptr, ev_join[S_NUM] = {};
+  cudaStream_t side = nullptr;          // weight-gradient stream lent to the backward tasks
+  cudaEvent_t side_ev[4] = {};
 };
 
 namespace {
@@ -126,6 +128,10 @@ void destroy(harmony_ctx* c) {
     if (c->st[s]) cudaStreamSynchronize(c->st[s]);
   drop_graph(c->g_plain);
   drop_graph(c->g_prof);
+  if (c->side) cudaStreamSynchronize(c->side);
+  for (auto e : c->side_ev)
+    if (e) cudaEventDestroy(e);
+  if (c->side) cudaStreamDestroy(c->side);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   for (int s = 0; s < S_NUM; ++s)
     if (c->ev_join[s]) cudaEventDestroy(c->ev_join[s]);
@@ -174,6 +180,14 @@ void issue_program(harmony_ctx* c, const float* x, const float* tg, bool x_dev, 
   uint8_t* A = c->arena;
   const int dt = p.dtype;
   const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
+  struct SideGuard {
+    SideGuard(harmony_ctx* c) {
+      void* ev[4] = {c->side_ev[0], c->side_ev[1], c->side_ev[2], c->side_ev[3]};
+      const char* e = getenv("HARMONY_NO_SIDE");
+      if (!(e && *e && *e != '0')) set_side_stream(c->side, ev);
+    }
+    ~SideGuard() { set_side_stream(nullptr, nullptr); }
+  } side_guard(c);
   // Adam's step t lives in device memory (read by the update kernels at execution time)
   HM_CUDA(cudaMemcpyAsync(A + p.tstep, c->h_step, sizeof(int), cudaMemcpyHostToDevice, c->st[S_COMPUTE]));
   for (size_t oi = 0; oi < p.ops.size(); ++oi) {
@@ -491,6 +505,8 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
   HM_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
   for (int s = 0; s < S_NUM; ++s) HM_CUDA(cudaEventCreateWithFlags(&c->ev_join[s], cudaEventDisableTiming));
   c->h_step = static_cast<int*>(alloc_host(sizeof(int)));
+  HM_CUDA(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+  for (auto& e : c->side_ev) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   {
     const char* e = getenv("HARMONY_NO_GRAPH");
     c->use_graph = !(e && *e && *e != '0');

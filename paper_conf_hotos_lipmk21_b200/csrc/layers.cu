@@ -125,9 +125,25 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   }
   bump(wb, bwd_scratch_bytes(g.rows, (int)D));
   if (stash_policy == 1) bump(wb, R * 4 * D * ts);  // recomputed G / U2 / U
+  // separate buffers read by the weight-gradient side stream (see bwd_core)
+  bump(wb, R * D * ts);      // dX2c
+  bump(wb, R * 3 * D * ts);  // dQKV
+  bump(wb, colsum_scratch_bytes(g.rows, (int)(4 * D)));  // side-stream column-sum scratch
   g.ws_bwd = wb;
   g.flops_fwd = 24.0 * (double)R * D * D + 4.0 * (double)b * g.S * g.S * D;
   return g;
+}
+
+// ------------------------------------------------------------------------------------------------ side stream
+// The executor lends the backward a second stream: the weight-gradient GEMMs and bias column sums
+// of a block (which feed only dW) run there, concurrently with the data-gradient chain
+// (dgrad -> LN backward -> attention -> dgrad) on the task's stream; the task joins it before it
+// ends, so to the planner a BWD task is still one op on the compute stream.
+static thread_local cudaStream_t t_side = nullptr;
+static thread_local cudaEvent_t t_side_ev[4] = {nullptr, nullptr, nullptr, nullptr};
+void set_side_stream(void* st, void* const* events) {
+  t_side = static_cast<cudaStream_t>(st);
+  for (int i = 0; i < 4; ++i) t_side_ev[i] = events ? static_cast<cudaEvent_t>(events[i]) : nullptr;
 }
 
 // ------------------------------------------------------------------------------------------------ helpers
@@ -316,6 +332,18 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   }
   float* scratch = reinterpret_cast<float*>(ws + bump(wc, bwd_scratch_bytes(R, D)));
   uint8_t* rec = g.stash_policy == 1 ? ws + bump(wc, R * 4 * D * ts) : nullptr;
+  uint8_t* dX2c_buf = ws + bump(wc, R * D * ts);
+  uint8_t* dQKV_buf = ws + bump(wc, R * 3 * D * ts);
+  float* side_scratch = reinterpret_cast<float*>(ws + bump(wc, colsum_scratch_bytes(R, 4 * D)));
+  // weight gradients on the side stream (not with policy 1: its recompute buffer is reused in place)
+  const bool overlap = t_side != nullptr && g.stash_policy != 1;
+  cudaStream_t sw = overlap ? t_side : st;     // stream of the weight-gradient work
+  float* wscratch = overlap ? side_scratch : scratch;
+  auto fork = [&](int k) {
+    if (!overlap) return;
+    HM_CUDA(cudaEventRecord(t_side_ev[k], st));
+    HM_CUDA(cudaStreamWaitEvent(t_side, t_side_ev[k], 0));
+  };
 
   // dY as a GEMM operand
   const void* dYop = dY;
@@ -328,8 +356,9 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   }
   const uint8_t* G = g.stash_policy == 0 ? stash + g.st.G : rec;
   if (g.stash_policy == 1) act_fwd_T(dt, HARMONY_ACT_GELU_TANH, R * 4 * D, Hh, rec, st);
-  gemm(lin_wgrad(g, R, D, 4 * D, G, dYop, gseg(g, dW, P_WFC2), first), st);
-  colsum(0, R, D, dY, D, gseg(g, dW, P_BFC2), acc, scratch, st);
+  fork(0);
+  gemm(lin_wgrad(g, R, D, 4 * D, G, dYop, gseg(g, dW, P_WFC2), first), sw);
+  colsum(0, R, D, dY, D, gseg(g, dW, P_BFC2), acc, wscratch, sw);
   // ---- FC1: dU2 = dH W_fc1^T (fp32 for the LN backward); dW_fc1 += U2^T dH
   {
     hk_gemm_args a = lin_dgrad(g, R, 4 * D, D, dHb, wseg(g, W, P_WFC1));
@@ -344,23 +373,25 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     layernorm_fwd(dt, R, D, X2, wseg(g, W, P_LN2_G), wseg(g, W, P_LN2_B), rec, tmp_mean, tmp_rstd, st);
     U2 = rec;
   }
-  gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), st);
-  colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, scratch, st);
+  if (g.stash_policy == 1) fork(0);
+  gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), sw);
+  colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, wscratch, sw);
   // ---- LN2 backward: dX2 = dY + LN2'(dU2), fused with the bf16 copy of dX2 (the O-projection
   // GEMM operand); db_o += sum_rows dX2
-  const void* dX2op = dt == 1 ? (const void*)dYc : (const void*)dX2;
+  const void* dX2op = dt == 1 ? (const void*)dX2c_buf : (const void*)dX2;
   layernorm_bwd_ex(dt, R, D, dUf, X2, mean2, rstd2, wseg(g, W, P_LN2_G), dY, dX2, gseg(g, dW, P_LN2_G),
-                   gseg(g, dW, P_LN2_B), acc, dt == 1 ? dYc : nullptr, nullptr, 0, scratch, st);
-  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, scratch, st);
+                   gseg(g, dW, P_LN2_B), acc, dt == 1 ? dX2c_buf : nullptr, nullptr, 0, scratch, st);
+  fork(1);
+  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, wscratch, sw);
   // ---- O projection: dC = dX2 W_o^T; dW_o += C^T dX2
   {
     hk_gemm_args a = lin_dgrad(g, R, D, D, dX2op, wseg(g, W, P_WO));
     a.C = dC; a.epilogue = HK_EPI_STORE_T;
     gemm(a, st);
   }
-  gemm(lin_wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first), st);
+  gemm(lin_wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first), sw);
   // ---- attention backward (batched over heads z0 and sequences z1)
-  uint8_t* dQKV = dHb;
+  uint8_t* dQKV = dQKV_buf;
   const float scale = 1.0f / std::sqrt((float)dh);
   if (g.fused_attn) {
     HM_CHECK(attention_bwd_fused(b, S, H, dh, d.causal, QKV, C, dC, reinterpret_cast<const float*>(P), dQKV,
@@ -419,11 +450,16 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     layernorm_fwd(dt, R, D, Xs, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), rec, tmp_mean, tmp_rstd, st);
     U = rec;
   }
-  gemm(lin_wgrad(g, R, 3 * D, D, U, dQKV, gseg(g, dW, P_WQKV), first), st);
-  colsum(dt, R, 3 * D, dQKV, 3 * D, gseg(g, dW, P_BQKV), acc, scratch, st);
+  fork(2);
+  gemm(lin_wgrad(g, R, 3 * D, D, U, dQKV, gseg(g, dW, P_WQKV), first), sw);
+  colsum(dt, R, 3 * D, dQKV, 3 * D, gseg(g, dW, P_BQKV), acc, wscratch, sw);
   // ---- LN1 backward: dX = dX2 + LN1'(dU)
   layernorm_bwd(dt, R, D, dUf, Xs, mean1, rstd1, wseg(g, W, P_LN1_G), dX2, dX, gseg(g, dW, P_LN1_G),
                 gseg(g, dW, P_LN1_B), acc, scratch, st);
+  if (overlap) {  // join: the task ends when its weight gradients are in dW
+    HM_CUDA(cudaEventRecord(t_side_ev[3], t_side));
+    HM_CUDA(cudaStreamWaitEvent(st, t_side_ev[3], 0));
+  }
 }
 
 // ------------------------------------------------------------------------------------------------ dispatch
