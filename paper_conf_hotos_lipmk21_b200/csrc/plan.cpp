@@ -213,6 +213,24 @@ int validate_program(const Plan& p, std::string* first) {
   std::vector<std::vector<Acc>> acc(n);
   for (size_t i = 0; i < n; ++i) acc[i] = accesses(p, p.ops[i]);
   int hazards = 0;
+  // dataflow rule: a spilled stash is produced and consumed within the step, so every read of a
+  // host stash buffer must be ordered after a write of it (else it would read the previous step's)
+  for (size_t j = 0; j < n; ++j)
+    for (const Acc& b : acc[j]) {
+      if (b.write || b.space != 1 + HB_STASH) continue;
+      bool produced = false;
+      for (size_t i = 0; i < n && !produced; ++i)
+        for (const Acc& a : acc[i])
+          if (a.write && a.space == b.space && a.idx == b.idx && a.lo <= b.lo && a.hi >= b.hi && i != j && hb(i, j)) {
+            produced = true;
+            break;
+          }
+      if (!produced) {
+        if (hazards == 0 && first)
+          *first = "op " + std::to_string(j) + " reads host stash " + std::to_string(b.idx) + " before it is written";
+        ++hazards;
+      }
+    }
   for (size_t j = 0; j < n; ++j)
     for (size_t i = 0; i < j; ++i) {
       if (p.ops[i].stream == p.ops[j].stream || hb(i, j)) continue;
@@ -323,14 +341,23 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     for (auto& c : pref) {
       if (fixed + c[0] * maxw + c[1] * maxs + c[2] * maxst <= p.cap) { nW = c[0]; nS = c[1]; nG = c[2]; break; }
     }
-    // fill residency, then reclaim slots of classes that became fully resident; iterate
-    for (int pass = 0; pass < 4; ++pass) {
+    // Fill residency with the room the slots leave, then shrink the slots to what is still streamed
+    // and repeat (the freed room lets more become resident).  Greedy filling is not monotone in
+    // the room, so every pass is checked: a pass whose streamed items fit its own slot sizes next
+    // to its residency is a consistent layout; the last consistent one is kept (pass 0 always is,
+    // its sizes are the global maxima).  Slot counts are upgraded (double buffering) only
+    // afterwards and only where they fit — the layout can never exceed the cap.
+    struct Res { std::vector<int> w, s, st; uint64_t mw, ms, mst, bytes; };
+    Res best{};
+    bool have_best = false;
+    for (int pass = 0; pass < 16; ++pass) {
       for (auto& lp : p.layers) {
         lp.wc_res = -1; lp.state_res = -1;
         std::fill(lp.stash_res.begin(), lp.stash_res.end(), -1);
       }
-      uint64_t used = fixed + nW * maxw + nS * maxs + nG * maxst;
+      const uint64_t used = fixed + nW * maxw + nS * maxs + nG * maxst;
       uint64_t room = p.cap > used ? p.cap - used : 0;
+      const uint64_t room0 = room;
       if (!baseline) {
         // compute weights: 3 B of transfer saved per resident byte; backward order
         for (int l = L - 1; l >= 0; --l) {
@@ -347,25 +374,43 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
           uint64_t sz = align_up(p.layers[l].g.st.total, ALIGN);
           if (sz <= room) { p.layers[l].stash_res[i] = 0; room -= sz; }
         }
-      // recompute the slot sizes from what is still streamed
-      uint64_t nmaxw = 0, nmaxs = 0, nmaxst = 0;
+      Res r{};
+      r.bytes = room0 - room;
+      r.mw = r.ms = r.mst = 0;
       for (auto& lp : p.layers) {
-        if (lp.wc_res < 0) nmaxw = std::max(nmaxw, align_up(lp.wc_bytes, ALIGN));
-        if (lp.state_res < 0) nmaxs = std::max(nmaxs, align_up(lp.state_bytes, ALIGN));
+        r.w.push_back(lp.wc_res); r.s.push_back(lp.state_res);
+        r.st.insert(r.st.end(), lp.stash_res.begin(), lp.stash_res.end());
+        if (lp.wc_res < 0) r.mw = std::max(r.mw, align_up(lp.wc_bytes, ALIGN));
+        if (lp.state_res < 0) r.ms = std::max(r.ms, align_up(lp.state_bytes, ALIGN));
         for (int i = 0; i < m; ++i)
-          if (lp.stash_res[i] < 0) nmaxst = std::max(nmaxst, align_up(lp.g.st.total, ALIGN));
+          if (lp.stash_res[i] < 0) r.mst = std::max(r.mst, align_up(lp.g.st.total, ALIGN));
       }
-      bool changed = nmaxw != maxw || nmaxs != maxs || nmaxst != maxst;
-      maxw = nmaxw; maxs = nmaxs; maxst = nmaxst;
-      if (maxw == 0) nW = 0;
-      if (maxs == 0) nS = 0;
-      if (maxst == 0) nG = 0;
-      if (!changed) break;
-      // slots shrank: retry preferences with the new sizes (never below one slot per streamed class)
-      for (auto& c : pref) {
-        int w = maxw ? c[0] : 0, s = maxs ? c[1] : 0, g2 = maxst ? c[2] : 0;
-        if (fixed + w * maxw + s * maxs + g2 * maxst <= p.cap) { nW = w; nS = s; nG = g2; break; }
+      const bool fits = r.mw <= maxw && r.ms <= maxs && r.mst <= maxst;  // streamed items fit the slots
+      const bool fixed_point = r.mw == maxw && r.ms == maxs && r.mst == maxst;
+      if (fits) { best = r; have_best = true; }
+      if (fixed_point || !fits) break;
+      maxw = r.mw; maxs = r.ms; maxst = r.mst;
+    }
+    HM_CHECK(have_best, HARMONY_E_CAP_TOO_SMALL, "internal: no consistent residency");
+    {
+      size_t k = 0, ks = 0;
+      for (auto& lp : p.layers) {
+        lp.wc_res = best.w[k]; lp.state_res = best.s[k]; ++k;
+        for (int i = 0; i < m; ++i) lp.stash_res[i] = best.st[ks++];
       }
+    }
+    maxw = best.mw; maxs = best.ms; maxst = best.mst;
+    const uint64_t resident_bytes = best.bytes;
+    nW = maxw ? std::max(nW, 1) : 0;
+    nS = maxs ? std::max(nS, 1) : 0;
+    nG = maxst ? std::max(nG, 1) : 0;
+    HM_CHECK(fixed + nW * maxw + nS * maxs + nG * maxst + resident_bytes <= p.cap, HARMONY_E_CAP_TOO_SMALL,
+             "internal: residency exceeds the cap");
+    // upgrade slot counts (double buffering) where the residency above still leaves room
+    for (auto& c : pref) {
+      const int w = maxw ? std::max(nW, c[0]) : 0, s2 = maxs ? std::max(nS, c[1]) : 0,
+                g2 = maxst ? std::max(nG, c[2]) : 0;
+      if (fixed + w * maxw + s2 * maxs + g2 * maxst + resident_bytes <= p.cap) { nW = w; nS = s2; nG = g2; break; }
     }
     p.wslot_bytes = maxw; p.sslot_bytes = maxs; p.stage_bytes = maxst;
   }
@@ -452,6 +497,8 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
 
   // ---- forward
   std::vector<int> fwd_wslot(L, -1);
+  // FWD task that spills each (l, i): a backward swap-in of that stash may not be issued before it
+  std::vector<int> spill_task((size_t)L * m, -1);
   {
     Task t;  // inputs are issued as the first ops (not prefetch items)
     (void)t;
@@ -483,6 +530,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
         d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + i; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
         t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, i)}}});
         stage_last[g] = (int)tasks.size();
+        spill_task[(size_t)l * m + i] = (int)tasks.size();
       }
       if (slot >= 0) wslot_last[slot] = (int)tasks.size();
       tasks.push_back(t);
@@ -607,7 +655,8 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
         gnext = (gnext + 1) % nG;
         Item it;
         it.need = (int)tasks.size();
-        it.release = stage_last[g];
+        // free staging slot AND the spill of this very stash already issued (read after write)
+        it.release = std::max(stage_last[g], spill_task[(size_t)l * m + i]);
         Op h;
         h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STASH; h.layer = l; h.mb = i;
         h.hbuf = HB_STASH; h.hidx = (int64_t)l * m + i; h.dev = p.stage[g]; h.bytes = lp.g.st.total;

@@ -81,12 +81,18 @@ def test_plans_are_hazard_free(kw):
     assert s.arena_bytes <= (kw["hbm_cap_bytes"] or 1 << 62)
 
 
-def test_transformer_plans_hazard_free_over_caps():
-    descs = synth.transformer_stack(6, 64, 4, 16, True)
-    base = min_cap(descs, microbatches=3, microbatch_size=2, precision=1)
-    for f in (1.0, 1.3, 2.0, 3.0, 6.0):
-        s, _ = plan(descs, microbatches=3, microbatch_size=2, precision=1, hbm_cap_bytes=int(base * f))
-        assert s.hazards == 0
+@pytest.mark.parametrize("policy", [0, 1, 2])
+@pytest.mark.parametrize("S,L,m", [(16, 6, 3), (64, 3, 2), (128, 4, 4)])
+def test_transformer_plans_hazard_free_over_caps(policy, S, L, m):
+    """Plan fuzz: every cap between the minimum working set and all-resident, for each stash policy,
+    gives a program without races and without a read of a spilled stash before its spill (the
+    independent validator; a regression of the latter was caught this way)."""
+    descs = synth.transformer_stack(L, 64, 4, S, True)
+    kw = dict(microbatches=m, microbatch_size=2, precision=1, stash_policy=policy)
+    base = min_cap(descs, **kw)
+    for f in (1.0, 1.05, 1.1, 1.2, 1.3, 1.5, 2.0, 3.0, 6.0):
+        s, _ = plan(descs, **dict(kw, hbm_cap_bytes=int(base * f)))
+        assert s.hazards == 0, (policy, S, f)
 
 
 def test_cap_too_small_is_reported():
