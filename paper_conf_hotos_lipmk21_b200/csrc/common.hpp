@@ -89,27 +89,58 @@ template <typename T> __device__ __forceinline__ T from_f32(float x);
 template <> __device__ __forceinline__ float from_f32<float>(float x) { return x; }
 template <> __device__ __forceinline__ __nv_bfloat16 from_f32<__nv_bfloat16>(float x) { return __float2bfloat16_rn(x); }
 
-// GeLU (tanh approximation, reading c12) and its derivative, fp32.
-__device__ __forceinline__ float gelu_tanh_f(float x) {
-  const float c = 0.7978845608028654f, a = 0.044715f;
-  float u = c * (x + a * x * x * x);
-  return 0.5f * x * (1.0f + tanhf(u));
+// GeLU (tanh approximation, reading c12) and its derivative.
+// FAST (the bf16 path): tanh u by the hardware tanh.approx.f32 (one MUFU op; relative error
+// ~2^-11, an order below the bf16 rounding of every value it feeds — reading c12a).
+// Exact (the fp32 path, 1e-5 budget): 0.5(1 + tanh u) written as the logistic
+// s = 1/(1 + e^{-2u}) (an identity) with ex2.approx and a fast divide, a few fp32 ulp;
+// tanh u = 2s - 1 and 1 - tanh^2 u = 4 s (1 - s).  Forward and recompute use the same
+// instance for a dtype, so a recomputed activation matches the stored one bit for bit.
+__device__ __forceinline__ float tanh_approx(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
 }
+__device__ __forceinline__ float gelu_sigmoid_f(float x) {
+  const float c2 = 2.0f * 0.7978845608028654f, a = 0.044715f;
+  const float u2 = c2 * (x + a * x * x * x);
+  return __fdividef(1.0f, 1.0f + __expf(-u2));
+}
+template <bool FAST>
+__device__ __forceinline__ float gelu_tanh_f(float x) {
+  if (FAST) {
+    const float c = 0.7978845608028654f, a = 0.044715f;
+    const float hx = 0.5f * x;
+    return fmaf(hx, tanh_approx(c * (x + a * x * x * x)), hx);
+  }
+  return x * gelu_sigmoid_f(x);
+}
+template <bool FAST>
 __device__ __forceinline__ float gelu_tanh_grad_f(float x) {
   const float c = 0.7978845608028654f, a = 0.044715f;
-  float u = c * (x + a * x * x * x);
-  float t = tanhf(u);
-  return 0.5f * (1.0f + t) + 0.5f * x * (1.0f - t * t) * c * (1.0f + 3.0f * a * x * x);
+  if (FAST) {
+    const float t = tanh_approx(c * (x + a * x * x * x));
+    return 0.5f * (1.0f + t) + 0.5f * x * (1.0f - t * t) * c * (1.0f + 3.0f * a * x * x);
+  }
+  const float s = gelu_sigmoid_f(x);
+  return s + 2.0f * x * s * (1.0f - s) * c * (1.0f + 3.0f * a * x * x);
 }
+template <bool FAST = false>
 __device__ __forceinline__ float act_f(int act, float z) {
   if (act == HARMONY_ACT_RELU) return z > 0.f ? z : 0.f;
-  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_f(z);
+  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_f<FAST>(z);
   return z;
 }
+template <bool FAST = false>
 __device__ __forceinline__ float act_grad_f(int act, float z) {
   if (act == HARMONY_ACT_RELU) return z > 0.f ? 1.f : 0.f;
-  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_grad_f(z);
+  if (act == HARMONY_ACT_GELU_TANH) return gelu_tanh_grad_f<FAST>(z);
   return 1.f;
 }
+// the instance a layer of activation type T uses (bf16: FAST)
+template <typename T>
+__device__ __forceinline__ float act_T(int act, float z) { return act_f<sizeof(T) == 2>(act, z); }
+template <typename T>
+__device__ __forceinline__ float act_grad_T(int act, float z) { return act_grad_f<sizeof(T) == 2>(act, z); }
 
 }  // namespace hm

@@ -42,22 +42,48 @@ __device__ __forceinline__ void epi_scalar(const EpiParams& e, int64_t off, int 
       // the stashed H (stash policies 1, 2) reproduces G bit for bit
       const T zt = from_f32<T>(acc + b);
       reinterpret_cast<T*>(e.C)[off] = zt;
-      reinterpret_cast<T*>(e.aux_out)[off] = from_f32<T>(act_f(e.act, to_f32(zt)));
+      reinterpret_cast<T*>(e.aux_out)[off] = from_f32<T>(act_T<T>(e.act, to_f32(zt)));
       break;
     }
     case HK_EPI_ACT_BWD: {
       float z = to_f32(reinterpret_cast<const T*>(e.aux)[off]);
-      reinterpret_cast<T*>(e.C)[off] = from_f32<T>(acc * act_grad_f(e.act, z));
+      reinterpret_cast<T*>(e.C)[off] = from_f32<T>(acc * act_grad_T<T>(e.act, z));
       break;
     }
     case HK_EPI_BIAS_ACT_F32: {
       float z = acc + b;
       reinterpret_cast<T*>(e.C)[off] = from_f32<T>(z);
-      reinterpret_cast<float*>(e.aux_out)[off] = act_f(e.act, z);
+      reinterpret_cast<float*>(e.aux_out)[off] = act_T<T>(e.act, z);
       break;
     }
     default:
       break;
+  }
+}
+
+// bias[n0 .. n0+31] (bf16) as fp32, zeros without a bias and past N; vector loads when aligned
+__device__ __forceinline__ void load_bias32(const EpiParams& e, int n0, float* bb) {
+  if (!e.bias) {
+#pragma unroll
+    for (int j = 0; j < 32; ++j) bb[j] = 0.f;
+    return;
+  }
+  const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(e.bias) + n0;
+  if (n0 + 32 > e.N) {
+#pragma unroll
+    for (int j = 0; j < 32; ++j) bb[j] = n0 + j < e.N ? __bfloat162float(b[j]) : 0.f;
+  } else if ((reinterpret_cast<uintptr_t>(b) & 15) == 0) {
+    const uint4* b4 = reinterpret_cast<const uint4*>(b);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint4 u = b4[q];
+      const __nv_bfloat16* h = reinterpret_cast<const __nv_bfloat16*>(&u);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) bb[8 * q + j] = __bfloat162float(h[j]);
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < 32; ++j) bb[j] = __bfloat162float(b[j]);
   }
 }
 
@@ -102,8 +128,8 @@ __device__ __forceinline__ void epi_row16(const EpiParams& e, int64_t row_off, i
         const __nv_bfloat16* h1 = reinterpret_cast<const __nv_bfloat16*>(&q1);
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          v[j] = acc[j] * act_grad_f(e.act, __bfloat162float(h0[j]));
-          v[8 + j] = acc[8 + j] * act_grad_f(e.act, __bfloat162float(h1[j]));
+          v[j] = acc[j] * act_grad_T<T>(e.act, __bfloat162float(h0[j]));
+          v[8 + j] = acc[8 + j] * act_grad_T<T>(e.act, __bfloat162float(h1[j]));
         }
       }
       uint4 o[2];
@@ -117,7 +143,7 @@ __device__ __forceinline__ void epi_row16(const EpiParams& e, int64_t row_off, i
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
           const float2 zr = __bfloat1622float2(op[j]);  // the stored (rounded) pre-activation
-          op[j] = __floats2bfloat162_rn(act_f(e.act, zr.x), act_f(e.act, zr.y));
+          op[j] = __floats2bfloat162_rn(act_T<T>(e.act, zr.x), act_T<T>(e.act, zr.y));
         }
         uint4* gp = reinterpret_cast<uint4*>(reinterpret_cast<T*>(e.aux_out) + off);
         gp[0] = o[0];

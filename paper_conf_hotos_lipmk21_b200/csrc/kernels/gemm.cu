@@ -95,37 +95,302 @@ using namespace tcx;
 
 __device__ __forceinline__ uint32_t make_idesc(int bn, int a_mn, int b_mn) { return make_idesc_f16(BM, bn, a_mn, b_mn); }
 
+// Epilogue inputs read from global memory: 1 = fp32 residual (aux), 2 = old fp32 C (dW accumulate),
+// 3 = bf16 stored pre-activation (aux of ACT_BWD), 0 = none.
+__device__ __forceinline__ int epi_in_kind(const EpiParams& e) {
+  if (e.epi == HK_EPI_RESID_F32) return 1;
+  if (e.epi == HK_EPI_ACC_F32 && e.accumulate) return 2;
+  if (e.epi == HK_EPI_ACT_BWD) return 3;
+  return 0;
+}
+
+// L2 prefetch of this thread's row segment [n_beg, n_end) of the epilogue input, issued before the
+// accumulator wait so the (cold, HBM) residual / dW / pre-activation read overlaps the mainloop.
+__device__ __forceinline__ void epi_prefetch(const EpiParams& e, int m, int n_beg, int n_end, int64_t zoff) {
+  const int kind = epi_in_kind(e);
+  if (!kind || m >= e.M || n_beg >= n_end) return;
+  const int esz = kind == 3 ? 2 : 4;
+  const char* base = static_cast<const char*>(kind == 2 ? e.C : e.aux);
+  const char* p = base + (zoff + (int64_t)m * e.ldc + n_beg) * esz;
+  const int bytes = (n_end - n_beg) * esz;
+  for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(p + o));
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p + bytes - 1));
+}
+
+__device__ __forceinline__ bool al16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
 // one epilogue warp's 32-column chunk: TMEM (thread = row) -> registers -> fused epilogue -> global in
-// 32-byte row pieces (full sectors).  A variant that transposed chunks through shared memory for
-// 128-byte row segments measured 6% slower in the step (profiles/r01_epilogue_ab.txt) and was dropped.
+// 32-byte row pieces (full sectors).  The chunk's global inputs are loaded before the TMEM load so
+// their latency overlaps it.  A variant that transposed chunks through shared memory for 128-byte
+// row segments measured 6% slower in the step (profiles/r01_epilogue_ab.txt) and was dropped.
 __device__ __forceinline__ void drain_chunk(const EpiParams& e, uint32_t taddr, bool have_acc, int lane, int mrow0,
                                             int n, int64_t zoff) {
+  const int m = mrow0 + lane;
+  const int64_t off = zoff + (int64_t)m * e.ldc + n;
+  const int kind = epi_in_kind(e);
+  const void* src = kind == 2 ? e.C : e.aux;
+  const bool fast = kind != 0 && m < e.M && n + 32 <= e.N && al16(static_cast<float*>(e.C) + (kind == 3 ? 0 : off)) &&
+                    (kind == 3 ? al16(static_cast<const __nv_bfloat16*>(src) + off) &&
+                                     al16(static_cast<__nv_bfloat16*>(e.C) + off)
+                               : al16(static_cast<const float*>(src) + off));
+  float4 in[8];
+  if (fast) {
+    if (kind == 3) {
+      const uint4* s4 = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(src) + off);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) { uint4 u = s4[q]; in[q] = *reinterpret_cast<float4*>(&u); }
+    } else {
+      const float4* s4 = reinterpret_cast<const float4*>(static_cast<const float*>(src) + off);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) in[q] = s4[q];
+    }
+  }
   float v[32];
   if (have_acc) {
-    tmem_ld16(taddr, v);
-    tmem_ld16(taddr + 16, v + 16);
+    tmem_ld32(taddr, v);
   } else {
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] = 0.f;
   }
-  const int m = mrow0 + lane;
-  if (m < e.M) {
-    epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n, v);
-    if (n + 16 < e.N) epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n + 16, v + 16);
+  if (m >= e.M) return;
+  if (fast) {
+    if (kind == 3) {  // dH = dG * act'(H), bf16 out
+      const __nv_bfloat16* h = reinterpret_cast<const __nv_bfloat16*>(in);
+      uint4 o[4];
+      __nv_bfloat162* op = reinterpret_cast<__nv_bfloat162*>(o);
+#pragma unroll
+      for (int j = 0; j < 16; ++j)
+        op[j] = __floats2bfloat162_rn(v[2 * j] * act_grad_f<true>(e.act, __bfloat162float(h[2 * j])),
+                                      v[2 * j + 1] * act_grad_f<true>(e.act, __bfloat162float(h[2 * j + 1])));
+      uint4* cp = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(e.C) + off);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) cp[q] = o[q];
+    } else {
+      float4* c4 = reinterpret_cast<float4*>(static_cast<float*>(e.C) + off);
+      if (kind == 1) {  // C = aux + (acc + b)
+        float bb[32];
+        load_bias32(e, n, bb);
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          c4[q] = make_float4(in[q].x + (v[4 * q] + bb[4 * q]), in[q].y + (v[4 * q + 1] + bb[4 * q + 1]),
+                              in[q].z + (v[4 * q + 2] + bb[4 * q + 2]), in[q].w + (v[4 * q + 3] + bb[4 * q + 3]));
+      } else {  // C = C + alpha * acc
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          c4[q] = make_float4(in[q].x + e.alpha * v[4 * q], in[q].y + e.alpha * v[4 * q + 1],
+                              in[q].z + e.alpha * v[4 * q + 2], in[q].w + e.alpha * v[4 * q + 3]);
+      }
+    }
+    return;
   }
+  epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n, v);
+  if (n + 16 < e.N) epi_row16<__nv_bfloat16>(e, zoff + (int64_t)m * e.ldc, n + 16, v + 16);
 }
 
 struct TcParams {
   int M, N, K, nz0, nz, a_mn, b_mn;
+  int tma_epi;  // 1: epilogue through shared-memory staging + TMA stores (maps tmC / tmIn / tmO2)
   EpiParams e;
 };
+
+// ------------------------------------------------------------------ TMA-store epilogue
+// Each epilogue warp owns two 4 KB staging boxes of 32 rows x 128 bytes (32 fp32 or 64 bf16
+// columns) in the 128-byte swizzle of the tensor map, so a thread writing its own row in 16-byte
+// pieces is bank-conflict free, plus its columns' bias as fp32.  Per box: TMEM -> registers ->
+// fused epilogue -> staging -> one TMA store (full-line writes, asynchronous: the warp moves on).
+// Epilogues that read global data (residual, old dW, stored pre-activation) TMA-load the box into
+// the staging buffer ahead of use: the first box before the accumulator wait (overlapping the
+// mainloop), each next one while the current one is processed.  BIAS_ACT writes its two bf16
+// outputs through both boxes.  (BIAS_ACT_F32, an fp32 second output, keeps the register path.)
+constexpr int EPI_BUF = 4096;
+constexpr int EPI_BIAS = 128 * 4;  // fp32 bias of a warp's (at most 128) columns
+constexpr int EPI_SMEM = EPI_WARPS * (2 * EPI_BUF + EPI_BIAS) + EPI_WARPS * 2 * 8;
+
+struct EpiWarp {
+  uint32_t buf;   // shared address of the two staging boxes
+  uint32_t bias;  // shared address of the fp32 bias
+  uint64_t* bar;  // input-load barriers of the two boxes
+  uint32_t ph;    // parity bit per box
+  uint32_t j;     // boxes processed
+};
+
+__device__ __forceinline__ uint32_t swz128(int r, int k) { return (uint32_t)(r * 128 + ((k ^ (r & 7)) << 4)); }
+__device__ __forceinline__ void sts128(uint32_t a, uint32_t x, uint32_t y, uint32_t z, uint32_t w) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
+}
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ float4 lds128f(uint32_t a) {
+  uint4 v = lds128(a);
+  return make_float4(__uint_as_float(v.x), __uint_as_float(v.y), __uint_as_float(v.z), __uint_as_float(v.w));
+}
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+__device__ __forceinline__ void tma_load_box(uint32_t dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                             int c3, uint32_t bytes) {
+  mbar_expect_tx(bar, bytes);
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(
+          dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+__device__ __forceinline__ void tma_store_box(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2, int c3) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(src), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+
+// Is the TMA epilogue usable for this epilogue kind / tile width (host and device agree)?
+__host__ __device__ __forceinline__ bool tma_epi_kind_ok(int epi) { return epi != HK_EPI_BIAS_ACT_F32; }
+
+// One warp's share of one tile: 32 rows (row0..) x columns [n_beg, n_end) (n_end - n_beg <= 128),
+// TMEM columns from tacc.  ESZ = output element size (4: fp32 outputs, 2: bf16 outputs).
+template <int ESZ>
+__device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMap* mC, const CUtensorMap* mIn,
+                                             const CUtensorMap* mO2, EpiWarp& w, uint32_t tacc, bool have_acc,
+                                             int lane, int row0, int n_beg, int n_end, int z0, int z1,
+                                             uint64_t* full_bar, uint32_t full_par) {
+  constexpr int CPB = 128 / ESZ;  // columns per box
+  const EpiParams& e = p.e;
+  const int kind = epi_in_kind(e);
+  const bool two = e.epi == HK_EPI_BIAS_ACT;
+  const int nbox = n_end > n_beg ? (n_end - n_beg + CPB - 1) / CPB : 0;
+  const bool has_bias = e.bias != nullptr && (e.epi == HK_EPI_STORE_T || e.epi == HK_EPI_BIAS_ACT ||
+                                              e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32);
+  if (kind && nbox > 0 && lane == 0) {
+    const int b = w.j & 1;
+    bulk_wait_read<1>();  // the store two boxes back has left this box
+    tma_load_box(w.buf + b * EPI_BUF, mIn, &w.bar[b], n_beg, row0, z0, z1, EPI_BUF);
+  }
+  if (has_bias) {  // this warp's bias columns as fp32 (while the mainloop runs)
+    const __nv_bfloat16* bp = static_cast<const __nv_bfloat16*>(e.bias);
+    for (int c = lane; c < nbox * CPB; c += 32) {
+      const int n = n_beg + c;
+      const float bv = n < e.N ? __bfloat162float(bp[n]) : 0.f;
+      asm volatile("st.shared.f32 [%0], %1;" ::"r"(w.bias + 4 * c), "f"(bv) : "memory");
+    }
+    __syncwarp();
+  }
+  mbar_wait(full_bar, full_par);
+  tc_fence_after();
+  const int r = lane;
+#pragma unroll 1
+  for (int bi = 0; bi < nbox; ++bi) {
+    const int b = w.j & 1;
+    const int n = n_beg + CPB * bi;
+    const uint32_t sb = two ? w.buf : w.buf + b * EPI_BUF;
+    if (kind) {
+      if (bi + 1 < nbox && lane == 0) {
+        bulk_wait_read<0>();  // the previous box's store has left the other buffer
+        tma_load_box(w.buf + (b ^ 1) * EPI_BUF, mIn, &w.bar[b ^ 1], n + CPB, row0, z0, z1, EPI_BUF);
+      }
+    } else if (lane == 0) {
+      if (two) bulk_wait_read<0>();
+      else bulk_wait_read<1>();
+    }
+    float v[CPB];
+    if (have_acc) {
+#pragma unroll
+      for (int h = 0; h < CPB / 32; ++h) tmem_ld32(tacc + CPB * bi + 32 * h, v + 32 * h);
+    } else {
+#pragma unroll
+      for (int i = 0; i < CPB; ++i) v[i] = 0.f;
+    }
+    if (kind) {
+      mbar_wait(&w.bar[b], (w.ph >> b) & 1);
+      w.ph ^= 1u << b;
+    } else {
+      __syncwarp();
+    }
+    const uint32_t bias_row = w.bias + 4 * CPB * bi;
+    if (ESZ == 4) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t ad = sb + swz128(r, k);
+        float o0 = e.alpha * v[4 * k], o1 = e.alpha * v[4 * k + 1], o2 = e.alpha * v[4 * k + 2],
+              o3 = e.alpha * v[4 * k + 3];
+        if (e.epi == HK_EPI_RESID_F32) {  // C = aux + (acc + b)
+          float4 bb = has_bias ? lds128f(bias_row + 16 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          const float4 in = lds128f(ad);
+          o0 = in.x + (v[4 * k] + bb.x); o1 = in.y + (v[4 * k + 1] + bb.y);
+          o2 = in.z + (v[4 * k + 2] + bb.z); o3 = in.w + (v[4 * k + 3] + bb.w);
+        } else if (e.epi == HK_EPI_ACC_F32) {  // C (+)= alpha * acc
+          if (kind) {
+            const float4 in = lds128f(ad);
+            o0 = in.x + o0; o1 = in.y + o1; o2 = in.z + o2; o3 = in.w + o3;
+          }
+        } else if (has_bias) {  // STORE_F32
+          float4 bb = lds128f(bias_row + 16 * k);
+          o0 += bb.x; o1 += bb.y; o2 += bb.z; o3 += bb.w;
+        }
+        sts128(ad, __float_as_uint(o0), __float_as_uint(o1), __float_as_uint(o2), __float_as_uint(o3));
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t ad = sb + swz128(r, k);
+        const float* x = v + 8 * k;
+        uint32_t o[4];
+        if (e.epi == HK_EPI_ACT_BWD) {  // dH = dG * act'(H)
+          const uint4 in = lds128(ad);
+          const uint32_t hw[4] = {in.x, in.y, in.z, in.w};
+#pragma unroll
+          for (int t = 0; t < 4; ++t) {
+            const float2 h = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hw[t]));
+            o[t] = pack_bf16(x[2 * t] * act_grad_f<true>(e.act, h.x), x[2 * t + 1] * act_grad_f<true>(e.act, h.y));
+          }
+        } else {
+          float bb[8];
+          if (has_bias) {
+            const float4 b0 = lds128f(bias_row + 32 * k), b1 = lds128f(bias_row + 32 * k + 16);
+            bb[0] = b0.x; bb[1] = b0.y; bb[2] = b0.z; bb[3] = b0.w; bb[4] = b1.x; bb[5] = b1.y; bb[6] = b1.z; bb[7] = b1.w;
+          } else {
+#pragma unroll
+            for (int t = 0; t < 8; ++t) bb[t] = 0.f;
+          }
+          if (e.epi == HK_EPI_STORE_T) {
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+              o[t] = pack_bf16(e.alpha * x[2 * t] + bb[2 * t], e.alpha * x[2 * t + 1] + bb[2 * t + 1]);
+          } else {  // BIAS_ACT: H = acc + b (bf16), G = act(H as stored) into the second box
+            uint32_t g[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              o[t] = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
+              const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&o[t]));
+              g[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
+            }
+            sts128(w.buf + EPI_BUF + swz128(r, k), g[0], g[1], g[2], g[3]);
+          }
+        }
+        sts128(ad, o[0], o[1], o[2], o[3]);
+      }
+    }
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+      tma_store_box(mC, sb, n, row0, z0, z1);
+      if (two) tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
+      bulk_commit();
+    }
+    ++w.j;
+  }
+}
 
 template <int BN, int STAGES>
 struct TcCfg {
   static constexpr int A_BYTES = BM * BK * 2;  // 16 KB
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_SMEM + 1024 /*align*/ + 256 /*barriers*/;
+  static_assert(SMEM <= 232448, "shared memory per CTA");
   static constexpr int ACC_COLS = BN;               // one fp32 accumulator = BN TMEM columns
   static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;  // double-buffered accumulator
 };
@@ -153,13 +418,17 @@ struct TileMap {
 
 template <int BN, int STAGES>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, TcParams p) {
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmIn,
+                   const __grid_constant__ CUtensorMap tmO2, TcParams p) {
   using Cfg = TcCfg<BN, STAGES>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint8_t* sE = smem + STAGES * Cfg::STAGE_BYTES;  // epilogue staging boxes
+  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * (2 * EPI_BUF + EPI_BIAS));
+  uint64_t* full = ebar + EPI_WARPS * 2;
   uint64_t* empty = full + STAGES;
   uint64_t* tmem_full = empty + STAGES;   // [2]
   uint64_t* tmem_empty = tmem_full + 2;   // [2]
@@ -178,6 +447,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     prefetch_tmap(&tmB);
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tmem_full[a], 1); mbar_init(&tmem_empty[a], 32 * EPI_WARPS); }
+    for (int i = 0; i < EPI_WARPS * 2; ++i) mbar_init(&ebar[i], 1);
+    if (p.tma_epi) { prefetch_tmap(&tmC); prefetch_tmap(&tmIn); prefetch_tmap(&tmO2); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -260,23 +531,37 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int half = (warp - 2) >> 2;  // which half of the tile's columns this warp drains
     const EpiParams& e = p.e;
+    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF + (warp - 2) * EPI_BIAS,
+               ebar + (warp - 2) * 2, 0u, 0u};
+    const bool out_f32 = e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32 || e.epi == HK_EPI_ACC_F32;
     int it = 0;
     for (int t = blockIdx.x; t < tm.total; t += gridDim.x, ++it) {
       int z, mb, nb;
       tm.get(t, z, mb, nb);
       const int z0 = z % p.nz0, z1 = z / p.nz0, m0 = mb * BM, n0 = nb * BN;
       const int acc = it & 1;
-      mbar_wait(&tmem_full[acc], (it >> 1) & 1);
-      tc_fence_after();
       const int64_t zoff = z0 * e.c_sz0 + z1 * e.c_sz1;
-      const uint32_t tacc = tmem_base + acc * Cfg::ACC_COLS + ((uint32_t)(q * 32) << 16);
       const int ncols = min(BN, p.N - n0);
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
+      const uint32_t tacc = tmem_base + acc * Cfg::ACC_COLS + ((uint32_t)(q * 32) << 16);
+      if (p.tma_epi) {
+        if (out_f32)
+          tma_epi_tile<4>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, m0 + q * 32, n0 + c_beg, n0 + c_end,
+                          z0, z1, &tmem_full[acc], (it >> 1) & 1);
+        else
+          tma_epi_tile<2>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, m0 + q * 32, n0 + c_beg, n0 + c_end,
+                          z0, z1, &tmem_full[acc], (it >> 1) & 1);
+      } else {
+        epi_prefetch(e, m0 + q * 32 + lane, n0 + c_beg, n0 + c_end, zoff);
+        mbar_wait(&tmem_full[acc], (it >> 1) & 1);
+        tc_fence_after();
 #pragma unroll 1
-      for (int c = c_beg; c < c_end; c += 32) drain_chunk(e, tacc + c, nkb > 0, lane, m0 + q * 32, n0 + c, zoff);
+        for (int c = c_beg; c < c_end; c += 32) drain_chunk(e, tacc + c, nkb > 0, lane, m0 + q * 32, n0 + c, zoff);
+      }
       tc_fence_before();
       mbar_arrive(&tmem_empty[acc]);
     }
+    if (p.tma_epi && lane == 0) bulk_wait_all();
   }
   tc_fence_before();
   __syncthreads();
@@ -289,6 +574,31 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
 // Operand (rows r, K) as a 4-D bf16 map (inner, outer, z0, z1).  K-major: inner = K, box (64, box_r);
 // MN-major: inner = r, box (64, BK).
+// Epilogue maps (C, input, second output); p.tma_epi = 0 when any is not TMA-addressable or
+// HARMONY_GEMM_TMA_EPI=0 (register epilogue).
+static void make_epi_maps(const hk_gemm_args& a, const EpiParams& e, int bn, CUtensorMap* mc, CUtensorMap* mi,
+                          CUtensorMap* mo, TcParams& p) {
+  static const int enabled = [] {
+    const char* v = getenv("HARMONY_GEMM_TMA_EPI");
+    return v ? atoi(v) : 1;
+  }();
+  memset(mc, 0, sizeof(CUtensorMap)); memset(mi, 0, sizeof(CUtensorMap)); memset(mo, 0, sizeof(CUtensorMap));
+  p.tma_epi = 0;
+  const int epi = e.epi;
+  const int esz = (epi == HK_EPI_STORE_F32 || epi == HK_EPI_RESID_F32 || epi == HK_EPI_ACC_F32) ? 4 : 2;
+  // a warp drains bn/2 columns: at least one 128-byte box of the output type
+  if (!enabled || !tma_epi_kind_ok(epi) || (bn / 2) * esz < 128) return;
+  auto mk = [&](CUtensorMap* m, const void* ptr, int sz) {
+    return make_epi_map(m, ptr, sz, a.N, a.M, e.ldc, a.nz0, e.c_sz0, a.nz1, e.c_sz1);
+  };
+  bool ok = mk(mc, e.C, esz);
+  if (epi == HK_EPI_RESID_F32) ok = ok && mk(mi, e.aux, 4);
+  else if (epi == HK_EPI_ACC_F32 && e.accumulate) ok = ok && mk(mi, e.C, 4);
+  else if (epi == HK_EPI_ACT_BWD) ok = ok && mk(mi, e.aux, 2);
+  if (epi == HK_EPI_BIAS_ACT) ok = ok && mk(mo, e.aux_out, 2);
+  p.tma_epi = ok ? 1 : 0;
+}
+
 static void make_operand_map(CUtensorMap* map, const void* ptr, int mn_major, int64_t rows, int64_t K, int64_t ld,
                              int64_t nz0, int64_t sz0, int64_t nz1, int64_t sz1, int box_r) {
   const int64_t inner = mn_major ? rows : K, outer = mn_major ? K : rows;
@@ -304,6 +614,8 @@ static void launch_tc(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
   p.e = e;
+  CUtensorMap mc, mi, mo;
+  make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
   static bool attr_set = false;  // per instantiation
   if (!attr_set) {
     HM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
@@ -319,7 +631,7 @@ static void launch_tc(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st
   dim3 grid((unsigned)std::min<int64_t>(tiles, num_sms));  // persistent: at most one CTA per SM
   // profiling events bracket only the device work (tensor maps are encoded before)
   const int e0 = g_prof.begin(st);
-  gemm_tc_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, p);
+  gemm_tc_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
   check_launch("gemm_tc_kernel");
   g_prof.end(PROF_GEMM, e0, st, 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1);
 }
@@ -392,19 +704,24 @@ struct Tc2Cfg {
   static constexpr int A_BYTES = 128 * BK * 2; // 16 KB
   static constexpr int B_BYTES = HB * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_SMEM + 1024 + 256;
+  static_assert(SMEM <= 232448, "shared memory per CTA");
   static constexpr int TMEM_COLS = 2 * BN;     // double-buffered accumulator (BN fp32 columns each)
 };
 
 template <int BN, int STAGES>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
-    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, TcParams p) {
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                    const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmIn,
+                    const __grid_constant__ CUtensorMap tmO2, TcParams p) {
   using Cfg = Tc2Cfg<BN, STAGES>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint8_t* sE = smem + STAGES * Cfg::STAGE_BYTES;  // epilogue staging boxes
+  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * (2 * EPI_BUF + EPI_BIAS));
+  uint64_t* full = ebar + EPI_WARPS * 2;
   uint64_t* empty = full + STAGES;
   uint64_t* tmem_full = empty + STAGES;  // [2]
   uint64_t* tmem_empty = tmem_full + 2;  // [2] (used in the leader)
@@ -426,6 +743,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     prefetch_tmap(&tmB);
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 2); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tmem_full[a], 1); mbar_init(&tmem_empty[a], 2 * 32 * EPI_WARPS); }
+    for (int i = 0; i < EPI_WARPS * 2; ++i) mbar_init(&ebar[i], 1);
+    if (p.tma_epi) { prefetch_tmap(&tmC); prefetch_tmap(&tmIn); prefetch_tmap(&tmO2); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -510,24 +829,38 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const int half = (warp - 2) >> 2;
     const EpiParams& e = p.e;
     const uint32_t te = mapa_leader(&tmem_empty[0]);
+    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF + (warp - 2) * EPI_BIAS,
+               ebar + (warp - 2) * 2, 0u, 0u};
+    const bool out_f32 = e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32 || e.epi == HK_EPI_ACC_F32;
     int it = 0;
     for (int t = pair; t < tm.total; t += npairs, ++it) {
       int z, mb, nb;
       tm.get(t, z, mb, nb);
       const int z0 = z % p.nz0, z1 = z / p.nz0, n0 = nb * BN;
       const int acc = it & 1;
-      mbar_wait(&tmem_full[acc], (it >> 1) & 1);
-      tc_fence_after();
       const int64_t zoff = z0 * e.c_sz0 + z1 * e.c_sz1;
-      const uint32_t tacc = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
       const int ncols = min(BN, p.N - n0);
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
+      const int row0 = mb * 256 + (int)rank * 128 + q * 32;
+      const uint32_t tacc = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
+      if (p.tma_epi) {
+        if (out_f32)
+          tma_epi_tile<4>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0, z1,
+                          &tmem_full[acc], (it >> 1) & 1);
+        else
+          tma_epi_tile<2>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0, z1,
+                          &tmem_full[acc], (it >> 1) & 1);
+      } else {
+        epi_prefetch(e, row0 + lane, n0 + c_beg, n0 + c_end, zoff);
+        mbar_wait(&tmem_full[acc], (it >> 1) & 1);
+        tc_fence_after();
 #pragma unroll 1
-      for (int c = c_beg; c < c_end; c += 32)
-        drain_chunk(e, tacc + c, nkb > 0, lane, mb * 256 + (int)rank * 128 + q * 32, n0 + c, zoff);
+        for (int c = c_beg; c < c_end; c += 32) drain_chunk(e, tacc + c, nkb > 0, lane, row0, n0 + c, zoff);
+      }
       tc_fence_before();
       mbar_arrive_cluster(te + acc * 8);
     }
+    if (p.tma_epi && lane == 0) bulk_wait_all();
   }
   tc_fence_before();
   cluster_sync_all();
@@ -547,6 +880,8 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
   p.e = e;
+  CUtensorMap mc, mi, mo;
+  make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
   static bool attr_set = false;
   if (!attr_set) {
     HM_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel<BN, STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
@@ -561,7 +896,7 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   const int64_t tiles = ceil_div(a.M, 256) * ceil_div(a.N, BN) * (int64_t)a.nz0 * a.nz1;
   dim3 grid((unsigned)(2 * std::min<int64_t>(tiles, num_sms / 2)));  // persistent pairs
   const int e0 = g_prof.begin(st);
-  gemm_tc2_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, p);
+  gemm_tc2_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
   check_launch("gemm_tc2_kernel");
   g_prof.end(PROF_GEMM, e0, st, 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1);
 }
@@ -599,15 +934,15 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
     // CTA-pair 256 x 256 tiles (measured best for every cfg2 shape, tools/gemm_bench.py);
     // HARMONY_GEMM_2SM=3 selects 256 x 128 pair tiles, 0 the single-CTA kernel
     if (mode == 3) tc::launch_tc2<128, 6>(a, e, st);
-    else tc::launch_tc2<256, 6>(a, e, st);
+    else tc::launch_tc2<256, 4>(a, e, st);
     return;
   }
   if (a.N <= 64)
-    tc::launch_tc<64, 8>(a, e, st);
+    tc::launch_tc<64, 6>(a, e, st);
   else if (a.N <= 128 || (int64_t)ceil_div(a.M, 128) * ceil_div(a.N, 256) * nz < 148)
-    tc::launch_tc<128, 6>(a, e, st);
+    tc::launch_tc<128, 4>(a, e, st);
   else
-    tc::launch_tc<256, 4>(a, e, st);
+    tc::launch_tc<256, 3>(a, e, st);
 }
 
 }  // namespace hm

@@ -283,13 +283,13 @@ __global__ void act_bwd_kernel(int act, int64_t n, const float* __restrict__ dY,
                                T* __restrict__ dZ) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
-    dZ[i] = from_f32<T>(dY[i] * act_grad_f(act, to_f32(Z[i])));
+    dZ[i] = from_f32<T>(dY[i] * act_grad_T<T>(act, to_f32(Z[i])));
 }
 template <typename T>
 __global__ void act_fwd_kernel(int act, int64_t n, const T* __restrict__ Z, T* __restrict__ out) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
-    out[i] = from_f32<T>(act_f(act, to_f32(Z[i])));
+    out[i] = from_f32<T>(act_T<T>(act, to_f32(Z[i])));
 }
 __global__ void copy_rows_kernel(int64_t n4, const float4* __restrict__ src, float4* __restrict__ dst) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;

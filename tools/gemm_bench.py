@@ -1,4 +1,5 @@
-"""Time the step's GEMM shapes (cfg2, one microbatch of 4096 tokens, d = 1024) through hk_gemm.
+"""Time the step's GEMMs (cfg2: one microbatch of 4096 tokens, d = 1024; the 12 linear GEMMs of a
+transformer layer with their in-step epilogues) through hk_gemm.
 
     python tools/gemm_bench.py [--reps 20] [--only NAME]
 
@@ -39,30 +40,73 @@ def shapes():
         a.B, a.b_mn_major, a.ldb, a.b_sz0, a.b_sz1 = Bm, bmn, ldb, kw.get("b_sz0", 0), kw.get("b_sz1", 0)
         a.C, a.ldc, a.c_sz0, a.c_sz1 = Cm, ldc, kw.get("c_sz0", 0), kw.get("c_sz1", 0)
         a.epilogue, a.alpha, a.accumulate = epi, 1.0, kw.get("acc", 0)
+        a.bias, a.aux, a.aux_out, a.act = kw.get("bias"), kw.get("aux"), kw.get("aux_out"), kw.get("act", 0)
         out.append((name, a, 2.0 * M * N * K * a.nz0 * a.nz1))
 
     X, W, Q, P, C32, C16 = (t.data_ptr() for t in (x, w, qkv, p, c32, c16))
-    g("fc1_fwd", T, 4 * D, D, X, 0, D, W, 1, 4 * D, C16, 4 * D, H.HK_EPI_STORE_T)
-    g("fc2_fwd", T, D, 4 * D, X, 0, 4 * D, W, 1, D, C32, D, H.HK_EPI_STORE_F32)
-    g("qkv_fwd", T, 3 * D, D, X, 0, D, W, 1, 3 * D, C16, 3 * D, H.HK_EPI_STORE_T)
-    g("fc1_dgrad", T, D, 4 * D, X, 0, 4 * D, W, 0, 4 * D, C32, D, H.HK_EPI_STORE_F32)
-    g("fc1_wgrad", D, 4 * D, T, X, 1, D, X, 1, 4 * D, C32, 4 * D, H.HK_EPI_ACC_F32, acc=1)
-    g("fc2_wgrad", 4 * D, D, T, X, 1, 4 * D, X, 1, D, C32, D, H.HK_EPI_ACC_F32, acc=1)
-    g("attn_qk", S, S, DH, Q, 0, 3 * D, Q + 2 * D, 0, 3 * D, C32, S, H.HK_EPI_STORE_F32, nz0=NH, nz1=B,
-      a_sz0=DH, a_sz1=S * 3 * D, b_sz0=DH, b_sz1=S * 3 * D, c_sz0=S * S, c_sz1=NH * S * S)
-    g("attn_pv", S, DH, S, P, 0, S, Q + 4 * D, 1, 3 * D, C16, D, H.HK_EPI_STORE_T, nz0=NH, nz1=B,
-      a_sz0=S * S, a_sz1=NH * S * S, b_sz0=DH, b_sz1=S * 3 * D, c_sz0=DH, c_sz1=S * D)
-    g("attn_dv", S, DH, S, P, 1, S, Q, 1, 3 * D, C16, D, H.HK_EPI_STORE_T, nz0=NH, nz1=B,
-      a_sz0=S * S, a_sz1=NH * S * S, b_sz0=DH, b_sz1=S * 3 * D, c_sz0=DH, c_sz1=S * D)
-    return out, (x, w, qkv, p, c32, c16)
+    bias = torch.randn(4 * D, device="cuda").to(bf)
+    aux32 = torch.randn(T * D, device="cuda")
+    aux16 = torch.randn(T * 4 * D, device="cuda").to(bf)
+    out16 = torch.zeros(T * 4 * D, device="cuda", dtype=bf)
+    keep = [bias, aux32, aux16, out16]
+    BI, A32, A16, O16 = (t.data_ptr() for t in keep)
+
+    def lin_fwd(name, n, k, C, epi, **kw):  # Y[T][n] = X[T][k] . W[k][n]
+        g(name, T, n, k, X, 0, k, W, 1, n, C, n, epi, **kw)
+
+    def lin_dgrad(name, n, k, C, epi, **kw):  # dX[T][k] = dY[T][n] . W^T
+        g(name, T, k, n, X, 0, n, W, 0, n, C, k, epi, **kw)
+
+    def lin_wgrad(name, n, k):  # dW[k][n] += X^T . dY
+        g(name, k, n, T, X, 1, k, X, 1, n, C32, n, H.HK_EPI_ACC_F32, acc=1)
+
+    # the per-microbatch GEMMs of one transformer layer, in-step epilogues (layers.cu fwd_core/bwd_core)
+    lin_fwd("qkv_fwd", 3 * D, D, C16, H.HK_EPI_STORE_T, bias=BI)
+    lin_fwd("out_fwd", D, D, C32, H.HK_EPI_RESID_F32, bias=BI, aux=A32)
+    lin_fwd("fc1_fwd", 4 * D, D, C16, H.HK_EPI_BIAS_ACT, bias=BI, act=2, aux_out=O16)
+    lin_fwd("fc2_fwd", D, 4 * D, C32, H.HK_EPI_RESID_F32, bias=BI, aux=A32)
+    lin_dgrad("fc2_dgrad", D, 4 * D, C16, H.HK_EPI_ACT_BWD, act=2, aux=A16)
+    lin_dgrad("fc1_dgrad", 4 * D, D, C32, H.HK_EPI_STORE_F32)
+    lin_dgrad("out_dgrad", D, D, C16, H.HK_EPI_STORE_T)
+    lin_dgrad("qkv_dgrad", 3 * D, D, C32, H.HK_EPI_STORE_F32)
+    lin_wgrad("fc2_wgrad", D, 4 * D)
+    lin_wgrad("fc1_wgrad", 4 * D, D)
+    lin_wgrad("out_wgrad", D, D)
+    lin_wgrad("qkv_wgrad", 3 * D, D)
+    return out, (x, w, qkv, p, c32, c16, keep)
+
+
+def sweep():
+    """M = 4096, N in {3072, 4096}, K in {256 .. 4096}: time = mainloop(K) + per-tile overhead."""
+    bf = torch.bfloat16
+    x = torch.randn(T, 4 * D, device="cuda").to(bf)
+    w = torch.randn(4 * D, 4 * D, device="cuda").to(bf) * 0.02
+    c16 = torch.zeros(T * 4 * D, device="cuda", dtype=bf)
+    o16 = torch.zeros(T * 4 * D, device="cuda", dtype=bf)
+    c32 = torch.zeros(T * 4 * D, device="cuda")
+    bias = torch.randn(4 * D, device="cuda").to(bf)
+    out = []
+    for n in (3072, 4096):
+        for k in (256, 512, 1024, 2048, 4096):
+            for epi, nm in ((H.HK_EPI_STORE_T, "T"), (H.HK_EPI_STORE_F32, "F32"), (H.HK_EPI_BIAS_ACT, "BACT")):
+                a = H.hk_gemm_args()
+                a.dtype, a.M, a.N, a.K, a.nz0, a.nz1 = 1, T, n, k, 1, 1
+                a.A, a.a_mn_major, a.lda = x.data_ptr(), 0, k
+                a.B, a.b_mn_major, a.ldb = w.data_ptr(), 1, n
+                a.C, a.ldc = (c32 if epi == H.HK_EPI_STORE_F32 else c16).data_ptr(), n
+                a.epilogue, a.alpha, a.accumulate = epi, 1.0, 0
+                a.bias, a.aux_out, a.act = bias.data_ptr(), o16.data_ptr(), 2
+                out.append((f"sweep_{nm}_n{n}_k{k}", a, 2.0 * T * n * k))
+    return out, (x, w, c16, o16, c32, bias)
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--only", default=None)
+    ap.add_argument("--sweep", action="store_true", help="K sweep of the QKV / FC1 shapes (epilogue vs mainloop)")
     args = ap.parse_args()
-    sh, keep = shapes()
+    sh, keep = sweep() if args.sweep else shapes()
     st = torch.cuda.current_stream()
     total_f = total_t = 0.0
     for name, a, fl in sh:
