@@ -40,62 +40,81 @@ struct FwdCfg {
   static constexpr int Q_BYTES = BQ * DH * 2;           // DH/64 K-atoms of 16 KB
   static constexpr int K_BYTES = BKV * DH * 2;
   static constexpr int V_BYTES = BKV * DH * 2;          // 2 key-atoms x DH/64 MN-chunks of 8 KB
-  static constexpr int P_BYTES = BQ * BKV * 2;          // 2 key-atoms of 16 KB
-  static constexpr int KST = 2, VST = DH == 64 ? 2 : 1, PST = 2;  // DH=128: fits 227 KB with 1 V stage
-  static constexpr int SMEM = Q_BYTES + KST * K_BYTES + VST * V_BYTES + PST * P_BYTES + 1024 + 512;
+  static constexpr int O_BYTES = BQ * DH * 2;           // output staging (DH/64 boxes of 64 columns)
+  static constexpr int QST = 2, KST = DH == 64 ? 4 : 2, VST = DH == 64 ? 4 : 2;
+  static constexpr int SMEM = QST * Q_BYTES + KST * K_BYTES + VST * V_BYTES + O_BYTES + 1024 + 256 + 2 * BQ * 4;
   static constexpr int S_COLS = BKV;                    // fp32 accumulator columns per S buffer
   static constexpr int O_COL = 2 * BKV;                 // O after the two S buffers
+  static constexpr int P_COL = 2 * BKV + DH;            // two P buffers (bf16 pairs: BKV/2 columns each)
   static constexpr int TMEM_COLS = 512;
+  static_assert(P_COL + BKV <= TMEM_COLS, "TMEM columns");
+  static_assert(SMEM <= 232448, "shared memory per CTA");
 };
 
 struct FwdParams {
-  int S, H, causal;
+  int S, H, B, causal;
   float scale_log2;  // scale * log2(e)
   float scale;
-  __nv_bfloat16* C;  // [b*S, H*DH]
   float* lse;        // [b, H, S]
-  int ldc;
 };
 
+// work item -> (sequence, head, query tile); query tiles in decreasing order so that, when causal,
+// the long rows are handed out first
+__device__ __forceinline__ void fwd_item(int item, int nq, int H, int& b, int& h, int& qt) {
+  qt = nq - 1 - item % nq;
+  h = (item / nq) % H;
+  b = item / (nq * H);
+}
+
+// Persistent: one CTA per SM loops over the (query tile, head, sequence) items.  All pipeline
+// counters (Q / K / V stages, S and P buffers) run on across items, so the producer loads the next
+// item's Q and K while the current one is in its second pass, the MMA issues the next item's
+// first-pass scores while the softmax warps drain O of the current one (O has its own full /
+// empty barriers), and the output leaves through shared memory with TMA stores.  P never touches
+// shared memory: the softmax warps store it (bf16 pairs) into TMEM and O += P V takes its A
+// operand from there.
 template <int DH>
 __global__ void __launch_bounds__(THREADS, 1)
     attn_fwd_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-                    const __grid_constant__ CUtensorMap tmV, FwdParams p) {
+                    const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmC, FwdParams p) {
   using Cfg = FwdCfg<DH>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
-  uint8_t* sK = sQ + Cfg::Q_BYTES;
+  uint8_t* sK = sQ + Cfg::QST * Cfg::Q_BYTES;
   uint8_t* sV = sK + Cfg::KST * Cfg::K_BYTES;
-  uint8_t* sP = sV + Cfg::VST * Cfg::V_BYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sP + Cfg::PST * Cfg::P_BYTES);
-  uint64_t* q_full = bars;
-  uint64_t* k_full = bars + 1;   // [2]
-  uint64_t* k_empty = bars + 3;  // [2]
-  uint64_t* v_full = bars + 5;   // [2]
-  uint64_t* v_empty = bars + 7;  // [2]
-  uint64_t* s_full = bars + 9;   // [2]
-  uint64_t* s_empty = bars + 11; // [2]
-  uint64_t* p_full = bars + 13;  // [2]
-  uint64_t* p_empty = bars + 15; // [2]
-  uint64_t* o_full = bars + 17;
-  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 18);
+  uint8_t* sO = sV + Cfg::VST * Cfg::V_BYTES;  // output staging
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sO + Cfg::O_BYTES);
+  uint64_t* q_full = bars;                      // [2]
+  uint64_t* q_empty = q_full + 2;               // [2]
+  uint64_t* k_full = q_empty + 2;               // [KST]
+  uint64_t* k_empty = k_full + Cfg::KST;        // [KST]
+  uint64_t* v_full = k_empty + Cfg::KST;        // [VST]
+  uint64_t* v_empty = v_full + Cfg::VST;        // [VST]
+  uint64_t* s_full = v_empty + Cfg::VST;        // [2]
+  uint64_t* s_empty = s_full + 2;               // [2]
+  uint64_t* p_full = s_empty + 2;               // [2]
+  uint64_t* p_empty = p_full + 2;               // [2]
+  uint64_t* o_full = p_empty + 2;
+  uint64_t* o_empty = o_full + 1;
+  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(o_empty + 1);
+  static_assert((14 + 2 * Cfg::KST + 2 * Cfg::VST) * 8 + 4 <= 256, "barrier area");
+  float(*sm_x)[BQ] = reinterpret_cast<float(*)[BQ]>(reinterpret_cast<uint8_t*>(bars) + 256);  // [2][BQ] row stats
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int qt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
-  const int q0 = qt * BQ;
-  const int ntiles = p.causal ? qt + 1 : p.S / BKV;
+  const int nq = p.S / BQ;
+  const int items = nq * p.H * p.B;
 
   if (warp == 0 && lane == 0) {
-    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV);
-    mbar_init(q_full, 1);
+    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmC);
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1);
-      mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1);
+      mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1);
       mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 256);
       mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1);
     }
-    mbar_init(o_full, 1);
+    for (int i = 0; i < Cfg::KST; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
+    for (int i = 0; i < Cfg::VST; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
+    mbar_init(o_full, 1); mbar_init(o_empty, 256);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -110,30 +129,39 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      // ===== TMA producer: Q once; K tiles for both passes; V tiles for pass 2 =====
-      mbar_expect_tx(q_full, Cfg::Q_BYTES);
-#pragma unroll
-      for (int a = 0; a < DH / 64; ++a) tma_load_4d(sQ + a * (BQ * 128), &tmQ, q_full, a * 64, q0, h, b);
+      // ===== TMA producer: per item Q once, K tiles for both passes, V tiles for pass 2 =====
       int ks = 0; uint32_t kph = 0;
       int vs = 0; uint32_t vph = 0;
-      for (int pass = 0; pass < 2; ++pass) {
-        for (int j = 0; j < ntiles; ++j) {
-          mbar_wait(&k_empty[ks], kph ^ 1);
-          mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
+      int n = 0;
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+        int b, h, qt;
+        fwd_item(item, nq, p.H, b, h, qt);
+        const int ntiles = p.causal ? qt + 1 : nq;
+        const int qs = n & 1;
+        mbar_wait(&q_empty[qs], ((n >> 1) & 1) ^ 1);
+        mbar_expect_tx(&q_full[qs], Cfg::Q_BYTES);
 #pragma unroll
-          for (int a = 0; a < DH / 64; ++a)
-            tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
-          if (++ks == 2) { ks = 0; kph ^= 1; }
-          if (pass == 1) {
-            mbar_wait(&v_empty[vs], vph ^ 1);
-            mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
+        for (int a = 0; a < DH / 64; ++a)
+          tma_load_4d(sQ + qs * Cfg::Q_BYTES + a * (BQ * 128), &tmQ, &q_full[qs], a * 64, qt * BQ, h, b);
+        for (int pass = 0; pass < 2; ++pass) {
+          for (int j = 0; j < ntiles; ++j) {
+            mbar_wait(&k_empty[ks], kph ^ 1);
+            mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
 #pragma unroll
-            for (int ka = 0; ka < 2; ++ka)
+            for (int a = 0; a < DH / 64; ++a)
+              tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
+            if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
+            if (pass == 1) {
+              mbar_wait(&v_empty[vs], vph ^ 1);
+              mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
 #pragma unroll
-              for (int c = 0; c < DH / 64; ++c)
-                tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
-                            j * BKV + ka * 64, h, b);
-            if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
+              for (int ka = 0; ka < 2; ++ka)
+#pragma unroll
+                for (int c = 0; c < DH / 64; ++c)
+                  tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
+                              j * BKV + ka * 64, h, b);
+              if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
+            }
           }
         }
       }
@@ -145,51 +173,62 @@ __global__ void __launch_bounds__(THREADS, 1)
       const uint32_t idesc_s = make_idesc_f16(128, BKV, 0, 0);
       // O += P V: M=128, N=DH, K=128 keys; P K-major (smem), V MN-major.
       const uint32_t idesc_o = make_idesc_f16(128, DH, 0, 1);
-      mbar_wait(q_full, 0);
-      const uint32_t qa = smem_u32(sQ);
       int ks = 0; uint32_t kph = 0;
       int vs = 0; uint32_t vph = 0;
-      int it = 0;  // S-buffer use counter across both passes
-      auto issue_s = [&](int sb) {
-        mbar_wait(&k_full[ks], kph);
-        mbar_wait(&s_empty[sb], (((it >> 1) & 1) ^ 1));
-        tc_fence_after();
-        const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
+      int it = 0;  // S-buffer uses
+      int pc = 0;  // P-buffer uses
+      int n = 0;
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+        int b, h, qt;
+        fwd_item(item, nq, p.H, b, h, qt);
+        const int ntiles = p.causal ? qt + 1 : nq;
+        const int qs = n & 1;
+        mbar_wait(&q_full[qs], (n >> 1) & 1);
+        const uint32_t qa = smem_u32(sQ + qs * Cfg::Q_BYTES);
+        auto issue_s = [&]() {
+          const int sb = it & 1;
+          mbar_wait(&k_full[ks], kph);
+          mbar_wait(&s_empty[sb], ((it >> 1) & 1) ^ 1);
+          tc_fence_after();
+          const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
 #pragma unroll
-        for (int kk = 0; kk < DH / 16; ++kk) {
-          const int atom = kk / 4, sub = kk % 4;
-          uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
-          uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
-          mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
-        }
-        mma_commit(&k_empty[ks]);
-        mma_commit(&s_full[sb]);
-        if (++ks == 2) { ks = 0; kph ^= 1; }
-        ++it;
-      };
-      for (int j = 0; j < ntiles; ++j) issue_s(it & 1);  // pass 1
-      // pass 2: S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
-      issue_s(it & 1);
-      for (int j = 0; j < ntiles; ++j) {
-        if (j + 1 < ntiles) issue_s(it & 1);
-        const int pb = j & 1;
-        mbar_wait(&p_full[pb], (j >> 1) & 1);
-        mbar_wait(&v_full[vs], vph);
-        tc_fence_after();
-        const uint32_t pa = smem_u32(sP + pb * Cfg::P_BYTES);
-        const uint32_t va = smem_u32(sV + vs * Cfg::V_BYTES);
+          for (int kk = 0; kk < DH / 16; ++kk) {
+            const int atom = kk / 4, sub = kk % 4;
+            uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
+            uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
+            mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
+          }
+          mma_commit(&k_empty[ks]);
+          mma_commit(&s_full[sb]);
+          if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
+          ++it;
+        };
+        for (int j = 0; j < ntiles; ++j) issue_s();  // pass 1
+        // pass 2: S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
+        issue_s();
+        for (int j = 0; j < ntiles; ++j) {
+          if (j + 1 < ntiles) issue_s();
+          const int pb = pc & 1;
+          mbar_wait(&p_full[pb], (pc >> 1) & 1);
+          mbar_wait(&v_full[vs], vph);
+          if (j == 0) mbar_wait(o_empty, (n & 1) ^ 1);  // the previous item's O has been drained
+          tc_fence_after();
+          const uint32_t pa = tmem + Cfg::P_COL + pb * (BKV / 2);
+          const uint32_t va = smem_u32(sV + vs * Cfg::V_BYTES);
 #pragma unroll
-        for (int kk = 0; kk < BKV / 16; ++kk) {
-          const int atom = kk / 4, sub = kk % 4;
-          uint64_t ad = make_sdesc(pa + atom * (BQ * 128) + sub * 32, 16, 1024);
-          uint64_t bd = make_sdesc(va + atom * (DH / 64) * 8192 + sub * 2048, 8192, 1024);
-          mma_bf16(tmem + Cfg::O_COL, ad, bd, idesc_o, (j | kk) ? 1u : 0u);
+          for (int kk = 0; kk < BKV / 16; ++kk) {
+            const int atom = kk / 4, sub = kk % 4;
+            uint64_t bd = make_sdesc(va + atom * (DH / 64) * 8192 + sub * 2048, 8192, 1024);
+            mma_bf16_ts(tmem + Cfg::O_COL, pa + kk * 8, bd, idesc_o, (j | kk) ? 1u : 0u);
+          }
+          mma_commit(&v_empty[vs]);
+          mma_commit(&p_empty[pb]);
+          if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
+          ++pc;
         }
-        mma_commit(&v_empty[vs]);
-        mma_commit(&p_empty[pb]);
-        if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
+        mma_commit(&q_empty[qs]);
+        mma_commit(o_full);
       }
-      mma_commit(o_full);
     }
     __syncwarp();
   } else {
@@ -199,89 +238,125 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int half = (warp - 2) >> 2;
     const int cb = half * 64;
     const int r = qd * 32 + lane;        // row within the tile
-    const int qrow = q0 + r;             // query index within the sequence
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
-    float m = -INFINITY, l = 0.f;
-    int it = 0;
-    // ---- pass 1: row max only (no exponentials)
-    for (int j = 0; j < ntiles; ++j, ++it) {
-      const int sb = it & 1;
-      mbar_wait(&s_full[sb], (it >> 1) & 1);
-      tc_fence_after();
-      const bool diag = p.causal && j == qt;
-#pragma unroll 1
-      for (int c = cb; c < cb + 64; c += 16) {
-        float v[16];
-        tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
+    const bool issuer = qd == 0 && lane == 0;  // of this half's TMA store of O
+    int it = 0, pc = 0, n = 0;
+    for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+      int b, h, qt;
+      fwd_item(item, nq, p.H, b, h, qt);
+      const int ntiles = p.causal ? qt + 1 : nq;
+      const int qrow = qt * BQ + r;  // query index within the sequence
+      float m = -INFINITY;
+      // ---- pass 1: row max only (no exponentials).  A thread's 64 columns come in one batch of
+      // TMEM loads and reduce in four independent chains (ILP); only the diagonal tile is masked.
+      for (int j = 0; j < ntiles; ++j, ++it) {
+        const int sb = it & 1;
+        mbar_wait(&s_full[sb], (it >> 1) & 1);
+        tc_fence_after();
+        const bool diag = p.causal && j == qt;
+        float v[64];
+        tmem_ld64(tmem + trow + sb * Cfg::S_COLS + cb, v);
+        tc_fence_before();
+        mbar_arrive_local(&s_empty[sb]);  // S is in registers: the MMA may overwrite the buffer
+        if (diag) {
+          const int lim = qrow - (j * BKV + cb);  // keys cb + i with i <= lim are visible
 #pragma unroll
-        for (int i = 0; i < 16; ++i)
-          if (!(diag && j * BKV + c + i > qrow)) m = fmaxf(m, v[i]);
+          for (int i = 0; i < 64; ++i)
+            if (i > lim) v[i] = -INFINITY;
+        }
+        float m4[4] = {m, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int i = 0; i < 64; ++i) m4[i & 3] = fmaxf(m4[i & 3], v[i]);
+        m = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
       }
-      tc_fence_before();
-      mbar_arrive_local(&s_empty[sb]);
-    }
-    __shared__ float sm_x[2][BQ];
-    sm_x[half][r] = m;
-    asm volatile("bar.sync 1, 256;" ::: "memory");
-    m = fmaxf(sm_x[0][r], sm_x[1][r]);  // the row max over all keys (the diagonal key is always valid)
-    // ---- pass 2: P = 2^((s - m) scale log2e) in (0, 1] (bf16) into shared memory, swizzled K-major
-    // (A operand of O += P V); the row sum l accumulates alongside and O is divided by it at the end
-    for (int j = 0; j < ntiles; ++j, ++it) {
-      const int sb = it & 1, pb = j & 1;
-      mbar_wait(&s_full[sb], (it >> 1) & 1);
-      mbar_wait(&p_empty[pb], ((j >> 1) & 1) ^ 1);
-      tc_fence_after();
-      const bool diag = p.causal && j == qt;
-      uint8_t* prow = sP + pb * Cfg::P_BYTES + r * 128;
-#pragma unroll 1
-      for (int c = cb; c < cb + 64; c += 16) {
-        float v[16];
-        tmem_ld16(tmem + trow + sb * Cfg::S_COLS + c, v);
-        uint32_t pk[8];
+      sm_x[half][r] = m;
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      m = fmaxf(sm_x[0][r], sm_x[1][r]);  // the row max over all keys (the diagonal key is always valid)
+      // ---- pass 2: P = 2^((s - m) scale log2e) in (0, 1] (bf16) into shared memory, swizzled
+      // K-major (A operand of O += P V); the row sum accumulates alongside, O is divided by it at the end
+      const float ms = m * p.scale_log2;
+      float l4[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int j = 0; j < ntiles; ++j, ++it, ++pc) {
+        const int sb = it & 1, pb = pc & 1;
+        mbar_wait(&s_full[sb], (it >> 1) & 1);
+        tc_fence_after();
+        const bool diag = p.causal && j == qt;
+        float v[64];
+        tmem_ld64(tmem + trow + sb * Cfg::S_COLS + cb, v);
+        tc_fence_before();
+        mbar_arrive_local(&s_empty[sb]);
+        const int lim = diag ? qrow - (j * BKV + cb) : 64;
+        uint32_t pk[32];
+        const float2 sl2 = make_float2(p.scale_log2, p.scale_log2), nms2 = make_float2(-ms, -ms);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          float a0 = (diag && j * BKV + c + 2 * i > qrow) ? 0.f : fast_exp2((v[2 * i] - m) * p.scale_log2);
-          float a1 = (diag && j * BKV + c + 2 * i + 1 > qrow) ? 0.f : fast_exp2((v[2 * i + 1] - m) * p.scale_log2);
-          l += a0 + a1;
+        for (int i = 0; i < 32; ++i) {
+          const float2 x = ffma2(make_float2(v[2 * i], v[2 * i + 1]), sl2, nms2);
+          float a0 = fast_exp2(x.x);
+          float a1 = fast_exp2(x.y);
+          if (diag) {
+            if (2 * i > lim) a0 = 0.f;
+            if (2 * i + 1 > lim) a1 = 0.f;
+          }
+          l4[i & 3] += a0 + a1;
           __nv_bfloat162 h2 = __floats2bfloat162_rn(a0, a1);
           pk[i] = *reinterpret_cast<uint32_t*>(&h2);
         }
-        // keys c..c+15 = two 16-byte chunks of key-atom (c / 64), chunk index (c % 64) / 8
-        const int atom = c / 64, ch = (c % 64) / 8;
-        uint8_t* base = prow + atom * (BQ * 128);
-        *reinterpret_cast<uint4*>(base + (((ch) ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-        *reinterpret_cast<uint4*>(base + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        mbar_wait(&p_empty[pb], ((pc >> 1) & 1) ^ 1);
+        tc_fence_after();
+        // this thread's 64 keys -> 32 TMEM columns (bf16 pairs) of P buffer pb, row = its lane
+        tmem_st32(tmem + trow + Cfg::P_COL + pb * (BKV / 2) + half * 32, pk);
+        tmem_wait_st();
+        tc_fence_before();
+        mbar_arrive_local(&p_full[pb]);
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async (UMMA) reads
-      tc_fence_before();
-      mbar_arrive_local(&s_empty[sb]);
-      mbar_arrive_local(&p_full[pb]);
-    }
-    asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
-    sm_x[half][r] = l;
-    asm volatile("bar.sync 1, 256;" ::: "memory");
-    l = sm_x[0][r] + sm_x[1][r];
-    const float inv_l = 1.f / l;
-    // ---- epilogue: O row -> bf16 C, LSE
-    mbar_wait(o_full, 0);
-    tc_fence_after();
-    __nv_bfloat16* crow = p.C + ((int64_t)b * p.S + qrow) * p.ldc + h * DH;
-#pragma unroll 1
-    for (int c = half * (DH / 2); c < (half + 1) * (DH / 2); c += 16) {
-      float v[16];
-      tmem_ld16(tmem + trow + Cfg::O_COL + c, v);
-      uint32_t pk[8];
+      float l = (l4[0] + l4[1]) + (l4[2] + l4[3]);
+      if (issuer) bulk_wait_read<0>();  // the previous item's O store has left the staging boxes
+      asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
+      sm_x[half][r] = l;
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      l = sm_x[0][r] + sm_x[1][r];
+      const float inv_l = 1.f / l;
+      // ---- epilogue: O row (normalised, bf16) -> this half's DH/2 columns in a swizzled staging
+      // box (P buffer `half`, free once O is complete) -> TMA store to C; then the LSE
+      mbar_wait(o_full, n & 1);
+      tc_fence_after();
+      float v[DH / 2];
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        __nv_bfloat162 h2 = __floats2bfloat162_rn(v[2 * i] * inv_l, v[2 * i + 1] * inv_l);
-        pk[i] = *reinterpret_cast<uint32_t*>(&h2);
+      for (int c = 0; c < DH / 2; c += 32) tmem_ld32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, v + c);
+      tc_fence_before();
+      mbar_arrive_local(o_empty);  // O is in registers: the next item's PV may start
+      // staging: boxes of 64 bf16 columns (128 B rows, 128B swizzle); DH=64: half h -> 32 columns
+      // of box 0 (chunks 4h..4h+3); DH=128: half h -> box h
+      uint8_t* box = sO + (DH == 64 ? 0 : half * (BQ * 128)) + r * 128;
+      const int ch0 = DH == 64 ? half * 4 : 0;
+#pragma unroll
+      for (int u = 0; u < DH / 16; ++u) {
+        uint32_t pk[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          __nv_bfloat162 h2 = __floats2bfloat162_rn(v[8 * u + 2 * t] * inv_l, v[8 * u + 2 * t + 1] * inv_l);
+          pk[t] = *reinterpret_cast<uint32_t*>(&h2);
+        }
+        *reinterpret_cast<uint4*>(box + (((ch0 + u) ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
       }
-      uint4* dst = reinterpret_cast<uint4*>(crow + c);
-      dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-      dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      if (DH == 64) {
+        asm volatile("bar.sync 1, 256;" ::: "memory");  // both halves wrote the box
+        if (half == 0 && issuer) {
+          tma_store_4d(&tmC, sO, 0, qt * BQ, h, b);
+          bulk_commit();
+        }
+      } else {
+        asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");
+        if (issuer) {
+          tma_store_4d(&tmC, sO + half * (BQ * 128), half * 64, qt * BQ, h, b);
+          bulk_commit();
+        }
+      }
+      // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
+      if (half == 0) p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
     }
-    // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
-    if (half == 0) p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
+    if (issuer) bulk_wait_all();
   }
   tc_fence_before();
   __syncthreads();
@@ -317,8 +392,9 @@ struct BwdCfg {
 struct BwdParams {
   int S, H, causal;
   float scale;
-  const float* lse;    // [b, H, S]
-  const float* D;      // [b, H, S]
+  float scale_log2;    // scale * log2(e)
+  const float* lse2;   // [b, H, S]: lse * log2(e)
+  const float* sD;     // [b, H, S]: scale * D
   __nv_bfloat16* dqkv; // [b*S, 3d]: dK, dV columns written here
   __nv_bfloat16* dst;  // [b, H, S(keys), S(queries)]: scale * dS^T
   int d;
@@ -327,7 +403,8 @@ struct BwdParams {
 template <int DH>
 __global__ void __launch_bounds__(THREADS, 1)
     attn_bwd_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-                    const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmdO, BwdParams p) {
+                    const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmdO,
+                    const __grid_constant__ CUtensorMap tmdS, BwdParams p) {
   using Cfg = BwdCfg<DH>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -353,7 +430,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   const int niter = nq - i0;
 
   if (warp == 0 && lane == 0) {
-    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO);
+    prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO); prefetch_tmap(&tmdS);
     mbar_init(kv_full, 1);
     for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
     mbar_init(s_full, 1);
@@ -448,9 +525,11 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int r = qd * 32 + lane;   // key row within the tile
     const int key = k0 + r;
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
-    const float* lse = p.lse + ((int64_t)b * p.H + h) * p.S;
-    const float* Dv = p.D + ((int64_t)b * p.H + h) * p.S;
-    __nv_bfloat16* dst_row = p.dst + (((int64_t)b * p.H + h) * p.S + key) * p.S;
+    const float* lse2 = p.lse2 + ((int64_t)b * p.H + h) * p.S;
+    const float* sDv = p.sD + ((int64_t)b * p.H + h) * p.S;
+    // this half's dS^T atom goes to global by one TMA store (the smem tile is already in the
+    // 128B-swizzled layout of a (64 queries x 128 keys) box); its issuer is lane 0 of quadrant 0
+    const bool issuer = qd == 0 && lane == 0;
     for (int n = 0; n < niter; ++n) {
       const int q0 = (i0 + n) * BQ;
       const int pb = n % Cfg::PB;
@@ -458,45 +537,64 @@ __global__ void __launch_bounds__(THREADS, 1)
       mbar_wait(&p_empty[pb], ((n / Cfg::PB) & 1) ^ 1);
       tc_fence_after();
       const bool diag = p.causal && (i0 + n) == kt;
-      uint8_t* prow = sPS + pb * 2 * Cfg::PS_BYTES + r * 128;
+      if (Cfg::PB == 1) {  // single buffer: the previous tile's dS^T store must have left it
+        if (issuer) bulk_wait_read<0>();
+        asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");
+      }
+      uint8_t* prow = sPS + pb * 2 * Cfg::PS_BYTES + half * (128 * 128) + r * 128;
       uint8_t* drow = prow + Cfg::PS_BYTES;
 #pragma unroll 1
-      for (int c = half * 64; c < half * 64 + 64; c += 16) {
-        float sv[16], dp[16];
-        tmem_ld16(tmem + trow + Cfg::ST_COL + c, sv);
-        tmem_ld16(tmem + trow + Cfg::DP_COL + c, dp);
-        uint32_t pk[8], dk[8];
+      for (int c = 0; c < 64; c += 32) {
+        const int qc = q0 + half * 64 + c;  // first query of this 32-column batch
+        // per-query statistics (same for every thread: L1 broadcast), loaded ahead of the TMEM reads
+        float l2[32], sd[32];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
+          const float4 a4 = __ldg(reinterpret_cast<const float4*>(lse2 + qc) + i);
+          const float4 d4 = __ldg(reinterpret_cast<const float4*>(sDv + qc) + i);
+          l2[4 * i] = a4.x; l2[4 * i + 1] = a4.y; l2[4 * i + 2] = a4.z; l2[4 * i + 3] = a4.w;
+          sd[4 * i] = d4.x; sd[4 * i + 1] = d4.y; sd[4 * i + 2] = d4.z; sd[4 * i + 3] = d4.w;
+        }
+        uint32_t rs[32], rd[32];
+        tmem_ld32_nw(tmem + trow + Cfg::ST_COL + half * 64 + c, rs);
+        tmem_ld32_nw(tmem + trow + Cfg::DP_COL + half * 64 + c, rd);
+        tmem_wait_ld();
+        uint32_t pk[16], dk[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
           float pr[2], dr[2];
 #pragma unroll
           for (int u = 0; u < 2; ++u) {
-            const int q = q0 + c + 2 * i + u;
-            const bool masked = diag && key > q;
-            const float pv = masked ? 0.f : __expf(sv[2 * i + u] * p.scale - __ldg(lse + q));
+            const int e = 2 * i + u;
+            float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, -l2[e]));
+            if (diag && key > qc + e) pv = 0.f;
             pr[u] = pv;
-            dr[u] = p.scale * pv * (dp[2 * i + u] - __ldg(Dv + q));
+            dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, -sd[e]);
           }
           __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
           __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
           pk[i] = *reinterpret_cast<uint32_t*>(&a2);
           dk[i] = *reinterpret_cast<uint32_t*>(&b2);
         }
-        const int atom = c / 64, ch = (c % 64) / 8;
-        uint8_t* pb = prow + atom * (128 * 128);
-        uint8_t* db = drow + atom * (128 * 128);
-        *reinterpret_cast<uint4*>(pb + ((ch ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-        *reinterpret_cast<uint4*>(pb + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-        *reinterpret_cast<uint4*>(db + ((ch ^ (r & 7)) << 4)) = make_uint4(dk[0], dk[1], dk[2], dk[3]);
-        *reinterpret_cast<uint4*>(db + (((ch + 1) ^ (r & 7)) << 4)) = make_uint4(dk[4], dk[5], dk[6], dk[7]);
-        uint4* g = reinterpret_cast<uint4*>(dst_row + q0 + c);
-        g[0] = make_uint4(dk[0], dk[1], dk[2], dk[3]);
-        g[1] = make_uint4(dk[4], dk[5], dk[6], dk[7]);
+        const int ch0 = c / 8;  // 16-byte chunk of the 128-byte row
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int sw = ((ch0 + u) ^ (r & 7)) << 4;
+          *reinterpret_cast<uint4*>(prow + sw) = make_uint4(pk[4 * u], pk[4 * u + 1], pk[4 * u + 2], pk[4 * u + 3]);
+          *reinterpret_cast<uint4*>(drow + sw) = make_uint4(dk[4 * u], dk[4 * u + 1], dk[4 * u + 2], dk[4 * u + 3]);
+        }
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       tc_fence_before();
+      if (issuer) bulk_wait_read<0>();  // the previous tile's dS^T store has left shared memory
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive_local(&p_full[pb]);
+      asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");  // the half's 128 rows are written
+      if (issuer) {
+        tma_store_4d(&tmdS, sPS + pb * 2 * Cfg::PS_BYTES + Cfg::PS_BYTES + half * (128 * 128), q0 + half * 64, k0, h, b);
+        bulk_commit();
+      }
     }
+    if (issuer) bulk_wait_all();
     // epilogue: dV_j, dK_j rows -> dQKV (bf16)
     mbar_wait(kd_full, 0);
     tc_fence_after();
@@ -529,29 +627,35 @@ __global__ void __launch_bounds__(THREADS, 1)
   }
 }
 
-// D[b, h, q] = sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e]   (one thread per (token, head))
-__global__ void attn_bwd_prep(int64_t ntok, int S, int H, int dh, const __nv_bfloat16* __restrict__ dO,
-                              const __nv_bfloat16* __restrict__ O, float* __restrict__ D) {
-  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= ntok * H) return;
-  const int64_t tok = t / H;
-  const int h = (int)(t % H);
+// sD[b, h, q] = scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = lse * log2(e)
+// (one thread per (token, head)): the per-query terms of dS = P (dP - D) in the forms the
+// backward's FFMAs take.
+__global__ void attn_bwd_prep(int64_t ntok, int S, int H, int dh, float scale, const __nv_bfloat16* __restrict__ dO,
+                              const __nv_bfloat16* __restrict__ O, const float* __restrict__ lse, float* __restrict__ sD,
+                              float* __restrict__ lse2) {
+  // thread i = ((b * H + h) * S + q): consecutive threads walk q, so the [b, H, S] statistics are
+  // read and written coalesced; each thread reads its (token, head) row of dO and O (dh * 2 bytes)
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= ntok * H) return;
+  const int64_t q = i % S, bh = i / S;
+  const int h = (int)(bh % H);
+  const int64_t tok = (bh / H) * S + q;
   const int d = H * dh;
   const uint4* a = reinterpret_cast<const uint4*>(dO + tok * d + h * dh);
   const uint4* o = reinterpret_cast<const uint4*>(O + tok * d + h * dh);
   float s = 0.f;
-  for (int i = 0; i < dh / 8; ++i) {
-    uint4 x = a[i], y = o[i];
+  for (int k8 = 0; k8 < dh / 8; ++k8) {
+    uint4 x = a[k8], y = o[k8];
     const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&x);
     const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&y);
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
+      const float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
       s += fx.x * fy.x + fx.y * fy.y;
     }
   }
-  const int64_t bb = tok / S, q = tok % S;
-  D[(bb * H + h) * S + q] = s;
+  sD[i] = scale * s;
+  lse2[i] = lse[i] * 1.4426950408889634f;
 }
 }  // namespace attn
 
@@ -561,29 +665,36 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   using namespace attn;
   if (S % BQ != 0 || (dh != 64 && dh != 128)) return false;
   const int d = H * dh;
-  CUtensorMap mq, mk, mv;
+  CUtensorMap mq, mk, mv, mc;
   // Q, K: K-major operands (inner = dh, rows = S, z0 = head, z1 = sequence); V: MN-major (inner = dh)
   tcx::make_map_4d(&mq, QKV, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BQ);
   tcx::make_map_4d(&mk, static_cast<const __nv_bfloat16*>(QKV) + d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
   tcx::make_map_4d(&mv, static_cast<const __nv_bfloat16*>(QKV) + 2 * d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64,
                    64);
+  // C [b*S][d], head h in columns h*dh..: stored in (64 columns x 128 rows) boxes
+  tcx::make_map_4d(&mc, C, dh, S, H, b, d, dh, (int64_t)S * d, 64, BQ);
   FwdParams p;
-  p.S = S; p.H = H; p.causal = causal;
+  p.S = S; p.H = H; p.B = (int)b; p.causal = causal;
   p.scale = 1.0f / std::sqrt((float)dh);
   p.scale_log2 = p.scale * 1.4426950408889634f;
-  p.C = static_cast<__nv_bfloat16*>(C);
   p.lse = lse;
-  p.ldc = d;
-  dim3 grid((unsigned)(S / BQ), (unsigned)H, (unsigned)b);
+  static int num_sms = 0;
+  if (!num_sms) {
+    int dev = 0;
+    HM_CUDA(cudaGetDevice(&dev));
+    HM_CUDA(cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const int64_t items = (int64_t)(S / BQ) * H * b;
+  dim3 grid((unsigned)std::min<int64_t>(items, num_sms));  // persistent
   const int e0 = g_prof.begin(st);
   if (dh == 64) {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<64>::SMEM)); set = true; }
-    attn_fwd_kernel<64><<<grid, THREADS, FwdCfg<64>::SMEM, st>>>(mq, mk, mv, p);
+    attn_fwd_kernel<64><<<grid, THREADS, FwdCfg<64>::SMEM, st>>>(mq, mk, mv, mc, p);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<128>::SMEM)); set = true; }
-    attn_fwd_kernel<128><<<grid, THREADS, FwdCfg<128>::SMEM, st>>>(mq, mk, mv, p);
+    attn_fwd_kernel<128><<<grid, THREADS, FwdCfg<128>::SMEM, st>>>(mq, mk, mv, mc, p);
   }
   check_launch("attn_fwd_kernel");
   // algorithmic FLOPs of the attention contractions (QK^T and PV, causal or not)
@@ -593,7 +704,7 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
 
 
 size_t attention_bwd_scratch_bytes(int64_t b, int S, int H) {
-  return align_up((uint64_t)b * H * S * S * 2, 256) + align_up((uint64_t)b * H * S * 4, 256);
+  return align_up((uint64_t)b * H * S * S * 2, 256) + 2 * align_up((uint64_t)b * H * S * 4, 256);
 }
 
 // Fused attention backward: dQKV (bf16 [b*S, 3d]) from QKV, O (= C), dO (= dC), lse.
@@ -604,23 +715,28 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   const int d = H * dh;
   uint8_t* sc = static_cast<uint8_t*>(scratch);
   __nv_bfloat16* dst = reinterpret_cast<__nv_bfloat16*>(sc);
-  float* D = reinterpret_cast<float*>(sc + align_up((uint64_t)b * H * S * S * 2, 256));
+  float* sD = reinterpret_cast<float*>(sc + align_up((uint64_t)b * H * S * S * 2, 256));
+  float* lse2 = sD + align_up((uint64_t)b * H * S * 4, 256) / 4;
+  const float scale = 1.0f / std::sqrt((float)dh);
   const int e0 = g_prof.begin(st);
   const int64_t n = b * S * H;
-  attn_bwd_prep<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(b * S, S, H, dh, static_cast<const __nv_bfloat16*>(dO),
-                                                           static_cast<const __nv_bfloat16*>(O), D);
+  attn_bwd_prep<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
+                                                           static_cast<const __nv_bfloat16*>(O), lse, sD, lse2);
   check_launch("attn_bwd_prep");
   if (causal) HM_CUDA(cudaMemsetAsync(dst, 0, (size_t)b * H * S * S * 2, st));  // key tiles never visited by a query tile
-  CUtensorMap mq, mk, mv, mo;
+  CUtensorMap mq, mk, mv, mo, mds;
   const __nv_bfloat16* q = static_cast<const __nv_bfloat16*>(QKV);
+  // dS^T [b][H][S keys][S queries]: stored from the kernel's swizzled (64 queries x 128 keys) atoms
+  tcx::make_map_4d(&mds, dst, S, S, H, b, S, (int64_t)S * S, (int64_t)H * S * S, 64, BKV);
   tcx::make_map_4d(&mq, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BQ);
   tcx::make_map_4d(&mk, q + d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
   tcx::make_map_4d(&mv, q + 2 * d, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BKV);
   tcx::make_map_4d(&mo, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BQ);
   BwdParams p;
   p.S = S; p.H = H; p.causal = causal;
-  p.scale = 1.0f / std::sqrt((float)dh);
-  p.lse = lse; p.D = D;
+  p.scale = scale;
+  p.scale_log2 = scale * 1.4426950408889634f;
+  p.lse2 = lse2; p.sD = sD;
   p.dqkv = static_cast<__nv_bfloat16*>(dQKV);
   p.dst = dst;
   p.d = d;
@@ -628,11 +744,11 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   if (dh == 64) {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<64>::SMEM)); set = true; }
-    attn_bwd_kernel<64><<<grid, THREADS, BwdCfg<64>::SMEM, st>>>(mq, mk, mv, mo, p);
+    attn_bwd_kernel<64><<<grid, THREADS, BwdCfg<64>::SMEM, st>>>(mq, mk, mv, mo, mds, p);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }
-    attn_bwd_kernel<128><<<grid, THREADS, BwdCfg<128>::SMEM, st>>>(mq, mk, mv, mo, p);
+    attn_bwd_kernel<128><<<grid, THREADS, BwdCfg<128>::SMEM, st>>>(mq, mk, mv, mo, mds, p);
   }
   check_launch("attn_bwd_kernel");
   g_prof.end(PROF_GEMM, e0, st, 8.0 * b * H * (double)S * S * dh);  // S^T, dP^T, dV, dK contractions

@@ -104,6 +104,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--only", default=None)
+    ap.add_argument("--graph", action="store_true", help="time a CUDA-graph replay of the reps")
     ap.add_argument("--sweep", action="store_true", help="K sweep of the QKV / FC1 shapes (epilogue vs mainloop)")
     args = ap.parse_args()
     sh, keep = sweep() if args.sweep else shapes()
@@ -116,10 +117,22 @@ def main():
             H.hk("hk_gemm", C.byref(a), C.c_void_p(st.cuda_stream))
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        for _ in range(args.reps):
-            H.hk("hk_gemm", C.byref(a), C.c_void_p(st.cuda_stream))
-        e1.record()
+        if args.graph:  # replay a captured sequence: no host launch cost between kernels (as in the step)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                cs = torch.cuda.current_stream()
+                for _ in range(args.reps):
+                    H.hk("hk_gemm", C.byref(a), C.c_void_p(cs.cuda_stream))
+            g.replay()
+            torch.cuda.synchronize()
+            e0.record()
+            g.replay()
+            e1.record()
+        else:
+            e0.record()
+            for _ in range(args.reps):
+                H.hk("hk_gemm", C.byref(a), C.c_void_p(st.cuda_stream))
+            e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / args.reps
         total_f += fl; total_t += ms
