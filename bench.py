@@ -33,6 +33,9 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+# per-launch DRAM traffic of the roofline kernel class, from the committed ncu launch list of the
+# same step (tools/traffic_summary.py); ncu replays cold, so this is the no-L2-reuse upper end
+TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2.json")}
 FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
 
 WORKLOADS = {
@@ -298,6 +301,16 @@ def main():
     gemm_tflops = g["work"] / g["seconds"] / 1e12 if g["seconds"] else 0.0
     gemm_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
     adam = prof["adam"]
+    traffic = traffic_src = None
+    try:
+        with open(TRAFFIC_FILES[args.workload]) as f:
+            tj = json.load(f)
+        traffic = tj["classes"]["gemm"]["dram_bytes_per_launch"]
+        traffic_src = (f"{os.path.relpath(TRAFFIC_FILES[args.workload], ROOT)}: ncu dram__bytes_read.sum + "
+                       f"dram__bytes_write.sum averaged over the {tj['classes']['gemm']['launches']} tensor-core "
+                       f"launches of the profiled step (cold-cache replay)")
+    except (KeyError, OSError, ValueError):
+        pass
     line = {
         "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
@@ -308,7 +321,9 @@ def main():
                    "l2": "inputs and per-step swap traffic (tens of GB) far larger than the 126 MB L2; no flush"},
         "roofline": {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05, all GEMM launches of the step)",
                      "achieved": gemm_tflops, "peak": gemm_peak, "unit": "TFLOP/s",
-                     "frac": gemm_tflops / gemm_peak if gemm_peak else None, "traffic": None,
+                     "frac": gemm_tflops / gemm_peak if gemm_peak else None, "traffic": traffic,
+                     "traffic_unit": "bytes per launch", "traffic_source": traffic_src,
+                     "algorithmic_flops_per_launch": g["work"] / g["launches"] if g["launches"] else None,
                      "peak_source": f"{peak_src} bf16_tflops_sustained (kernel timed inside a long step)",
                      "launches_per_step": g["launches"] / args.steps,
                      "flops_per_step": g["work"] / args.steps},

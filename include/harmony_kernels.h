@@ -30,7 +30,9 @@ typedef enum {
   HK_EPI_ACC_F32 = 3,     /* C(f32) = (accumulate ? C : 0) + alpha*acc  (wgrad, dW += .)   */
   HK_EPI_BIAS_ACT = 4,    /* C(T) = z = acc + bias[n];  aux_out(T) = act(z)   (FC1: H, G)  */
   HK_EPI_ACT_BWD = 5,     /* C(T) = acc * act'(aux_T[m][n])                  (dG -> dH)   */
-  HK_EPI_BIAS_ACT_F32 = 6 /* C(T) = z = acc + bias[n]; aux_out(f32) = act(z)   (MLP layer)  */
+  HK_EPI_BIAS_ACT_F32 = 6, /* C(T) = z = acc + bias[n]; aux_out(f32) = act(z)  (MLP layer)  */
+  HK_EPI_ACT_T = 7        /* C(T) = act(RN_T(acc + bias[n]))   (FC1 when only G is needed;
+                             bit-identical to the aux_out of HK_EPI_BIAS_ACT)             */
 } hk_epilogue;
 
 /* C[z0,z1][m][n] = epilogue( sum_k A[z0,z1](m,k) * B[z0,z1](n,k) )

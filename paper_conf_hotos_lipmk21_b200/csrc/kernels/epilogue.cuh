@@ -45,6 +45,11 @@ __device__ __forceinline__ void epi_scalar(const EpiParams& e, int64_t off, int 
       reinterpret_cast<T*>(e.aux_out)[off] = from_f32<T>(act_T<T>(e.act, to_f32(zt)));
       break;
     }
+    case HK_EPI_ACT_T: {
+      const T zt = from_f32<T>(acc + b);
+      reinterpret_cast<T*>(e.C)[off] = from_f32<T>(act_T<T>(e.act, to_f32(zt)));
+      break;
+    }
     case HK_EPI_ACT_BWD: {
       float z = to_f32(reinterpret_cast<const T*>(e.aux)[off]);
       reinterpret_cast<T*>(e.C)[off] = from_f32<T>(acc * act_grad_T<T>(e.act, z));

@@ -263,7 +263,8 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
   const bool two = e.epi == HK_EPI_BIAS_ACT;
   const int nbox = n_end > n_beg ? (n_end - n_beg + CPB - 1) / CPB : 0;
   const bool has_bias = e.bias != nullptr && (e.epi == HK_EPI_STORE_T || e.epi == HK_EPI_BIAS_ACT ||
-                                              e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32);
+                                              e.epi == HK_EPI_ACT_T || e.epi == HK_EPI_STORE_F32 ||
+                                              e.epi == HK_EPI_RESID_F32);
   if (kind && nbox > 0 && lane == 0) {
     const int b = w.j & 1;
     bulk_wait_read<1>();  // the store two boxes back has left this box
@@ -365,6 +366,13 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
 #pragma unroll
             for (int t = 0; t < 4; ++t)
               o[t] = pack_bf16(e.alpha * x[2 * t] + bb[2 * t], e.alpha * x[2 * t + 1] + bb[2 * t + 1]);
+          } else if (e.epi == HK_EPI_ACT_T) {  // G = act(H as it would be stored), H not written
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              const uint32_t hz = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
+              const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hz));
+              o[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
+            }
           } else {  // BIAS_ACT: H = acc + b (bf16), G = act(H as stored) into the second box
             uint32_t g[4];
 #pragma unroll
@@ -936,7 +944,10 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
     return v ? atoi(v) : 1;
   }();
   const int64_t nz = (int64_t)a.nz0 * a.nz1;
-  if (mode && a.M >= 256 && a.N >= 256) {
+  // CTA-pair tiles unless they would leave most pairs idle (e.g. the d x d weight gradient: 16 pair
+  // tiles on 74 pairs) — then 128 x 128 single-CTA tiles spread the work over 4x more SMs
+  const int64_t pair_tiles = ceil_div(a.M, 256) * ceil_div(a.N, 256) * nz;
+  if (mode && a.M >= 256 && a.N >= 256 && pair_tiles >= 37) {
     // CTA-pair 256 x 256 tiles (measured best for every cfg2 shape, tools/gemm_bench.py);
     // HARMONY_GEMM_2SM=3 selects 256 x 128 pair tiles, 0 the single-CTA kernel
     if (mode == 3) tc::launch_tc2<128, 6>(a, e, st);

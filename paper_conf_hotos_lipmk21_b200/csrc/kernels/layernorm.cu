@@ -170,22 +170,31 @@ __global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const fl
   }
 }
 
-// fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 8 warps per block
+// fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 8 warps per block,
+// blockIdx.y selects which of the np interleaved partial sets (dgamma, dbeta[, sum dX]) -> one launch
+struct ColOuts {
+  float* out[3];
+  int acc[3];
+};
 __global__ void __launch_bounds__(256) colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial,
-                                                         int64_t stride, float* __restrict__ out, int accumulate) {
+                                                         int64_t stride, ColOuts outs) {
   __shared__ float sh[8][33];
   const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
+  const float* pp = partial + (int64_t)blockIdx.y * n;
   float s = 0.f;
-  if (c < n)
-    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];
+  if (c < n) {
+#pragma unroll 8
+    for (int j = g; j < nchunks; j += 8) s += pp[(int64_t)j * stride + c];  // loads hoisted, adds in order
+  }
   sh[g][cl] = s;
   __syncthreads();
   if (g == 0 && c < n) {
     float t = sh[0][cl];
 #pragma unroll
     for (int k = 1; k < 8; ++k) t += sh[k][cl];
-    out[c] = accumulate ? out[c] + t : t;
+    float* out = outs.out[blockIdx.y];
+    out[c] = outs.acc[blockIdx.y] ? out[c] + t : t;
   }
 }
 
@@ -255,15 +264,10 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
 #undef HM_LNB_ALL
 #undef HM_LNB
   check_launch("layernorm_bwd_vec");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch, np * (int64_t)d, dg, accumulate);
-  check_launch("colreduce(dgamma)");
-  colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + d, np * (int64_t)d, db, accumulate);
-  check_launch("colreduce(dbeta)");
-  if (dsum) {
-    colreduce2_kernel<<<(unsigned)ceil_div(d, 32), 256, 0, st>>>(nblk, d, scratch + 2 * d, np * (int64_t)d, dsum,
-                                                                dsum_acc);
-    check_launch("colreduce(sum dX)");
-  }
+  ColOuts outs{{dg, db, dsum}, {accumulate, accumulate, dsum_acc}};
+  colreduce2_kernel<<<dim3((unsigned)ceil_div(d, 32), (unsigned)np), 256, 0, st>>>(nblk, d, scratch, np * (int64_t)d,
+                                                                                 outs);
+  check_launch("colreduce(dgamma, dbeta[, sum dX])");
   return true;
 }
 

@@ -113,8 +113,10 @@ __global__ void __launch_bounds__(256) colreduce_kernel(int nchunks, int n, cons
   const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
   float s = 0.f;
-  if (c < n)
-    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];
+  if (c < n) {
+#pragma unroll 8
+    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];  // loads hoisted, adds in order
+  }
   sh[g][cl] = s;
   __syncthreads();
   if (g == 0 && c < n) {
@@ -131,7 +133,9 @@ static void colreduce(int nchunks, int n, const float* partial, int64_t stride, 
 }
 
 // ------------------------------------------------------------------------------------- column sums
-constexpr int CS_ROWS = 64;
+// partial[chunk][c] = sum of rows [chunk*CS_ROWS, ...) of column c, rows in increasing order; each
+// thread owns VEC adjacent columns (16-byte loads) and keeps CS_ROWS independent loads in flight.
+constexpr int CS_ROWS = 32;
 template <typename Tin>
 __global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict__ X, int64_t ld,
                                       float* __restrict__ partial) {
@@ -141,6 +145,27 @@ __global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict
   float s = 0.f;
   for (int64_t r = r0; r < r1; ++r) s += to_f32(X[r * ld + c]);
   partial[(int64_t)blockIdx.y * n + c] = s;
+}
+template <typename Tin>
+__global__ void __launch_bounds__(128) colsum_partial_vec_kernel(int64_t rows, int n, const Tin* __restrict__ X,
+                                                                 int64_t ld, float* __restrict__ partial) {
+  constexpr int VEC = 16 / sizeof(Tin);
+  const int c0 = (blockIdx.x * blockDim.x + threadIdx.x) * VEC;
+  if (c0 >= n) return;
+  const int64_t r0 = (int64_t)blockIdx.y * CS_ROWS, r1 = min(rows, r0 + CS_ROWS);
+  float s[VEC];
+#pragma unroll
+  for (int v = 0; v < VEC; ++v) s[v] = 0.f;
+#pragma unroll 8
+  for (int64_t r = r0; r < r1; ++r) {
+    const uint4 u = __ldg(reinterpret_cast<const uint4*>(X + r * ld + c0));
+    const Tin* e = reinterpret_cast<const Tin*>(&u);
+#pragma unroll
+    for (int v = 0; v < VEC; ++v) s[v] += to_f32(e[v]);
+  }
+  float* p = partial + (int64_t)blockIdx.y * n + c0;
+#pragma unroll
+  for (int v = 0; v < VEC; v += 4) *reinterpret_cast<float4*>(p + v) = make_float4(s[v], s[v + 1], s[v + 2], s[v + 3]);
 }
 
 // ------------------------------------------------------------------------------------- softmax
@@ -365,9 +390,16 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
     if (!accumulate) HM_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * n, st));
     return;
   }
-  dim3 grid((unsigned)ceil_div(n, 128), (unsigned)nch);
+  const int vec = 16 / (in_dtype ? 2 : 4);
+  const bool vok = n % vec == 0 && ld % vec == 0 && (reinterpret_cast<uintptr_t>(X) & 15) == 0;
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+  if (vok) {
+    dim3 grid((unsigned)ceil_div(n / vec, 128), (unsigned)nch);
+    HM_DISPATCH_T(in_dtype, (colsum_partial_vec_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+  } else {
+    dim3 grid((unsigned)ceil_div(n, 128), (unsigned)nch);
+    HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+  }
   check_launch("colsum_partial");
   colreduce(nch, n, scratch, n, out, accumulate, st);
   g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (in_dtype ? 2 : 4));

@@ -182,7 +182,7 @@ static hk_gemm_args lin_wgrad(const LayerGeom& g, int64_t rows, int n, int k, co
 
 // ------------------------------------------------------------------------------------------------ forward
 static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws,
-                     void* stv) {
+                     void* stv, bool stash_x = true) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   if (d.kind == HARMONY_LAYER_MLP) {
@@ -216,8 +216,8 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   } else {
     U = ws + bump(wc, R * D * ts); U2 = ws + bump(wc, R * D * ts); G = ws + bump(wc, R * 4 * D * ts);
   }
-  // stash the layer input (Fig. 5(a) "Stashed X")
-  copy_f32(R * D, X, Xs, st);
+  // stash the layer input (Fig. 5(a) "Stashed X"); under block recompute the caller keeps X itself
+  if (stash_x) copy_f32(R * D, X, Xs, st);
   // U = LN1(X)
   layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st);
   // QKV = U W_qkv + b_qkv
@@ -262,10 +262,16 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   }
   // U2 = LN2(X2)
   layernorm_fwd(g.dtype, R, D, X2, wseg(g, W, P_LN2_G), wseg(g, W, P_LN2_B), U2, mean2, rstd2, st);
-  // H = U2 W_fc1 + b_fc1 ; G = GeLU(H)
+  // H = U2 W_fc1 + b_fc1 ; G = GeLU(H).  The block-recompute forward (stash_x false, output wanted)
+  // needs only G: H is recomputed in the backward, so it is not written (identical G bits)
   {
     hk_gemm_args a = lin_fwd(g, R, 4 * D, D, U2, wseg(g, W, P_WFC1));
-    a.C = Hh; a.epilogue = HK_EPI_BIAS_ACT; a.act = HARMONY_ACT_GELU_TANH; a.bias = wseg(g, W, P_BFC1); a.aux_out = G;
+    a.act = HARMONY_ACT_GELU_TANH; a.bias = wseg(g, W, P_BFC1);
+    if (!stash_x && Y && g.dtype == 1) {
+      a.C = G; a.epilogue = HK_EPI_ACT_T;
+    } else {
+      a.C = Hh; a.epilogue = HK_EPI_BIAS_ACT; a.aux_out = G;
+    }
     gemm(a, st);
   }
   // Y = X2 + G W_fc2 + b_fc2   (skipped when Y == nullptr: the backward's recompute needs only
@@ -279,7 +285,7 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
 
 // ------------------------------------------------------------------------------------------------ backward
 static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
-                     int first, uint8_t* ws, void* stv) {
+                     int first, uint8_t* ws, void* stv, const float* Xs_in = nullptr) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   const int acc = first ? 0 : 1;
@@ -303,7 +309,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   const int D = g.d, S = g.S, H = g.h, dh = g.dh, b = g.b;
   const size_t ts = g.ts;
   const int dt = g.dtype;
-  const float* Xs = reinterpret_cast<const float*>(stash + g.st.X);
+  const float* Xs = Xs_in ? Xs_in : reinterpret_cast<const float*>(stash + g.st.X);
   const float* mean1 = reinterpret_cast<const float*>(stash + g.st.mean1);
   const float* rstd1 = reinterpret_cast<const float*>(stash + g.st.rstd1);
   const uint8_t* QKV = stash + g.st.QKV;
@@ -477,7 +483,7 @@ void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
   uint8_t* rest = ws + align_up(c.st.total, 256);
-  fwd_core(c, W, X, Y, full, rest, st);
+  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false);
   copy_f32(g.rows * g.d, X, reinterpret_cast<float*>(stash + g.st.X), static_cast<cudaStream_t>(st));
 }
 
@@ -487,9 +493,11 @@ void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const fl
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
   uint8_t* rest = ws + align_up(c.st.total, 256);
-  // recompute the block's forward from its stashed input: the same kernels, hence the same bits
-  fwd_core(c, W, reinterpret_cast<const float*>(stash + g.st.X), nullptr, full, rest, st);
-  bwd_core(c, W, full, dY, dX, dW, first, rest, st);
+  // recompute the block's forward from its stashed input: the same kernels, hence the same bits;
+  // the LN1 backward reads the stashed input in place
+  const float* Xst = reinterpret_cast<const float*>(stash + g.st.X);
+  fwd_core(c, W, Xst, nullptr, full, rest, st, /*stash_x=*/false);
+  bwd_core(c, W, full, dY, dX, dW, first, rest, st, Xst);
 }
 
 }  // namespace hm

@@ -23,7 +23,7 @@ HARMONY_ACT_NONE, HARMONY_ACT_RELU, HARMONY_ACT_GELU_TANH = 0, 1, 2
 HARMONY_PARAM, HARMONY_GRAD, HARMONY_ADAM_M, HARMONY_ADAM_V = 0, 1, 2, 3
 HARMONY_SCHED_HARMONY_DP, HARMONY_SCHED_PER_GPU_VIRT = 0, 1
 HK_EPI_STORE_T, HK_EPI_STORE_F32, HK_EPI_RESID_F32, HK_EPI_ACC_F32 = 0, 1, 2, 3
-HK_EPI_BIAS_ACT, HK_EPI_ACT_BWD, HK_EPI_BIAS_ACT_F32 = 4, 5, 6
+HK_EPI_BIAS_ACT, HK_EPI_ACT_BWD, HK_EPI_BIAS_ACT_F32, HK_EPI_ACT_T = 4, 5, 6, 7
 
 
 class harmony_config(C.Structure):

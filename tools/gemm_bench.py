@@ -106,6 +106,7 @@ def main():
     ap.add_argument("--only", default=None)
     ap.add_argument("--graph", action="store_true", help="time a CUDA-graph replay of the reps")
     ap.add_argument("--sweep", action="store_true", help="K sweep of the QKV / FC1 shapes (epilogue vs mainloop)")
+    ap.add_argument("--cublas", action="store_true", help="also time torch.matmul (cuBLAS) on the same shape/majors")
     args = ap.parse_args()
     sh, keep = sweep() if args.sweep else shapes()
     st = torch.cuda.current_stream()
@@ -136,8 +137,25 @@ def main():
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / args.reps
         total_f += fl; total_t += ms
-        print(json.dumps({"gemm": name, "M": a.M, "N": a.N, "K": a.K, "batch": a.nz0 * a.nz1, "us": ms * 1e3,
-                          "tflops": fl / (ms * 1e-3) / 1e12}))
+        rec = {"gemm": name, "M": a.M, "N": a.N, "K": a.K, "batch": a.nz0 * a.nz1, "us": ms * 1e3,
+               "tflops": fl / (ms * 1e-3) / 1e12}
+        if args.cublas and a.nz0 * a.nz1 == 1:
+            bf = torch.bfloat16
+            A_ = (torch.randn(a.K, a.M, device="cuda").to(bf).t() if a.a_mn_major else torch.randn(a.M, a.K, device="cuda").to(bf))
+            B_ = (torch.randn(a.K, a.N, device="cuda").to(bf) if a.b_mn_major else torch.randn(a.N, a.K, device="cuda").to(bf).t())
+            C_ = torch.empty(a.M, a.N, device="cuda", dtype=bf)
+            for _ in range(3):
+                torch.matmul(A_, B_, out=C_)
+            torch.cuda.synchronize()
+            e0.record()
+            for _ in range(args.reps):
+                torch.matmul(A_, B_, out=C_)
+            e1.record()
+            torch.cuda.synchronize()
+            cms = e0.elapsed_time(e1) / args.reps
+            rec["cublas_us"] = cms * 1e3
+            rec["cublas_tflops"] = fl / (cms * 1e-3) / 1e12
+        print(json.dumps(rec))
     print(json.dumps({"gemm": "ALL", "tflops": total_f / (total_t * 1e-3) / 1e12}))
 
 
