@@ -113,32 +113,38 @@ __global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const fl
   for (int i = warp; i < LNV_ROWS; i += 8) {
     const int64_t row = r0 + i;
     if (row >= rows) break;
-    const float mu = mean[row], rs = rstd[row];
     const float* x = X + row * d;
     const float* du = dU + row * d;
-    float4 xv[VPT], dv[VPT];
+    const float* dr = dres ? dres + row * d : nullptr;
+    // all of the row's global loads first (x, dU and the residual gradient), so the warp waits for
+    // one memory round trip per row; the shared-memory partials are touched only afterwards
+    // (wide rows, VPT > 8: the residual gradient is loaded in the second pass, to stay in registers)
+    constexpr bool PRE = VPT <= 8;
+    float4 xv[VPT], dv[VPT], rv[PRE ? VPT : 1];
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int c = (j * 32 + lane) * 4;
+      const bool in = c < d;
+      xv[j] = in ? __ldg(reinterpret_cast<const float4*>(x + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      dv[j] = in ? __ldg(reinterpret_cast<const float4*>(du + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      if (PRE) rv[PRE ? j : 0] = in && dr ? __ldg(reinterpret_cast<const float4*>(dr + c)) : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    const float mu = mean[row], rs = rstd[row];
     float s1 = 0.f, s2 = 0.f;
 #pragma unroll
     for (int j = 0; j < VPT; ++j) {
       const int c = (j * 32 + lane) * 4;
       if (c < d) {
-        xv[j] = *reinterpret_cast<const float4*>(x + c);
-        dv[j] = *reinterpret_cast<const float4*>(du + c);
         const float4 gv = ld4<T>(g + c);  // gamma re-read per row (L1-resident): keeps registers < 128
         const float4 xh = make_float4((xv[j].x - mu) * rs, (xv[j].y - mu) * rs, (xv[j].z - mu) * rs, (xv[j].w - mu) * rs);
         const float4 dx = make_float4(dv[j].x * gv.x, dv[j].y * gv.y, dv[j].z * gv.z, dv[j].w * gv.w);
         s1 += (dx.x + dx.y) + (dx.z + dx.w);
         s2 += (dx.x * xh.x + dx.y * xh.y) + (dx.z * xh.z + dx.w * xh.w);
-        float4 a = *reinterpret_cast<float4*>(sg + c), bq = *reinterpret_cast<float4*>(sb + c);
-        *reinterpret_cast<float4*>(sg + c) =
-            make_float4(a.x + dv[j].x * xh.x, a.y + dv[j].y * xh.y, a.z + dv[j].z * xh.z, a.w + dv[j].w * xh.w);
-        *reinterpret_cast<float4*>(sb + c) = make_float4(bq.x + dv[j].x, bq.y + dv[j].y, bq.z + dv[j].z, bq.w + dv[j].w);
       }
     }
     s1 = wsum(s1) / (float)d;
     s2 = wsum(s2) / (float)d;
     float* dxr = dX + row * d;
-    const float* dr = dres ? dres + row * d : nullptr;
 #pragma unroll
     for (int j = 0; j < VPT; ++j) {
       const int c = (j * 32 + lane) * 4;
@@ -148,14 +154,18 @@ __global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const fl
         float4 o = make_float4(rs * (dv[j].x * gv.x - s1 - xh.x * s2), rs * (dv[j].y * gv.y - s1 - xh.y * s2),
                                rs * (dv[j].z * gv.z - s1 - xh.z * s2), rs * (dv[j].w * gv.w - s1 - xh.w * s2));
         if (dr) {
-          float4 rr = *reinterpret_cast<const float4*>(dr + c);
+          const float4 rr = PRE ? rv[PRE ? j : 0] : __ldg(reinterpret_cast<const float4*>(dr + c));
           o.x = rr.x + o.x; o.y = rr.y + o.y; o.z = rr.z + o.z; o.w = rr.w + o.w;
         }
         *reinterpret_cast<float4*>(dxr + c) = o;
         if (dXt) st4<T>(dXt + row * d + c, o);  // the bf16 GEMM operand copy of dX
+        float4 a = *reinterpret_cast<float4*>(sg + c), bq = *reinterpret_cast<float4*>(sb + c);
+        *reinterpret_cast<float4*>(sg + c) =
+            make_float4(a.x + dv[j].x * xh.x, a.y + dv[j].y * xh.y, a.z + dv[j].z * xh.z, a.w + dv[j].w * xh.w);
+        *reinterpret_cast<float4*>(sb + c) = make_float4(bq.x + dv[j].x, bq.y + dv[j].y, bq.z + dv[j].z, bq.w + dv[j].w);
         if (ss) {
-          float4 a = *reinterpret_cast<float4*>(ss + c);
-          *reinterpret_cast<float4*>(ss + c) = make_float4(a.x + o.x, a.y + o.y, a.z + o.z, a.w + o.w);
+          float4 q = *reinterpret_cast<float4*>(ss + c);
+          *reinterpret_cast<float4*>(ss + c) = make_float4(q.x + o.x, q.y + o.y, q.z + o.z, q.w + o.w);
         }
       }
     }
@@ -170,29 +180,29 @@ __global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const fl
   }
 }
 
-// fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 8 warps per block,
+// fixed-order tree column reduction (as colreduce_kernel in ops.cu): 32 columns x 32 warps per block,
 // blockIdx.y selects which of the np interleaved partial sets (dgamma, dbeta[, sum dX]) -> one launch
 struct ColOuts {
   float* out[3];
   int acc[3];
 };
-__global__ void __launch_bounds__(256) colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial,
-                                                         int64_t stride, ColOuts outs) {
-  __shared__ float sh[8][33];
+__global__ void __launch_bounds__(1024) colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial,
+                                                          int64_t stride, ColOuts outs) {
+  __shared__ float sh[32][33];
   const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
   const float* pp = partial + (int64_t)blockIdx.y * n;
   float s = 0.f;
   if (c < n) {
 #pragma unroll 8
-    for (int j = g; j < nchunks; j += 8) s += pp[(int64_t)j * stride + c];  // loads hoisted, adds in order
+    for (int j = g; j < nchunks; j += 32) s += pp[(int64_t)j * stride + c];  // loads hoisted, adds in order
   }
   sh[g][cl] = s;
   __syncthreads();
   if (g == 0 && c < n) {
     float t = sh[0][cl];
 #pragma unroll
-    for (int k = 1; k < 8; ++k) t += sh[k][cl];
+    for (int k = 1; k < 32; ++k) t += sh[k][cl];
     float* out = outs.out[blockIdx.y];
     out[c] = outs.acc[blockIdx.y] ? out[c] + t : t;
   }
@@ -265,7 +275,7 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
 #undef HM_LNB
   check_launch("layernorm_bwd_vec");
   ColOuts outs{{dg, db, dsum}, {accumulate, accumulate, dsum_acc}};
-  colreduce2_kernel<<<dim3((unsigned)ceil_div(d, 32), (unsigned)np), 256, 0, st>>>(nblk, d, scratch, np * (int64_t)d,
+  colreduce2_kernel<<<dim3((unsigned)ceil_div(d, 32), (unsigned)np), 1024, 0, st>>>(nblk, d, scratch, np * (int64_t)d,
                                                                                  outs);
   check_launch("colreduce(dgamma, dbeta[, sum dX])");
   return true;

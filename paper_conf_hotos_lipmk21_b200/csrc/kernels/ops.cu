@@ -104,38 +104,40 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(int64_t rows, int d,
   }
 }
 
-// out[c] (+)= sum over chunks of partial[j][c] (row stride `stride`): 32 columns per block, 8 warps
-// each summing every 8th chunk, then the 8 warp sums in warp order — a fixed tree (deterministic),
-// coalesced along the columns and 8x more memory-level parallelism than one thread per column.
-__global__ void __launch_bounds__(256) colreduce_kernel(int nchunks, int n, const float* __restrict__ partial,
-                                                        int64_t stride, float* __restrict__ out, int accumulate) {
-  __shared__ float sh[8][33];
+// out[c] (+)= sum over chunks of partial[j][c] (row stride `stride`): 32 columns per block, 32 warps
+// each summing every 32nd chunk, then the 32 warp sums in warp order — a fixed tree (deterministic),
+// coalesced along the columns, every load of a warp in flight at once.
+__global__ void __launch_bounds__(1024) colreduce_kernel(int nchunks, int n, const float* __restrict__ partial,
+                                                         int64_t stride, float* __restrict__ out, int accumulate) {
+  // 32 columns x 32 warps per block: warp g sums chunks g, g+32, ... in order (a handful of loads,
+  // all in flight at once), then the 32 warp sums are added in warp order — a fixed tree
+  __shared__ float sh[32][33];
   const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
   float s = 0.f;
   if (c < n) {
 #pragma unroll 8
-    for (int j = g; j < nchunks; j += 8) s += partial[(int64_t)j * stride + c];  // loads hoisted, adds in order
+    for (int j = g; j < nchunks; j += 32) s += partial[(int64_t)j * stride + c];
   }
   sh[g][cl] = s;
   __syncthreads();
   if (g == 0 && c < n) {
     float t = sh[0][cl];
 #pragma unroll
-    for (int k = 1; k < 8; ++k) t += sh[k][cl];
+    for (int k = 1; k < 32; ++k) t += sh[k][cl];
     out[c] = accumulate ? out[c] + t : t;
   }
 }
 static void colreduce(int nchunks, int n, const float* partial, int64_t stride, float* out, int accumulate,
                       cudaStream_t st) {
-  colreduce_kernel<<<(unsigned)ceil_div(n, 32), 256, 0, st>>>(nchunks, n, partial, stride, out, accumulate);
+  colreduce_kernel<<<(unsigned)ceil_div(n, 32), 1024, 0, st>>>(nchunks, n, partial, stride, out, accumulate);
   check_launch("colreduce");
 }
 
 // ------------------------------------------------------------------------------------- column sums
 // partial[chunk][c] = sum of rows [chunk*CS_ROWS, ...) of column c, rows in increasing order; each
 // thread owns VEC adjacent columns (16-byte loads) and keeps CS_ROWS independent loads in flight.
-constexpr int CS_ROWS = 32;
+constexpr int CS_ROWS = 16;
 template <typename Tin>
 __global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict__ X, int64_t ld,
                                       float* __restrict__ partial) {
@@ -156,10 +158,13 @@ __global__ void __launch_bounds__(128) colsum_partial_vec_kernel(int64_t rows, i
   float s[VEC];
 #pragma unroll
   for (int v = 0; v < VEC; ++v) s[v] = 0.f;
-#pragma unroll 8
-  for (int64_t r = r0; r < r1; ++r) {
-    const uint4 u = __ldg(reinterpret_cast<const uint4*>(X + r * ld + c0));
-    const Tin* e = reinterpret_cast<const Tin*>(&u);
+  uint4 u[CS_ROWS];  // every load in flight before the first add (one memory round trip per thread)
+#pragma unroll
+  for (int i = 0; i < CS_ROWS; ++i)
+    u[i] = r0 + i < r1 ? __ldg(reinterpret_cast<const uint4*>(X + (r0 + i) * ld + c0)) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+  for (int i = 0; i < CS_ROWS; ++i) {
+    const Tin* e = reinterpret_cast<const Tin*>(&u[i]);
 #pragma unroll
     for (int v = 0; v < VEC; ++v) s[v] += to_f32(e[v]);
   }

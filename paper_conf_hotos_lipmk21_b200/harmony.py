@@ -13,7 +13,8 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libharmony.so")
+# HARMONY_LIB: an alternative in-tree build of the same library (A/B experiments)
+LIB_PATH = os.environ.get("HARMONY_LIB") or os.path.join(_PKG, "libharmony.so")
 
 HARMONY_OK, HARMONY_E_INVALID_ARG, HARMONY_E_BAD_STATE, HARMONY_E_CAP_TOO_SMALL = 0, 1, 2, 3
 HARMONY_E_HOST_OOM, HARMONY_E_CUDA, HARMONY_E_NCCL, HARMONY_E_UNSUPPORTED = 4, 5, 6, 7
