@@ -45,6 +45,9 @@ WORKLOADS = {
     "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=4 x b=2), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
                  per_gpu_batch=8, m=4, cap=16 << 30, S=1024),
+    "cfg5": dict(name="cfg5: one 16384 x 16384 x 65536 (M x N x K) bf16 GEMM fwd+bwd, operator split along K into "
+                      "8 row-chunk tile subtasks per GPU (harmony_split_gemm_*)", model="gemm-16384x16384x65536",
+                 M=16384, N=16384, K=65536, chunks=8, S=1, per_gpu_batch=1, m=1, cap=0),
     "cfg1": dict(name="cfg1: 4-layer MLP d256, batch 32 as 4 microbatches, fp32, cap = 2 layers' state",
                  model="mlp4-d256", descs=lambda: synth.mlp_stack(4, 256), per_gpu_batch=32, m=4,
                  cap=2 * 16 * (256 * 256 + 256), S=1, precision=0),
@@ -165,6 +168,81 @@ def cpu_oracle_sample(wl, budget_s=20.0):
     return B / step, desc, (len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count())
 
 
+def run_cfg5(args, wl, world, rank, local, torch, H):
+    """Row a15: Y = X.W fwd + dX, dW bwd of one large GEMM, K split over the ranks (reading c19);
+    each rank runs its K-slice as `chunks` row-chunk tile subtasks (reduce-scatter of the fp32
+    partials over NCCL when world > 1, all-gather of dY).  Metric: whole-job TFLOP/s (3 x 2MNK
+    per step), device time (CUDA events on the library's compute stream), max over ranks."""
+    torch.cuda.set_device(local)
+    device = torch.device("cuda", local)
+    dist = None
+    nccl_id = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo", init_method="env://")
+        obj = [H.harmony_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    M, N, K = wl["M"], wl["N"], wl["K"]
+    Kr, Mr = K // world, M // world
+    g = torch.Generator(device=device)
+    g.manual_seed(7 + rank)
+    bf = torch.bfloat16
+    X = torch.randn(M, Kr, device=device, generator=g).to(bf)
+    W = (torch.randn(Kr, N, device=device, generator=g) / (K ** 0.5)).to(bf)
+    dY = torch.randn(Mr, N, device=device, generator=g).to(bf)
+    Y = torch.empty(Mr, N, device=device)
+    dX = torch.empty(M, Kr, device=device, dtype=bf)
+    dW = torch.empty(Kr, N, device=device)
+    flops = 3 * 2.0 * M * N * K  # whole job per step
+    with H.SplitGemm(M, N, K, chunks=wl["chunks"], rank=rank, world_size=world, device=local, precision=1,
+                     nccl_id=nccl_id) as sg:
+        for _ in range(args.warmup):
+            sg.run(X, W, dY, Y, dX, dW)
+        clocks = ClockSampler(local)
+        clocks.start()
+        torch.cuda.synchronize(device)
+        if dist is not None:
+            dist.barrier()
+        dev_s = sum(sg.run(X, W, dY, Y, dX, dW) for _ in range(args.steps))
+        torch.cuda.synchronize(device)
+        clk = clocks.stop()
+        # e2e: this rank's operand slices from pinned host memory, Y shard back, host wall clock
+        Xh, Wh, dYh = X.cpu().pin_memory(), W.cpu().pin_memory(), dY.cpu().pin_memory()
+        Yh = torch.empty(Mr, N).pin_memory()
+        torch.cuda.synchronize(device)
+        t0 = time.perf_counter()
+        for _ in range(max(1, args.steps // 2)):
+            X.copy_(Xh, non_blocking=True); W.copy_(Wh, non_blocking=True); dY.copy_(dYh, non_blocking=True)
+            sg.run(X, W, dY, Y, dX, dW)
+            Yh.copy_(Y, non_blocking=True)
+            torch.cuda.synchronize(device)
+        e2e_s = (time.perf_counter() - t0) / max(1, args.steps // 2)
+    if dist is not None:
+        t = torch.tensor([dev_s, e2e_s], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev_s, e2e_s = t.tolist()
+    if rank != 0:
+        return
+    peaks, peak_src = load_peaks()
+    tflops = flops * args.steps / dev_s / 1e12
+    peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]) * world
+    line = {"metric": "TFLOP/s of the operator-split GEMM fwd+bwd (cfg5)", "value": tflops, "unit": "TFLOP/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dev_s / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic (torch.randn on device, seeded)",
+            "config": {"workload": wl["name"], "M": M, "N": N, "K": K, "chunks": wl["chunks"], "parallelism": f"ksplit{world}",
+                       "l2": "operands 4.3 GB + outputs 7 GB per step, far larger than L2; no flush"},
+            "roofline": {"bound": "tensor", "kernel": "gemm_tc2_kernel (all GEMM launches of the step)",
+                         "achieved": tflops, "peak": peak, "unit": "TFLOP/s", "frac": tflops / peak, "traffic": None,
+                         "peak_source": f"{peak_src} bf16_tflops_sustained x {world} GPU(s)"},
+            "e2e": {"value": flops / e2e_s / 1e12, "unit": "TFLOP/s",
+                    "h2d_bytes_per_step": (X.numel() + W.numel() + dY.numel()) * 2, "d2h_bytes_per_step": Y.numel() * 4,
+                    "timing": "host wall clock: pinned H2D of this rank's operands + run + D2H of its Y shard"},
+            "gpu_launches": None, "clocks": clk}
+    print(json.dumps(line))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -207,6 +285,8 @@ def main():
     import torch
     from paper_conf_hotos_lipmk21_b200 import harmony as H
 
+    if args.workload == "cfg5":
+        return run_cfg5(args, wl, world, rank, local, torch, H)
     torch.cuda.set_device(local)
     device = torch.device("cuda", local)
     dist = None

@@ -99,7 +99,11 @@ typedef struct {
                                 backward (24d+2hS+16 B/token/block);
                                 2 = block recompute: stash only the fp32 block
                                 input (4d B/token/block), the backward re-runs the block's
-                                forward first (4/3 of the GEMM FLOPs, far fewer swap bytes)  */
+                                forward first (4/3 of the GEMM FLOPs, far fewer swap bytes);
+                                3 = as 2, plus the fused attention's output C (bf16) and row
+                                log-sum-exp (6d+4h B/token/block): the recompute skips the
+                                attention forward (falls back to 2 when attention is unfused).
+                                All four give bit-identical results (reading c13).           */
   double lr, beta1, beta2, eps, weight_decay; /* Adam; weight_decay must be 0 (reading c3).  Doubles:
                                 the kernel uses fp32 b and (1-b) each rounded once from these */
   uint8_t nccl_id[128];      /* ncclUniqueId from harmony_get_unique_id() on rank 0, broadcast
@@ -166,6 +170,21 @@ typedef struct {
   double seconds[5];
   double work[5];
 } harmony_kernel_profile;
+
+/* The step timeline of the last profiled step (profiling on): one record per op of the static
+ * program, in issue order — kind (OP_INPUT 0, H2D 1, D2H 2, FWD 3, LOSS 4, BWD 5, UPD 6,
+ * ALLGATHER 7, REDUCESCATTER 8, LOSS_GATHER 9, LOSS_OUT 10), stream (0 compute, 1 h2d, 2 d2h,
+ * 3 comm), tensor class of a copy (0 weight, 1 state, 2 stash, 3 input, 4 output, 5 grad, 6 none),
+ * layer, microbatch, bytes moved, and [t0, t1] in seconds from the step's start: CUDA events
+ * recorded on the op's stream around it (after its cross-stream waits), so the span is the op's
+ * own time on its stream.  The evidence for swap/compute overlap and achieved host-link GB/s.
+ * Writes min(n, cap) records to out (nullable) and the count to *n_out. */
+typedef struct {
+  int32_t op, kind, stream, cat, layer, micro;
+  uint64_t bytes;
+  double t0, t1;
+} harmony_timeline_rec;
+harmony_status harmony_read_timeline(const harmony_ctx* ctx, harmony_timeline_rec* out, int32_t cap, int32_t* n_out);
 
 harmony_status harmony_set_profiling(harmony_ctx* ctx, int32_t on);
 harmony_status harmony_read_profile(const harmony_ctx* ctx, harmony_kernel_profile* out);

@@ -49,6 +49,8 @@ struct KProf {
   size_t used = 0;
   struct Rec { int cat, e0, e1; double work; };
   std::vector<Rec> recs;
+  struct OpRec { int op, e0, e1; };  // the step timeline: events around every op of the program
+  std::vector<OpRec> oprecs;
   int begin(cudaStream_t st) {
     if (!on) return -1;
     if (used == pool.size()) {

@@ -49,6 +49,7 @@ struct StepGraph {
   harmony_step_stats stats{};
   uint64_t launches = 0;
   std::vector<KProf::Rec> recs;           // profiled graph: timing-event pairs of its kernels
+  std::vector<KProf::OpRec> oprecs;       // profiled graph: timing-event pairs of its ops
 };
 
 struct harmony_ctx {
@@ -72,6 +73,7 @@ struct harmony_ctx {
   harmony_step_stats last{};
   bool profiling = false;
   harmony_kernel_profile prof{};
+  std::vector<harmony_timeline_rec> timeline;  // last profiled step, one record per op
   int* h_step = nullptr;  // pinned: Adam's t, copied to the device at the start of every step
   bool use_graph = true;
   StepGraph g_plain, g_prof;  // the step as CUDA graphs: plain, and with per-kernel timing events
@@ -194,6 +196,7 @@ void issue_program(harmony_ctx* c, const float* x, const float* tg, bool x_dev, 
     const Op& o = p.ops[oi];
     cudaStream_t st = c->st[o.stream];
     for (int w : o.waits) HM_CUDA(cudaStreamWaitEvent(st, c->events[p.ops[w].event], 0));
+    const int op_e0 = g_prof.begin(st);  // profiling: the op's span on its stream (after its waits)
     switch (o.kind) {
       case OP_INPUT: {
         const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)x : (const void*)tg);
@@ -290,6 +293,10 @@ void issue_program(harmony_ctx* c, const float* x, const float* tg, bool x_dev, 
       default:
         throw Error{HARMONY_E_INVALID_ARG, "unknown op kind in plan"};
     }
+    if (op_e0 >= 0) {
+      const int op_e1 = g_prof.begin(st);
+      if (op_e1 >= 0) g_prof.oprecs.push_back({(int)oi, op_e0, op_e1});
+    }
     if (o.event >= 0) HM_CUDA(cudaEventRecord(c->events[o.event], st));
   }
 }
@@ -318,6 +325,7 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg
   g_prof.external = profiled;
   g_prof.used = 0;
   g_prof.recs.clear();
+  g_prof.oprecs.clear();
   HM_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
   try {
     HM_CUDA(cudaEventRecord(c->ev_fork, cs));
@@ -337,10 +345,11 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg
   }
   g_prof.on = g_prof.external = false;
   HM_CUDA(cudaStreamEndCapture(cs, &G.graph));
-  HM_CUDA(cudaGraphInstantiate(&G.exec, G.graph, 0));
+  HM_CUDA(cudaGraphInstantiate(&G.exec, G.graph, cudaGraphInstantiateFlagUseNodePriority));
   G.stats = s;
   G.launches = g_kernel_launches;
   G.recs = g_prof.recs;
+  G.oprecs = g_prof.oprecs;
   // find the input memcpy nodes by their destinations
   size_t n = 0;
   HM_CUDA(cudaGraphGetNodes(G.graph, nullptr, &n));
@@ -378,8 +387,10 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
   g_prof.external = false;
   g_prof.used = 0;
   g_prof.recs.clear();
+  g_prof.oprecs.clear();
   cudaStream_t cs = c->st[S_COMPUTE];
   std::vector<KProf::Rec>* recs = &g_prof.recs;
+  std::vector<KProf::OpRec>* oprecs = &g_prof.oprecs;
   if (use_graph) {
     StepGraph& G = c->profiling ? c->g_prof : c->g_plain;
     const int sig = (x_dev ? 1 : 0) | (t_dev ? 2 : 0);
@@ -400,6 +411,7 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     s.kernel_launches = G.launches;
     s.step_seconds = ms * 1e-3;
     recs = &G.recs;
+    oprecs = &G.oprecs;
   } else {
     HM_CUDA(cudaEventRecord(c->ev_begin, cs));
     for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_begin, 0));
@@ -423,6 +435,17 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
       c->prof.launches[rc.cat] += 1;
       c->prof.seconds[rc.cat] += e * 1e-3;
       c->prof.work[rc.cat] += rc.work;
+    }
+    c->timeline.clear();
+    for (auto& orc : *oprecs) {
+      const Op& o = p.ops[orc.op];
+      float t0 = 0.f, t1 = 0.f;
+      HM_CUDA(cudaEventElapsedTime(&t0, c->ev_begin, g_prof.pool[orc.e0]));
+      HM_CUDA(cudaEventElapsedTime(&t1, c->ev_begin, g_prof.pool[orc.e1]));
+      harmony_timeline_rec r{};
+      r.op = orc.op; r.kind = o.kind; r.stream = o.stream; r.cat = o.cat; r.layer = o.layer; r.micro = o.mb;
+      r.bytes = o.bytes; r.t0 = t0 * 1e-3; r.t1 = t1 * 1e-3;
+      c->timeline.push_back(r);
     }
     g_prof.on = false;
   }
@@ -497,15 +520,24 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
   HM_CUDA(cudaGetDeviceProperties(&prop, cfg->device));
   HM_CHECK(prop.major == 10, HARMONY_E_UNSUPPORTED,
            std::string("libharmony is built for sm_100a (B200); device is ") + prop.name);
+  // Stream priorities: the compute stream carries the step's critical path (the dgrad chain), the
+  // side stream the weight-gradient work that only feeds dW — when SMs free up, the block scheduler
+  // places the compute stream's CTAs first (HARMONY_PRIO=0: all default priority)
+  int prio_lo = 0, prio_hi = 0;
+  HM_CUDA(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
+  {
+    const char* e = getenv("HARMONY_PRIO");
+    if (e && *e == '0') prio_lo = prio_hi = 0;
+  }
   for (int s = 0; s < S_NUM; ++s) {
-    HM_CUDA(cudaStreamCreateWithFlags(&c->st[s], cudaStreamNonBlocking));
+    HM_CUDA(cudaStreamCreateWithPriority(&c->st[s], cudaStreamNonBlocking, s == S_COMPUTE ? prio_hi : 0));
     HM_CUDA(cudaEventCreate(&c->ev_end[s]));
   }
   HM_CUDA(cudaEventCreate(&c->ev_begin));
   HM_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
   for (int s = 0; s < S_NUM; ++s) HM_CUDA(cudaEventCreateWithFlags(&c->ev_join[s], cudaEventDisableTiming));
   c->h_step = static_cast<int*>(alloc_host(sizeof(int)));
-  HM_CUDA(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+  HM_CUDA(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio_lo));
   for (auto& e : c->side_ev) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   {
     const char* e = getenv("HARMONY_NO_GRAPH");
@@ -673,6 +705,15 @@ harmony_status harmony_set_profiling(harmony_ctx* c, int32_t on) {
   if (!c) return HARMONY_E_INVALID_ARG;
   c->profiling = on != 0;
   c->prof = harmony_kernel_profile{};
+  return HARMONY_OK;
+}
+
+harmony_status harmony_read_timeline(const harmony_ctx* c, harmony_timeline_rec* out, int32_t cap, int32_t* n_out) {
+  if (!c || !n_out || cap < 0) return HARMONY_E_INVALID_ARG;
+  const int32_t n = (int32_t)c->timeline.size();
+  *n_out = n;
+  if (out)
+    for (int32_t i = 0; i < std::min(n, cap); ++i) out[i] = c->timeline[i];
   return HARMONY_OK;
 }
 

@@ -911,35 +911,51 @@ __global__ void __launch_bounds__(THREADS, 1)
   }
 }
 
-// sD[b, h, q] = scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = lse * log2(e)
-// (one thread per (token, head)): the per-query terms of dS = P (dP - D) in the forms the
-// backward's FFMAs take.
-__global__ void attn_bwd_prep(int64_t ntok, int S, int H, int dh, float scale, const __nv_bfloat16* __restrict__ dO,
-                              const __nv_bfloat16* __restrict__ O, const float* __restrict__ lse, float* __restrict__ sD,
-                              float* __restrict__ lse2) {
-  // thread i = ((b * H + h) * S + q): consecutive threads walk q, so the [b, H, S] statistics are
-  // read and written coalesced; each thread reads its (token, head) row of dO and O (dh * 2 bytes)
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= ntok * H) return;
-  const int64_t q = i % S, bh = i / S;
-  const int h = (int)(bh % H);
-  const int64_t tok = (bh / H) * S + q;
-  const int d = H * dh;
-  const uint4* a = reinterpret_cast<const uint4*>(dO + tok * d + h * dh);
-  const uint4* o = reinterpret_cast<const uint4*>(O + tok * d + h * dh);
-  float s = 0.f;
-  for (int k8 = 0; k8 < dh / 8; ++k8) {
-    uint4 x = a[k8], y = o[k8];
-    const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&x);
-    const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&y);
+// sD[b, h, q] = scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = lse * log2(e): the
+// per-query terms of dS = P (dP - D) in the forms the backward's FFMAs take.  One warp per token:
+// the token's dO and O rows are read once, contiguously (lane l takes elements 8l.. of every
+// 256-element chunk; 256 % dh == 0, so a chunk holds whole heads), and each head's dh/8 lanes
+// reduce with shuffles in a fixed order.
+__global__ void __launch_bounds__(256) attn_bwd_prep(int64_t ntok, int S, int H, int dh, float scale,
+                                                     const __nv_bfloat16* __restrict__ dO,
+                                                     const __nv_bfloat16* __restrict__ O, const float* __restrict__ lse,
+                                                     float* __restrict__ sD, float* __restrict__ lse2) {
+  const int lane = threadIdx.x & 31;
+  const int64_t tok = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (tok >= ntok) return;
+  const int d = H * dh, lph = dh / 8;  // lanes per head
+  const int64_t bseq = tok / S, q = tok % S;
+  const uint4* a = reinterpret_cast<const uint4*>(dO + tok * d);
+  const uint4* o = reinterpret_cast<const uint4*>(O + tok * d);
+  for (int j0 = 0; 256 * j0 < d; j0 += 8) {  // 2048 elements per round, every load in flight at once
+    uint4 xa[8], ya[8];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
-      s += fx.x * fy.x + fx.y * fy.y;
+    for (int j = 0; j < 8; ++j) {
+      const int e = 256 * (j0 + j) + 8 * lane;
+      xa[j] = e < d ? a[e / 8] : make_uint4(0, 0, 0, 0);
+      ya[j] = e < d ? o[e / 8] : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int e = 256 * (j0 + j) + 8 * lane;
+      if (256 * (j0 + j) >= d) break;
+      const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&xa[j]);
+      const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&ya[j]);
+      float s = 0.f;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
+        s += fx.x * fy.x + fx.y * fy.y;
+      }
+      for (int w = lph / 2; w > 0; w >>= 1) s += __shfl_xor_sync(0xffffffffu, s, w);
+      if (e < d && (lane % lph) == 0) {
+        const int h = e / dh;
+        const int64_t i = (bseq * H + h) * S + q;
+        sD[i] = scale * s;
+        lse2[i] = lse[i] * 1.4426950408889634f;
+      }
     }
   }
-  sD[i] = scale * s;
-  lse2[i] = lse[i] * 1.4426950408889634f;
 }
 }  // namespace attn
 
@@ -1003,9 +1019,8 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   float* lse2 = sD + align_up((uint64_t)b * H * S * 4, 256) / 4;
   const float scale = 1.0f / std::sqrt((float)dh);
   const int e0 = g_prof.begin(st);
-  const int64_t n = b * S * H;
-  attn_bwd_prep<<<(unsigned)ceil_div(n, 256), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
-                                                           static_cast<const __nv_bfloat16*>(O), lse, sD, lse2);
+  attn_bwd_prep<<<(unsigned)ceil_div(b * S, 8), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
+                                                             static_cast<const __nv_bfloat16*>(O), lse, sD, lse2);
   check_launch("attn_bwd_prep");
   if (causal) HM_CUDA(cudaMemsetAsync(dst, 0, (size_t)b * H * S * S * 2, st));  // key tiles never visited by a query tile
   CUtensorMap mq, mk, mv, mo, mds;

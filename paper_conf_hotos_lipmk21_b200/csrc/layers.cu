@@ -30,18 +30,24 @@ static uint64_t bump(uint64_t& cur, uint64_t bytes) {
 }
 
 LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_policy) {
-  if (stash_policy == 2 && desc.kind == HARMONY_LAYER_TRANSFORMER) {
+  if ((stash_policy == 2 || stash_policy == 3) && desc.kind == HARMONY_LAYER_TRANSFORMER) {
     // Block recompute ([7] P:881): the stash is the block input X; the forward and the
     // backward both run the policy-0 block on a workspace-resident copy of the full stash.
+    // Policy 3 also stashes the fused attention's output C (bf16) and row log-sum-exp, so the
+    // recompute skips the attention forward (8.25 MB more per cfg2 task, usually host-swapped).
     LayerGeom core = make_geom(desc, b, dtype, 0);
     LayerGeom g = core;
-    g.stash_policy = 2;
+    g.stash_policy = stash_policy == 3 && core.fused_attn ? 3 : 2;
     g.core_st = core.st;
     g.core_ws_fwd = core.ws_fwd;
     g.core_ws_bwd = core.ws_bwd;
     g.st = StashLayout{};
     uint64_t c = 0;
     g.st.X = bump(c, (uint64_t)core.rows * core.d * 4);
+    if (g.stash_policy == 3) {
+      g.st.C = bump(c, (uint64_t)core.rows * core.d * core.ts);
+      g.st.P = bump(c, (uint64_t)core.b * core.h * core.S * 4);  // row log-sum-exp
+    }
     g.st.total = c;
     const uint64_t full = align_up(core.st.total, 256);
     g.core_off = 0;
@@ -49,7 +55,7 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
     g.ws_bwd = full + std::max(core.ws_fwd, core.ws_bwd) + align_up((uint64_t)core.rows * core.d * 4, 256);
     return g;
   }
-  if (stash_policy == 2) stash_policy = 0;  // MLP: the op-input stash is already minimal
+  if (stash_policy >= 2) stash_policy = 0;  // MLP: the op-input stash is already minimal
   LayerGeom g;
   g.desc = desc;
   g.dtype = dtype;
@@ -181,8 +187,16 @@ static hk_gemm_args lin_wgrad(const LayerGeom& g, int64_t rows, int n, int k, co
 }
 
 // ------------------------------------------------------------------------------------------------ forward
+// Attention output C and row LSE kept outside the core stash (stash policy 3): where they live and
+// whether they already hold this block's values (the backward's recompute skips the attention)
+struct AttnStash {
+  uint8_t* C;
+  float* lse;
+  bool have;
+};
+
 static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws,
-                     void* stv, bool stash_x = true) {
+                     void* stv, bool stash_x = true, const AttnStash* as = nullptr) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   if (d.kind == HARMONY_LAYER_MLP) {
@@ -202,8 +216,8 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   float* mean1 = reinterpret_cast<float*>(stash + g.st.mean1);
   float* rstd1 = reinterpret_cast<float*>(stash + g.st.rstd1);
   uint8_t* QKV = stash + g.st.QKV;
-  uint8_t* P = stash + g.st.P;
-  uint8_t* C = stash + g.st.C;
+  uint8_t* P = as ? reinterpret_cast<uint8_t*>(as->lse) : stash + g.st.P;
+  uint8_t* C = as ? as->C : stash + g.st.C;
   float* X2 = reinterpret_cast<float*>(stash + g.st.X2);
   float* mean2 = reinterpret_cast<float*>(stash + g.st.mean2);
   float* rstd2 = reinterpret_cast<float*>(stash + g.st.rstd2);
@@ -226,7 +240,9 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
     a.C = QKV; a.epilogue = HK_EPI_STORE_T; a.bias = wseg(g, W, P_BQKV);
     gemm(a, st);
   }
-  if (g.fused_attn) {
+  if (as && as->have) {
+    // C and the LSE of this block are in the stash (policy 3): the recompute needs only Q, K, V
+  } else if (g.fused_attn) {
     // C = softmax(Q K^T / sqrt(dh)) V per head, scores kept in TMEM; stash the row LSE
     HM_CHECK(attention_fwd_fused(b, S, H, dh, d.causal, QKV, C, reinterpret_cast<float*>(P), st), HARMONY_E_INVALID_ARG,
              "fused attention rejected a qualifying shape");
@@ -285,7 +301,8 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
 
 // ------------------------------------------------------------------------------------------------ backward
 static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
-                     int first, uint8_t* ws, void* stv, const float* Xs_in = nullptr) {
+                     int first, uint8_t* ws, void* stv, const float* Xs_in = nullptr,
+                     const AttnStash* as = nullptr) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   const int acc = first ? 0 : 1;
@@ -313,8 +330,8 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   const float* mean1 = reinterpret_cast<const float*>(stash + g.st.mean1);
   const float* rstd1 = reinterpret_cast<const float*>(stash + g.st.rstd1);
   const uint8_t* QKV = stash + g.st.QKV;
-  const uint8_t* P = stash + g.st.P;
-  const uint8_t* C = stash + g.st.C;
+  const uint8_t* P = as ? reinterpret_cast<const uint8_t*>(as->lse) : stash + g.st.P;
+  const uint8_t* C = as ? as->C : stash + g.st.C;
   const float* X2 = reinterpret_cast<const float*>(stash + g.st.X2);
   const float* mean2 = reinterpret_cast<const float*>(stash + g.st.mean2);
   const float* rstd2 = reinterpret_cast<const float*>(stash + g.st.rstd2);
@@ -479,25 +496,30 @@ static LayerGeom core_geom(const LayerGeom& g) {
 }
 
 void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* st) {
-  if (g.stash_policy != 2) return fwd_core(g, W, X, Y, stash, ws, st);
+  if (g.stash_policy < 2) return fwd_core(g, W, X, Y, stash, ws, st);
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
   uint8_t* rest = ws + align_up(c.st.total, 256);
-  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false);
+  // policy 3: the attention writes C and its LSE straight into the stash
+  const AttnStash as{stash + g.st.C, reinterpret_cast<float*>(stash + g.st.P), false};
+  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false, g.stash_policy == 3 ? &as : nullptr);
   copy_f32(g.rows * g.d, X, reinterpret_cast<float*>(stash + g.st.X), static_cast<cudaStream_t>(st));
 }
 
 void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
                int first, uint8_t* ws, void* st) {
-  if (g.stash_policy != 2) return bwd_core(g, W, stash, dY, dX, dW, first, ws, st);
+  if (g.stash_policy < 2) return bwd_core(g, W, stash, dY, dX, dW, first, ws, st);
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
   uint8_t* rest = ws + align_up(c.st.total, 256);
   // recompute the block's forward from its stashed input: the same kernels, hence the same bits;
-  // the LN1 backward reads the stashed input in place
+  // the LN1 backward reads the stashed input in place (policy 3: and the stashed C / LSE)
   const float* Xst = reinterpret_cast<const float*>(stash + g.st.X);
-  fwd_core(c, W, Xst, nullptr, full, rest, st, /*stash_x=*/false);
-  bwd_core(c, W, full, dY, dX, dW, first, rest, st, Xst);
+  const AttnStash as{const_cast<uint8_t*>(stash) + g.st.C, reinterpret_cast<float*>(const_cast<uint8_t*>(stash) + g.st.P),
+                     true};
+  const AttnStash* asp = g.stash_policy == 3 ? &as : nullptr;
+  fwd_core(c, W, Xst, nullptr, full, rest, st, /*stash_x=*/false, asp);
+  bwd_core(c, W, full, dY, dX, dW, first, rest, st, Xst, asp);
 }
 
 }  // namespace hm

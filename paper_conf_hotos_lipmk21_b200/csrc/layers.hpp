@@ -26,8 +26,9 @@ struct LayerGeom {
   int dtype = 0;            // 0 = fp32 activations / SIMT GEMM, 1 = bf16 / tcgen05
   int ts = 4;               // bytes per activation element
   int stash_policy = 0;     // 0 = all op inputs, 1 = recompute LN outputs and GeLU in the backward,
-                            // 2 = stash only the block input; the backward recomputes the block
-  int64_t core_off = 0;     // policy 2: offset of the full (policy-0) stash inside the workspace
+                            // 2 = stash only the block input; the backward recomputes the block,
+                            // 3 = 2 + the attention output and LSE (the recompute skips attention)
+  int64_t core_off = 0;     // policy 2/3: offset of the full (policy-0) stash inside the workspace
   int b = 0;                // samples per microbatch
   int64_t rows = 0;         // tokens per microbatch (b*S; MLP: b)
   int d = 0, dh = 0, h = 0, S = 1;

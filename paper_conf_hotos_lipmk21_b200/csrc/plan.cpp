@@ -27,7 +27,7 @@ void validate_config(const harmony_config& c) {
            "unknown schedule");
   HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
            "the per-GPU-virtualization baseline schedule is not built yet (SURVEY NEXT-3)");
-  HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 2, HARMONY_E_INVALID_ARG, "stash_policy must be 0, 1 or 2");
+  HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 3, HARMONY_E_INVALID_ARG, "stash_policy must be 0..3");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");

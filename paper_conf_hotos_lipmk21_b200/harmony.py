@@ -73,6 +73,14 @@ class harmony_kernel_profile(C.Structure):
                 for i, c in enumerate(self.CLASSES)}
 
 
+class harmony_timeline_rec(C.Structure):
+    _fields_ = [(n, C.c_int32) for n in ("op", "kind", "stream", "cat", "layer", "micro")] + [
+        ("bytes", C.c_uint64), ("t0", C.c_double), ("t1", C.c_double)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
 class hk_gemm_args(C.Structure):
     _fields_ = [("dtype", C.c_int32), ("M", C.c_int32), ("N", C.c_int32), ("K", C.c_int32), ("nz0", C.c_int32),
                 ("nz1", C.c_int32),
@@ -124,6 +132,7 @@ def lib() -> C.CDLL:
         "harmony_plan_dry": (st, [C.POINTER(harmony_config), C.c_int32, C.POINTER(harmony_layer_desc),
                                   C.POINTER(harmony_plan_summary), P, C.c_uint64]),
         "harmony_finalize": (st, [P]),
+        "harmony_read_timeline": (st, [P, P, C.c_int32, C.POINTER(C.c_int32)]),
         "hk_gemm": (st, [C.POINTER(hk_gemm_args), P]),
         "hk_layernorm_fwd": (st, [C.c_int32, C.c_int64, C.c_int32, P, P, P, P, P, P, P]),
         "hk_layernorm_bwd": (st, [C.c_int32, C.c_int64, C.c_int32, P, P, P, P, P, P, P, P, P, C.c_int32, P]),
@@ -261,6 +270,15 @@ def harmony_read_profile(ctx):
     p = harmony_kernel_profile()
     _check(lib().harmony_read_profile(ctx, C.byref(p)), ctx)
     return p
+
+
+def harmony_read_timeline(ctx):
+    """Per-op timeline of the last profiled step (list of dicts; see harmony.h)."""
+    n = C.c_int32()
+    _check(lib().harmony_read_timeline(ctx, None, 0, C.byref(n)), ctx)
+    arr = (harmony_timeline_rec * max(n.value, 1))()
+    _check(lib().harmony_read_timeline(ctx, arr, n.value, C.byref(n)), ctx)
+    return [arr[i].as_dict() for i in range(n.value)]
 
 
 def harmony_finalize(ctx):
