@@ -39,9 +39,9 @@ TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2.json")
 FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
 
 WORKLOADS = {
-    "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=8 x b=8), bf16/fp32-master Adam, "
+    "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=4 x b=16), bf16/fp32-master Adam, "
                       "HBM cap 8 GiB/GPU", model="bert-large-like-preLN", descs=lambda: synth.transformer_stack(24, 1024, 16, 512, False),
-                 per_gpu_batch=64, m=8, cap=8 << 30, S=512),
+                 per_gpu_batch=64, m=4, cap=8 << 30, S=512),
     "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=4 x b=2), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
                  per_gpu_batch=8, m=4, cap=16 << 30, S=1024),
@@ -251,6 +251,8 @@ def main():
     ap.add_argument("--workload", default="cfg2", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--stash-policy", type=int, default=2)
+    ap.add_argument("--microbatches", type=int, default=0,
+                    help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
@@ -296,7 +298,7 @@ def main():
     precision = wl.get("precision", 1)
     descs = wl["descs"]()
     B = wl["per_gpu_batch"]
-    m = wl["m"]
+    m = args.microbatches or wl["m"]
     nccl_id = None
     if world > 1:
         obj = [H.harmony_get_unique_id() if rank == 0 else None]
@@ -396,10 +398,11 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "bf16" if precision else "f32", "data": "synthetic (seeded, paper-shaped)",
         "config": {"workload": wl["name"], "global_batch": B * world, "seq_len": wl["S"],
+                   "microbatches": m, "microbatch_size": B // m,
                    "parallelism": f"dp{world}", "hbm_cap_bytes_per_gpu": wl["cap"],
                    "arena_bytes": plan["arena_bytes"], "stash_policy": cfg["stash_policy"],
                    "l2": "inputs and per-step swap traffic (tens of GB) far larger than the 126 MB L2; no flush"},
-        "roofline": {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05, all GEMM launches of the step)",
+        "roofline": {"bound": "tensor", "kernel": "gemm_tc2_kernel / gemm_tc_kernel (tcgen05, all GEMM launches of the step)",
                      "achieved": gemm_tflops, "peak": gemm_peak, "unit": "TFLOP/s",
                      "frac": gemm_tflops / gemm_peak if gemm_peak else None, "traffic": traffic,
                      "traffic_unit": "bytes per launch", "traffic_source": traffic_src,
@@ -416,6 +419,9 @@ def main():
                           "host_link_gbs_measured": bw, "flops_per_step": F},
         "kernels": {k: dict(v, per_launch_us=(v["seconds"] / v["launches"] * 1e6 if v["launches"] else None))
                     for k, v in prof.items()},
+        "attention": {"achieved_tflops": (prof["attention"]["work"] / prof["attention"]["seconds"] / 1e12
+                                          if prof["attention"]["seconds"] else None),
+                      "peak_tflops": gemm_peak, "kernel": "attn_fwd_kernel / attn_bwd_kernel (fused, tcgen05)"},
         "adam_hbm": {"achieved_gbs": adam["work"] / adam["seconds"] / 1e9 if adam["seconds"] else None,
                      "peak_gbs": peaks["hbm_gbs"]},
         "e2e": {"value": samples / e2e_wall, "unit": unit, "h2d_bytes_per_step": e2e_stats[-1]["h2d_input_bytes"],

@@ -164,11 +164,12 @@ void harmony_abi_sizes(uint64_t out[6]);
 /* Per-kernel-class timing (CUDA events recorded on the launching stream around every launch
  * while profiling is on).  Classes: 0 GEMM (work = algorithmic FLOPs 2MNK), 1 Adam (work =
  * algorithmic HBM bytes, 30 B/param bf16 / 32 fp32), 2 LayerNorm fwd+bwd (bytes), 3 softmax
- * fwd+bwd (bytes), 4 other.  Totals accumulate over steps since harmony_set_profiling(ctx, 1). */
+ * fwd+bwd (bytes), 4 other, 5 fused attention fwd/bwd (work = algorithmic FLOPs of its QK^T, PV
+ * (and backward) contractions).  Totals accumulate over steps since harmony_set_profiling(ctx, 1). */
 typedef struct {
-  uint64_t launches[5];
-  double seconds[5];
-  double work[5];
+  uint64_t launches[6];
+  double seconds[6];
+  double work[6];
 } harmony_kernel_profile;
 
 /* The step timeline of the last profiled step (profiling on): one record per op of the static

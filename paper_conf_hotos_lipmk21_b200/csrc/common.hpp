@@ -41,7 +41,7 @@ extern thread_local uint64_t g_kernel_launches;
 
 // Optional per-launch timing (harmony_set_profiling): CUDA events recorded on the launching
 // stream around each kernel of a class, with the launch's algorithmic work (FLOPs or bytes).
-enum ProfCat { PROF_GEMM = 0, PROF_ADAM = 1, PROF_LN = 2, PROF_SOFTMAX = 3, PROF_OTHER = 4, PROF_NUM = 5 };
+enum ProfCat { PROF_GEMM = 0, PROF_ADAM = 1, PROF_LN = 2, PROF_SOFTMAX = 3, PROF_OTHER = 4, PROF_ATTN = 5, PROF_NUM = 6 };
 struct KProf {
   bool on = false;
   bool external = false;  // inside a stream capture: record event nodes into the graph

@@ -628,23 +628,28 @@ __global__ void __launch_bounds__(THREADS, 1)
 }
 
 // ------------------------------------------------------------------ persistent backward (dh = 64)
-// Same per-tile mathematics as attn_bwd_kernel; one CTA per SM loops over the (key tile, head,
-// sequence) items with every pipeline counter running on across items: K_j / V_j double-buffered
-// (the next item's load overlaps the current one), (Q_i, dO_i) in a 3-deep ring, P^T stored by the
-// softmax warps into TMEM (two buffers) as the A operand of dV += P^T dO, dS^T in shared memory
-// (A operand of dK += dS^T Q and source of its TMA store), dK / dV drained with their own
-// full / empty barriers so the next item's scores start while they are written out.
+// Same per-element mathematics as attn_bwd_kernel; one CTA per SM loops over the (key tile, head,
+// sequence) items, and each item over 64-query sub-tiles, with every pipeline counter running on
+// across items.  TMEM holds TWO S^T / dP^T buffer pairs (128 keys x 64 queries each), so the MMA
+// computes the scores of sub-tile g+2 while the softmax warps turn sub-tile g+1 into P^T / dS^T:
+//   MMA:     S(0) S(1) | per g: [wait P(g)] dV += P^T(g) dO, dK += dS^T(g) Q, S(g+2)
+//   softmax: per g: [wait S(g)] P^T -> TMEM (A operand of dV), dS^T -> smem (A operand of dK and
+//            the source of its TMA store for the deterministic dQ GEMM)
+// K_j / V_j are double-buffered (the next item's load overlaps the current one), (Q_i, dO_i, the
+// sub-tile's statistics) run in a 4-deep ring, and dK / dV drain with their own full / empty
+// barriers so the next item's scores start while they are written out.
 struct BwdPCfg {
   static constexpr int DH = 64;
+  static constexpr int BQS = 64;                  // queries per sub-tile
   static constexpr int KV_BYTES = BKV * DH * 2;   // K_j or V_j
-  static constexpr int QT_BYTES = BQ * DH * 2;    // Q_i or dO_i
-  static constexpr int KVST = 2, QST = 2, DSB = 2;
-  static constexpr int DS_BYTES = BKV * BQ * 2;   // dS^T tile
-  static constexpr int STAT_BYTES = 2 * BQ * 4;   // lse2 and sD of a query tile
+  static constexpr int QT_BYTES = BQS * DH * 2;   // Q_i or dO_i sub-tile
+  static constexpr int KVST = 2, QST = 4, DSB = 2;
+  static constexpr int DS_BYTES = BKV * BQS * 2;  // dS^T sub-tile (128 keys x 128 B)
+  static constexpr int STAT_BYTES = 2 * BQS * 4;  // lse2 and sD of a sub-tile
   static constexpr int SMEM = KVST * 2 * KV_BYTES + QST * (2 * QT_BYTES + STAT_BYTES) + DSB * DS_BYTES + 1024 + 256;
-  static constexpr int ST_COL = 0, DP_COL = 128, DV_COL = 256, DK_COL = 256 + DH, PT_COL = 256 + 2 * DH;
+  static constexpr int ST_COL = 0, DP_COL = 2 * BQS, DV_COL = 4 * BQS, DK_COL = 4 * BQS + DH, PT_COL = 4 * BQS + 2 * DH;
   static constexpr int TMEM_COLS = 512;
-  static_assert(PT_COL + 2 * (BQ / 2) <= TMEM_COLS, "TMEM columns");
+  static_assert(PT_COL + 2 * (BQS / 2) <= TMEM_COLS, "TMEM columns");
   static_assert(SMEM <= 232448, "shared memory per CTA");
 };
 
@@ -659,37 +664,37 @@ __global__ void __launch_bounds__(THREADS, 1)
                         const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmdO,
                         const __grid_constant__ CUtensorMap tmdS, BwdParams p, int B) {
   using Cfg = BwdPCfg;
-  constexpr int DH = Cfg::DH;
+  constexpr int DH = Cfg::DH, BQS = Cfg::BQS;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sKV = smem;                                   // [KVST] (K_j, V_j)
   uint8_t* sQ = sKV + Cfg::KVST * 2 * Cfg::KV_BYTES;     // [QST] (Q_i, dO_i)
   uint8_t* sDS = sQ + Cfg::QST * 2 * Cfg::QT_BYTES;      // [DSB] dS^T
-  float* sStat = reinterpret_cast<float*>(sDS + Cfg::DSB * Cfg::DS_BYTES);  // [QST] (lse2[BQ], sD[BQ])
+  float* sStat = reinterpret_cast<float*>(sDS + Cfg::DSB * Cfg::DS_BYTES);  // [QST] (lse2[BQS], sD[BQS])
   uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(sStat) + Cfg::QST * Cfg::STAT_BYTES);
   uint64_t* kv_full = bars;          // [2]
   uint64_t* kv_empty = bars + 2;     // [2]
-  uint64_t* q_full = bars + 4;       // [QST <= 3]
-  uint64_t* q_empty = bars + 7;      // [QST <= 3]
-  uint64_t* s_full = bars + 10;
-  uint64_t* p_full = bars + 11;      // [2]: P^T in TMEM, dS^T in smem, S^T / dP^T read
-  uint64_t* p_empty = bars + 13;     // [2]
-  uint64_t* kd_full = bars + 15;
-  uint64_t* kd_empty = bars + 16;
-  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 17);
+  uint64_t* q_full = bars + 4;       // [QST]
+  uint64_t* q_empty = bars + 8;      // [QST]
+  uint64_t* s_full = bars + 12;      // [2]: S^T / dP^T buffer pair written by the MMA
+  uint64_t* p_full = bars + 14;      // [2]: P^T in TMEM, dS^T in smem, S^T / dP^T pair read
+  uint64_t* p_empty = bars + 16;     // [2]: dV / dK MMAs of the buffer's sub-tile done
+  uint64_t* kd_full = bars + 18;
+  uint64_t* kd_empty = bars + 19;
+  uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(bars + 20);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int nk = p.S / BKV, nq = p.S / BQ;
+  const int nk = p.S / BKV, nqs = p.S / BQS;
   const int items = nk * p.H * B;
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmdO); prefetch_tmap(&tmdS);
     for (int i = 0; i < 2; ++i) {
       mbar_init(&kv_full[i], 1); mbar_init(&kv_empty[i], 1);
+      mbar_init(&s_full[i], 1);
       mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1);
     }
     for (int i = 0; i < Cfg::QST; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
-    mbar_init(s_full, 1);
     mbar_init(kd_full, 1); mbar_init(kd_empty, 256);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -710,175 +715,180 @@ __global__ void __launch_bounds__(THREADS, 1)
       for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
         int b, h, kt;
         bwd_item(item, nk, p.H, b, h, kt);
-        const int i0 = p.causal ? kt : 0;
+        const int i0 = p.causal ? kt * (BKV / BQS) : 0;
         const int kvs = n & 1;
         mbar_wait(&kv_empty[kvs], ((n >> 1) & 1) ^ 1);
         mbar_expect_tx(&kv_full[kvs], 2 * Cfg::KV_BYTES);
         uint8_t* kb = sKV + kvs * 2 * Cfg::KV_BYTES;
         tma_load_4d(kb, &tmK, &kv_full[kvs], 0, kt * BKV, h, b);
         tma_load_4d(kb + Cfg::KV_BYTES, &tmV, &kv_full[kvs], 0, kt * BKV, h, b);
-        for (int i = i0; i < nq; ++i) {
+        for (int i = i0; i < nqs; ++i) {
           mbar_wait(&q_empty[qs], qph ^ 1);
           mbar_expect_tx(&q_full[qs], 2 * Cfg::QT_BYTES + Cfg::STAT_BYTES);
           uint8_t* q = sQ + qs * 2 * Cfg::QT_BYTES;
-          tma_load_4d(q, &tmQ, &q_full[qs], 0, i * BQ, h, b);
-          tma_load_4d(q + Cfg::QT_BYTES, &tmdO, &q_full[qs], 0, i * BQ, h, b);
-          // the tile's per-query statistics (lse2, sD: 512 B each) ride on the same barrier
-          const int64_t so = ((int64_t)b * p.H + h) * p.S + i * BQ;
-          float* st = sStat + qs * (2 * BQ);
-          bulk_load_1d(st, p.lse2 + so, BQ * 4, &q_full[qs]);
-          bulk_load_1d(st + BQ, p.sD + so, BQ * 4, &q_full[qs]);
+          tma_load_4d(q, &tmQ, &q_full[qs], 0, i * BQS, h, b);
+          tma_load_4d(q + Cfg::QT_BYTES, &tmdO, &q_full[qs], 0, i * BQS, h, b);
+          // the sub-tile's per-query statistics (lse2, sD: 256 B each) ride on the same barrier
+          const int64_t so = ((int64_t)b * p.H + h) * p.S + i * BQS;
+          float* st = sStat + qs * (2 * BQS);
+          bulk_load_1d(st, p.lse2 + so, BQS * 4, &q_full[qs]);
+          bulk_load_1d(st + BQS, p.sD + so, BQS * 4, &q_full[qs]);
           if (++qs == Cfg::QST) { qs = 0; qph ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc_s = make_idesc_f16(128, BQ, 0, 0);   // S^T, dP^T: M=keys, N=queries, K=DH
+      const uint32_t idesc_s = make_idesc_f16(128, BQS, 0, 0);  // S^T, dP^T: M=keys, N=queries, K=DH
       const uint32_t idesc_g = make_idesc_f16(128, DH, 0, 1);   // dV, dK: M=keys, N=DH, K=queries
-      int qs = 0; uint32_t qph = 0;  // (Q, dO) ring position of the next S issue
-      int gq = 0;                    // (Q, dO) ring position of the next dV/dK
-      int sc = 0;                    // S issues (s_full phase)
-      int pc = 0;                    // P/dS buffer uses
+      // score-issue cursor (runs two sub-tiles ahead of the gradient cursor, across items)
+      int s_item = blockIdx.x, s_sub = 0, s_n = 0;
+      int qs = 0; uint32_t qph = 0;  // (Q, dO) ring position of the next score issue
+      int sc = 0;                    // score issues (buffer pair sc & 1)
+      auto issue_s = [&]() {
+        if (s_item >= items) return;
+        int b, h, kt;
+        bwd_item(s_item, nk, p.H, b, h, kt);
+        const int nt = nqs - (p.causal ? kt * (BKV / BQS) : 0);
+        const int kvs = s_n & 1;
+        if (s_sub == 0) mbar_wait(&kv_full[kvs], (s_n >> 1) & 1);
+        mbar_wait(&q_full[qs], qph);
+        tc_fence_after();
+        const uint32_t ka = smem_u32(sKV + kvs * 2 * Cfg::KV_BYTES), va = ka + Cfg::KV_BYTES;
+        const uint32_t qa = smem_u32(sQ + qs * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
+        const int sb = sc & 1;
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t off = kk * 32;
+          mma_bf16(tmem + Cfg::ST_COL + sb * BQS, make_sdesc(ka + off, 16, 1024), make_sdesc(qa + off, 16, 1024),
+                   idesc_s, kk ? 1u : 0u);
+          mma_bf16(tmem + Cfg::DP_COL + sb * BQS, make_sdesc(va + off, 16, 1024), make_sdesc(oa + off, 16, 1024),
+                   idesc_s, kk ? 1u : 0u);
+        }
+        mma_commit(&s_full[sb]);
+        if (++qs == Cfg::QST) { qs = 0; qph ^= 1; }
+        ++sc;
+        if (++s_sub == nt) { s_sub = 0; s_item += gridDim.x; ++s_n; }
+      };
+      issue_s();
+      issue_s();
+      int gq = 0;  // (Q, dO) ring position of the next dV/dK
+      int pc = 0;  // sub-tiles whose gradients were issued (P/dS buffer pc & 1)
       int n = 0;
       for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
         int b, h, kt;
         bwd_item(item, nk, p.H, b, h, kt);
-        const int i0 = p.causal ? kt : 0;
-        const int niter = nq - i0;
+        const int nt = nqs - (p.causal ? kt * (BKV / BQS) : 0);
         const int kvs = n & 1;
-        mbar_wait(&kv_full[kvs], (n >> 1) & 1);
-        const uint32_t ka = smem_u32(sKV + kvs * 2 * Cfg::KV_BYTES), va = ka + Cfg::KV_BYTES;
-        auto issue_s = [&]() {
-          mbar_wait(&q_full[qs], qph);
-          tc_fence_after();
-          const uint32_t qa = smem_u32(sQ + qs * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
-#pragma unroll
-          for (int kk = 0; kk < DH / 16; ++kk) {
-            const uint32_t off = kk * 32;
-            mma_bf16(tmem + Cfg::ST_COL, make_sdesc(ka + off, 16, 1024), make_sdesc(qa + off, 16, 1024), idesc_s,
-                     kk ? 1u : 0u);
-            mma_bf16(tmem + Cfg::DP_COL, make_sdesc(va + off, 16, 1024), make_sdesc(oa + off, 16, 1024), idesc_s,
-                     kk ? 1u : 0u);
-          }
-          mma_commit(s_full);
-          if (++qs == Cfg::QST) { qs = 0; qph ^= 1; }
-          ++sc;
-        };
-        issue_s();
-        for (int t = 0; t < niter; ++t) {
+        for (int t = 0; t < nt; ++t) {
           const int pb = pc & 1;
-          mbar_wait(&p_full[pb], (pc >> 1) & 1);  // P^T / dS^T of tile t ready, S^T / dP^T read
-          tc_fence_after();
-          if (t + 1 < niter) issue_s();  // next scores overlap this tile's gradient MMAs
+          mbar_wait(&p_full[pb], (pc >> 1) & 1);  // P^T / dS^T of this sub-tile ready, its S^T / dP^T read
           if (t == 0) mbar_wait(kd_empty, (n & 1) ^ 1);  // previous item's dK / dV drained
           tc_fence_after();
           const uint32_t qa = smem_u32(sQ + gq * 2 * Cfg::QT_BYTES), oa = qa + Cfg::QT_BYTES;
-          const uint32_t pa = tmem + Cfg::PT_COL + pb * (BQ / 2);
+          const uint32_t pa = tmem + Cfg::PT_COL + pb * (BQS / 2);
           const uint32_t da = smem_u32(sDS + pb * Cfg::DS_BYTES);
 #pragma unroll
-          for (int kk = 0; kk < BQ / 16; ++kk) {
-            const int atom = kk / 4, sub = kk % 4;
+          for (int kk = 0; kk < BQS / 16; ++kk) {
             const uint32_t boff = kk * 2048;  // dO / Q as MN-major B (k = query rows)
             const uint32_t acc = (t | kk) ? 1u : 0u;
             mma_bf16_ts(tmem + Cfg::DV_COL, pa + kk * 8, make_sdesc(oa + boff, 128 * 128, 1024), idesc_g, acc);
-            mma_bf16(tmem + Cfg::DK_COL, make_sdesc(da + atom * (128 * 128) + sub * 32, 16, 1024),
-                     make_sdesc(qa + boff, 128 * 128, 1024), idesc_g, acc);
+            mma_bf16(tmem + Cfg::DK_COL, make_sdesc(da + kk * 32, 16, 1024), make_sdesc(qa + boff, 128 * 128, 1024),
+                     idesc_g, acc);
           }
           mma_commit(&p_empty[pb]);
           mma_commit(&q_empty[gq]);
           if (++gq == Cfg::QST) gq = 0;
           ++pc;
+          if (t == nt - 1) {
+            mma_commit(&kv_empty[kvs]);
+            mma_commit(kd_full);
+          }
+          issue_s();  // the scores two sub-tiles ahead go into the pair this sub-tile just released
         }
-        mma_commit(&kv_empty[kvs]);
-        mma_commit(kd_full);
       }
     }
     __syncwarp();
   } else {
     const int qd = warp & 3;
-    const int half = (warp - 2) >> 2;  // which 64 queries of the tile (= which atom of dS^T)
+    const int half = (warp - 2) >> 2;  // which 32 queries of the sub-tile
     const int r = qd * 32 + lane;      // key row within the tile
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
-    const bool issuer = qd == 0 && lane == 0;
-    int sc = 0, pc = 0, n = 0;
-    int qsl = 0;        // (Q, dO, statistics) ring position of the current tile
+    const bool issuer = warp == 2 && lane == 0;
+    int g = 0, n = 0;
+    int qsl = 0;        // (Q, dO, statistics) ring position of the current sub-tile
     uint32_t qslph = 0; // its phase
     for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
       int b, h, kt;
       bwd_item(item, nk, p.H, b, h, kt);
-      const int i0 = p.causal ? kt : 0;
-      const int niter = nq - i0;
+      const int i0 = p.causal ? kt * (BKV / BQS) : 0;
+      const int nt = nqs - i0;
       const int key = kt * BKV + r;
-      for (int t = 0; t < niter; ++t, ++sc, ++pc) {
-        const float* sl2 = sStat + qsl * (2 * BQ);
-        const float* ssd = sl2 + BQ;
+      for (int t = 0; t < nt; ++t, ++g) {
+        const float* sl2 = sStat + qsl * (2 * BQS) + half * 32;
+        const float* ssd = sl2 + BQS;
         mbar_wait(&q_full[qsl], qslph);  // the TMA-written statistics are visible to this thread
         if (++qsl == Cfg::QST) { qsl = 0; qslph ^= 1; }
-        const int q0 = (i0 + t) * BQ;
-        const int pb = pc & 1;
-        mbar_wait(s_full, sc & 1);
-        mbar_wait(&p_empty[pb], ((pc >> 1) & 1) ^ 1);
+        const int q0 = (i0 + t) * BQS;
+        const int buf = g & 1;
+        mbar_wait(&s_full[buf], (g >> 1) & 1);
+        mbar_wait(&p_empty[buf], ((g >> 1) & 1) ^ 1);
         tc_fence_after();
-        const bool diag = p.causal && (i0 + t) == kt;
-        uint8_t* drow = sDS + pb * Cfg::DS_BYTES + half * (128 * 128) + r * 128;
-#pragma unroll 1
-        for (int c = 0; c < 64; c += 32) {
-          const int qc = q0 + half * 64 + c;  // first query of this 32-column batch
-          uint32_t rs[32], rd[32];
-          tmem_ld32_nw(tmem + trow + Cfg::ST_COL + half * 64 + c, rs);
-          tmem_ld32_nw(tmem + trow + Cfg::DP_COL + half * 64 + c, rd);
-          float l2[32], sd[32];  // broadcast reads of the staged statistics
+        const bool diag = p.causal && q0 < kt * BKV + BKV;  // the sub-tile overlaps the key range
+        const int qc = q0 + half * 32;  // first query of this thread's 32 columns
+        uint32_t rs[32], rd[32];
+        tmem_ld32_nw(tmem + trow + Cfg::ST_COL + buf * BQS + half * 32, rs);
+        tmem_ld32_nw(tmem + trow + Cfg::DP_COL + buf * BQS + half * 32, rd);
+        float l2[32], sd[32];  // broadcast reads of the staged statistics
 #pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            const float4 a4 = reinterpret_cast<const float4*>(sl2 + half * 64 + c)[i];
-            const float4 d4 = reinterpret_cast<const float4*>(ssd + half * 64 + c)[i];
-            l2[4 * i] = a4.x; l2[4 * i + 1] = a4.y; l2[4 * i + 2] = a4.z; l2[4 * i + 3] = a4.w;
-            sd[4 * i] = d4.x; sd[4 * i + 1] = d4.y; sd[4 * i + 2] = d4.z; sd[4 * i + 3] = d4.w;
-          }
-          tmem_wait_ld();
-          uint32_t pk[16], dk[16];
-#pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            float pr[2], dr[2];
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-              const int e = 2 * i + u;
-              float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, -l2[e]));
-              if (diag && key > qc + e) pv = 0.f;
-              pr[u] = pv;
-              dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, -sd[e]);
-            }
-            __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
-            __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
-            pk[i] = *reinterpret_cast<uint32_t*>(&a2);
-            dk[i] = *reinterpret_cast<uint32_t*>(&b2);
-          }
-          // P^T: this thread's 32 queries -> 16 TMEM columns (bf16 pairs) of P buffer pb
-          uint32_t pk32[32];
-#pragma unroll
-          for (int i = 0; i < 16; ++i) pk32[i] = pk[i];
-          asm volatile(
-              "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
-                  tmem + trow + Cfg::PT_COL + pb * (BQ / 2) + half * 32 + c / 2),
-              "r"(pk32[0]), "r"(pk32[1]), "r"(pk32[2]), "r"(pk32[3]), "r"(pk32[4]), "r"(pk32[5]), "r"(pk32[6]),
-              "r"(pk32[7]), "r"(pk32[8]), "r"(pk32[9]), "r"(pk32[10]), "r"(pk32[11]), "r"(pk32[12]), "r"(pk32[13]),
-              "r"(pk32[14]), "r"(pk32[15])
-              : "memory");
-          const int ch0 = c / 8;  // 16-byte chunk of the 128-byte dS^T row
-#pragma unroll
-          for (int u = 0; u < 4; ++u)
-            *reinterpret_cast<uint4*>(drow + (((ch0 + u) ^ (r & 7)) << 4)) =
-                make_uint4(dk[4 * u], dk[4 * u + 1], dk[4 * u + 2], dk[4 * u + 3]);
+        for (int i = 0; i < 8; ++i) {
+          const float4 a4 = reinterpret_cast<const float4*>(sl2)[i];
+          const float4 d4 = reinterpret_cast<const float4*>(ssd)[i];
+          l2[4 * i] = a4.x; l2[4 * i + 1] = a4.y; l2[4 * i + 2] = a4.z; l2[4 * i + 3] = a4.w;
+          sd[4 * i] = d4.x; sd[4 * i + 1] = d4.y; sd[4 * i + 2] = d4.z; sd[4 * i + 3] = d4.w;
         }
+        tmem_wait_ld();
+        uint32_t pk[16], dk[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          float pr[2], dr[2];
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const int e = 2 * i + u;
+            float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, -l2[e]));
+            if (diag && key > qc + e) pv = 0.f;
+            pr[u] = pv;
+            dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, -sd[e]);
+          }
+          __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
+          pk[i] = *reinterpret_cast<uint32_t*>(&a2);
+          dk[i] = *reinterpret_cast<uint32_t*>(&b2);
+        }
+        // P^T: this thread's 32 queries -> 16 TMEM columns (bf16 pairs) of P buffer `buf`
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+                tmem + trow + Cfg::PT_COL + buf * (BQS / 2) + half * 16),
+            "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]), "r"(pk[8]),
+            "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]), "r"(pk[15])
+            : "memory");
+        // dS^T: the row's 16-byte chunks 4*half .. 4*half+3 of the 128-byte (64-query) row, swizzled
+        uint8_t* drow = sDS + buf * Cfg::DS_BYTES + r * 128;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          *reinterpret_cast<uint4*>(drow + (((4 * half + u) ^ (r & 7)) << 4)) =
+              make_uint4(dk[4 * u], dk[4 * u + 1], dk[4 * u + 2], dk[4 * u + 3]);
         tmem_wait_st();
         tc_fence_before();
-        if (issuer) bulk_wait_read<0>();  // the previous tile's dS^T store has left shared memory
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_arrive_local(&p_full[pb]);
-        asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");  // the half's 128 rows are written
+        mbar_arrive_local(&p_full[buf]);
+        // the whole (128 keys x 64 queries) box is written: one TMA store.  The store of the
+        // sub-tile two back (same buffer) was waited for at the previous sub-tile's store, before
+        // this barrier's previous instance, so the buffer was free when it was written above.
+        if (issuer) bulk_wait_read<0>();
+        asm volatile("bar.sync 1, 256;" ::: "memory");
         if (issuer) {
-          tma_store_4d(&tmdS, sDS + pb * Cfg::DS_BYTES + half * (128 * 128), q0 + half * 64, kt * BKV, h, b);
+          tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES, q0, kt * BKV, h, b);
           bulk_commit();
         }
       }
@@ -912,49 +922,39 @@ __global__ void __launch_bounds__(THREADS, 1)
 }
 
 // sD[b, h, q] = scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = lse * log2(e): the
-// per-query terms of dS = P (dP - D) in the forms the backward's FFMAs take.  One warp per token:
-// the token's dO and O rows are read once, contiguously (lane l takes elements 8l.. of every
-// 256-element chunk; 256 % dh == 0, so a chunk holds whole heads), and each head's dh/8 lanes
-// reduce with shuffles in a fixed order.
+// per-query terms of dS = P (dP - D) in the forms the backward's FFMAs take.  One thread per 8
+// consecutive elements of the [tokens, d] rows (one 16-byte load of dO and of O, fully coalesced,
+// a few registers, so the grid is many small resident blocks); each head's dh/8 adjacent lanes
+// reduce their 8-term partial sums with shuffles in a fixed order.
 __global__ void __launch_bounds__(256) attn_bwd_prep(int64_t ntok, int S, int H, int dh, float scale,
                                                      const __nv_bfloat16* __restrict__ dO,
                                                      const __nv_bfloat16* __restrict__ O, const float* __restrict__ lse,
                                                      float* __restrict__ sD, float* __restrict__ lse2) {
-  const int lane = threadIdx.x & 31;
-  const int64_t tok = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
-  if (tok >= ntok) return;
-  const int d = H * dh, lph = dh / 8;  // lanes per head
-  const int64_t bseq = tok / S, q = tok % S;
-  const uint4* a = reinterpret_cast<const uint4*>(dO + tok * d);
-  const uint4* o = reinterpret_cast<const uint4*>(O + tok * d);
-  for (int j0 = 0; 256 * j0 < d; j0 += 8) {  // 2048 elements per round, every load in flight at once
-    uint4 xa[8], ya[8];
+  const int d = H * dh, lph = dh / 8;  // lanes per head (8 or 16: a head never straddles a warp)
+  const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;  // 8-element vector index
+  const int64_t nvec = ntok * (d / 8);
+  const bool in = v < nvec;
+  const int64_t tok = in ? v / (d / 8) : 0;
+  const int e = in ? (int)(v - tok * (d / 8)) * 8 : 0;
+  float s = 0.f;
+  if (in) {
+    const uint4 xa = __ldg(reinterpret_cast<const uint4*>(dO) + v);
+    const uint4 ya = __ldg(reinterpret_cast<const uint4*>(O) + v);
+    const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&xa);
+    const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&ya);
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int e = 256 * (j0 + j) + 8 * lane;
-      xa[j] = e < d ? a[e / 8] : make_uint4(0, 0, 0, 0);
-      ya[j] = e < d ? o[e / 8] : make_uint4(0, 0, 0, 0);
+    for (int k = 0; k < 4; ++k) {
+      const float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
+      s += fx.x * fy.x + fx.y * fy.y;
     }
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int e = 256 * (j0 + j) + 8 * lane;
-      if (256 * (j0 + j) >= d) break;
-      const __nv_bfloat162* xp = reinterpret_cast<const __nv_bfloat162*>(&xa[j]);
-      const __nv_bfloat162* yp = reinterpret_cast<const __nv_bfloat162*>(&ya[j]);
-      float s = 0.f;
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const float2 fx = __bfloat1622float2(xp[k]), fy = __bfloat1622float2(yp[k]);
-        s += fx.x * fy.x + fx.y * fy.y;
-      }
-      for (int w = lph / 2; w > 0; w >>= 1) s += __shfl_xor_sync(0xffffffffu, s, w);
-      if (e < d && (lane % lph) == 0) {
-        const int h = e / dh;
-        const int64_t i = (bseq * H + h) * S + q;
-        sD[i] = scale * s;
-        lse2[i] = lse[i] * 1.4426950408889634f;
-      }
-    }
+  }
+  for (int w = lph / 2; w > 0; w >>= 1) s += __shfl_xor_sync(0xffffffffu, s, w);
+  if (in && (threadIdx.x % lph) == 0) {
+    const int h = e / dh;
+    const int64_t bseq = tok / S, q = tok % S;
+    const int64_t i = (bseq * H + h) * S + q;
+    sD[i] = scale * s;
+    lse2[i] = lse[i] * 1.4426950408889634f;
   }
 }
 }  // namespace attn
@@ -998,7 +998,7 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   }
   check_launch("attn_fwd_kernel");
   // algorithmic FLOPs of the attention contractions (QK^T and PV, causal or not)
-  g_prof.end(PROF_GEMM, e0, st, 4.0 * b * H * (double)S * S * dh);
+  g_prof.end(PROF_ATTN, e0, st, 4.0 * b * H * (double)S * S * dh);
   return true;
 }
 
@@ -1019,7 +1019,7 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   float* lse2 = sD + align_up((uint64_t)b * H * S * 4, 256) / 4;
   const float scale = 1.0f / std::sqrt((float)dh);
   const int e0 = g_prof.begin(st);
-  attn_bwd_prep<<<(unsigned)ceil_div(b * S, 8), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
+  attn_bwd_prep<<<(unsigned)ceil_div(b * S * (d / 8), 256), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
                                                              static_cast<const __nv_bfloat16*>(O), lse, sD, lse2);
   check_launch("attn_bwd_prep");
   if (causal) HM_CUDA(cudaMemsetAsync(dst, 0, (size_t)b * H * S * S * 2, st));  // key tiles never visited by a query tile
@@ -1053,15 +1053,19 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
       HM_CUDA(cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev));
     }
     const int64_t items = (int64_t)(S / BKV) * H * b;
-    attn_bwd_persistent<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq, mk, mv, mo, mds,
-                                                                                                    p, (int)b);
+    // Q / dO in 64-query sub-tiles
+    CUtensorMap mq64, mo64;
+    tcx::make_map_4d(&mq64, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BwdPCfg::BQS);
+    tcx::make_map_4d(&mo64, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BwdPCfg::BQS);
+    attn_bwd_persistent<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq64, mk, mv, mo64,
+                                                                                                    mds, p, (int)b);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }
     attn_bwd_kernel<128><<<grid, THREADS, BwdCfg<128>::SMEM, st>>>(mq, mk, mv, mo, mds, p);
   }
   check_launch("attn_bwd_kernel");
-  g_prof.end(PROF_GEMM, e0, st, 8.0 * b * H * (double)S * S * dh);  // S^T, dP^T, dV, dK contractions
+  g_prof.end(PROF_ATTN, e0, st, 8.0 * b * H * (double)S * S * dh);  // S^T, dP^T, dV, dK contractions
   // dQ = dS K: A(m=q, k=key) = dS^T[key][q] (MN-major), B(n=e, k=key) = K[key][e] (MN-major)
   hk_gemm_args a = gemm_args(1, S, dh, S);
   a.nz0 = H; a.nz1 = (int)b;

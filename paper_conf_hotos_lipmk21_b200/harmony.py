@@ -65,8 +65,8 @@ class harmony_plan_summary(C.Structure):
 
 
 class harmony_kernel_profile(C.Structure):
-    _fields_ = [("launches", C.c_uint64 * 5), ("seconds", C.c_double * 5), ("work", C.c_double * 5)]
-    CLASSES = ("gemm", "adam", "layernorm", "softmax", "other")
+    _fields_ = [("launches", C.c_uint64 * 6), ("seconds", C.c_double * 6), ("work", C.c_double * 6)]
+    CLASSES = ("gemm", "adam", "layernorm", "softmax", "other", "attention")
 
     def as_dict(self):
         return {c: dict(launches=self.launches[i], seconds=self.seconds[i], work=self.work[i])

@@ -264,7 +264,10 @@ def test_fused_attention_forward(S, dh, h, b, causal):
 
 
 @pytest.mark.parametrize("S,dh,h,b,causal", [(128, 64, 2, 1, 0), (256, 64, 2, 2, 1), (512, 64, 2, 1, 0),
-                                             (384, 128, 2, 1, 1), (512, 64, 1, 1, 1)])
+                                             (384, 128, 2, 1, 1), (512, 64, 1, 1, 1),
+                                             # more (key tile, head, sequence) items than SMs: every
+                                             # pipeline counter of the persistent kernel wraps across items
+                                             (512, 64, 16, 4, 0), (512, 64, 16, 4, 1)])
 def test_fused_attention_backward(S, dh, h, b, causal):
     """dQKV of the fused backward (S^T, dP^T in TMEM; P^T, dS^T in smem; dQ by GEMM on dS^T) vs the
     oracle's attention_bwd on the same inputs."""

@@ -1,4 +1,4 @@
-"""Fused attention on the cfg2 per-microbatch shape (b=8 sequences, S=512, 16 heads, dh=64).
+"""Fused attention on the cfg2 per-microbatch shape (b=16 sequences, S=512, 16 heads, dh=64).
 
     python tools/attn_bench.py [--reps 20] [--causal 0]
 
@@ -24,7 +24,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--causal", type=int, default=0)
-    ap.add_argument("--b", type=int, default=8)
+    ap.add_argument("--b", type=int, default=16)
     ap.add_argument("--S", type=int, default=512)
     ap.add_argument("--h", type=int, default=16)
     ap.add_argument("--dh", type=int, default=64)

@@ -4,7 +4,7 @@
         python tools/profile_step.py --layers 2 --steps 2
 
 Same per-layer shapes and launch configuration as `bench.py` (cfg2: d=1024, h=16, S=512,
-m=8 x b=8, stash policy 2); `--layers` trims the stack depth so the list stays short (every layer
+m=4 x b=16 by default, stash policy 2); `--layers` trims the stack depth so the list stays short (every layer
 runs the identical kernel sequence).  Eager issue (HARMONY_NO_GRAPH=1 is set) so each kernel is
 one launch record.
 """
@@ -27,12 +27,13 @@ def main():
     ap.add_argument("--layers", type=int, default=2)
     ap.add_argument("--steps", type=int, default=2)
     ap.add_argument("--policy", type=int, default=2)
+    ap.add_argument("--microbatches", type=int, default=4)
     a = ap.parse_args()
     descs = synth.transformer_stack(a.layers, 1024, 16, 512, False)
     params = synth.gen_params(descs, 1)
     X, T = synth.gen_batch(descs, 64, 1, 1)
     Xd, Td = torch.tensor(X, device="cuda"), torch.tensor(T, device="cuda")
-    with H.Harmony(descs, params, microbatches=8, microbatch_size=8, precision=1, stash_policy=a.policy,
+    with H.Harmony(descs, params, microbatches=a.microbatches, microbatch_size=64 // a.microbatches, precision=1, stash_policy=a.policy,
                    hbm_cap_bytes=8 << 30, lr=1e-4) as h:
         for _ in range(a.steps):
             loss, st = h.step(Xd, Td)
