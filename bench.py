@@ -42,9 +42,9 @@ WORKLOADS = {
     "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=4 x b=16), bf16/fp32-master Adam, "
                       "HBM cap 8 GiB/GPU", model="bert-large-like-preLN", descs=lambda: synth.transformer_stack(24, 1024, 16, 512, False),
                  per_gpu_batch=64, m=4, cap=8 << 30, S=512),
-    "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=4 x b=2), bf16/fp32-master Adam, "
+    "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=2 x b=4), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
-                 per_gpu_batch=8, m=4, cap=16 << 30, S=1024),
+                 per_gpu_batch=8, m=2, cap=16 << 30, S=1024),
     "cfg5": dict(name="cfg5: one 16384 x 16384 x 65536 (M x N x K) bf16 GEMM fwd+bwd, operator split along K into "
                       "8 row-chunk tile subtasks per GPU (harmony_split_gemm_*)", model="gemm-16384x16384x65536",
                  M=16384, N=16384, K=65536, chunks=8, S=1, per_gpu_batch=1, m=1, cap=0),

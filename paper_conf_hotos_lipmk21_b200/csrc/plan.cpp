@@ -364,9 +364,27 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
           uint64_t sz = align_up(p.layers[l].wc_bytes, ALIGN);
           if (sz <= room) { p.layers[l].wc_res = 0; room -= sz; }
         }
-        for (int l = L - 1; l >= 0; --l) {  // master/m/v: 2 B saved per byte
-          uint64_t sz = align_up(p.layers[l].state_bytes, ALIGN);
-          if (sz <= room) { p.layers[l].state_res = 0; room -= sz; }
+        // master/m/v: 2 B saved per byte, both in the backward (swap-in before the JIT update,
+        // swap-out after it).  With equal per-layer state sizes the streamed layers are spread
+        // evenly over the backward order instead of being the last ones updated: each streamed
+        // layer's swap-in then overlaps the backward of the resident layers before it, rather
+        // than a run of consecutive updates waiting on the host link.
+        bool uniform = true;
+        for (int l = 1; l < L; ++l) uniform = uniform && p.layers[l].state_bytes == p.layers[0].state_bytes;
+        const uint64_t ssz = align_up(p.layers[0].state_bytes, ALIGN);
+        if (uniform && ssz > 0 && (uint64_t)L * ssz > room) {
+          const int keep = (int)std::min<uint64_t>(room / ssz, (uint64_t)L);
+          const int nstream = L - keep;
+          // backward position j (0 = layer L-1) is streamed iff floor((j+1) n / L) > floor(j n / L)
+          for (int j = 0; j < L; ++j) {
+            const bool streamed = (int64_t)(j + 1) * nstream / L > (int64_t)j * nstream / L;
+            if (!streamed) { p.layers[L - 1 - j].state_res = 0; room -= ssz; }
+          }
+        } else {
+          for (int l = L - 1; l >= 0; --l) {
+            uint64_t sz = align_up(p.layers[l].state_bytes, ALIGN);
+            if (sz <= room) { p.layers[l].state_res = 0; room -= sz; }
+          }
         }
       }
       for (int l = L - 1; l >= 0; --l)  // stash: LIFO (consumed first in the backward)

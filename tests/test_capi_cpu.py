@@ -174,6 +174,30 @@ def test_stash_residency_is_lifo():
         assert max(l for l, _ in spilled) < 7
 
 
+@pytest.mark.parametrize("extra", [6, 8, 10, 12])
+def test_streamed_state_is_spread_over_the_backward(extra):
+    """With equal per-layer state, the layers whose master/m/v stream through the host are spread
+    evenly over the backward order (each one's swap-in overlaps the backward of resident layers
+    before it) instead of being the last ones updated; the plan stays hazard free."""
+    L = 12
+    descs = synth.transformer_stack(L, 256, 4, 128, True)
+    kw = dict(microbatches=2, microbatch_size=2, precision=1, stash_policy=2)
+    base = min_cap(descs, **kw)
+    state = 12 * (12 * 256 * 256 + 13 * 256)
+    s, ops = plan(descs, **dict(kw, hbm_cap_bytes=base + extra * state))
+    streamed = sorted({o["l"] for o in ops if o["kind"] == "H2D" and o["cat"] == "state"}, reverse=True)
+    n = len(streamed)
+    assert 0 < n < L, streamed
+    padded = next(o["bytes"] for o in ops if o["kind"] == "H2D" and o["cat"] == "state")
+    assert s.resident_state_bytes == (L - n) * padded
+    expect = sorted([L - 1 - j for j in range(L) if (j + 1) * n // L > j * n // L], reverse=True)
+    assert streamed == expect
+    pos = [L - 1 - l for l in streamed]  # backward positions
+    gaps = [b - a for a, b in zip(pos, pos[1:])]
+    assert not gaps or max(gaps) - min(gaps) <= 1, gaps
+    assert s.hazards == 0
+
+
 def test_config_validation_errors():
     with pytest.raises(H.HarmonyError) as e:
         plan([synth.LayerDesc(1, 64, 64, n_heads=5, seq_len=8)], microbatches=1, microbatch_size=1)

@@ -91,10 +91,11 @@ def main():
     ap.add_argument("--workload", default="cfg3", choices=[k for k in bench.WORKLOADS if k != "cfg5"])
     ap.add_argument("--stash-policy", type=int, default=2)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--microbatches", type=int, default=0)
     a = ap.parse_args()
     wl = bench.WORKLOADS[a.workload]
     descs = wl["descs"]()
-    B, m = wl["per_gpu_batch"], wl["m"]
+    B, m = wl["per_gpu_batch"], a.microbatches or wl["m"]
     prec = wl.get("precision", 1)
     params = synth.gen_params(descs, prec)
     X, T = synth.gen_batch(descs, B, 1, prec)
