@@ -1,19 +1,19 @@
 // attention.cu — fused multi-head attention forward on tcgen05 (SURVEY §8(a) rows a4/a5, K4 + K9).
 //
-// One CTA per (128-query tile, head, sequence).  The scores never touch HBM: S = Q K^T lands in
-// TMEM, four softmax warps (one query row per thread) read it with tcgen05.ld, and the
-// probabilities go to shared memory in the UMMA K-major 128B-swizzled layout where they are the A
-// operand of O += P V (accumulated in TMEM).  Softmax is exact and two-pass over the key tiles:
-// pass 1 computes each row's max and sum (online, scalars only), pass 2 recomputes S and
-// normalises P with the final statistics, so O needs no rescaling (1.5x the QK^T FLOPs of a
-// one-pass kernel, in exchange for no TMEM read-modify-write of O).  Pass 1 needs only the row max;
-// pass 2 forms P = exp(s - max) in (0, 1], accumulates the row sum beside it and O is divided by
-// the sum in the epilogue.  Outputs: C (bf16, heads
+// Persistent CTAs loop over (128-query tile, head, sequence) items.  The scores never touch HBM:
+// S = Q K^T lands in TMEM, eight softmax warps (two per TMEM lane quadrant, 64 keys each) read it
+// with tcgen05.ld, and the bf16 probabilities are stored back into TMEM where they are the A
+// operand of O += P V (accumulated in TMEM).  One pass over the key tiles with a lazily raised
+// running max: S is read from TMEM once per tile (the TMEM read bandwidth, not the tensor pipe, is
+// what bounds a dh = 64 tile), O is rescaled in TMEM only when a tile raises the row max by more
+// than 2^8, and O is divided by the row sum in the epilogue.  Outputs: C (bf16, heads
 // interleaved in [T, d]) and the row log-sum-exp (fp32 [b, h, S]) the backward needs.
 // Numerics match the unfused path's reading c11: P = softmax(scale * Q K^T) with causal rows
 // masked to exactly 0 above the diagonal.
 #include <cuda.h>
 #include <cudaTypedefs.h>
+
+#include <type_traits>
 
 #include "../common.hpp"
 #include "kernels.hpp"
@@ -41,8 +41,8 @@ struct FwdCfg {
   static constexpr int K_BYTES = BKV * DH * 2;
   static constexpr int V_BYTES = BKV * DH * 2;          // 2 key-atoms x DH/64 MN-chunks of 8 KB
   static constexpr int O_BYTES = BQ * DH * 2;           // output staging (DH/64 boxes of 64 columns)
-  static constexpr int QST = 2, KST = DH == 64 ? 4 : 2, VST = DH == 64 ? 4 : 2;
-  static constexpr int SMEM = QST * Q_BYTES + KST * K_BYTES + VST * V_BYTES + O_BYTES + 1024 + 256 + 2 * BQ * 4;
+  static constexpr int QST = DH == 64 ? 2 : 1, KST = DH == 64 ? 4 : 2, VST = DH == 64 ? 4 : 2;
+  static constexpr int SMEM = QST * Q_BYTES + KST * K_BYTES + VST * V_BYTES + O_BYTES + 1024 + 256 + 2 * BQ * 4 + 4 * BQ * 4;
   static constexpr int S_COLS = BKV;                    // fp32 accumulator columns per S buffer
   static constexpr int O_COL = 2 * BKV;                 // O after the two S buffers
   static constexpr int P_COL = 2 * BKV + DH;            // two P buffers (bf16 pairs: BKV/2 columns each)
@@ -58,12 +58,21 @@ struct FwdParams {
   float* lse;        // [b, H, S]
 };
 
-// work item -> (sequence, head, query tile); query tiles in decreasing order so that, when causal,
-// the long rows are handed out first
-__device__ __forceinline__ void fwd_item(int item, int nq, int H, int& b, int& h, int& qt) {
-  qt = nq - 1 - item % nq;
-  h = (item / nq) % H;
-  b = item / (nq * H);
+// Persistent item order.  Items are numbered by decreasing work (causal: query tile nq-1 first,
+// whose rows see every key tile) and dealt to the CTAs in a snake (round r: CTA c takes
+// r*G + c, or r*G + G-1-c on odd rounds), so every CTA gets a mix of long and short items.  (A
+// plain stride-G walk hands CTA c only items with one tile index when G is a multiple of the
+// tile count — 148 = 37 * 4 — which left the causal kernels as slow as the non-causal ones.)
+__device__ __forceinline__ int snake(int r) {
+  return r * (int)gridDim.x + ((r & 1) ? (int)(gridDim.x - 1 - blockIdx.x) : (int)blockIdx.x);
+}
+// sorted item -> (sequence, head, query tile)
+__device__ __forceinline__ void fwd_item(int item, int nq, int H, int B, int& b, int& h, int& qt) {
+  const int hb = H * B;
+  qt = nq - 1 - item / hb;
+  const int rem = item % hb;
+  h = rem % H;
+  b = rem / H;
 }
 
 // Persistent: one CTA per SM loops over the (query tile, head, sequence) items.  All pipeline
@@ -100,6 +109,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(o_empty + 1);
   static_assert((14 + 2 * Cfg::KST + 2 * Cfg::VST) * 8 + 4 <= 256, "barrier area");
   float(*sm_x)[BQ] = reinterpret_cast<float(*)[BQ]>(reinterpret_cast<uint8_t*>(bars) + 256);  // [2][BQ] row stats
+  float(*sm_t)[2][BQ] = reinterpret_cast<float(*)[2][BQ]>(reinterpret_cast<uint8_t*>(bars) + 256 + 2 * BQ * 4);  // [2][2][BQ]
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int nq = p.S / BQ;
@@ -129,40 +139,36 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      // ===== TMA producer: per item Q once, K tiles for both passes, V tiles for pass 2 =====
+      // ===== TMA producer: per item Q once, then a K and a V tile per key tile =====
       int ks = 0; uint32_t kph = 0;
       int vs = 0; uint32_t vph = 0;
       int n = 0;
-      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+      for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
         int b, h, qt;
-        fwd_item(item, nq, p.H, b, h, qt);
+        fwd_item(item, nq, p.H, p.B, b, h, qt);
         const int ntiles = p.causal ? qt + 1 : nq;
-        const int qs = n & 1;
-        mbar_wait(&q_empty[qs], ((n >> 1) & 1) ^ 1);
+        const int qs = n % Cfg::QST;
+        mbar_wait(&q_empty[qs], ((n / Cfg::QST) & 1) ^ 1);
         mbar_expect_tx(&q_full[qs], Cfg::Q_BYTES);
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a)
           tma_load_4d(sQ + qs * Cfg::Q_BYTES + a * (BQ * 128), &tmQ, &q_full[qs], a * 64, qt * BQ, h, b);
-        for (int pass = 0; pass < 2; ++pass) {
-          for (int j = 0; j < ntiles; ++j) {
-            mbar_wait(&k_empty[ks], kph ^ 1);
-            mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
+        for (int j = 0; j < ntiles; ++j) {
+          mbar_wait(&k_empty[ks], kph ^ 1);
+          mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
 #pragma unroll
-            for (int a = 0; a < DH / 64; ++a)
-              tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
-            if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
-            if (pass == 1) {
-              mbar_wait(&v_empty[vs], vph ^ 1);
-              mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
+          for (int a = 0; a < DH / 64; ++a)
+            tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
+          if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
+          mbar_wait(&v_empty[vs], vph ^ 1);
+          mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
 #pragma unroll
-              for (int ka = 0; ka < 2; ++ka)
+          for (int ka = 0; ka < 2; ++ka)
 #pragma unroll
-                for (int c = 0; c < DH / 64; ++c)
-                  tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
-                              j * BKV + ka * 64, h, b);
-              if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
-            }
-          }
+            for (int c = 0; c < DH / 64; ++c)
+              tma_load_4d(sV + vs * Cfg::V_BYTES + ka * (DH / 64) * 8192 + c * 8192, &tmV, &v_full[vs], c * 64,
+                          j * BKV + ka * 64, h, b);
+          if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
         }
       }
     }
@@ -178,12 +184,12 @@ __global__ void __launch_bounds__(THREADS, 1)
       int it = 0;  // S-buffer uses
       int pc = 0;  // P-buffer uses
       int n = 0;
-      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+      for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
         int b, h, qt;
-        fwd_item(item, nq, p.H, b, h, qt);
+        fwd_item(item, nq, p.H, p.B, b, h, qt);
         const int ntiles = p.causal ? qt + 1 : nq;
-        const int qs = n & 1;
-        mbar_wait(&q_full[qs], (n >> 1) & 1);
+        const int qs = n % Cfg::QST;
+        mbar_wait(&q_full[qs], (n / Cfg::QST) & 1);
         const uint32_t qa = smem_u32(sQ + qs * Cfg::Q_BYTES);
         auto issue_s = [&]() {
           const int sb = it & 1;
@@ -203,8 +209,7 @@ __global__ void __launch_bounds__(THREADS, 1)
           if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
           ++it;
         };
-        for (int j = 0; j < ntiles; ++j) issue_s();  // pass 1
-        // pass 2: S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
+        // S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
         issue_s();
         for (int j = 0; j < ntiles; ++j) {
           if (j + 1 < ntiles) issue_s();
@@ -240,65 +245,81 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int r = qd * 32 + lane;        // row within the tile
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
     const bool issuer = qd == 0 && lane == 0;  // of this half's TMA store of O
-    int it = 0, pc = 0, n = 0;
-    for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+    int it = 0, pc = 0, n = 0, tp = 0;
+    for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
       int b, h, qt;
-      fwd_item(item, nq, p.H, b, h, qt);
+      fwd_item(item, nq, p.H, p.B, b, h, qt);
       const int ntiles = p.causal ? qt + 1 : nq;
       const int qrow = qt * BQ + r;  // query index within the sequence
+      // ---- one pass over the key tiles (online softmax with lazy rescaling): the row's running
+      // max m is raised only when a tile's max exceeds it by more than 8 (log2 units of the
+      // scaled scores), so P = 2^((s - m) scale log2e) stays in (0, 256] and O (in TMEM) is
+      // rescaled only on those rare raises; O and the row sum l carry the same shift, so O / l and
+      // the LSE are the softmax of reading c11 whatever m ends up being.
       float m = -INFINITY;
-      // ---- pass 1: row max only (no exponentials).  A thread's 64 columns come in one batch of
-      // TMEM loads and reduce in four independent chains (ILP); only the diagonal tile is masked.
-      for (int j = 0; j < ntiles; ++j, ++it) {
-        const int sb = it & 1;
+      float2 l2a = make_float2(0.f, 0.f), l2b = make_float2(0.f, 0.f);  // row-sum partials
+      // one key tile; DIAG (the causal diagonal tile) is a compile-time copy of the body, so the
+      // other tiles carry no masking instructions at all (masked scores are -inf, whose
+      // exponential is exactly 0)
+      auto tile = [&](int j, auto diag_tag) {
+        constexpr bool DIAG = decltype(diag_tag)::value;
+        const int sb = it & 1, pb = pc & 1;
         mbar_wait(&s_full[sb], (it >> 1) & 1);
         tc_fence_after();
-        const bool diag = p.causal && j == qt;
         float v[64];
         tmem_ld64(tmem + trow + sb * Cfg::S_COLS + cb, v);
         tc_fence_before();
         mbar_arrive_local(&s_empty[sb]);  // S is in registers: the MMA may overwrite the buffer
-        if (diag) {
+        if constexpr (DIAG) {
           const int lim = qrow - (j * BKV + cb);  // keys cb + i with i <= lim are visible
 #pragma unroll
           for (int i = 0; i < 64; ++i)
             if (i > lim) v[i] = -INFINITY;
         }
-        float m4[4] = {m, -INFINITY, -INFINITY, -INFINITY};
+        float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
         for (int i = 0; i < 64; ++i) m4[i & 3] = fmaxf(m4[i & 3], v[i]);
-        m = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
-      }
-      sm_x[half][r] = m;
-      asm volatile("bar.sync 1, 256;" ::: "memory");
-      m = fmaxf(sm_x[0][r], sm_x[1][r]);  // the row max over all keys (the diagonal key is always valid)
-      // ---- pass 2: P = 2^((s - m) scale log2e) in (0, 1] (bf16) into shared memory, swizzled
-      // K-major (A operand of O += P V); the row sum accumulates alongside, O is divided by it at the end
-      const float ms = m * p.scale_log2;
-      float l4[4] = {0.f, 0.f, 0.f, 0.f};
-      for (int j = 0; j < ntiles; ++j, ++it, ++pc) {
-        const int sb = it & 1, pb = pc & 1;
-        mbar_wait(&s_full[sb], (it >> 1) & 1);
-        tc_fence_after();
-        const bool diag = p.causal && j == qt;
-        float v[64];
-        tmem_ld64(tmem + trow + sb * Cfg::S_COLS + cb, v);
-        tc_fence_before();
-        mbar_arrive_local(&s_empty[sb]);
-        const int lim = diag ? qrow - (j * BKV + cb) : 64;
+        float tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
+        // the other half of the row (the partner warp of this lane quadrant)
+        sm_t[tp][half][r] = tm;
+        asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
+        tm = fmaxf(tm, sm_t[tp][half ^ 1][r]);
+        tp ^= 1;
+        const bool raise = (tm - m) * p.scale_log2 > 8.f;  // true on the first tile (m = -inf)
+        float f = 1.f;
+        if (raise) {
+          f = j == 0 ? 0.f : fast_exp2((m - tm) * p.scale_log2);
+          m = tm;
+          l2a = make_float2(l2a.x * f, l2a.y * f);
+          l2b = make_float2(l2b.x * f, l2b.y * f);
+        }
+        if (__any_sync(0xffffffffu, raise && j > 0)) {
+          // rescale this warp's rows of O (its DH/2 columns) once PV_{j-1} has landed
+          const int u = pc - 1;
+          mbar_wait(&p_empty[u & 1], (u >> 1) & 1);
+          tc_fence_after();
+#pragma unroll
+          for (int c = 0; c < DH / 2; c += 32) {
+            float o[32];
+            tmem_ld32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, o);
+            uint32_t ou[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i) ou[i] = __float_as_uint(o[i] * f);
+            tmem_st32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, ou);
+          }
+          tmem_wait_st();
+        }
+        const float ms = m * p.scale_log2;
         uint32_t pk[32];
         const float2 sl2 = make_float2(p.scale_log2, p.scale_log2), nms2 = make_float2(-ms, -ms);
+        const float2 one2 = make_float2(1.f, 1.f);
 #pragma unroll
         for (int i = 0; i < 32; ++i) {
           const float2 x = ffma2(make_float2(v[2 * i], v[2 * i + 1]), sl2, nms2);
-          float a0 = fast_exp2(x.x);
-          float a1 = fast_exp2(x.y);
-          if (diag) {
-            if (2 * i > lim) a0 = 0.f;
-            if (2 * i + 1 > lim) a1 = 0.f;
-          }
-          l4[i & 3] += a0 + a1;
-          __nv_bfloat162 h2 = __floats2bfloat162_rn(a0, a1);
+          const float2 e2 = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+          if (i & 1) l2b = ffma2(e2, one2, l2b);
+          else l2a = ffma2(e2, one2, l2a);
+          __nv_bfloat162 h2 = __floats2bfloat162_rn(e2.x, e2.y);
           pk[i] = *reinterpret_cast<uint32_t*>(&h2);
         }
         mbar_wait(&p_empty[pb], ((pc >> 1) & 1) ^ 1);
@@ -308,8 +329,12 @@ __global__ void __launch_bounds__(THREADS, 1)
         tmem_wait_st();
         tc_fence_before();
         mbar_arrive_local(&p_full[pb]);
-      }
-      float l = (l4[0] + l4[1]) + (l4[2] + l4[3]);
+        ++it; ++pc;
+      };
+      const int nfull = p.causal ? ntiles - 1 : ntiles;
+      for (int j = 0; j < nfull; ++j) tile(j, std::false_type{});
+      if (p.causal) tile(ntiles - 1, std::true_type{});
+      float l = (l2a.x + l2a.y) + (l2b.x + l2b.y);
       if (issuer) bulk_wait_read<0>();  // the previous item's O store has left the staging boxes
       asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
       sm_x[half][r] = l;
@@ -653,10 +678,13 @@ struct BwdPCfg {
   static_assert(SMEM <= 232448, "shared memory per CTA");
 };
 
-__device__ __forceinline__ void bwd_item(int item, int nk, int H, int& b, int& h, int& kt) {
-  kt = item % nk;  // causal: small key tiles see the most query tiles, handed out first
-  h = (item / nk) % H;
-  b = item / (nk * H);
+// sorted item -> (sequence, head, key tile); causal: small key tiles see the most query tiles
+__device__ __forceinline__ void bwd_item(int item, int nk, int H, int B, int& b, int& h, int& kt) {
+  const int hb = H * B;
+  kt = item / hb;
+  const int rem = item % hb;
+  h = rem % H;
+  b = rem / H;
 }
 
 __global__ void __launch_bounds__(THREADS, 1)
@@ -712,9 +740,9 @@ __global__ void __launch_bounds__(THREADS, 1)
     if (lane == 0) {
       int qs = 0; uint32_t qph = 0;
       int n = 0;
-      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+      for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
         int b, h, kt;
-        bwd_item(item, nk, p.H, b, h, kt);
+        bwd_item(item, nk, p.H, B, b, h, kt);
         const int i0 = p.causal ? kt * (BKV / BQS) : 0;
         const int kvs = n & 1;
         mbar_wait(&kv_empty[kvs], ((n >> 1) & 1) ^ 1);
@@ -742,13 +770,13 @@ __global__ void __launch_bounds__(THREADS, 1)
       const uint32_t idesc_s = make_idesc_f16(128, BQS, 0, 0);  // S^T, dP^T: M=keys, N=queries, K=DH
       const uint32_t idesc_g = make_idesc_f16(128, DH, 0, 1);   // dV, dK: M=keys, N=DH, K=queries
       // score-issue cursor (runs two sub-tiles ahead of the gradient cursor, across items)
-      int s_item = blockIdx.x, s_sub = 0, s_n = 0;
+      int s_item = snake(0), s_sub = 0, s_n = 0;
       int qs = 0; uint32_t qph = 0;  // (Q, dO) ring position of the next score issue
       int sc = 0;                    // score issues (buffer pair sc & 1)
       auto issue_s = [&]() {
         if (s_item >= items) return;
         int b, h, kt;
-        bwd_item(s_item, nk, p.H, b, h, kt);
+        bwd_item(s_item, nk, p.H, B, b, h, kt);
         const int nt = nqs - (p.causal ? kt * (BKV / BQS) : 0);
         const int kvs = s_n & 1;
         if (s_sub == 0) mbar_wait(&kv_full[kvs], (s_n >> 1) & 1);
@@ -768,16 +796,16 @@ __global__ void __launch_bounds__(THREADS, 1)
         mma_commit(&s_full[sb]);
         if (++qs == Cfg::QST) { qs = 0; qph ^= 1; }
         ++sc;
-        if (++s_sub == nt) { s_sub = 0; s_item += gridDim.x; ++s_n; }
+        if (++s_sub == nt) { s_sub = 0; s_item = snake(s_n + 1); ++s_n; }
       };
       issue_s();
       issue_s();
       int gq = 0;  // (Q, dO) ring position of the next dV/dK
       int pc = 0;  // sub-tiles whose gradients were issued (P/dS buffer pc & 1)
       int n = 0;
-      for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+      for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
         int b, h, kt;
-        bwd_item(item, nk, p.H, b, h, kt);
+        bwd_item(item, nk, p.H, B, b, h, kt);
         const int nt = nqs - (p.causal ? kt * (BKV / BQS) : 0);
         const int kvs = n & 1;
         for (int t = 0; t < nt; ++t) {
@@ -818,9 +846,9 @@ __global__ void __launch_bounds__(THREADS, 1)
     int g = 0, n = 0;
     int qsl = 0;        // (Q, dO, statistics) ring position of the current sub-tile
     uint32_t qslph = 0; // its phase
-    for (int item = blockIdx.x; item < items; item += gridDim.x, ++n) {
+    for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
       int b, h, kt;
-      bwd_item(item, nk, p.H, b, h, kt);
+      bwd_item(item, nk, p.H, B, b, h, kt);
       const int i0 = p.causal ? kt * (BKV / BQS) : 0;
       const int nt = nqs - i0;
       const int key = kt * BKV + r;
