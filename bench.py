@@ -39,9 +39,9 @@ TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2.json")
 FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
 
 WORKLOADS = {
-    "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=4 x b=16), bf16/fp32-master Adam, "
+    "cfg2": dict(name="cfg2: BERT-Large 24L d1024 h16 S512, 64 seq/GPU (m=2 x b=32), bf16/fp32-master Adam, "
                       "HBM cap 8 GiB/GPU", model="bert-large-like-preLN", descs=lambda: synth.transformer_stack(24, 1024, 16, 512, False),
-                 per_gpu_batch=64, m=4, cap=8 << 30, S=512),
+                 per_gpu_batch=64, m=2, cap=8 << 30, S=512),
     "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=2 x b=4), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
                  per_gpu_batch=8, m=2, cap=16 << 30, S=1024),

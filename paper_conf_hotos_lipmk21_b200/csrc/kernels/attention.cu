@@ -418,8 +418,8 @@ struct BwdParams {
   int S, H, causal;
   float scale;
   float scale_log2;    // scale * log2(e)
-  const float* lse2;   // [b, H, S]: lse * log2(e)
-  const float* sD;     // [b, H, S]: scale * D
+  const float* lse2;   // [b, H, S]: -lse * log2(e)
+  const float* sD;     // [b, H, S]: -scale * D
   __nv_bfloat16* dqkv; // [b*S, 3d]: dK, dV columns written here
   __nv_bfloat16* dst;  // [b, H, S(keys), S(queries)]: scale * dS^T
   int d;
@@ -591,10 +591,10 @@ __global__ void __launch_bounds__(THREADS, 1)
 #pragma unroll
           for (int u = 0; u < 2; ++u) {
             const int e = 2 * i + u;
-            float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, -l2[e]));
+            float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, l2[e]));
             if (diag && key > qc + e) pv = 0.f;
             pr[u] = pv;
-            dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, -sd[e]);
+            dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, sd[e]);
           }
           __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
           __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
@@ -842,7 +842,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int half = (warp - 2) >> 2;  // which 32 queries of the sub-tile
     const int r = qd * 32 + lane;      // key row within the tile
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
-    const bool issuer = warp == 2 && lane == 0;
+    const bool issuer = half == 0 && lane == 0;  // of this lane quadrant's dS^T store
     int g = 0, n = 0;
     int qsl = 0;        // (Q, dO, statistics) ring position of the current sub-tile
     uint32_t qslph = 0; // its phase
@@ -867,29 +867,34 @@ __global__ void __launch_bounds__(THREADS, 1)
         uint32_t rs[32], rd[32];
         tmem_ld32_nw(tmem + trow + Cfg::ST_COL + buf * BQS + half * 32, rs);
         tmem_ld32_nw(tmem + trow + Cfg::DP_COL + buf * BQS + half * 32, rd);
-        float l2[32], sd[32];  // broadcast reads of the staged statistics
+        float2 l2[16], sd[16];  // broadcast reads of the staged statistics (-lse2, -sD), in pairs
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-          const float4 a4 = reinterpret_cast<const float4*>(sl2)[i];
-          const float4 d4 = reinterpret_cast<const float4*>(ssd)[i];
-          l2[4 * i] = a4.x; l2[4 * i + 1] = a4.y; l2[4 * i + 2] = a4.z; l2[4 * i + 3] = a4.w;
-          sd[4 * i] = d4.x; sd[4 * i + 1] = d4.y; sd[4 * i + 2] = d4.z; sd[4 * i + 3] = d4.w;
+          float4 a4, d4;
+          asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(a4.x), "=f"(a4.y), "=f"(a4.z), "=f"(a4.w)
+                       : "r"(smem_u32(sl2) + 16 * i));
+          asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(d4.x), "=f"(d4.y), "=f"(d4.z), "=f"(d4.w)
+                       : "r"(smem_u32(ssd) + 16 * i));
+          l2[2 * i] = make_float2(a4.x, a4.y); l2[2 * i + 1] = make_float2(a4.z, a4.w);
+          sd[2 * i] = make_float2(d4.x, d4.y); sd[2 * i + 1] = make_float2(d4.z, d4.w);
         }
         tmem_wait_ld();
+        if (diag) {  // keys after the query: score -inf, so P = 0 and dS = 0 exactly
+#pragma unroll
+          for (int e = 0; e < 32; ++e)
+            if (key > qc + e) rs[e] = __float_as_uint(-INFINITY);
+        }
         uint32_t pk[16], dk[16];
+        const float2 sl2v = make_float2(p.scale_log2, p.scale_log2), sc2 = make_float2(p.scale, p.scale);
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
-          float pr[2], dr[2];
-#pragma unroll
-          for (int u = 0; u < 2; ++u) {
-            const int e = 2 * i + u;
-            float pv = fast_exp2(fmaf(__uint_as_float(rs[e]), p.scale_log2, -l2[e]));
-            if (diag && key > qc + e) pv = 0.f;
-            pr[u] = pv;
-            dr[u] = pv * fmaf(__uint_as_float(rd[e]), p.scale, -sd[e]);
-          }
-          __nv_bfloat162 a2 = __floats2bfloat162_rn(pr[0], pr[1]);
-          __nv_bfloat162 b2 = __floats2bfloat162_rn(dr[0], dr[1]);
+          // P = 2^(s scale log2e - lse2); dS = P (dp scale - sD): three packed FP ops per pair
+          const float2 x = ffma2(make_float2(__uint_as_float(rs[2 * i]), __uint_as_float(rs[2 * i + 1])), sl2v, l2[i]);
+          const float2 pv = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+          const float2 t = ffma2(make_float2(__uint_as_float(rd[2 * i]), __uint_as_float(rd[2 * i + 1])), sc2, sd[i]);
+          const float2 dr = fmul2(pv, t);
+          __nv_bfloat162 a2 = __floats2bfloat162_rn(pv.x, pv.y);
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(dr.x, dr.y);
           pk[i] = *reinterpret_cast<uint32_t*>(&a2);
           dk[i] = *reinterpret_cast<uint32_t*>(&b2);
         }
@@ -901,22 +906,24 @@ __global__ void __launch_bounds__(THREADS, 1)
             "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]), "r"(pk[15])
             : "memory");
         // dS^T: the row's 16-byte chunks 4*half .. 4*half+3 of the 128-byte (64-query) row, swizzled
-        uint8_t* drow = sDS + buf * Cfg::DS_BYTES + r * 128;
+        const uint32_t drow = smem_u32(sDS + buf * Cfg::DS_BYTES + r * 128);
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-          *reinterpret_cast<uint4*>(drow + (((4 * half + u) ^ (r & 7)) << 4)) =
-              make_uint4(dk[4 * u], dk[4 * u + 1], dk[4 * u + 2], dk[4 * u + 3]);
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(drow + (((4 * half + u) ^ (r & 7)) << 4)),
+                       "r"(dk[4 * u]), "r"(dk[4 * u + 1]), "r"(dk[4 * u + 2]), "r"(dk[4 * u + 3])
+                       : "memory");
         tmem_wait_st();
         tc_fence_before();
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_arrive_local(&p_full[buf]);
-        // the whole (128 keys x 64 queries) box is written: one TMA store.  The store of the
-        // sub-tile two back (same buffer) was waited for at the previous sub-tile's store, before
-        // this barrier's previous instance, so the buffer was free when it was written above.
+        // this lane quadrant's 32 keys x 64 queries are written (both halves): one TMA store per
+        // quadrant, synchronised by the quadrant's two warps only.  The quadrant's store of the
+        // sub-tile two back (same buffer) was waited for before the previous instance of this
+        // barrier, so its rows were free when they were written above.
         if (issuer) bulk_wait_read<0>();
-        asm volatile("bar.sync 1, 256;" ::: "memory");
+        asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
         if (issuer) {
-          tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES, q0, kt * BKV, h, b);
+          tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES + qd * 32 * 128, q0, kt * BKV + qd * 32, h, b);
           bulk_commit();
         }
       }
@@ -949,7 +956,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   }
 }
 
-// sD[b, h, q] = scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = lse * log2(e): the
+// sD[b, h, q] = -scale * sum_e dO[b*S+q][h*dh+e] * O[b*S+q][h*dh+e] and lse2 = -lse * log2(e): the
 // per-query terms of dS = P (dP - D) in the forms the backward's FFMAs take.  One thread per 8
 // consecutive elements of the [tokens, d] rows (one 16-byte load of dO and of O, fully coalesced,
 // a few registers, so the grid is many small resident blocks); each head's dh/8 adjacent lanes
@@ -981,8 +988,8 @@ __global__ void __launch_bounds__(256) attn_bwd_prep(int64_t ntok, int S, int H,
     const int h = e / dh;
     const int64_t bseq = tok / S, q = tok % S;
     const int64_t i = (bseq * H + h) * S + q;
-    sD[i] = scale * s;
-    lse2[i] = lse[i] * 1.4426950408889634f;
+    sD[i] = -(scale * s);                     // -scale * D
+    lse2[i] = -(lse[i] * 1.4426950408889634f);  // -lse * log2(e)
   }
 }
 }  // namespace attn
@@ -1082,11 +1089,12 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
     }
     const int64_t items = (int64_t)(S / BKV) * H * b;
     // Q / dO in 64-query sub-tiles
-    CUtensorMap mq64, mo64;
+    CUtensorMap mq64, mo64, mds32;
+    tcx::make_map_4d(&mds32, dst, S, S, H, b, S, (int64_t)S * S, (int64_t)H * S * S, 64, 32);  // per-quadrant boxes
     tcx::make_map_4d(&mq64, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BwdPCfg::BQS);
     tcx::make_map_4d(&mo64, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BwdPCfg::BQS);
     attn_bwd_persistent<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq64, mk, mv, mo64,
-                                                                                                    mds, p, (int)b);
+                                                                                                    mds32, p, (int)b);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }

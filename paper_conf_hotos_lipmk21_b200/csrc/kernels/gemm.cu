@@ -293,8 +293,9 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
         tma_load_box(w.buf + (b ^ 1) * EPI_BUF, mIn, &w.bar[b ^ 1], n + CPB, row0, z0, z1, EPI_BUF);
       }
     } else if (lane == 0) {
-      if (two) bulk_wait_read<0>();
-      else bulk_wait_read<1>();
+      // <= 1 store group pending: one buffer back (plain), or for BIAS_ACT the previous box's G
+      // store may still be reading buffer B while this box's H goes into buffer A
+      bulk_wait_read<1>();
     }
     float v[CPB];
     if (p.tma_epi == 2) {  // DEBUG
@@ -373,15 +374,9 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
               const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hz));
               o[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
             }
-          } else {  // BIAS_ACT: H = acc + b (bf16), G = act(H as stored) into the second box
-            uint32_t g[4];
+          } else {  // BIAS_ACT: H = acc + b (bf16) now; G = act(H as stored) after H's store is issued
 #pragma unroll
-            for (int t = 0; t < 4; ++t) {
-              o[t] = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
-              const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&o[t]));
-              g[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
-            }
-            sts128(w.buf + EPI_BUF + swz128(r, k), g[0], g[1], g[2], g[3]);
+            for (int t = 0; t < 4; ++t) o[t] = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
           }
         }
         sts128(ad, o[0], o[1], o[2], o[3]);
@@ -391,8 +386,31 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
     __syncwarp();
     if (lane == 0) {
       tma_store_box(mC, sb, n, row0, z0, z1);
-      if (two) tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
       bulk_commit();
+    }
+    if (ESZ == 2 && two) {
+      // G = act(H as stored): H is read back from buffer A (which the H store only reads) and G
+      // goes into buffer B once the previous box's G store has left it
+      if (lane == 0) bulk_wait_read<1>();
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint4 hq = lds128(sb + swz128(r, k));
+        const uint32_t hw[4] = {hq.x, hq.y, hq.z, hq.w};
+        uint32_t g[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hw[t]));
+          g[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
+        }
+        sts128(w.buf + EPI_BUF + swz128(r, k), g[0], g[1], g[2], g[3]);
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) {
+        tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
+        bulk_commit();
+      }
     }
     ++w.j;
   }

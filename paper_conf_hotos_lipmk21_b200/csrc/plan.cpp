@@ -387,11 +387,28 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
           }
         }
       }
-      for (int l = L - 1; l >= 0; --l)  // stash: LIFO (consumed first in the backward)
-        for (int i = 0; i < m; ++i) {
-          uint64_t sz = align_up(p.layers[l].g.st.total, ALIGN);
-          if (sz <= room) { p.layers[l].stash_res[i] = 0; room -= sz; }
+      // stash: 2 B saved per byte.  Equal-size entries: the spilled (layer, microbatch) entries are
+      // spread evenly over the backward order (as the streamed state above), so each one's swap-in
+      // overlaps the backward of resident entries instead of a run of spilled entries at the end
+      // of the backward waiting on the host link; otherwise LIFO (consumed first in the backward).
+      bool st_uniform = true;
+      for (int l = 1; l < L; ++l) st_uniform = st_uniform && p.layers[l].g.st.total == p.layers[0].g.st.total;
+      const uint64_t gsz = align_up(p.layers[0].g.st.total, ALIGN);
+      const int nent = L * m;
+      if (st_uniform && gsz > 0 && (uint64_t)nent * gsz > room && !baseline) {
+        const int keep = (int)std::min<uint64_t>(room / gsz, (uint64_t)nent);
+        const int nspill = nent - keep;
+        for (int j = 0; j < nent; ++j) {  // backward position j: layer L-1-j/m, microbatch j%m
+          const bool spilled = (int64_t)(j + 1) * nspill / nent > (int64_t)j * nspill / nent;
+          if (!spilled) { p.layers[L - 1 - j / m].stash_res[j % m] = 0; room -= gsz; }
         }
+      } else {
+        for (int l = L - 1; l >= 0; --l)
+          for (int i = 0; i < m; ++i) {
+            uint64_t sz = align_up(p.layers[l].g.st.total, ALIGN);
+            if (sz <= room) { p.layers[l].stash_res[i] = 0; room -= sz; }
+          }
+      }
       Res r{};
       r.bytes = room0 - room;
       r.mw = r.ms = r.mst = 0;

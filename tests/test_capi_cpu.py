@@ -164,14 +164,24 @@ def test_uncapped_moves_only_inputs_and_loss():
     assert s.pred_h2d_bytes == 2 * 32 * 256 * 4 and s.pred_d2h_bytes == 4 * 8
 
 
-def test_stash_residency_is_lifo():
-    """The last layers' stash (consumed first by the backward) is the one kept resident."""
-    descs = synth.transformer_stack(8, 64, 4, 16, False)
-    base = min_cap(descs, microbatches=2, microbatch_size=2, precision=1)
-    s, ops = plan(descs, microbatches=2, microbatch_size=2, precision=1, hbm_cap_bytes=int(base * 8))
-    spilled = {(o["l"], o["i"]) for o in ops if o["kind"] == "D2H" and o["cat"] == "stash"}
-    if spilled and s.resident_stash_bytes:
-        assert max(l for l, _ in spilled) < 7
+@pytest.mark.parametrize("mult", [4, 6, 8])
+def test_spilled_stash_is_spread_over_the_backward(mult):
+    """Equal-size stash entries: the spilled (layer, microbatch) entries are spread evenly over the
+    backward order (layer L-1 first, microbatches in canonical order), so each one's swap-in
+    overlaps the backward of resident entries; every spilled entry leaves once (D2H) and comes
+    back once (H2D)."""
+    L, m = 8, 2
+    descs = synth.transformer_stack(L, 64, 4, 16, False)
+    base = min_cap(descs, microbatches=m, microbatch_size=2, precision=1)
+    s, ops = plan(descs, microbatches=m, microbatch_size=2, precision=1, hbm_cap_bytes=int(base * mult))
+    out = sorted((o["l"], o["i"]) for o in ops if o["kind"] == "D2H" and o["cat"] == "stash")
+    back = sorted((o["l"], o["i"]) for o in ops if o["kind"] == "H2D" and o["cat"] == "stash")
+    assert out == back
+    n = len(out)
+    if 0 < n < L * m:
+        expect = sorted((L - 1 - j // m, j % m) for j in range(L * m) if (j + 1) * n // (L * m) > j * n // (L * m))
+        assert out == expect
+    assert s.hazards == 0
 
 
 @pytest.mark.parametrize("extra", [6, 8, 10, 12])

@@ -1,5 +1,6 @@
-"""Time the step's GEMMs (cfg2: one microbatch of 4096 tokens, d = 1024; the 12 linear GEMMs of a
-transformer layer with their in-step epilogues) through hk_gemm.
+"""Time the step's GEMMs (cfg2: one microbatch of T tokens, d = 1024 — T = 16384 for the bench's
+m=2 x b=32, --tokens to change; the 12 linear GEMMs of a transformer layer with their in-step
+epilogues) through hk_gemm.
 
     python tools/gemm_bench.py [--reps 20] [--only NAME]
 
@@ -19,7 +20,7 @@ import torch  # noqa: E402
 
 from paper_conf_hotos_lipmk21_b200 import harmony as H  # noqa: E402
 
-T, D, S, B, NH = 4096, 1024, 512, 8, 16
+T, D, S, B, NH = int(os.environ.get("GEMM_BENCH_TOKENS", "16384")), 1024, 512, 8, 16
 DH = D // NH
 
 

@@ -4,7 +4,7 @@
         python tools/profile_step.py --layers 2 --steps 2
 
 Same per-layer shapes and launch configuration as `bench.py` (cfg2: d=1024, h=16, S=512,
-m=4 x b=16 by default, stash policy 2); `--layers` trims the stack depth so the list stays short (every layer
+m=2 x b=32 by default, stash policy 2); `--layers` trims the stack depth so the list stays short (every layer
 runs the identical kernel sequence).  Eager issue (HARMONY_NO_GRAPH=1 is set) so each kernel is
 one launch record.
 """
@@ -27,7 +27,7 @@ def main():
     ap.add_argument("--layers", type=int, default=2)
     ap.add_argument("--steps", type=int, default=2)
     ap.add_argument("--policy", type=int, default=2)
-    ap.add_argument("--microbatches", type=int, default=4)
+    ap.add_argument("--microbatches", type=int, default=2)
     a = ap.parse_args()
     descs = synth.transformer_stack(a.layers, 1024, 16, 512, False)
     params = synth.gen_params(descs, 1)
