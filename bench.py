@@ -35,7 +35,7 @@ import synth  # noqa: E402
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 # per-launch DRAM traffic of the roofline kernel class, from the committed ncu launch list of the
 # same step (tools/traffic_summary.py); ncu replays cold, so this is the no-L2-reuse upper end
-TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2.json")}
+TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2_m2.json")}
 FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
 
 WORKLOADS = {
@@ -389,7 +389,7 @@ def main():
             tj = json.load(f)
         traffic = tj["classes"]["gemm"]["dram_bytes_per_launch"]
         traffic_src = (f"{os.path.relpath(TRAFFIC_FILES[args.workload], ROOT)}: ncu dram__bytes_read.sum + "
-                       f"dram__bytes_write.sum averaged over the {tj['classes']['gemm']['launches']} tensor-core "
+                       f"dram__bytes_write.sum averaged over the {tj['classes']['gemm']['launches']} tcgen05 GEMM "
                        f"launches of the profiled step (cold-cache replay)")
     except (KeyError, OSError, ValueError):
         pass

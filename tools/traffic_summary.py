@@ -6,8 +6,8 @@
 
 ncu replays every kernel with its caches flushed (cold), so `dram_bytes_per_launch` is the traffic a
 launch moves from HBM when nothing it reads is L2-resident — the upper end of what the step sees.
-The "gemm" class matches the bench's roofline kernel class (all tensor-core contractions of the
-step: the tcgen05 GEMMs and the fused attention kernels).
+The "gemm" class matches the bench's roofline kernel class (the tcgen05 GEMMs of the step); the
+fused attention kernels are their own class, as in the bench's profile.
 """
 import csv
 import json
@@ -15,7 +15,8 @@ import re
 import sys
 from collections import defaultdict
 
-CLASSES = [("gemm", re.compile(r"gemm_tc|attn_fwd|attn_bwd_persistent|attn_bwd_kernel")),
+CLASSES = [("gemm", re.compile(r"gemm_tc")),
+           ("attention", re.compile(r"attn_fwd|attn_bwd_persistent|attn_bwd_kernel")),
            ("layernorm", re.compile(r"ln_fwd|ln_bwd|colreduce2")),
            ("adam", re.compile(r"adam")),
            ("other", re.compile(r"."))]
