@@ -425,7 +425,9 @@ def main():
         "adam_hbm": {"achieved_gbs": adam["work"] / adam["seconds"] / 1e9 if adam["seconds"] else None,
                      "peak_gbs": peaks["hbm_gbs"]},
         "e2e": {"value": samples / e2e_wall, "unit": unit, "h2d_bytes_per_step": e2e_stats[-1]["h2d_input_bytes"],
-                "d2h_bytes_per_step": e2e_stats[-1]["d2h_output_bytes"], "timing": "host wall clock around harmony_step"},
+                "d2h_bytes_per_step": e2e_stats[-1]["d2h_output_bytes"], "timing": "host wall clock around harmony_step",
+                "ms_per_step": e2e_wall / args.steps * 1e3,
+                "device_ms_per_step": sum(x["step_seconds"] for x in e2e_stats) / len(e2e_stats) * 1e3},
         "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
         "graph_replay": bool(stats[-1]["graph"]),
         "profiled_pass_ms_per_step": prof_s / args.steps * 1e3,

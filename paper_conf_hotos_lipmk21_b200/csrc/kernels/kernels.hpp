@@ -11,11 +11,11 @@ namespace hm {
 void gemm(const hk_gemm_args& a, cudaStream_t st);
 
 void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
-                   float* rstd, cudaStream_t st);
+                   float* rstd, cudaStream_t st, float* Xcopy = nullptr);
 size_t layernorm_bwd_scratch_bytes(int64_t rows, int d);
 // register-resident variants (d % 4 == 0, d <= 2048); return false when not applicable
 bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U,
-                       float* mean, float* rstd, cudaStream_t st);
+                       float* mean, float* rstd, cudaStream_t st, float* Xcopy = nullptr);
 size_t layernorm_bwd_vec_scratch_bytes(int64_t rows, int d);
 bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const float* X, const float* mean,
                        const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db,
@@ -29,6 +29,8 @@ void layernorm_bwd(int dtype, int64_t rows, int d, const float* dU, const float*
                    const float* rstd, const void* g, const float* dres, float* dX, float* dg, float* db, int accumulate,
                    float* scratch, cudaStream_t st);
 size_t colsum_scratch_bytes(int64_t rows, int n);
+// C (+)= sum of S fp32 split-K partials ws[z][n] in z order (deterministic)
+void splitk_sum(int S, int64_t n, const float* ws, float* C, int accumulate, cudaStream_t st);
 void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float* out, int accumulate, float* scratch,
             cudaStream_t st);
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st);

@@ -47,7 +47,8 @@ __device__ __forceinline__ void st4<__nv_bfloat16>(__nv_bfloat16* p, float4 v) {
 template <typename T, int VPT>
 __global__ void __launch_bounds__(256) ln_fwd_v(int64_t rows, int d, const float* __restrict__ X,
                                                const T* __restrict__ g, const T* __restrict__ b, T* __restrict__ U,
-                                               float* __restrict__ mean, float* __restrict__ rstd) {
+                                               float* __restrict__ mean, float* __restrict__ rstd,
+                                               float* __restrict__ Xcopy) {
   const int lane = threadIdx.x & 31;
   const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (row >= rows) return;
@@ -59,6 +60,13 @@ __global__ void __launch_bounds__(256) ln_fwd_v(int64_t rows, int d, const float
     const int c = (j * 32 + lane) * 4;
     v[j] = c < d ? *reinterpret_cast<const float4*>(x + c) : make_float4(0.f, 0.f, 0.f, 0.f);
     s += (v[j].x + v[j].y) + (v[j].z + v[j].w);
+  }
+  if (Xcopy) {  // the block input stashed by the same pass that normalises it (block recompute)
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int c = (j * 32 + lane) * 4;
+      if (c < d) *reinterpret_cast<float4*>(Xcopy + row * d + c) = v[j];
+    }
   }
   const float mu = wsum(s) / (float)d;
   float q = 0.f;
@@ -221,11 +229,11 @@ static int ln_vpt(int d) {
 }
 
 bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U,
-                       float* mean, float* rstd, cudaStream_t st) {
+                       float* mean, float* rstd, cudaStream_t st, float* Xcopy) {
   const int v = ln_vpt(d);
   if (!v) return false;
   const unsigned grid = (unsigned)ceil_div(rows, 8);
-#define HM_LNF(T, V) ln_fwd_v<T, V><<<grid, 256, 0, st>>>(rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)
+#define HM_LNF(T, V) ln_fwd_v<T, V><<<grid, 256, 0, st>>>(rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd, Xcopy)
 #define HM_LNF_ALL(T)                   \
   switch (v) {                          \
     case 1: HM_LNF(T, 1); break;        \

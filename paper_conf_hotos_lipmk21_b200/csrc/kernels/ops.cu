@@ -128,6 +128,32 @@ __global__ void __launch_bounds__(1024) colreduce_kernel(int nchunks, int n, con
     out[c] = accumulate ? out[c] + t : t;
   }
 }
+// Split-K reduction: C[i] (+)= sum_{z < S} ws[z * n + i], the S partial products added in z order
+// (a fixed order: deterministic), four elements per thread with 16-byte loads.
+__global__ void __launch_bounds__(256) splitk_sum_kernel(int S, int64_t n4, const float4* __restrict__ ws,
+                                                        float4* __restrict__ C, int accumulate) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n4) return;
+  float4 t = ws[i];
+  for (int z = 1; z < S; ++z) {
+    const float4 u = ws[(int64_t)z * n4 + i];
+    t.x += u.x; t.y += u.y; t.z += u.z; t.w += u.w;
+  }
+  if (accumulate) {
+    const float4 c = C[i];
+    t = make_float4(c.x + t.x, c.y + t.y, c.z + t.z, c.w + t.w);
+  }
+  C[i] = t;
+}
+void splitk_sum(int S, int64_t n, const float* ws, float* C, int accumulate, cudaStream_t st) {
+  HM_CHECK(n % 4 == 0, HARMONY_E_INVALID_ARG, "splitk_sum: n % 4 != 0");
+  const int e0 = g_prof.begin(st);
+  splitk_sum_kernel<<<(unsigned)ceil_div(n / 4, 256), 256, 0, st>>>(S, n / 4, reinterpret_cast<const float4*>(ws),
+                                                                   reinterpret_cast<float4*>(C), accumulate);
+  check_launch("splitk_sum");
+  g_prof.end(PROF_OTHER, e0, st, (double)n * 4 * (S + 1 + (accumulate ? 1 : 0)));
+}
+
 static void colreduce(int nchunks, int n, const float* partial, int64_t stride, float* out, int accumulate,
                       cudaStream_t st) {
   colreduce_kernel<<<(unsigned)ceil_div(n, 32), 1024, 0, st>>>(nchunks, n, partial, stride, out, accumulate);
@@ -339,13 +365,14 @@ __global__ void copy_rows_kernel(int64_t n4, const float4* __restrict__ src, flo
   } while (0)
 
 void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
-                   float* rstd, cudaStream_t st) {
+                   float* rstd, cudaStream_t st, float* Xcopy) {
   if (rows == 0) return;
   const int e0 = g_prof.begin(st);
-  if (layernorm_fwd_vec(dtype, rows, d, X, g, b, U, mean, rstd, st)) {
-    g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 + (dtype ? 2 : 4)) + rows * 8.0);
+  if (layernorm_fwd_vec(dtype, rows, d, X, g, b, U, mean, rstd, st, Xcopy)) {
+    g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 + (dtype ? 2 : 4) + (Xcopy ? 4 : 0)) + rows * 8.0);
     return;
   }
+  if (Xcopy) copy_f32(rows * d, X, Xcopy, st);
   HM_DISPATCH_T(dtype, (layernorm_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(
                            rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)));
   check_launch("layernorm_fwd");

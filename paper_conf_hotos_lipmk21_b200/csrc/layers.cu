@@ -29,6 +29,22 @@ static uint64_t bump(uint64_t& cur, uint64_t bytes) {
   return o;
 }
 
+// Split-K factor of a weight gradient dW[k][n] += X^T dY over `rows` tokens: when its 256 x 256
+// CTA-pair tiles would leave most of the 74 pairs idle (the d x d output projection: 16 tiles),
+// the token (K) range is cut into S slices computed as S batched GEMMs into a workspace and added
+// in slice order by splitk_sum (deterministic; shape-only, so capped == uncapped).
+static int wgrad_splits(const LayerGeom& g, int64_t rows, int n, int k) {
+  if (g.dtype != 1) return 1;
+  const int64_t tiles = ceil_div(k, 256) * ceil_div(n, 256);
+  if (k < 256 || n < 256 || tiles >= 37) return 1;
+  int S = 1;
+  while (S < 4 && tiles * S * 2 <= 74 && rows % (S * 2 * 64) == 0) S *= 2;
+  return S;
+}
+static uint64_t wgrad_split_ws_bytes(const LayerGeom& g, int64_t rows, int n, int k) {
+  const int S = wgrad_splits(g, rows, n, k);
+  return S > 1 ? (uint64_t)S * k * n * 4 : 0;
+}
 LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_policy) {
   if ((stash_policy == 2 || stash_policy == 3) && desc.kind == HARMONY_LAYER_TRANSFORMER) {
     // Block recompute ([7] P:881): the stash is the block input X; the forward and the
@@ -135,6 +151,7 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   bump(wb, R * D * ts);      // dX2c
   bump(wb, R * 3 * D * ts);  // dQKV
   bump(wb, colsum_scratch_bytes(g.rows, (int)(4 * D)));  // side-stream column-sum scratch
+  bump(wb, std::max<uint64_t>(wgrad_split_ws_bytes(g, g.rows, (int)D, (int)D), 256));  // split-K dW_o partials
   g.ws_bwd = wb;
   g.flops_fwd = 24.0 * (double)R * D * D + 4.0 * (double)b * g.S * g.S * D;
   return g;
@@ -186,6 +203,22 @@ static hk_gemm_args lin_wgrad(const LayerGeom& g, int64_t rows, int n, int k, co
   return a;
 }
 
+static void wgrad(const LayerGeom& g, int64_t rows, int n, int k, const void* X, const void* dY, float* dW, int first,
+                  float* ws, cudaStream_t st) {
+  const int S = wgrad_splits(g, rows, n, k);
+  if (S == 1) return gemm(lin_wgrad(g, rows, n, k, X, dY, dW, first), st);
+  const int64_t ks = rows / S;
+  hk_gemm_args a = lin_wgrad(g, ks, n, k, X, dY, ws, 1);
+  a.nz0 = S;
+  a.a_sz0 = ks * k;  // X^T slice z: token rows [z ks, (z+1) ks) of X[rows][k]
+  a.b_sz0 = ks * n;
+  a.c_sz0 = (int64_t)k * n;
+  a.epilogue = HK_EPI_STORE_F32;
+  a.accumulate = 0;
+  gemm(a, st);
+  splitk_sum(S, (int64_t)k * n, ws, dW, first ? 0 : 1, st);
+}
+
 // ------------------------------------------------------------------------------------------------ forward
 // Attention output C and row LSE kept outside the core stash (stash policy 3): where they live and
 // whether they already hold this block's values (the backward's recompute skips the attention)
@@ -196,7 +229,7 @@ struct AttnStash {
 };
 
 static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws,
-                     void* stv, bool stash_x = true, const AttnStash* as = nullptr) {
+                     void* stv, bool stash_x = true, const AttnStash* as = nullptr, float* x_copy = nullptr) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   if (d.kind == HARMONY_LAYER_MLP) {
@@ -233,7 +266,8 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   // stash the layer input (Fig. 5(a) "Stashed X"); under block recompute the caller keeps X itself
   if (stash_x) copy_f32(R * D, X, Xs, st);
   // U = LN1(X)
-  layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st);
+  // (block recompute: the LN reads X once and also writes the stashed copy of the block input)
+  layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st, x_copy);
   // QKV = U W_qkv + b_qkv
   {
     hk_gemm_args a = lin_fwd(g, R, 3 * D, D, U, wseg(g, W, P_WQKV));
@@ -358,6 +392,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   uint8_t* dX2c_buf = ws + bump(wc, R * D * ts);
   uint8_t* dQKV_buf = ws + bump(wc, R * 3 * D * ts);
   float* side_scratch = reinterpret_cast<float*>(ws + bump(wc, colsum_scratch_bytes(R, 4 * D)));
+  float* split_ws = reinterpret_cast<float*>(ws + bump(wc, std::max<uint64_t>(wgrad_split_ws_bytes(g, R, D, D), 256)));
   // weight gradients on the side stream (not with policy 1: its recompute buffer is reused in place)
   const bool overlap = t_side != nullptr && g.stash_policy != 1;
   cudaStream_t sw = overlap ? t_side : st;     // stream of the weight-gradient work
@@ -412,7 +447,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     a.C = dC; a.epilogue = HK_EPI_STORE_T;
     gemm(a, st);
   }
-  gemm(lin_wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first), sw);
+  wgrad(g, R, D, D, C, dX2op, gseg(g, dW, P_WO), first, split_ws, sw);
   // ---- attention backward (batched over heads z0 and sequences z1)
   uint8_t* dQKV = dQKV_buf;
   const float scale = 1.0f / std::sqrt((float)dh);
@@ -502,8 +537,8 @@ void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint
   uint8_t* rest = ws + align_up(c.st.total, 256);
   // policy 3: the attention writes C and its LSE straight into the stash
   const AttnStash as{stash + g.st.C, reinterpret_cast<float*>(stash + g.st.P), false};
-  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false, g.stash_policy == 3 ? &as : nullptr);
-  copy_f32(g.rows * g.d, X, reinterpret_cast<float*>(stash + g.st.X), static_cast<cudaStream_t>(st));
+  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false, g.stash_policy == 3 ? &as : nullptr,
+           reinterpret_cast<float*>(stash + g.st.X));
 }
 
 void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
