@@ -20,7 +20,7 @@ import torch  # noqa: E402
 
 from paper_conf_hotos_lipmk21_b200 import harmony as H  # noqa: E402
 
-T, D, S, B, NH = int(os.environ.get("GEMM_BENCH_TOKENS", "16384")), 1024, 512, 8, 16
+T, D, S, B, NH = int(os.environ.get("GEMM_BENCH_TOKENS", "16384")), int(os.environ.get("GEMM_BENCH_D", "1024")), 512, 8, 16
 DH = D // NH
 
 

@@ -28,13 +28,17 @@ def main():
     ap.add_argument("--steps", type=int, default=2)
     ap.add_argument("--policy", type=int, default=2)
     ap.add_argument("--microbatches", type=int, default=2)
+    ap.add_argument("--cfg3", action="store_true", help="GPT-2 XL geometry (d=1600, h=25, S=1024 causal, 8 seq, 16 GiB)")
     a = ap.parse_args()
-    descs = synth.transformer_stack(a.layers, 1024, 16, 512, False)
+    if a.cfg3:
+        descs, B, cap = synth.transformer_stack(a.layers, 1600, 25, 1024, True), 8, 16 << 30
+    else:
+        descs, B, cap = synth.transformer_stack(a.layers, 1024, 16, 512, False), 64, 8 << 30
     params = synth.gen_params(descs, 1)
-    X, T = synth.gen_batch(descs, 64, 1, 1)
+    X, T = synth.gen_batch(descs, B, 1, 1)
     Xd, Td = torch.tensor(X, device="cuda"), torch.tensor(T, device="cuda")
-    with H.Harmony(descs, params, microbatches=a.microbatches, microbatch_size=64 // a.microbatches, precision=1, stash_policy=a.policy,
-                   hbm_cap_bytes=8 << 30, lr=1e-4) as h:
+    with H.Harmony(descs, params, microbatches=a.microbatches, microbatch_size=B // a.microbatches, precision=1,
+                   stash_policy=a.policy, hbm_cap_bytes=cap, lr=1e-4) as h:
         for _ in range(a.steps):
             loss, st = h.step(Xd, Td)
             print("step", loss, st.step_seconds, st.kernel_launches)
