@@ -860,7 +860,6 @@ __global__ void __launch_bounds__(THREADS, 1)
         const int q0 = (i0 + t) * BQS;
         const int buf = g & 1;
         mbar_wait(&s_full[buf], (g >> 1) & 1);
-        mbar_wait(&p_empty[buf], ((g >> 1) & 1) ^ 1);
         tc_fence_after();
         const bool diag = p.causal && q0 < kt * BKV + BKV;  // the sub-tile overlaps the key range
         const int qc = q0 + half * 32;  // first query of this thread's 32 columns
@@ -898,6 +897,10 @@ __global__ void __launch_bounds__(THREADS, 1)
           pk[i] = *reinterpret_cast<uint32_t*>(&a2);
           dk[i] = *reinterpret_cast<uint32_t*>(&b2);
         }
+        // the P^T / dS^T buffers are free once the dV / dK MMAs of sub-tile g-2 are done (waited only
+        // now, so the score loads and the exponentials above overlap those MMAs)
+        mbar_wait(&p_empty[buf], ((g >> 1) & 1) ^ 1);
+        tc_fence_after();
         // P^T: this thread's 32 queries -> 16 TMEM columns (bf16 pairs) of P buffer `buf`
         asm volatile(
             "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
