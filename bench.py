@@ -251,6 +251,8 @@ def main():
     ap.add_argument("--workload", default="cfg2", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--stash-policy", type=int, default=2)
+    ap.add_argument("--schedule", default="harmony", choices=["harmony", "baseline"],
+                    help="harmony: Harmony-DP; baseline: the paper's per-GPU-virtualization comparison (Fig. 5(b))")
     ap.add_argument("--microbatches", type=int, default=0,
                     help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -308,7 +310,8 @@ def main():
     params = synth.gen_params(descs, precision)
     cfg = dict(rank=rank, world_size=world, device=local, hbm_cap_bytes=wl["cap"], microbatches=m,
                microbatch_size=B // m, precision=precision, stash_policy=args.stash_policy if precision else 0,
-               lr=1e-4, nccl_id=nccl_id)
+               lr=1e-4, nccl_id=nccl_id,
+               schedule=H.HARMONY_SCHED_PER_GPU_VIRT if args.schedule == "baseline" else H.HARMONY_SCHED_HARMONY_DP)
     h = H.Harmony(descs, params, **cfg)
     del params
     plan = h.plan().as_dict()
@@ -398,7 +401,7 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "bf16" if precision else "f32", "data": "synthetic (seeded, paper-shaped)",
         "config": {"workload": wl["name"], "global_batch": B * world, "seq_len": wl["S"],
-                   "microbatches": m, "microbatch_size": B // m,
+                   "microbatches": m, "microbatch_size": B // m, "schedule": args.schedule,
                    "parallelism": f"dp{world}", "hbm_cap_bytes_per_gpu": wl["cap"],
                    "arena_bytes": plan["arena_bytes"], "stash_policy": cfg["stash_policy"],
                    "l2": "inputs and per-step swap traffic (tens of GB) far larger than the 126 MB L2; no flush"},

@@ -601,7 +601,7 @@ harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const h
     const int64_t sh = lp.shard, P = lp.P;
     c->h_wc[l] = static_cast<uint8_t*>(alloc_host((size_t)sh * ts));
     c->h_state[l] = static_cast<float*>(alloc_host((size_t)lp.state_bytes));
-    if (p.retain_grads) c->h_grad[l] = static_cast<float*>(alloc_host((size_t)sh * 4));
+    if (p.retain_grads || p.schedule == HARMONY_SCHED_PER_GPU_VIRT) c->h_grad[l] = static_cast<float*>(alloc_host((size_t)sh * 4));
     float* master = c->h_state[l];
     memset(master, 0, lp.state_bytes);  // m = v = 0 (reading c3), padding = 0
     const int64_t lo = (int64_t)r * sh, hi = std::min<int64_t>(P, lo + sh);

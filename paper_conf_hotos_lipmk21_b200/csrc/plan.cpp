@@ -25,8 +25,6 @@ void validate_config(const harmony_config& c) {
            "unknown precision");
   HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP || c.schedule == HARMONY_SCHED_PER_GPU_VIRT, HARMONY_E_INVALID_ARG,
            "unknown schedule");
-  HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
-           "the per-GPU-virtualization baseline schedule is not built yet (SURVEY NEXT-3)");
   HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 3, HARMONY_E_INVALID_ARG, "stash_policy must be 0..3");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
@@ -568,6 +566,12 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
         spill_task[(size_t)l * m + i] = (int)tasks.size();
       }
       if (slot >= 0) wslot_last[slot] = (int)tasks.size();
+      if (baseline && slot >= 0) {  // per-GPU virtualization: weights out again after each forward
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
+        d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
+        t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
+      }
       tasks.push_back(t);
     }
   }
@@ -611,6 +615,18 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     if (N > 1) { t.op.grad = p.gsh[l % 2]; gkey = key(R_GSH, l % 2); }
     else t.op.grad = p.dw[j];
     t.rd = {gkey};
+    if (baseline) {
+      // the baseline updates after the whole backward: this layer's gradient was
+      // swapped out after its backward and comes back now
+      Item it;
+      it.need = (int)tasks.size();
+      it.release = (int)tasks.size() - 1;
+      Op h;
+      h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_GRAD; h.layer = l;
+      h.hbuf = HB_GRAD; h.hidx = l; h.dev = t.op.grad; h.bytes = (uint64_t)lp.shard * 4;
+      it.ops.push_back({h, {{key(H_GRAD, l)}, {gkey}}});
+      items.push_back(it);
+    }
     int sslot = -1;
     if (lp.state_res >= 0) {
       t.op.state = (uint64_t)lp.state_res;
@@ -636,8 +652,10 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
       t.post.push_back({d, {{key(R_SSLOT, sslot)}, {key(H_STATE, l)}}});
       sslot_last[sslot] = (int)tasks.size();
     }
-    // the compute copy this rank's shard is written into
-    const int wsl = bwd_wslot[l];
+    // the compute copy this rank's shard is written into (the baseline's backward slot of this layer
+    // was reused long ago: it takes the next slot in turn)
+    int wsl = bwd_wslot[l];
+    if (baseline && lp.wc_res < 0) { wsl = wnext; wnext = (wnext + 1) % nW; }
     const uint64_t sh_bytes = (uint64_t)lp.shard * ts;
     if (lp.wc_res >= 0) {
       t.op.w = (uint64_t)lp.wc_res;
@@ -708,6 +726,24 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
         rs.dev = p.dw[j]; rs.grad = p.gsh[l % 2]; rs.count = (uint64_t)lp.shard;
         rs.bytes = (uint64_t)lp.shard * 4 * (N - 1);
         t.post.push_back({rs, {{key(R_DW, j)}, {key(R_GSH, l % 2)}}});
+      }
+      if (baseline) {
+        // per-GPU virtualization swaps the layer's weights out again after every microbatch's
+        // backward (Fig. 5(b); clean, so the bytes are those already on the host), and
+        // parks the finished gradient on the host until the update at the end of the backward
+        if (slot >= 0) {
+          Op d;
+          d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
+          d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
+          t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
+        }
+        if (i == m - 1) {
+          const uint64_t gk = N > 1 ? key(R_GSH, l % 2) : key(R_DW, j);
+          Op d;
+          d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_GRAD; d.layer = l;
+          d.hbuf = HB_GRAD; d.hidx = l; d.dev = N > 1 ? p.gsh[l % 2] : p.dw[j]; d.bytes = (uint64_t)lp.shard * 4;
+          t.post.push_back({d, {{gk}, {key(H_GRAD, l)}}});
+        }
       }
       tasks.push_back(t);
     }

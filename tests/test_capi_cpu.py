@@ -116,6 +116,30 @@ def test_harmony_dp_weight_swap_volume_is_3W():
     assert s.pred_h2d_weight_bytes + s.pred_d2h_weight_bytes < oracle.weight_swap_baseline_dp(Wb, 4, 1)
 
 
+@pytest.mark.parametrize("m", [1, 2, 4])
+def test_baseline_schedule_weight_swap_volume(m):
+    """P:726-731 (Fig. 5(b)): DP with per-GPU memory virtualization swaps W in and out for the
+    forward and the backward of every microbatch, plus in and out for the update: (4m+2)N|W| in the
+    paper's count.  Here the update's swap-in of W is the fp32 master copy inside the Adam state, so
+    the compute-copy ledger is (4m+1)|W| — against Harmony-DP's 3|W| at the same cap.  The baseline
+    updates after the whole backward, so each layer's gradient is parked on the host and comes back."""
+    kw = dict(CFG1, microbatches=m, microbatch_size=32 // m)
+    cap = min_cap(MLP, **dict(kw, schedule=H.HARMONY_SCHED_PER_GPU_VIRT))
+    s, ops = plan(MLP, **dict(kw, hbm_cap_bytes=cap, schedule=H.HARMONY_SCHED_PER_GPU_VIRT))
+    Wb = s.total_weight_bytes
+    assert s.resident_weight_bytes == 0 and s.hazards == 0
+    assert s.pred_h2d_weight_bytes == 2 * m * Wb and s.pred_d2h_weight_bytes == (2 * m + 1) * Wb
+    assert s.pred_h2d_weight_bytes + s.pred_d2h_weight_bytes + Wb == oracle.weight_swap_baseline_dp(Wb, m, 1)
+    grad = [o for o in ops if o["cat"] == "grad"]
+    assert sorted((o["kind"], o["l"]) for o in grad) == sorted([("D2H", l) for l in range(4)] + [("H2D", l) for l in range(4)])
+    # every update after the last backward (P:351-353)
+    comp = [(o["kind"], o["l"]) for o in ops if o["stream"] == "compute"]
+    last_bwd = max(k for k, (kind, _) in enumerate(comp) if kind == "BWD")
+    assert all(k > last_bwd for k, (kind, _) in enumerate(comp) if kind == "UPD")
+    s2, _ = plan(MLP, **dict(kw, hbm_cap_bytes=cap))
+    assert s2.pred_h2d_weight_bytes + s2.pred_d2h_weight_bytes == oracle.weight_swap_harmony_dp(Wb, m, 1)
+
+
 @pytest.mark.parametrize("m", [1, 2, 4, 8])
 def test_grouping_weight_traffic_independent_of_m(m):
     """a task runs over its group of m microbatches back to back, so W is swapped once."""

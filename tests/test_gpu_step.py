@@ -185,6 +185,30 @@ def test_transformer_bf16_matches_oracle_and_capped_bitwise(causal, S):
     bitwise_equal(capped, uncapped)
 
 
+@pytest.mark.parametrize("bf16", [False, True])
+def test_baseline_schedule_is_bitwise_identical_to_harmony_dp(bf16):
+    """The per-GPU-virtualization baseline (Fig. 5(b): per-microbatch weight swaps, updates after the
+    whole backward, gradients parked on the host) computes exactly what Harmony-DP computes (reading
+    c4: no layer's W is read after its own backward), while moving (4m+1)|W| of weights instead of 3|W|."""
+    if bf16:
+        descs, params, batches, kw = tiny_transformer(True, 1, L=3, d=128, h=2, S=128, B=4, m=2)
+    else:
+        descs = CFG1["descs"]()
+        params = synth.gen_params(descs)
+        batches = batches_for(descs, CFG1["batch"], 2, 0)
+        kw = dict(microbatches=CFG1["m"], microbatch_size=CFG1["batch"] // CFG1["m"])
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, schedule=H.HARMONY_SCHED_PER_GPU_VIRT, **kw),
+                              descs, text_len=0)
+    cap = int(s.min_working_set_bytes * 1.2)
+    a, pa = run_gpu(descs, params, batches, hbm_cap_bytes=cap, **kw)
+    b, pb = run_gpu(descs, params, batches, hbm_cap_bytes=cap, schedule=H.HARMONY_SCHED_PER_GPU_VIRT, **kw)
+    bitwise_equal(a, b)
+    wa = a[-1]["stats"]["h2d_weight_bytes"] + a[-1]["stats"]["d2h_weight_bytes"]
+    wb = b[-1]["stats"]["h2d_weight_bytes"] + b[-1]["stats"]["d2h_weight_bytes"]
+    assert wb > wa, (wa, wb)
+    assert b[-1]["stats"]["d2h_grad_bytes"] > 0
+
+
 @pytest.mark.parametrize("S", [64, 128])
 @pytest.mark.parametrize("policy", [1, 2, 3])
 def test_transformer_bf16_recompute_policies_are_bitwise_identical(policy, S):
