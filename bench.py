@@ -253,6 +253,8 @@ def main():
     ap.add_argument("--stash-policy", type=int, default=2)
     ap.add_argument("--schedule", default="harmony", choices=["harmony", "baseline"],
                     help="harmony: Harmony-DP; baseline: the paper's per-GPU-virtualization comparison (Fig. 5(b))")
+    ap.add_argument("--tune", action="store_true",
+                    help="pick the microbatch count by the tuner (plan feasibility + 2 timed steps per candidate)")
     ap.add_argument("--microbatches", type=int, default=0,
                     help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -308,6 +310,18 @@ def main():
         nccl_id = obj[0]
     t_setup = time.perf_counter()
     params = synth.gen_params(descs, precision)
+    tuning = None
+    if args.tune and world == 1:
+        from paper_conf_hotos_lipmk21_b200 import tuner
+        Xt, Tt = synth.gen_batch(descs, B, 1, precision)
+        Xt, Tt = torch.tensor(Xt, device=device), torch.tensor(Tt, device=device)
+        tcfg = dict(hbm_cap_bytes=wl["cap"], precision=precision, stash_policy=args.stash_policy if precision else 0,
+                    lr=1e-4)
+        res = tuner.tune_microbatches(descs, B, tcfg, tuner.measure_on_device(descs, params, Xt, Tt, tcfg))
+        m = res.best
+        tuning = res.as_dict()
+        del Xt, Tt
+        torch.cuda.empty_cache()
     cfg = dict(rank=rank, world_size=world, device=local, hbm_cap_bytes=wl["cap"], microbatches=m,
                microbatch_size=B // m, precision=precision, stash_policy=args.stash_policy if precision else 0,
                lr=1e-4, nccl_id=nccl_id,
@@ -402,6 +416,7 @@ def main():
         "vs_baseline": None, "dtype": "bf16" if precision else "f32", "data": "synthetic (seeded, paper-shaped)",
         "config": {"workload": wl["name"], "global_batch": B * world, "seq_len": wl["S"],
                    "microbatches": m, "microbatch_size": B // m, "schedule": args.schedule,
+                   **({"tuning": tuning} if tuning else {}),
                    "parallelism": f"dp{world}", "hbm_cap_bytes_per_gpu": wl["cap"],
                    "arena_bytes": plan["arena_bytes"], "stash_policy": cfg["stash_policy"],
                    "l2": "inputs and per-step swap traffic (tens of GB) far larger than the 126 MB L2; no flush"},

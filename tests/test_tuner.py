@@ -1,0 +1,45 @@
+"""Microbatch-size tuner: host logic on CPU with a synthetic step-time model; the
+planner decides feasibility under the cap (harmony_plan_dry), the measurement picks the winner."""
+import pytest
+
+import synth
+from paper_conf_hotos_lipmk21_b200 import harmony as H
+from paper_conf_hotos_lipmk21_b200 import tuner
+
+
+def test_candidates_divide_the_batch():
+    assert tuner.candidates(64) == [1, 2, 4, 8, 16]
+    assert tuner.candidates(6) == [1, 2]
+    assert tuner.candidates(1) == [1]
+
+
+def test_tuner_skips_infeasible_and_picks_fastest():
+    descs = synth.transformer_stack(4, 64, 4, 16, False)
+    cfg = dict(precision=1, stash_policy=2)
+    # a cap the widest microbatch (m=1, 8 sequences) cannot meet, but m >= 2 can
+    s1, _ = H.harmony_plan_dry(H.make_config(microbatches=1, microbatch_size=8, hbm_cap_bytes=1 << 40, **cfg), descs,
+                               text_len=0)
+    s2, _ = H.harmony_plan_dry(H.make_config(microbatches=2, microbatch_size=4, hbm_cap_bytes=1 << 40, **cfg), descs,
+                               text_len=0)
+    assert s2.min_working_set_bytes < s1.min_working_set_bytes
+    cap = s2.min_working_set_bytes
+    seen = []
+
+    def measure(m, b):  # per-launch overhead vs. nothing else: fewer, larger microbatches win
+        seen.append(m)
+        return 1e-3 * m + 1e-4
+
+    r = tuner.tune_microbatches(descs, 8, dict(cfg, hbm_cap_bytes=cap), measure)
+    trials = {t.microbatches: t for t in r.trials}
+    assert not trials[1].feasible and trials[1].reason
+    assert 1 not in seen and r.best == 2
+    d = r.as_dict()
+    assert d["best_microbatches"] == 2 and len(d["trials"]) == len(tuner.candidates(8))
+
+
+def test_tuner_breaks_ties_toward_larger_microbatches_and_raises_when_nothing_fits():
+    descs = synth.mlp_stack(4, 256)
+    r = tuner.tune_microbatches(descs, 32, dict(hbm_cap_bytes=0), lambda m, b: 1.0)
+    assert r.best == 1
+    with pytest.raises(H.HarmonyError):
+        tuner.tune_microbatches(descs, 32, dict(hbm_cap_bytes=1024), lambda m, b: 1.0)
