@@ -298,12 +298,6 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       bulk_wait_read<1>();
     }
     float v[CPB];
-    if (p.tma_epi == 2) {  // DEBUG
-      tmem_ld32(tacc + CPB * bi, v);
-      if (v[0] == 123.f && lane == 99) printf("x");
-      ++w.j;
-      continue;
-    }
     if (have_acc) {
 #pragma unroll
       for (int h = 0; h < CPB / 32; ++h) tmem_ld32(tacc + CPB * bi + 32 * h, v + 32 * h);
@@ -628,7 +622,7 @@ static void make_epi_maps(const hk_gemm_args& a, const EpiParams& e, int bn, CUt
   else if (epi == HK_EPI_ACC_F32 && e.accumulate) ok = ok && mk(mi, e.C, 4);
   else if (epi == HK_EPI_ACT_BWD) ok = ok && mk(mi, e.aux, 2);
   if (epi == HK_EPI_BIAS_ACT) ok = ok && mk(mo, e.aux_out, 2);
-  p.tma_epi = ok ? (enabled == 2 ? 2 : 1) : 0;  // DEBUG 2: drain TMEM only
+  p.tma_epi = ok ? 1 : 0;
 }
 
 static void make_operand_map(CUtensorMap* map, const void* ptr, int mn_major, int64_t rows, int64_t K, int64_t ld,

@@ -3,6 +3,7 @@
 
 #include <algorithm>
 #include <array>
+#include <cstdlib>
 #include <deque>
 #include <map>
 #include <sstream>
@@ -335,7 +336,12 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     HM_CHECK(p.min_ws_bytes <= p.cap, HARMONY_E_CAP_TOO_SMALL,
              "hbm_cap_bytes " + std::to_string(p.cap) + " < minimum working set " + std::to_string(p.min_ws_bytes));
     // slot counts in order of preference (double buffering needs memory)
-    const int pref[][3] = {{2, 2, 2}, {2, 1, 2}, {2, 1, 1}, {1, 1, 2}, {1, 1, 1}};
+    // Small stash entries get four staging slots: a stash swap-in waits for its slot to be released
+    // by the backward two entries back, and on the one H2D stream that wait would hold up the
+    // state swap-ins queued behind it (head-of-line blocking; cfg3: 26 MB entries, 16 GiB cap)
+    int gq = maxst > 0 && maxst * 4 <= p.cap / 64 ? 4 : 2;
+    if (const char* e = getenv("HARMONY_STAGE_SLOTS")) gq = std::max(1, std::min(8, atoi(e)));  // experiments
+    const int pref[][3] = {{2, 2, gq}, {2, 2, std::min(gq, 2)}, {2, 1, 2}, {2, 1, 1}, {1, 1, 2}, {1, 1, 1}};
     for (auto& c : pref) {
       if (fixed + c[0] * maxw + c[1] * maxs + c[2] * maxst <= p.cap) { nW = c[0]; nS = c[1]; nG = c[2]; break; }
     }
