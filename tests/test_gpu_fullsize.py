@@ -70,6 +70,40 @@ def test_cfg3_block_full_width_matches_oracle():
     one_block_vs_oracle(1600, 25, 1024, True, m=2, b=4, cap=16 << 30)
 
 
+@pytest.mark.slow
+def test_cfg4_blocks_full_width_streamed_match_oracle():
+    """cfg4's 11B-class block geometry (d=5120, h=40, S=1024, causal; 314.6M parameters per block),
+    two blocks at full width with every bf16 weight and every fp32 master/m/v streamed from pinned
+    host memory (a cap that holds one layer's slots and nothing resident), against the oracle."""
+    descs = synth.transformer_stack(2, 5120, 40, 1024, True)
+    kw = dict(microbatches=2, microbatch_size=1, precision=1, stash_policy=2)
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, **kw), descs, text_len=0)
+    cap = int(s.min_working_set_bytes * 1.05)
+    s2, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=cap, **kw), descs, text_len=0)
+    assert s2.resident_state_bytes == 0 and s2.resident_weight_bytes == 0 and s2.hazards == 0
+    params = synth.gen_params(descs, synth.BF16)
+    X, T = synth.gen_batch(descs, 2, 1, synth.BF16)
+    with H.Harmony(descs, params, retain_grads=1, hbm_cap_bytes=cap, **kw) as hm:
+        loss, st = hm.step(torch.tensor(X, device="cuda"), torch.tensor(T, device="cuda"))
+        got = [(hm.read(l, H.HARMONY_GRAD), hm.read(l), hm.read(l, H.HARMONY_ADAM_M), hm.read(l, H.HARMONY_ADAM_V))
+               for l in range(2)]
+    assert st.h2d_weight_bytes > 0 and st.h2d_state_bytes > 0
+    P = [p.astype(np.float64) for p in params]
+    del params
+    ref_loss, ref_g, ref_P, ref_st = oracle.train_step(descs, P, oracle.AdamState.zeros(P), X.astype(np.float64),
+                                                       T.astype(np.float64))
+    errs = {"loss": abs(loss - ref_loss) / abs(ref_loss)}
+    for l in range(2):
+        g, W, mm, v = got[l]
+        errs[f"g{l}"] = rel(g, ref_g[l])
+        errs[f"W{l}"] = rel(W, ref_P[l])
+        errs[f"m{l}"] = rel(mm, ref_st.m[l])
+        errs[f"sqrt_v{l}"] = rel(np.sqrt(v), np.sqrt(ref_st.v[l]))
+    print({k: f"{v_:.2e}" for k, v_ in errs.items()})
+    for k, e in errs.items():
+        assert e <= 2e-2, (k, e, errs)
+
+
 def _digests(hm, n_layers):
     out = []
     for l in range(n_layers):
