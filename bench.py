@@ -45,6 +45,10 @@ WORKLOADS = {
     "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=2 x b=4), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
                  per_gpu_batch=8, m=2, cap=16 << 30, S=1024),
+    "cfg4s": dict(name="cfg4s: 8 of cfg4's 36 GPT blocks (d5120 h40 S1024 causal, 2.5B params), 8 seq/GPU (m=4 x b=2), "
+                       "bf16/fp32-master Adam, weights + Adam state streamed from pinned host (HBM cap 12 GiB/GPU)",
+                  model="gpt-11b-like-preLN-8-of-36", descs=lambda: synth.transformer_stack(8, 5120, 40, 1024, True),
+                  per_gpu_batch=8, m=4, cap=12 << 30, S=1024),
     "cfg5": dict(name="cfg5: one 16384 x 16384 x 65536 (M x N x K) bf16 GEMM fwd+bwd, operator split along K into "
                       "8 row-chunk tile subtasks per GPU (harmony_split_gemm_*)", model="gemm-16384x16384x65536",
                  M=16384, N=16384, K=65536, chunks=8, S=1, per_gpu_batch=1, m=1, cap=0),
