@@ -61,7 +61,7 @@ def build(force: bool = False, jobs: int = 0, verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
     flags = ARCH + ["-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
                     "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
-                    "-I", nccl_include(), "-DNDEBUG"]
+                    "-I", nccl_include(), "-DNDEBUG"] + os.environ.get("HARMONY_NVCC_EXTRA", "").split()
     hdr_mtime = max([os.path.getmtime(h) for h in headers()] + [os.path.getmtime(__file__)])
     srcs = sources()
     objs, todo = [], []
