@@ -190,6 +190,7 @@ __device__ __forceinline__ void drain_chunk(const EpiParams& e, uint32_t taddr, 
 struct TcParams {
   int M, N, K, nz0, nz, a_mn, b_mn;
   int tma_epi;  // 1: epilogue through shared-memory staging + TMA stores (maps tmC / tmIn / tmO2)
+  int group_m;  // tile raster: GROUP_M consecutive m-tiles per n sweep (order only; results unchanged)
   EpiParams e;
 };
 
@@ -427,10 +428,19 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 
 // Persistent tile walk shared by the three roles: tile t -> (z, m_blk, n_blk), grouped along M
 // (GROUP_M row-blocks share their B column panels in L2).
+// HARMONY_GEMM_GROUP_M (default 8): raster width of the persistent tile order, an A/B knob
+static int gemm_group_m() {
+  static const int g = [] {
+    const char* v = getenv("HARMONY_GEMM_GROUP_M");
+    const int x = v ? atoi(v) : 8;
+    return x >= 1 ? x : 8;
+  }();
+  return g;
+}
+
 struct TileMap {
-  int tiles_m, tiles_n, per_z, total;
+  int tiles_m, tiles_n, per_z, total, GROUP_M;
   __device__ __forceinline__ void get(int t, int& z, int& mb, int& nb) const {
-    constexpr int GROUP_M = 8;
     z = t / per_z;
     int r = t - z * per_z;
     int group = r / (GROUP_M * tiles_n);
@@ -467,6 +477,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   tm.tiles_n = (p.N + BN - 1) / BN;
   tm.per_z = tm.tiles_m * tm.tiles_n;
   tm.total = tm.per_z * p.nz;
+  tm.GROUP_M = p.group_m;
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmA);
@@ -639,6 +650,7 @@ static void launch_tc(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st
   make_operand_map(&mb, a.B, a.b_mn_major, a.N, a.K, a.ldb, a.nz0, a.b_sz0, a.nz1, a.b_sz1, BN);
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
+  p.group_m = gemm_group_m();
   p.e = e;
   CUtensorMap mc, mi, mo;
   make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
@@ -762,6 +774,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   tm.tiles_n = (p.N + BN - 1) / BN;
   tm.per_z = tm.tiles_m * tm.tiles_n;
   tm.total = tm.per_z * p.nz;
+  tm.GROUP_M = p.group_m;
   const int pair = (int)cluster_id_x(), npairs = (int)nclusters_x();
 
   if (warp == 0 && lane == 0) {
@@ -905,6 +918,7 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   make_operand_map(&mb, a.B, a.b_mn_major, a.N, a.K, a.ldb, a.nz0, a.b_sz0, a.nz1, a.b_sz1, Cfg::HB);
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
+  p.group_m = gemm_group_m();
   p.e = e;
   CUtensorMap mc, mi, mo;
   make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
