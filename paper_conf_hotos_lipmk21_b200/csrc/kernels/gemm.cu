@@ -728,6 +728,22 @@ __device__ __forceinline__ void mma_bf16_2sm(uint32_t tmem_d, uint64_t adesc, ui
       "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
       "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
 }
+// the four K=16 UMMAs of one 64-deep k-block in one asm block (one operand hand-off to the
+// uniform datapath instead of four); the first accumulates only if acc != 0, the rest always
+__device__ __forceinline__ void mma4_bf16_2sm(uint32_t tmem_d, uint64_t ad, uint64_t bd, uint32_t a_kst, uint32_t b_kst,
+                                              uint32_t idesc, uint32_t acc) {
+  const uint64_t a1 = ad + a_kst, a2 = ad + 2 * a_kst, a3 = ad + 3 * a_kst;
+  const uint64_t b1 = bd + b_kst, b2 = bd + 2 * b_kst, b3 = bd + 3 * b_kst;
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t"
+      "setp.ne.b32 p, %10, 0;\n\t"
+      "setp.eq.b32 q, %0, %0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %9, p;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %3, %4, %9, q;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %5, %6, %9, q;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %7, %8, %9, q;\n\t}" ::"r"(tmem_d),
+      "l"(ad), "l"(bd), "l"(a1), "l"(b1), "l"(a2), "l"(b2), "l"(a3), "l"(b3), "r"(idesc), "r"(acc));
+}
 __device__ __forceinline__ void mma_commit_2sm_mc(uint64_t* bar) {
   asm volatile(
       "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
@@ -836,6 +852,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       // ===== MMA issuer (leader CTA, single thread): M=256 x N=BN UMMAs over the pair =====
       const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)p.a_mn << 15) |
                              ((uint32_t)p.b_mn << 16) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+      // descriptors built once: stage s, sub-step kk is base + s * stage stride + kk * k-step in the
+      // 14-bit start-address field (shared addresses < 2^18, so the adds never carry out of it)
+      const uint64_t a_d0 = make_sdesc(smem_u32(sA), p.a_mn ? BK * 128 : 16, 1024);
+      const uint64_t b_d0 = make_sdesc(smem_u32(sB), p.b_mn ? BK * 128 : 16, 1024);
+      const uint32_t a_kst = p.a_mn ? 2048 >> 4 : 32 >> 4, b_kst = p.b_mn ? 2048 >> 4 : 32 >> 4;
+      static_assert(BK / 16 == 4, "four UMMAs per k-block");
       int s = 0;
       uint32_t ph = 0;
       int it = 0;
@@ -847,14 +869,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&full[s], ph);
           tc_fence_after();
-          const uint32_t a = smem_u32(sA + s * Cfg::A_BYTES);
-          const uint32_t b = smem_u32(sB + s * Cfg::B_BYTES);
-#pragma unroll
-          for (int kk = 0; kk < BK / 16; ++kk) {
-            uint64_t ad = p.a_mn ? make_sdesc(a + kk * 2048, BK * 128, 1024) : make_sdesc(a + kk * 32, 16, 1024);
-            uint64_t bd = p.b_mn ? make_sdesc(b + kk * 2048, BK * 128, 1024) : make_sdesc(b + kk * 32, 16, 1024);
-            mma_bf16_2sm(tmem_d, ad, bd, idesc, (kb | kk) ? 1u : 0u);
-          }
+          const uint64_t ad = a_d0 + (uint64_t)(s * (Cfg::A_BYTES >> 4));
+          const uint64_t bd = b_d0 + (uint64_t)(s * (Cfg::B_BYTES >> 4));
+          mma4_bf16_2sm(tmem_d, ad, bd, a_kst, b_kst, idesc, kb ? 1u : 0u);
           mma_commit_2sm_mc(&empty[s]);  // frees this stage in both CTAs
           if (++s == STAGES) { s = 0; ph ^= 1; }
         }
