@@ -411,6 +411,22 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
   }
 }
 
+// the four K=16 UMMAs of one 64-deep k-block in one asm block (see mma4_bf16_2sm)
+__device__ __forceinline__ void mma4_bf16(uint32_t tmem_d, uint64_t ad, uint64_t bd, uint32_t a_kst, uint32_t b_kst,
+                                          uint32_t idesc, uint32_t acc) {
+  const uint64_t a1 = ad + a_kst, a2 = ad + 2 * a_kst, a3 = ad + 3 * a_kst;
+  const uint64_t b1 = bd + b_kst, b2 = bd + 2 * b_kst, b3 = bd + 3 * b_kst;
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t"
+      "setp.ne.b32 p, %10, 0;\n\t"
+      "setp.eq.b32 q, %0, %0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %9, p;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %3, %4, %9, q;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %5, %6, %9, q;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %7, %8, %9, q;\n\t}" ::"r"(tmem_d),
+      "l"(ad), "l"(bd), "l"(a1), "l"(b1), "l"(a2), "l"(b2), "l"(a3), "l"(b3), "r"(idesc), "r"(acc));
+}
+
 template <int BN, int STAGES>
 struct TcCfg {
   static constexpr int A_BYTES = BM * BK * 2;  // 16 KB
@@ -537,6 +553,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       int it = 0;
+      const uint64_t a_d0 = make_sdesc(smem_u32(sA), p.a_mn ? BK * 128 : 16, 1024);
+      const uint64_t b_d0 = make_sdesc(smem_u32(sB), p.b_mn ? BK * 128 : 16, 1024);
+      const uint32_t a_kst = p.a_mn ? 2048 >> 4 : 32 >> 4, b_kst = p.b_mn ? 2048 >> 4 : 32 >> 4;
+      static_assert(BK / 16 == 4, "four UMMAs per k-block");
       for (int t = blockIdx.x; t < tm.total; t += gridDim.x, ++it) {
         const int acc = it & 1;
         const uint32_t aph = (it >> 1) & 1;
@@ -546,16 +566,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&full[s], ph);
           tc_fence_after();
-          const uint32_t a = smem_u32(sA + s * Cfg::A_BYTES);
-          const uint32_t b = smem_u32(sB + s * Cfg::B_BYTES);
-#pragma unroll
-          for (int kk = 0; kk < BK / 16; ++kk) {
-            // K-major: 16 k = 32 bytes along the swizzled row; SBO = 8 rows * 128 B.
-            // MN-major: 16 k = 16 rows of 128 B; LBO = next 64-wide MN chunk (BK*128 B), SBO = 8 k-rows.
-            uint64_t ad = p.a_mn ? make_sdesc(a + kk * 2048, BK * 128, 1024) : make_sdesc(a + kk * 32, 16, 1024);
-            uint64_t bd = p.b_mn ? make_sdesc(b + kk * 2048, BK * 128, 1024) : make_sdesc(b + kk * 32, 16, 1024);
-            mma_bf16(tmem_d, ad, bd, idesc, (kb | kk) ? 1u : 0u);
-          }
+          // K-major: 16 k = 32 bytes along the swizzled row; SBO = 8 rows * 128 B.
+          // MN-major: 16 k = 16 rows of 128 B; LBO = next 64-wide MN chunk (BK*128 B), SBO = 8 k-rows.
+          const uint64_t ad = a_d0 + (uint64_t)(s * (Cfg::A_BYTES >> 4));
+          const uint64_t bd = b_d0 + (uint64_t)(s * (Cfg::B_BYTES >> 4));
+          mma4_bf16(tmem_d, ad, bd, a_kst, b_kst, idesc, kb ? 1u : 0u);
           mma_commit(&empty[s]);  // frees the smem stage once these MMAs complete
           if (++s == STAGES) { s = 0; ph ^= 1; }
         }
