@@ -197,12 +197,16 @@ __global__ void __launch_bounds__(THREADS, 1)
           mbar_wait(&s_empty[sb], ((it >> 1) & 1) ^ 1);
           tc_fence_after();
           const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
+          if constexpr (DH == 64) {  // one swizzle atom: the four K=16 steps from one asm block
+            mma4_bf16(tmem + sb * Cfg::S_COLS, make_sdesc(qa, 16, 1024), make_sdesc(ka, 16, 1024), 2, 2, idesc_s, 0u);
+          } else {
 #pragma unroll
-          for (int kk = 0; kk < DH / 16; ++kk) {
-            const int atom = kk / 4, sub = kk % 4;
-            uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
-            uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
-            mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
+            for (int kk = 0; kk < DH / 16; ++kk) {
+              const int atom = kk / 4, sub = kk % 4;
+              uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
+              uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
+              mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
+            }
           }
           mma_commit(&k_empty[ks]);
           mma_commit(&s_full[sb]);

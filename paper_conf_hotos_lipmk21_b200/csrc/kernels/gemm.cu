@@ -411,22 +411,6 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
   }
 }
 
-// the four K=16 UMMAs of one 64-deep k-block in one asm block (see mma4_bf16_2sm)
-__device__ __forceinline__ void mma4_bf16(uint32_t tmem_d, uint64_t ad, uint64_t bd, uint32_t a_kst, uint32_t b_kst,
-                                          uint32_t idesc, uint32_t acc) {
-  const uint64_t a1 = ad + a_kst, a2 = ad + 2 * a_kst, a3 = ad + 3 * a_kst;
-  const uint64_t b1 = bd + b_kst, b2 = bd + 2 * b_kst, b3 = bd + 3 * b_kst;
-  asm volatile(
-      "{\n\t.reg .pred p, q;\n\t"
-      "setp.ne.b32 p, %10, 0;\n\t"
-      "setp.eq.b32 q, %0, %0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %9, p;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %3, %4, %9, q;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %5, %6, %9, q;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %7, %8, %9, q;\n\t}" ::"r"(tmem_d),
-      "l"(ad), "l"(bd), "l"(a1), "l"(b1), "l"(a2), "l"(b2), "l"(a3), "l"(b3), "r"(idesc), "r"(acc));
-}
-
 template <int BN, int STAGES>
 struct TcCfg {
   static constexpr int A_BYTES = BM * BK * 2;  // 16 KB
