@@ -4,15 +4,17 @@ swap GB/s and % of roofline).
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload cfg2] [--impl ours|reference]
 
 N=1: the workload BASELINE.json's metric is quoted on that fits one GPU — configs[1], BERT-Large
-(24 pre-LN blocks, d=1024, h=16, S=512), 64 sequences per GPU as 8 microbatches, bf16 tensor-core
+(24 pre-LN blocks, d=1024, h=16, S=512), 64 sequences per GPU as 2 microbatches of 32, bf16 tensor-core
 compute with fp32 master weights + Adam, per-GPU HBM cap 8 GiB.  N>1 (torchrun, one process per
-GPU): the same per-GPU work on every rank (weak scaling), data-parallel with NCCL reduce-scatter
-of gradients and all-gather of weight shards inside the library.
+GPU; `--gpus N` without torchrun re-launches itself under torchrun): the same per-GPU work on every
+rank (weak scaling), data-parallel with NCCL reduce-scatter of gradients and all-gather of weight
+shards inside the library.
 
 `value` = samples / device time of the K timed steps (CUDA events on the library's streams,
 inputs resident in HBM, max over ranks).  `e2e` = the same through the C ABI with pinned HOST
 inputs (the H2D of X and T and the D2H of the loss inside the timed region), host wall clock.
-`--impl reference` times the CPU oracle (fp64 NumPy) on a bounded sample of the same workload.
+`--impl reference` times the CPU oracle (fp64 NumPy): one complete full-depth step at batch 1,
+split over the K timed steps; `cpu_baseline` is the same complete step, timed once.
 """
 from __future__ import annotations
 
@@ -141,35 +143,103 @@ def host_link_bandwidth(torch, device):
     return out
 
 
-def cpu_oracle_sample(wl, budget_s=20.0):
-    """Time the fp64 oracle (as it stands) on a bounded sample of the workload: forward+backward
-    of ONE sample through `ls` of the L layers, plus Adam on those layers' parameters; scale to the
-    full step (per-sample cost x batch + Adam) x L/ls.  Returns (samples/s, description, cores)."""
+def oracle_step_work(wl, batch=1):
+    """One complete oracle training step of the workload's full stack (every layer: forward, the
+    loss, backward, Adam) on `batch` sequences, as a list of work items in the step's order (the
+    oracle's own block functions, called as oracle.stack_loss_and_grads / train_step call them).
+    Returns (items, n_samples); each item is a no-argument callable."""
     import oracle
+    from oracle.layers import transformer_block_bwd, mlp_layer_bwd
     descs = wl["descs"]()
+    prec = wl.get("precision", 1)
+    params = [p.astype(np.float64) for p in synth.gen_params(descs, prec)]
+    X, T = synth.gen_batch(descs, batch, 1, prec)
+    X, T = X.astype(np.float64), T.astype(np.float64)
+    st = {"A": X, "caches": [None] * len(descs), "grads": [None] * len(descs)}
+    state = oracle.AdamState.zeros(params)
+    items = []
+
+    def fwd(l):
+        def f():
+            A, caches = oracle.stack_forward([descs[l]], [params[l]], st["A"].reshape(batch, -1, descs[l].d_in))
+            st["A"], st["caches"][l] = A, caches[0]
+        return f
+
+    def loss():
+        st["loss"], st["A"] = oracle.mse_loss(st["A"], T, batch)
+
+    def bwd(l):
+        def f():
+            p, c = st["caches"][l]
+            if descs[l].kind == synth.LAYER_MLP:
+                st["A"], g = mlp_layer_bwd(st["A"], c, p, descs[l].act)
+            else:
+                st["A"], g = transformer_block_bwd(st["A"], c, p)
+            st["grads"][l] = synth.pack(descs[l], g)
+            st["caches"][l] = None
+        return f
+
+    def adam(l):
+        def f():
+            params[l], state.m[l], state.v[l] = oracle.adam_update(params[l], st["grads"][l], state.m[l], state.v[l],
+                                                                   1, 1e-4, 0.9, 0.999, 1e-8)
+        return f
+
     L = len(descs)
-    ls = 1 if descs[0].kind == synth.LAYER_TRANSFORMER else L
-    sub = descs[:ls]
-    params = [p.astype(np.float64) for p in synth.gen_params(sub, wl.get("precision", 1))]
-    X, T = synth.gen_batch(sub, 1, 1, wl.get("precision", 1))
+    items += [fwd(l) for l in range(L)] + [loss] + [bwd(l) for l in range(L - 1, -1, -1)] + [adam(l) for l in range(L)]
+    return items, batch
+
+
+def cores_used():
+    return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+
+
+def cpu_oracle_full_step(wl, batch=1):
+    """The fp64 oracle (as it stands) timed on one COMPLETE training step of the full-depth workload
+    at a batch of `batch` sequences: every layer's forward and backward, the loss and Adam over all
+    parameters (about 40 s for cfg2 on a 16-core host).  value = batch / measured seconds."""
+    items, n = oracle_step_work(wl, batch)
     t0 = time.perf_counter()
-    reps = 0
-    while True:
-        _, grads, _ = oracle.stack_loss_and_grads(sub, params, X.astype(np.float64), T.astype(np.float64))
-        reps += 1
-        if time.perf_counter() - t0 > budget_s * 0.6 or reps >= 50:
-            break
-    t_fb = (time.perf_counter() - t0) / reps
-    st = oracle.AdamState.zeros(params)
-    t1 = time.perf_counter()
-    for W, g, m, v in zip(params, grads, st.m, st.v):
-        oracle.adam_update(W, g, m, v, 1, 1e-3, 0.9, 0.999, 1e-8)
-    t_adam = time.perf_counter() - t1
+    for f in items:
+        f()
+    dt = time.perf_counter() - t0
+    L = len(wl["descs"]())
     B = wl["per_gpu_batch"]
-    step = (B * t_fb + t_adam) * (L / ls)
-    desc = (f"fp64 NumPy oracle: fwd+bwd of 1 sample through {ls} of {L} layers ({reps} reps, {t_fb:.3f} s each) "
-            f"+ Adam on those layers ({t_adam:.3f} s); scaled x{B} samples x{L // ls} layers = {step:.1f} s/step")
-    return B / step, desc, (len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count())
+    desc = (f"fp64 NumPy oracle, one complete step of all {L} layers (fwd, loss, bwd, Adam on every parameter) at "
+            f"batch {n} sequence(s) of the workload's shape: {dt:.1f} s measured")
+    return n / dt, desc, cores_used(), dt
+
+
+def run_reference(args, wl, metric, unit):
+    """--impl reference: the oracle on the box's host cores.  The K timed steps together run ONE
+    complete full-depth oracle training step at batch 1 (its work items — layer forwards, loss, layer
+    backwards, Adam per layer — split into K consecutive slices, one per timed step), so the run stays
+    within minutes and `value` = 1 sample / the measured time of that whole step (no extrapolation)."""
+    items, n = oracle_step_work(wl, 1)
+    warm, _ = oracle_step_work(dict(wl, descs=lambda: wl["descs"]()[:1]), 1)
+    for f in warm[:max(0, min(args.warmup, len(warm)))]:
+        f()
+    K = max(1, args.steps)
+    bounds = [round(i * len(items) / K) for i in range(K + 1)]
+    times = []
+    for k in range(K):
+        t0 = time.perf_counter()
+        for f in items[bounds[k]:bounds[k + 1]]:
+            f()
+        times.append(time.perf_counter() - t0)
+    total = sum(times)
+    value = n / total
+    L = len(wl["descs"]())
+    desc = (f"fp64 NumPy oracle, one complete step of all {L} layers (fwd, loss, bwd, Adam) at batch 1 sequence, "
+            f"its {len(items)} work items split over the {K} timed steps: {total:.1f} s measured")
+    line = {"impl": "reference", "metric": metric, "value": value, "unit": unit, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / K * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": wl["name"], "global_batch": wl["per_gpu_batch"] * max(args.gpus, 1),
+                       "seq_len": wl["S"], "parallelism": f"dp{args.gpus}"},
+            "cpu_baseline": {"value": value, "unit": unit, "cores": cores_used(), "kind": "oracle", "sample": desc},
+            "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
 
 
 def run_cfg5(args, wl, world, rank, local, torch, H):
@@ -265,31 +335,33 @@ def main():
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     wl = WORKLOADS[args.workload]
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: launch this script under torchrun with args.gpus ranks
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+        sys.exit(subprocess.call(cmd))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch one rank per GPU)")
+    # NCCL (one process per GPU): a fixed algorithm and protocol keep the reduce-scatter's summation
+    # order the same from run to run (reading c21); the caller's environment wins
+    os.environ.setdefault("NCCL_ALGO", "Ring")
+    os.environ.setdefault("NCCL_PROTO", "Simple")
     metric = "samples/sec/step under HBM cap"
     unit = "samples/s"
 
     if args.impl == "reference":
-        if rank != 0:
-            return
-        vals = []
-        desc = cores = None
-        for _ in range(args.warmup):
-            cpu_oracle_sample(wl, budget_s=2.0)
-        for _ in range(args.steps):
-            v, desc, cores = cpu_oracle_sample(wl, budget_s=8.0)
-            vals.append(v)
-        value = statistics.median(vals)
-        line = {"impl": "reference", "metric": metric, "value": value, "unit": unit, "n_gpus": args.gpus,
-                "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
-                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": wl["name"], "global_batch": wl["per_gpu_batch"] * max(args.gpus, 1),
-                           "seq_len": wl["S"], "parallelism": f"dp{args.gpus}"},
-                "cpu_baseline": {"value": value, "unit": unit, "cores": cores, "kind": "oracle", "sample": desc},
-                "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-        print(json.dumps(line))
+        if rank == 0 and args.workload != "cfg5":
+            run_reference(args, wl, metric, unit)
+        elif rank == 0:
+            print(json.dumps({"impl": "reference", "unavailable": "cfg5 is a single GEMM; its oracle is sampled dot "
+                                                                  "products (tests), not a throughput program"}))
         return
 
     import torch
@@ -346,7 +418,14 @@ def main():
         if dist is not None:
             dist.barrier()
 
-    bw = host_link_bandwidth(torch, device) if rank == 0 else None
+    # host link measured concurrently on every rank (they share the host's PCIe / memory system);
+    # the slowest rank's figures bound the step
+    barrier()
+    bw = host_link_bandwidth(torch, device)
+    if dist is not None:
+        t = torch.tensor([-bw["h2d"], -bw["d2h"], -bw["duplex"]], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        bw = {"h2d": -t[0].item(), "d2h": -t[1].item(), "duplex": -t[2].item(), "ranks": world}
     for _ in range(args.warmup):
         h.step(Xd, Td)
     # ---- timed region: device-resident inputs, CUDA-graph replay of the step program
@@ -461,8 +540,9 @@ def main():
                                       "pred_d2h_bytes", "n_ops", "hazards")},
     }
     if world == 1 and not args.no_cpu_baseline:
-        v, desc, cores = cpu_oracle_sample(wl)
-        line["cpu_baseline"] = {"value": v, "unit": unit, "cores": cores, "kind": "oracle", "sample": desc}
+        v, desc, cores, dt = cpu_oracle_full_step(wl, 1)
+        line["cpu_baseline"] = {"value": v, "unit": unit, "cores": cores, "kind": "oracle", "sample": desc,
+                                "measured_step_s": dt}
     txt = json.dumps(line)
     print(txt)
     if args.out:

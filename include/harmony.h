@@ -16,9 +16,16 @@
  * and inserts collectives to keep the result that of the plain single-device
  * step.
  *
- * Process model: ONE process per GPU (rank r of world_size).  Every rank calls
- * the same functions in the same order; collectives (NCCL, loaded with dlopen)
- * run inside harmony_step / harmony_read_state.
+ * Process models (both run the same planner and executor):
+ *  - ONE process per GPU (harmony_init; rank r of world_size).  Every rank calls
+ *    the same functions in the same order; collectives (NCCL, loaded with dlopen)
+ *    run inside harmony_step / harmony_read_state.
+ *  - ONE process, N ranks: "a single virtual accelerator device" (
+ *    harmony_init_group).  The caller holds one context and passes the global
+ *    batch; the library drives the N rank programs itself and runs the collectives
+ *    (reduce-scatter of dW, all-gather of weight shards and loss partials) as its own
+ *    pulls from the peers' HBM — over NVLink between GPUs, or inside one GPU when
+ *    ranks share it (a loopback that runs the N > 1 data path on a single B200).
  *
  * Conventions for every call:
  *  - Status codes only; no exception or abort crosses the ABI.  On failure
@@ -197,6 +204,21 @@ harmony_status harmony_get_unique_id(uint8_t out[128]);
  * the arena and, for world_size > 1, the NCCL communicator.  *out owns everything. */
 harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out);
 
+/* Single-process group: one context driving num_ranks data-parallel ranks (1..16), rank r on
+ * CUDA device devices[r] (NULL = all on device 0; repeated ordinals = ranks sharing a GPU, each
+ * with its own arena of cfg->hbm_cap_bytes).  cfg->rank, cfg->world_size, cfg->device and
+ * cfg->nccl_id are ignored; cfg->arena must be NULL.  Ranks on different GPUs need peer access
+ * (HARMONY_E_UNSUPPORTED otherwise).  Afterwards the context is used like a rank context:
+ * harmony_register_layers, harmony_step with the GLOBAL batch (x, target: num_ranks*m*b rows;
+ * rank r takes rows r*m*b .. (r+1)*m*b-1, reading c14), harmony_read_state (no collective),
+ * harmony_finalize.  harmony_step's stats are box totals (bytes summed over ranks); per-rank
+ * ledgers via harmony_read_rank_stats.  Collectives: rank r's reduced-gradient shard is the sum
+ * of the N ranks' fp32 partials in rank order 0..N-1 (deterministic, the same on one GPU or many);
+ * all-gathers are copies.  Per-kernel profiling is not available for num_ranks > 1. */
+harmony_status harmony_init_group(const harmony_config* cfg, int32_t num_ranks, const int32_t* devices,
+                                  harmony_ctx** out);
+harmony_status harmony_read_rank_stats(const harmony_ctx* ctx, int32_t rank, harmony_step_stats* out);
+
 /* Registers the layer stack and its initial fp32 parameters (canonical packing, one
  * host array per layer, identical on every rank).  Decomposes the step into tasks,
  * plans residency / slots / swap sets / the per-stream program, and fills the pinned
@@ -214,7 +236,11 @@ harmony_status harmony_register_layers(harmony_ctx* ctx, int32_t n_layers, const
  *  batch:  must equal m*b
  *  loss_out (nullable): the GLOBAL loss (rank partials summed in rank order, c22)
  *  stats (nullable): this rank's ledger for the step
- * Synchronous: returns when the update of every layer has finished on this GPU. */
+ * Synchronous: returns when the update of every layer has finished on this GPU.
+ * Ordering: the step's first copy waits for work the caller queued on the legacy default stream
+ * (e.g. torch ops on its default stream writing x / target); work on other caller streams must be
+ * synchronised by the caller before the call.  On any failure after work was issued the context
+ * is marked broken (only harmony_finalize is valid) and Adam's t is not advanced. */
 harmony_status harmony_step(harmony_ctx* ctx, const float* x, const float* target, int64_t batch, double* loss_out,
                             harmony_step_stats* stats);
 

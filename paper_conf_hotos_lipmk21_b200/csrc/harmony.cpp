@@ -3,9 +3,17 @@
 // Runtime pieces: the capped device arena (one block, laid out by the planner),
 // the pinned host store (this rank's shards of the fp32 master W, Adam m and v, the compute copy
 // of W, and the spilled activation stash), four CUDA streams {compute, h2d, d2h, comm} with the
-// plan's events, the NCCL communicator, and the copy ledger (bytes per tensor class, per step).
+// plan's events, the collectives, and the copy ledger (bytes per tensor class, per step).
 // The executor replays the static program of plan.cpp every step: for each op it waits on the
 // events of its cross-stream dependencies, issues the op on its stream, and records its event.
+//
+// Two process models share the executor:
+//  - one process per GPU (harmony_init; rank r of world_size, NCCL loaded with dlopen);
+//  - one process driving N ranks as "one virtual device" (harmony_init_group; SURVEY §8(b)
+//    primary mode): the context the caller holds owns N rank contexts, issues their
+//    programs op by op in lock step from one thread, and runs the collectives itself as pulls
+//    from the peers' arenas (kernels/collective.cu) — over NVLink between GPUs, or inside one
+//    GPU when ranks share it (the loopback that exercises N > 1 on a single B200).
 #include <cuda_runtime.h>
 #include <string.h>
 
@@ -39,14 +47,14 @@ static inline uint16_t f32_to_bf16_rne(float f) {
 
 using namespace hm;
 
-// One captured instance of the step program.
+// One captured instance of the step program (all ranks of a group in one graph).
 struct StepGraph {
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
   int sig = -1;                           // (x on device) | (target on device) << 1 at capture
-  std::vector<cudaGraphNode_t> in_nodes;  // input copies, re-pointed every step
-  std::vector<int> in_ops;
-  harmony_step_stats stats{};
+  struct In { int rank, op; cudaGraphNode_t node; };
+  std::vector<In> in_nodes;               // input copies, re-pointed every step
+  std::vector<harmony_step_stats> stats;  // per rank
   uint64_t launches = 0;
   std::vector<KProf::Rec> recs;           // profiled graph: timing-event pairs of its kernels
   std::vector<KProf::OpRec> oprecs;       // profiled graph: timing-event pairs of its ops
@@ -59,6 +67,7 @@ struct harmony_ctx {
   cudaStream_t st[S_NUM] = {};
   std::vector<cudaEvent_t> events;
   cudaEvent_t ev_begin = nullptr, ev_end[S_NUM] = {};
+  cudaEvent_t ev_caller = nullptr;  // caller's default-stream work the step's input copies wait for
   uint8_t* arena = nullptr;
   bool own_arena = false;
   ncclComm_t comm = nullptr;
@@ -69,6 +78,7 @@ struct harmony_ctx {
   std::vector<uint8_t*> h_stash;  // per (layer, microbatch): spilled stash, nullptr if resident
   std::vector<float*> h_grad;     // retain_grads: reduced gradient shard
   double* h_loss = nullptr;
+  float* h_gather = nullptr;      // read_state at world_size > 1: pinned staging of the gathered tensor
   int t = 0;
   harmony_step_stats last{};
   bool profiling = false;
@@ -80,6 +90,11 @@ struct harmony_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[S_NUM] = {};
   cudaStream_t side = nullptr;          // weight-gradient stream lent to the backward tasks
   cudaEvent_t side_ev[4] = {};
+  // group mode: the caller's context owns the rank contexts (members); a member knows its group
+  std::vector<harmony_ctx*> members;
+  harmony_ctx* group = nullptr;
+  bool one_device = true;               // group: every rank on the same GPU (loopback)
+  cudaEvent_t lb_ready = nullptr, lb_done = nullptr;  // member: rendezvous of a group collective
 };
 
 namespace {
@@ -123,18 +138,38 @@ harmony_status fail(harmony_ctx* ctx, const Error& e) {
 
 void drop_graph(StepGraph& g);
 
+// The rank contexts a context drives: itself, or a group's members.
+std::vector<harmony_ctx*> ranks_of(harmony_ctx* c) {
+  if (c->members.empty()) return {c};
+  return c->members;
+}
+
+void sync_all(harmony_ctx* c) {
+  for (harmony_ctx* r : ranks_of(c)) {
+    if (r->st[0] == nullptr) continue;
+    cudaSetDevice(r->cfg.device);
+    for (int s = 0; s < S_NUM; ++s)
+      if (r->st[s]) cudaStreamSynchronize(r->st[s]);
+    if (r->side) cudaStreamSynchronize(r->side);
+  }
+}
+
 void destroy(harmony_ctx* c) {
   if (!c) return;
-  cudaSetDevice(c->cfg.device);
-  for (int s = 0; s < S_NUM; ++s)
-    if (c->st[s]) cudaStreamSynchronize(c->st[s]);
-  drop_graph(c->g_plain);
+  sync_all(c);
+  drop_graph(c->g_plain);  // a group's graphs span its ranks' streams: dropped before the ranks
   drop_graph(c->g_prof);
+  for (harmony_ctx* m : c->members) destroy(m);
+  c->members.clear();
+  cudaSetDevice(c->cfg.device);
   if (c->side) cudaStreamSynchronize(c->side);
   for (auto e : c->side_ev)
     if (e) cudaEventDestroy(e);
   if (c->side) cudaStreamDestroy(c->side);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_caller) cudaEventDestroy(c->ev_caller);
+  if (c->lb_ready) cudaEventDestroy(c->lb_ready);
+  if (c->lb_done) cudaEventDestroy(c->lb_done);
   for (int s = 0; s < S_NUM; ++s)
     if (c->ev_join[s]) cudaEventDestroy(c->ev_join[s]);
   free_host(c->h_step);
@@ -151,6 +186,7 @@ void destroy(harmony_ctx* c) {
   for (auto p : c->h_stash) free_host(p);
   for (auto p : c->h_grad) free_host(p);
   free_host(c->h_loss);
+  free_host(c->h_gather);
   delete c;
 }
 
@@ -161,6 +197,51 @@ bool is_device_ptr(const void* p) {
     return false;
   }
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// Streams, events and (world_size > 1, one process per GPU) the NCCL communicator of one rank.
+void init_rank(harmony_ctx* c, const harmony_config& cfg, bool want_nccl) {
+  c->cfg = cfg;
+  int ndev = 0;
+  HM_CUDA(cudaGetDeviceCount(&ndev));
+  HM_CHECK(cfg.device >= 0 && cfg.device < ndev, HARMONY_E_INVALID_ARG, "device ordinal out of range");
+  HM_CUDA(cudaSetDevice(cfg.device));
+  cudaDeviceProp prop;
+  HM_CUDA(cudaGetDeviceProperties(&prop, cfg.device));
+  HM_CHECK(prop.major == 10, HARMONY_E_UNSUPPORTED,
+           std::string("libharmony is built for sm_100a (B200); device is ") + prop.name);
+  // Stream priorities: the compute stream carries the step's critical path (the dgrad chain), the
+  // side stream the weight-gradient work that only feeds dW — when SMs free up, the block scheduler
+  // places the compute stream's CTAs first (HARMONY_PRIO=0: all default priority)
+  int prio_lo = 0, prio_hi = 0;
+  HM_CUDA(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
+  {
+    const char* e = getenv("HARMONY_PRIO");
+    if (e && *e == '0') prio_lo = prio_hi = 0;
+  }
+  for (int s = 0; s < S_NUM; ++s) {
+    HM_CUDA(cudaStreamCreateWithPriority(&c->st[s], cudaStreamNonBlocking, s == S_COMPUTE ? prio_hi : 0));
+    HM_CUDA(cudaEventCreate(&c->ev_end[s]));
+  }
+  HM_CUDA(cudaEventCreate(&c->ev_begin));
+  HM_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+  HM_CUDA(cudaEventCreateWithFlags(&c->ev_caller, cudaEventDisableTiming));
+  HM_CUDA(cudaEventCreateWithFlags(&c->lb_ready, cudaEventDisableTiming));
+  HM_CUDA(cudaEventCreateWithFlags(&c->lb_done, cudaEventDisableTiming));
+  for (int s = 0; s < S_NUM; ++s) HM_CUDA(cudaEventCreateWithFlags(&c->ev_join[s], cudaEventDisableTiming));
+  c->h_step = static_cast<int*>(alloc_host(sizeof(int)));
+  HM_CUDA(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio_lo));
+  for (auto& e : c->side_ev) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  {
+    const char* e = getenv("HARMONY_NO_GRAPH");
+    c->use_graph = !(e && *e && *e != '0');
+  }
+  if (want_nccl && cfg.world_size > 1) {
+    HM_CHECK(nccl().load(), HARMONY_E_NCCL, nccl().err);
+    ncclUniqueId id;
+    memcpy(&id, cfg.nccl_id, 128);
+    check_nccl(nccl().CommInitRank(&c->comm, cfg.world_size, id, cfg.rank), "ncclCommInitRank");
+  }
 }
 
 // ---------------------------------------------------------------------------------------- executor
@@ -176,129 +257,237 @@ PtrKind ptr_kind(const void* p) {
   return PTR_PAGEABLE;
 }
 
-// Issue the static program once on the four streams (eagerly, or inside a stream capture).
-void issue_program(harmony_ctx* c, const float* x, const float* tg, bool x_dev, bool t_dev, harmony_step_stats& s) {
+// This rank's view of the step's user inputs.
+struct RankIn {
+  const float* x = nullptr;
+  const float* tg = nullptr;
+  bool x_dev = false, t_dev = false;
+};
+
+bool is_group_collective(int kind) {
+  return kind == OP_ALLGATHER || kind == OP_REDUCESCATTER || kind == OP_LOSS_GATHER;
+}
+
+void issue_prologue(harmony_ctx* c) {
+  // Adam's step t lives in device memory (read by the update kernels at execution time)
+  HM_CUDA(cudaMemcpyAsync(c->arena + c->plan.tstep, c->h_step, sizeof(int), cudaMemcpyHostToDevice, c->st[S_COMPUTE]));
+}
+
+// cross-stream waits of op oi; returns the profiling event opened after them (-1: not profiling)
+int op_pre(harmony_ctx* c, size_t oi) {
+  const Plan& p = c->plan;
+  const Op& o = p.ops[oi];
+  cudaStream_t st = c->st[o.stream];
+  for (int w : o.waits) HM_CUDA(cudaStreamWaitEvent(st, c->events[p.ops[w].event], 0));
+  return g_prof.begin(st);  // profiling: the op's span on its stream (after its waits)
+}
+
+void op_post(harmony_ctx* c, size_t oi, int op_e0) {
+  const Op& o = c->plan.ops[oi];
+  cudaStream_t st = c->st[o.stream];
+  if (op_e0 >= 0) {
+    const int op_e1 = g_prof.begin(st);
+    if (op_e1 >= 0) g_prof.oprecs.push_back({(int)oi, op_e0, op_e1});
+  }
+  if (o.event >= 0) HM_CUDA(cudaEventRecord(c->events[o.event], st));
+}
+
+// The zero padding of a dW buffer beyond the layer's P parameters is part of every rank's reduce-
+// scatter input: keep it zero (another layer of a larger P may have left values there).
+void zero_dw_padding(harmony_ctx* c, const Op& o) {
+  const LayerPlan& lp = c->plan.layers[o.layer];
+  const uint64_t tot = (uint64_t)c->plan.N * o.count;
+  if (tot > (uint64_t)lp.P)
+    HM_CUDA(cudaMemsetAsync(c->arena + o.dev + (uint64_t)lp.P * 4, 0, (tot - (uint64_t)lp.P) * 4, c->st[o.stream]));
+}
+
+void op_body(harmony_ctx* c, size_t oi, const RankIn& in, harmony_step_stats& s) {
   Plan& p = c->plan;
+  const Op& o = p.ops[oi];
   uint8_t* A = c->arena;
   const int dt = p.dtype;
-  const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
-  struct SideGuard {
-    SideGuard(harmony_ctx* c) {
-      void* ev[4] = {c->side_ev[0], c->side_ev[1], c->side_ev[2], c->side_ev[3]};
-      const char* e = getenv("HARMONY_NO_SIDE");
-      if (!(e && *e && *e != '0')) set_side_stream(c->side, ev);
+  cudaStream_t st = c->st[o.stream];
+  switch (o.kind) {
+    case OP_INPUT: {
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)in.x : (const void*)in.tg);
+      const bool dev = o.hbuf == HB_USER_X ? in.x_dev : in.t_dev;
+      HM_CUDA(cudaMemcpyAsync(A + o.dev, src + o.hoff, o.bytes, cudaMemcpyDefault, st));
+      if (!dev) { s.h2d_bytes += o.bytes; s.h2d_input_bytes += o.bytes; }
+      break;
     }
-    ~SideGuard() { set_side_stream(nullptr, nullptr); }
-  } side_guard(c);
-  // Adam's step t lives in device memory (read by the update kernels at execution time)
-  HM_CUDA(cudaMemcpyAsync(A + p.tstep, c->h_step, sizeof(int), cudaMemcpyHostToDevice, c->st[S_COMPUTE]));
-  for (size_t oi = 0; oi < p.ops.size(); ++oi) {
-    const Op& o = p.ops[oi];
-    cudaStream_t st = c->st[o.stream];
-    for (int w : o.waits) HM_CUDA(cudaStreamWaitEvent(st, c->events[p.ops[w].event], 0));
-    const int op_e0 = g_prof.begin(st);  // profiling: the op's span on its stream (after its waits)
-    switch (o.kind) {
-      case OP_INPUT: {
-        const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)x : (const void*)tg);
-        const bool dev = o.hbuf == HB_USER_X ? x_dev : t_dev;
-        HM_CUDA(cudaMemcpyAsync(A + o.dev, src + o.hoff, o.bytes, cudaMemcpyDefault, st));
-        if (!dev) { s.h2d_bytes += o.bytes; s.h2d_input_bytes += o.bytes; }
-        break;
+    case OP_H2D:
+    case OP_D2H: {
+      uint8_t* h = nullptr;
+      switch (o.hbuf) {
+        case HB_WC: h = c->h_wc[o.hidx]; break;
+        case HB_STATE: h = reinterpret_cast<uint8_t*>(c->h_state[o.hidx]); break;
+        case HB_STASH: h = c->h_stash[o.hidx]; break;
+        case HB_GRAD: h = reinterpret_cast<uint8_t*>(c->h_grad[o.hidx]); break;
+        default: throw Error{HARMONY_E_INVALID_ARG, "bad host buffer in plan"};
       }
-      case OP_H2D:
-      case OP_D2H: {
-        uint8_t* h = nullptr;
-        switch (o.hbuf) {
-          case HB_WC: h = c->h_wc[o.hidx]; break;
-          case HB_STATE: h = reinterpret_cast<uint8_t*>(c->h_state[o.hidx]); break;
-          case HB_STASH: h = c->h_stash[o.hidx]; break;
-          case HB_GRAD: h = reinterpret_cast<uint8_t*>(c->h_grad[o.hidx]); break;
-          default: throw Error{HARMONY_E_INVALID_ARG, "bad host buffer in plan"};
-        }
-        h += o.hoff;
-        if (o.kind == OP_H2D) {
-          HM_CUDA(cudaMemcpyAsync(A + o.dev, h, o.bytes, cudaMemcpyHostToDevice, st));
-          s.h2d_bytes += o.bytes;
-          if (o.cat == CAT_WEIGHT) s.h2d_weight_bytes += o.bytes;
-          else if (o.cat == CAT_STATE) s.h2d_state_bytes += o.bytes;
-          else if (o.cat == CAT_STASH) s.h2d_stash_bytes += o.bytes;
-          else if (o.cat == CAT_GRAD) s.h2d_grad_bytes += o.bytes;
-        } else {
-          HM_CUDA(cudaMemcpyAsync(h, A + o.dev, o.bytes, cudaMemcpyDeviceToHost, st));
-          s.d2h_bytes += o.bytes;
-          if (o.cat == CAT_WEIGHT) s.d2h_weight_bytes += o.bytes;
-          else if (o.cat == CAT_STATE) s.d2h_state_bytes += o.bytes;
-          else if (o.cat == CAT_STASH) s.d2h_stash_bytes += o.bytes;
-          else if (o.cat == CAT_GRAD) s.d2h_grad_bytes += o.bytes;
-        }
-        break;
-      }
-      case OP_FWD: {
-        const LayerPlan& lp = p.layers[o.layer];
-        layer_fwd(lp.g, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
-                  A + o.stash, A + o.ws, st);
-        break;
-      }
-      case OP_LOSS: {
-        mse(p.out_elems_per_mb, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<const float*>(A + o.tgt),
-            inv_batch, reinterpret_cast<float*>(A + o.out), reinterpret_cast<double*>(A + o.loss),
-            reinterpret_cast<double*>(A + p.loss_scratch), st);
-        break;
-      }
-      case OP_BWD: {
-        const LayerPlan& lp = p.layers[o.layer];
-        layer_bwd(lp.g, A + o.w, A + o.stash, reinterpret_cast<const float*>(A + o.in),
-                  reinterpret_cast<float*>(A + o.out), reinterpret_cast<float*>(A + o.dw), o.first, A + o.ws, st);
-        break;
-      }
-      case OP_UPD: {
-        const LayerPlan& lp = p.layers[o.layer];
-        float* state = reinterpret_cast<float*>(A + o.state);
-        const uint64_t sh = (uint64_t)lp.shard;
-        uint8_t* wc = A + o.w + (uint64_t)p.rank * sh * (dt ? 2 : 4);
-        adam(dt, (int64_t)sh, state, state + sh, state + 2 * sh, reinterpret_cast<const float*>(A + o.grad), wc,
-             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->t, reinterpret_cast<const int*>(A + p.tstep), st);
-        break;
-      }
-      case OP_ALLGATHER: {
-        const size_t esz = dt ? 2 : 4;
-        uint8_t* buf = A + o.dev;
-        check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * esz, buf, o.count, dt ? ncclBfloat16 : ncclFloat32,
-                                    c->comm, st),
-                   "ncclAllGather");
-        s.nvlink_bytes += o.bytes;
-        break;
-      }
-      case OP_REDUCESCATTER: {
-        check_nccl(nccl().ReduceScatter(A + o.dev, A + o.grad, o.count, ncclFloat32, ncclSum, c->comm, st),
-                   "ncclReduceScatter");
-        s.nvlink_bytes += o.bytes;
-        break;
-      }
-      case OP_LOSS_GATHER: {
-        uint8_t* buf = A + o.dev;
-        check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * 8, buf, o.count, ncclFloat64, c->comm, st),
-                   "ncclAllGather(loss)");
-        s.nvlink_bytes += o.bytes;
-        break;
-      }
-      case OP_LOSS_OUT: {
-        const uint64_t off = p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8;
-        HM_CUDA(cudaMemcpyAsync(reinterpret_cast<uint8_t*>(c->h_loss) + off, A + o.dev + off, o.bytes,
-                                cudaMemcpyDeviceToHost, st));
+      h += o.hoff;
+      if (o.kind == OP_H2D) {
+        HM_CUDA(cudaMemcpyAsync(A + o.dev, h, o.bytes, cudaMemcpyHostToDevice, st));
+        s.h2d_bytes += o.bytes;
+        if (o.cat == CAT_WEIGHT) s.h2d_weight_bytes += o.bytes;
+        else if (o.cat == CAT_STATE) s.h2d_state_bytes += o.bytes;
+        else if (o.cat == CAT_STASH) s.h2d_stash_bytes += o.bytes;
+        else if (o.cat == CAT_GRAD) s.h2d_grad_bytes += o.bytes;
+      } else {
+        HM_CUDA(cudaMemcpyAsync(h, A + o.dev, o.bytes, cudaMemcpyDeviceToHost, st));
         s.d2h_bytes += o.bytes;
-        s.d2h_output_bytes += o.bytes;
-        break;
+        if (o.cat == CAT_WEIGHT) s.d2h_weight_bytes += o.bytes;
+        else if (o.cat == CAT_STATE) s.d2h_state_bytes += o.bytes;
+        else if (o.cat == CAT_STASH) s.d2h_stash_bytes += o.bytes;
+        else if (o.cat == CAT_GRAD) s.d2h_grad_bytes += o.bytes;
       }
-      default:
-        throw Error{HARMONY_E_INVALID_ARG, "unknown op kind in plan"};
+      break;
     }
-    if (op_e0 >= 0) {
-      const int op_e1 = g_prof.begin(st);
-      if (op_e1 >= 0) g_prof.oprecs.push_back({(int)oi, op_e0, op_e1});
+    case OP_FWD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      layer_fwd(lp.g, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
+                A + o.stash, A + o.ws, st);
+      break;
     }
-    if (o.event >= 0) HM_CUDA(cudaEventRecord(c->events[o.event], st));
+    case OP_LOSS: {
+      const float inv_batch = 1.0f / (float)((int64_t)p.N * p.m * p.b);
+      mse(p.out_elems_per_mb, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<const float*>(A + o.tgt),
+          inv_batch, reinterpret_cast<float*>(A + o.out), reinterpret_cast<double*>(A + o.loss),
+          reinterpret_cast<double*>(A + p.loss_scratch), st);
+      break;
+    }
+    case OP_BWD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      const char* e = getenv("HARMONY_NO_SIDE");
+      if (!(e && *e && *e != '0')) {
+        void* ev[4] = {c->side_ev[0], c->side_ev[1], c->side_ev[2], c->side_ev[3]};
+        set_side_stream(c->side, ev);
+      } else {
+        set_side_stream(nullptr, nullptr);
+      }
+      layer_bwd(lp.g, A + o.w, A + o.stash, reinterpret_cast<const float*>(A + o.in),
+                reinterpret_cast<float*>(A + o.out), reinterpret_cast<float*>(A + o.dw), o.first, A + o.ws, st);
+      set_side_stream(nullptr, nullptr);
+      break;
+    }
+    case OP_UPD: {
+      const LayerPlan& lp = p.layers[o.layer];
+      float* state = reinterpret_cast<float*>(A + o.state);
+      const uint64_t sh = (uint64_t)lp.shard;
+      uint8_t* wc = A + o.w + (uint64_t)p.rank * sh * (dt ? 2 : 4);
+      adam(dt, (int64_t)sh, state, state + sh, state + 2 * sh, reinterpret_cast<const float*>(A + o.grad), wc,
+           c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->t, reinterpret_cast<const int*>(A + p.tstep), st);
+      break;
+    }
+    case OP_ALLGATHER: {
+      const size_t esz = dt ? 2 : 4;
+      uint8_t* buf = A + o.dev;
+      check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * esz, buf, o.count, dt ? ncclBfloat16 : ncclFloat32,
+                                  c->comm, st),
+                 "ncclAllGather");
+      s.nvlink_bytes += o.bytes;
+      break;
+    }
+    case OP_REDUCESCATTER: {
+      zero_dw_padding(c, o);
+      check_nccl(nccl().ReduceScatter(A + o.dev, A + o.grad, o.count, ncclFloat32, ncclSum, c->comm, st),
+                 "ncclReduceScatter");
+      s.nvlink_bytes += o.bytes;
+      break;
+    }
+    case OP_LOSS_GATHER: {
+      uint8_t* buf = A + o.dev;
+      check_nccl(nccl().AllGather(buf + (uint64_t)p.rank * o.count * 8, buf, o.count, ncclFloat64, c->comm, st),
+                 "ncclAllGather(loss)");
+      s.nvlink_bytes += o.bytes;
+      break;
+    }
+    case OP_LOSS_OUT: {
+      const uint64_t off = p.N > 1 ? 0 : (uint64_t)p.rank * p.m * 8;
+      HM_CUDA(cudaMemcpyAsync(reinterpret_cast<uint8_t*>(c->h_loss) + off, A + o.dev + off, o.bytes,
+                              cudaMemcpyDeviceToHost, st));
+      s.d2h_bytes += o.bytes;
+      s.d2h_output_bytes += o.bytes;
+      break;
+    }
+    default:
+      throw Error{HARMONY_E_INVALID_ARG, "unknown op kind in plan"};
   }
+}
+
+// A collective of a group, as three lock-step phases over the ranks: (1) every rank reaches the op
+// (its plan waits) and marks its inputs ready; (2) every rank waits for all inputs and pulls what it
+// receives from its peers' arenas; (3) every rank waits until all peers have finished pulling before
+// its program may overwrite the buffers (the same ordering NCCL gives the one-process-per-GPU path).
+void issue_group_collective(const std::vector<harmony_ctx*>& R, bool one_device, size_t oi,
+                            std::vector<harmony_step_stats>& s) {
+  const int N = (int)R.size();
+  std::vector<int> e0(N);
+  for (int r = 0; r < N; ++r) {
+    harmony_ctx* c = R[r];
+    if (!one_device) HM_CUDA(cudaSetDevice(c->cfg.device));
+    e0[r] = op_pre(c, oi);
+    const Op& o = c->plan.ops[oi];
+    if (o.kind == OP_REDUCESCATTER) zero_dw_padding(c, o);
+    HM_CUDA(cudaEventRecord(c->lb_ready, c->st[o.stream]));
+  }
+  for (int r = 0; r < N; ++r) {
+    harmony_ctx* c = R[r];
+    if (!one_device) HM_CUDA(cudaSetDevice(c->cfg.device));
+    const Op& o = c->plan.ops[oi];
+    cudaStream_t st = c->st[o.stream];
+    for (int q = 0; q < N; ++q)
+      if (q != r) HM_CUDA(cudaStreamWaitEvent(st, R[q]->lb_ready, 0));
+    if (o.kind == OP_REDUCESCATTER) {
+      const float* src[HM_MAX_GROUP];
+      for (int q = 0; q < N; ++q)
+        src[q] = reinterpret_cast<const float*>(R[q]->arena + R[q]->plan.ops[oi].dev) + (uint64_t)r * o.count;
+      rank_sum(N, src, (int64_t)o.count, reinterpret_cast<float*>(c->arena + o.grad), st);
+    } else {
+      const size_t esz = o.kind == OP_LOSS_GATHER ? 8 : (c->plan.dtype ? 2 : 4);
+      const uint64_t sh = o.count * esz;
+      for (int q = 0; q < N; ++q) {
+        if (q == r) continue;
+        HM_CUDA(cudaMemcpyAsync(c->arena + o.dev + (uint64_t)q * sh, R[q]->arena + R[q]->plan.ops[oi].dev + (uint64_t)q * sh,
+                                sh, cudaMemcpyDefault, st));
+      }
+    }
+    s[r].nvlink_bytes += o.bytes;
+    HM_CUDA(cudaEventRecord(c->lb_done, st));
+  }
+  for (int r = 0; r < N; ++r) {
+    harmony_ctx* c = R[r];
+    if (!one_device) HM_CUDA(cudaSetDevice(c->cfg.device));
+    const Op& o = c->plan.ops[oi];
+    for (int q = 0; q < N; ++q)
+      if (q != r) HM_CUDA(cudaStreamWaitEvent(c->st[o.stream], R[q]->lb_done, 0));
+    op_post(c, oi, e0[r]);
+  }
+}
+
+// Issue the static program once on every rank's streams (eagerly, or inside a stream capture).
+void issue_program(harmony_ctx* c, const std::vector<RankIn>& in, std::vector<harmony_step_stats>& s) {
+  const std::vector<harmony_ctx*> R = ranks_of(c);
+  const bool group = !c->members.empty();
+  const bool one_device = c->one_device;
+  for (size_t r = 0; r < R.size(); ++r) {
+    if (!one_device) HM_CUDA(cudaSetDevice(R[r]->cfg.device));
+    issue_prologue(R[r]);
+  }
+  const size_t n = R[0]->plan.ops.size();
+  for (size_t oi = 0; oi < n; ++oi) {
+    if (group && is_group_collective(R[0]->plan.ops[oi].kind)) {
+      issue_group_collective(R, one_device, oi, s);
+      continue;
+    }
+    for (size_t r = 0; r < R.size(); ++r) {
+      if (!one_device) HM_CUDA(cudaSetDevice(R[r]->cfg.device));
+      const int e0 = op_pre(R[r], oi);
+      op_body(R[r], oi, in[r], s[r]);
+      op_post(R[r], oi, e0);
+    }
+  }
+  if (!one_device) HM_CUDA(cudaSetDevice(R[0]->cfg.device));
 }
 
 void drop_graph(StepGraph& g) {
@@ -308,18 +497,20 @@ void drop_graph(StepGraph& g) {
   g.graph = nullptr;
   g.in_nodes.clear();
   g.recs.clear();
+  g.oprecs.clear();
   g.sig = -1;
 }
 
-// Capture the whole step (all four streams, NCCL included) as one CUDA graph; later steps only
-// patch the source pointers of the input copies and replay it (one launch per step).  With
-// `profiled`, every kernel of the step is bracketed by external event-record nodes, so the
-// per-kernel durations come from the real step without host-issue gaps.
-void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg, bool x_dev, bool t_dev, bool profiled) {
+// Capture the whole step (every rank's four streams, collectives included) as one CUDA graph;
+// later steps only patch the source pointers of the input copies and replay it (one launch per
+// step).  With `profiled`, every kernel of the step is bracketed by external event-record nodes, so
+// the per-kernel durations come from the real step without host-issue gaps.
+void capture_graph(harmony_ctx* c, StepGraph& G, const std::vector<RankIn>& in, bool profiled) {
   drop_graph(G);
-  Plan& p = c->plan;
-  cudaStream_t cs = c->st[S_COMPUTE];
-  harmony_step_stats s{};
+  const std::vector<harmony_ctx*> R = ranks_of(c);
+  harmony_ctx* c0 = R[0];
+  cudaStream_t cs = c0->st[S_COMPUTE];
+  std::vector<harmony_step_stats> s(R.size());
   g_kernel_launches = 0;
   g_prof.on = profiled;
   g_prof.external = profiled;
@@ -328,13 +519,17 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg
   g_prof.oprecs.clear();
   HM_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
   try {
-    HM_CUDA(cudaEventRecord(c->ev_fork, cs));
-    for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_fork, 0));
-    issue_program(c, x, tg, x_dev, t_dev, s);
-    for (int k = 1; k < S_NUM; ++k) {
-      HM_CUDA(cudaEventRecord(c->ev_join[k], c->st[k]));
-      HM_CUDA(cudaStreamWaitEvent(cs, c->ev_join[k], 0));
-    }
+    HM_CUDA(cudaEventRecord(c0->ev_fork, cs));
+    for (harmony_ctx* r : R)
+      for (int k = 0; k < S_NUM; ++k)
+        if (r->st[k] != cs) HM_CUDA(cudaStreamWaitEvent(r->st[k], c0->ev_fork, 0));
+    issue_program(c, in, s);
+    for (harmony_ctx* r : R)
+      for (int k = 0; k < S_NUM; ++k) {
+        if (r->st[k] == cs) continue;
+        HM_CUDA(cudaEventRecord(r->ev_join[k], r->st[k]));
+        HM_CUDA(cudaStreamWaitEvent(cs, r->ev_join[k], 0));
+      }
   } catch (...) {
     cudaGraph_t g = nullptr;
     cudaStreamEndCapture(cs, &g);
@@ -350,15 +545,15 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg
   G.launches = g_kernel_launches;
   G.recs = g_prof.recs;
   G.oprecs = g_prof.oprecs;
-  // find the input memcpy nodes by their destinations
+  // find the input memcpy nodes by their destinations (every rank's arena is its own allocation)
   size_t n = 0;
   HM_CUDA(cudaGraphGetNodes(G.graph, nullptr, &n));
   std::vector<cudaGraphNode_t> nodes(n);
   HM_CUDA(cudaGraphGetNodes(G.graph, nodes.data(), &n));
-  G.in_ops.clear();
-  for (size_t i = 0; i < p.ops.size(); ++i)
-    if (p.ops[i].kind == OP_INPUT) G.in_ops.push_back((int)i);
-  G.in_nodes.assign(G.in_ops.size(), nullptr);
+  G.in_nodes.clear();
+  for (size_t r = 0; r < R.size(); ++r)
+    for (size_t i = 0; i < R[r]->plan.ops.size(); ++i)
+      if (R[r]->plan.ops[i].kind == OP_INPUT) G.in_nodes.push_back({(int)r, (int)i, nullptr});
   for (auto nd : nodes) {
     cudaGraphNodeType ty;
     HM_CUDA(cudaGraphNodeGetType(nd, &ty));
@@ -366,68 +561,113 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const float* x, const float* tg
     cudaMemcpy3DParms mp;
     HM_CUDA(cudaGraphMemcpyNodeGetParams(nd, &mp));
     const uint8_t* dst = static_cast<const uint8_t*>(mp.dstPtr.ptr);
-    for (size_t j = 0; j < G.in_ops.size(); ++j)
-      if (dst == c->arena + p.ops[G.in_ops[j]].dev) G.in_nodes[j] = nd;
+    for (auto& e : G.in_nodes)
+      if (dst == R[e.rank]->arena + R[e.rank]->plan.ops[e.op].dev) e.node = nd;
   }
-  for (auto nd : G.in_nodes) HM_CHECK(nd != nullptr, HARMONY_E_CUDA, "graph capture: input copy node not found");
-  G.sig = (x_dev ? 1 : 0) | (t_dev ? 2 : 0);
+  for (auto& e : G.in_nodes) HM_CHECK(e.node != nullptr, HARMONY_E_CUDA, "graph capture: input copy node not found");
+  G.sig = (in[0].x_dev ? 1 : 0) | (in[0].t_dev ? 2 : 0);
 }
 
+// One step of a rank context or a group.  x / tg: this context's rows (a group: the global batch).
 void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out, harmony_step_stats* out) {
-  Plan& p = c->plan;
-  c->t += 1;
-  *c->h_step = c->t;
+  const std::vector<harmony_ctx*> R = ranks_of(c);
+  const int NR = (int)R.size();
+  harmony_ctx* c0 = R[0];
+  const Plan& p0 = c0->plan;
+  const int t_next = c->t + 1;
+  for (harmony_ctx* r : R) {
+    r->t = t_next;  // the value the update kernels of this step read (reverted below on failure)
+    *r->h_step = t_next;
+  }
   const PtrKind xk = ptr_kind(x), tk = ptr_kind(tg);
-  const bool x_dev = xk == PTR_DEVICE, t_dev = tk == PTR_DEVICE;
-  // graphs need pinned or device inputs (a pageable copy cannot be captured)
-  const bool use_graph = c->use_graph && xk != PTR_PAGEABLE && tk != PTR_PAGEABLE;
-  harmony_step_stats s{};
+  std::vector<RankIn> in(NR);
+  for (int r = 0; r < NR; ++r) {
+    in[r].x = x + (size_t)r * p0.m * p0.in_elems_per_mb;
+    in[r].tg = tg + (size_t)r * p0.m * p0.out_elems_per_mb;
+    in[r].x_dev = xk == PTR_DEVICE;
+    in[r].t_dev = tk == PTR_DEVICE;
+  }
+  // graphs need pinned or device inputs (a pageable copy cannot be captured); one graph spans the
+  // ranks of a group only when they share a GPU
+  const bool use_graph = c0->use_graph && xk != PTR_PAGEABLE && tk != PTR_PAGEABLE && c->one_device;
+  std::vector<harmony_step_stats> s(NR);
   g_kernel_launches = 0;
   g_prof.on = c->profiling;
   g_prof.external = false;
   g_prof.used = 0;
   g_prof.recs.clear();
   g_prof.oprecs.clear();
-  cudaStream_t cs = c->st[S_COMPUTE];
+  cudaStream_t cs = c0->st[S_COMPUTE];
   std::vector<KProf::Rec>* recs = &g_prof.recs;
   std::vector<KProf::OpRec>* oprecs = &g_prof.oprecs;
-  if (use_graph) {
-    StepGraph& G = c->profiling ? c->g_prof : c->g_plain;
-    const int sig = (x_dev ? 1 : 0) | (t_dev ? 2 : 0);
-    if (!G.exec || G.sig != sig) capture_graph(c, G, x, tg, x_dev, t_dev, c->profiling);
-    for (size_t j = 0; j < G.in_nodes.size(); ++j) {
-      const Op& o = p.ops[G.in_ops[j]];
-      const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)x : (const void*)tg);
-      HM_CUDA(cudaGraphExecMemcpyNodeSetParams1D(G.exec, G.in_nodes[j], c->arena + o.dev, src + o.hoff, o.bytes,
-                                                 cudaMemcpyDefault));
+  uint64_t launches = 0;
+  bool issued = false;
+  try {
+    // the caller's work on the legacy default stream (e.g. torch ops writing x / target) first
+    HM_CUDA(cudaEventRecord(c0->ev_caller, cudaStreamLegacy));
+    HM_CUDA(cudaStreamWaitEvent(cs, c0->ev_caller, 0));
+    if (use_graph) {
+      StepGraph& G = c->profiling ? c->g_prof : c->g_plain;
+      const int sig = (in[0].x_dev ? 1 : 0) | (in[0].t_dev ? 2 : 0);
+      issued = true;
+      if (!G.exec || G.sig != sig) capture_graph(c, G, in, c->profiling);
+      for (auto& e : G.in_nodes) {
+        const Op& o = R[e.rank]->plan.ops[e.op];
+        const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)in[e.rank].x
+                                                                                  : (const void*)in[e.rank].tg);
+        HM_CUDA(cudaGraphExecMemcpyNodeSetParams1D(G.exec, e.node, R[e.rank]->arena + o.dev, src + o.hoff, o.bytes,
+                                                   cudaMemcpyDefault));
+      }
+      HM_CUDA(cudaEventRecord(c0->ev_begin, cs));
+      HM_CUDA(cudaGraphLaunch(G.exec, cs));
+      HM_CUDA(cudaEventRecord(c0->ev_end[0], cs));
+      HM_CUDA(cudaEventSynchronize(c0->ev_end[0]));
+      float ms = 0.f;
+      HM_CUDA(cudaEventElapsedTime(&ms, c0->ev_begin, c0->ev_end[0]));
+      s = G.stats;
+      for (auto& x2 : s) x2.step_seconds = ms * 1e-3;
+      launches = G.launches;
+      recs = &G.recs;
+      oprecs = &G.oprecs;
+    } else {
+      HM_CUDA(cudaEventRecord(c0->ev_begin, cs));
+      for (harmony_ctx* r : R) {
+        if (!c->one_device) HM_CUDA(cudaSetDevice(r->cfg.device));
+        for (int k = 0; k < S_NUM; ++k)
+          if (r->st[k] != cs) HM_CUDA(cudaStreamWaitEvent(r->st[k], c0->ev_begin, 0));
+      }
+      issued = true;
+      issue_program(c, in, s);
+      float ms = 0.f;
+      for (harmony_ctx* r : R) {
+        if (!c->one_device) HM_CUDA(cudaSetDevice(r->cfg.device));
+        for (int k = 0; k < S_NUM; ++k) HM_CUDA(cudaEventRecord(r->ev_end[k], r->st[k]));
+      }
+      for (harmony_ctx* r : R)
+        for (int k = 0; k < S_NUM; ++k) {
+          HM_CUDA(cudaEventSynchronize(r->ev_end[k]));
+          float e = 0.f;
+          HM_CUDA(cudaEventElapsedTime(&e, c0->ev_begin, r->ev_end[k]));
+          ms = std::max(ms, e);
+        }
+      HM_CUDA(cudaSetDevice(c0->cfg.device));
+      for (auto& x2 : s) x2.step_seconds = ms * 1e-3;
+      launches = g_kernel_launches;
     }
-    HM_CUDA(cudaEventRecord(c->ev_begin, cs));
-    HM_CUDA(cudaGraphLaunch(G.exec, cs));
-    HM_CUDA(cudaEventRecord(c->ev_end[0], cs));
-    HM_CUDA(cudaEventSynchronize(c->ev_end[0]));
-    float ms = 0.f;
-    HM_CUDA(cudaEventElapsedTime(&ms, c->ev_begin, c->ev_end[0]));
-    s = G.stats;
-    s.kernel_launches = G.launches;
-    s.step_seconds = ms * 1e-3;
-    recs = &G.recs;
-    oprecs = &G.oprecs;
-  } else {
-    HM_CUDA(cudaEventRecord(c->ev_begin, cs));
-    for (int k = 1; k < S_NUM; ++k) HM_CUDA(cudaStreamWaitEvent(c->st[k], c->ev_begin, 0));
-    issue_program(c, x, tg, x_dev, t_dev, s);
-    for (int k = 0; k < S_NUM; ++k) HM_CUDA(cudaEventRecord(c->ev_end[k], c->st[k]));
-    float ms = 0.f;
-    for (int k = 0; k < S_NUM; ++k) {
-      HM_CUDA(cudaEventSynchronize(c->ev_end[k]));
-      float e = 0.f;
-      HM_CUDA(cudaEventElapsedTime(&e, c->ev_begin, c->ev_end[k]));
-      ms = std::max(ms, e);
+    HM_CUDA(cudaGetLastError());
+  } catch (...) {
+    // nothing of this step may count: t back, and — once work was issued — the context is unusable
+    g_prof.on = g_prof.external = false;
+    for (harmony_ctx* r : R) r->t = t_next - 1;
+    if (issued) {
+      sync_all(c);
+      cudaGetLastError();
+      c->broken = true;
+      for (harmony_ctx* r : R) r->broken = true;
     }
-    s.step_seconds = ms * 1e-3;
-    s.kernel_launches = g_kernel_launches;
+    throw;
   }
-  HM_CUDA(cudaGetLastError());
+  c->t = t_next;
   if (c->profiling) {
     for (auto& rc : *recs) {
       float e = 0.f;
@@ -438,10 +678,10 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     }
     c->timeline.clear();
     for (auto& orc : *oprecs) {
-      const Op& o = p.ops[orc.op];
+      const Op& o = p0.ops[orc.op];
       float t0 = 0.f, t1 = 0.f;
-      HM_CUDA(cudaEventElapsedTime(&t0, c->ev_begin, g_prof.pool[orc.e0]));
-      HM_CUDA(cudaEventElapsedTime(&t1, c->ev_begin, g_prof.pool[orc.e1]));
+      HM_CUDA(cudaEventElapsedTime(&t0, c0->ev_begin, g_prof.pool[orc.e0]));
+      HM_CUDA(cudaEventElapsedTime(&t1, c0->ev_begin, g_prof.pool[orc.e1]));
       harmony_timeline_rec r{};
       r.op = orc.op; r.kind = o.kind; r.stream = o.stream; r.cat = o.cat; r.layer = o.layer; r.micro = o.mb;
       r.bytes = o.bytes; r.t0 = t0 * 1e-3; r.t1 = t1 * 1e-3;
@@ -450,14 +690,112 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     g_prof.on = false;
   }
   double loss = 0.0;  // rank partials summed in rank order, microbatches in order (reading c22)
-  for (int r = 0; r < p.N; ++r)
-    for (int i = 0; i < p.m; ++i) loss += c->h_loss[r * p.m + i];
+  for (int r = 0; r < p0.N; ++r)
+    for (int i = 0; i < p0.m; ++i) loss += c0->h_loss[r * p0.m + i];
   if (loss_out) *loss_out = loss;
-  s.n_ops = p.ops.size();
-  s.peak_arena_bytes = p.arena_bytes;
-  s.graph = use_graph ? 1 : 0;
-  c->last = s;
-  if (out) *out = s;
+  // a rank's ledger, or a group's box totals (bytes summed over ranks)
+  harmony_step_stats tot = s[0];
+  for (int r = 1; r < NR; ++r) {
+    tot.h2d_bytes += s[r].h2d_bytes; tot.d2h_bytes += s[r].d2h_bytes;
+    tot.h2d_weight_bytes += s[r].h2d_weight_bytes; tot.d2h_weight_bytes += s[r].d2h_weight_bytes;
+    tot.h2d_state_bytes += s[r].h2d_state_bytes; tot.d2h_state_bytes += s[r].d2h_state_bytes;
+    tot.h2d_stash_bytes += s[r].h2d_stash_bytes; tot.d2h_stash_bytes += s[r].d2h_stash_bytes;
+    tot.h2d_input_bytes += s[r].h2d_input_bytes; tot.d2h_output_bytes += s[r].d2h_output_bytes;
+    tot.h2d_grad_bytes += s[r].h2d_grad_bytes; tot.d2h_grad_bytes += s[r].d2h_grad_bytes;
+    tot.nvlink_bytes += s[r].nvlink_bytes;
+  }
+  tot.kernel_launches = launches;
+  tot.n_ops = p0.ops.size() * NR;
+  tot.peak_arena_bytes = 0;
+  for (harmony_ctx* r : R) tot.peak_arena_bytes = std::max<uint64_t>(tot.peak_arena_bytes, r->plan.arena_bytes);
+  tot.graph = use_graph ? 1 : 0;
+  for (int r = 0; r < NR; ++r) {
+    R[r]->last = s[r];
+    R[r]->last.kernel_launches = launches;
+  }
+  c->last = tot;
+  if (out) *out = tot;
+}
+
+// Fill one rank's pinned host store and resident HBM tensors from the caller's fp32 parameters.
+void register_rank(harmony_ctx* c, Plan&& p_in, const float* const* init_params) {
+  Plan p = std::move(p_in);
+  const int L = (int)p.layers.size(), m = p.m, N = p.N, r = p.rank;
+  const size_t ts = p.dtype ? 2 : 4;
+  HM_CUDA(cudaSetDevice(c->cfg.device));
+  // arena
+  if (c->arena) {
+    HM_CHECK(p.arena_bytes <= c->cfg.hbm_cap_bytes, HARMONY_E_CAP_TOO_SMALL, "plan exceeds the adopted arena");
+  } else {
+    HM_CUDA(cudaMalloc(&c->arena, p.arena_bytes));
+    c->own_arena = true;
+  }
+  // every arena byte starts at zero (the dW padding every rank's reduce-scatter reads among them)
+  HM_CUDA(cudaMemset(c->arena, 0, p.arena_bytes));
+  // events of the program
+  c->events.resize(p.n_events);
+  for (auto& e : c->events) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  // pinned host store
+  c->h_wc.assign(L, nullptr);
+  c->h_state.assign(L, nullptr);
+  c->h_stash.assign((size_t)L * m, nullptr);
+  c->h_grad.assign(L, nullptr);
+  c->h_loss = static_cast<double*>(alloc_host((size_t)N * m * 8));
+  if (N > 1) {
+    int64_t maxPpad = 0;
+    for (auto& lp : p.layers) maxPpad = std::max(maxPpad, lp.Ppad);
+    c->h_gather = static_cast<float*>(alloc_host((size_t)maxPpad * 4));
+  }
+  std::vector<uint8_t> full;  // staging of a full compute copy for resident layers
+  for (int l = 0; l < L; ++l) {
+    const LayerPlan& lp = p.layers[l];
+    const int64_t sh = lp.shard, P = lp.P;
+    c->h_wc[l] = static_cast<uint8_t*>(alloc_host((size_t)sh * ts));
+    c->h_state[l] = static_cast<float*>(alloc_host((size_t)lp.state_bytes));
+    if (p.retain_grads || p.schedule == HARMONY_SCHED_PER_GPU_VIRT) c->h_grad[l] = static_cast<float*>(alloc_host((size_t)sh * 4));
+    float* master = c->h_state[l];
+    memset(master, 0, lp.state_bytes);  // m = v = 0 (reading c3), padding = 0
+    const int64_t lo = (int64_t)r * sh, hi = std::min<int64_t>(P, lo + sh);
+    if (hi > lo) memcpy(master, init_params[l] + lo, (size_t)(hi - lo) * 4);
+    if (ts == 2) {
+      uint16_t* w = reinterpret_cast<uint16_t*>(c->h_wc[l]);
+      for (int64_t i = 0; i < sh; ++i) w[i] = f32_to_bf16_rne(master[i]);
+    } else {
+      memcpy(c->h_wc[l], master, (size_t)sh * 4);
+    }
+    for (int i = 0; i < m; ++i)
+      if (lp.stash_res[i] < 0) c->h_stash[(size_t)l * m + i] = static_cast<uint8_t*>(alloc_host(lp.g.st.total));
+    // resident tensors go to HBM now
+    if (lp.wc_res >= 0) {
+      full.assign((size_t)lp.Ppad * ts, 0);
+      if (ts == 2) {
+        uint16_t* w = reinterpret_cast<uint16_t*>(full.data());
+        for (int64_t i = 0; i < P; ++i) w[i] = f32_to_bf16_rne(init_params[l][i]);
+      } else {
+        memcpy(full.data(), init_params[l], (size_t)P * 4);
+      }
+      HM_CUDA(cudaMemcpy(c->arena + lp.wc_res, full.data(), full.size(), cudaMemcpyHostToDevice));
+    }
+    if (lp.state_res >= 0)
+      HM_CUDA(cudaMemcpy(c->arena + lp.state_res, c->h_state[l], lp.state_bytes, cudaMemcpyHostToDevice));
+  }
+  HM_CUDA(cudaDeviceSynchronize());
+  c->plan = std::move(p);
+  c->registered = true;
+}
+
+// This rank's shard of one fp32 state tensor into host memory (n = shard elements).
+void read_shard(harmony_ctx* c, int layer, int which, float* dst) {
+  const LayerPlan& lp = c->plan.layers[layer];
+  const uint64_t sh = (uint64_t)lp.shard;
+  HM_CUDA(cudaSetDevice(c->cfg.device));
+  if (which == HARMONY_GRAD) {
+    memcpy(dst, c->h_grad[layer], sh * 4);
+  } else {
+    const uint64_t off = (which == HARMONY_PARAM ? 0 : which == HARMONY_ADAM_M ? 1 : 2) * sh * 4;
+    if (lp.state_res >= 0) HM_CUDA(cudaMemcpy(dst, c->arena + lp.state_res + off, sh * 4, cudaMemcpyDeviceToHost));
+    else memcpy(dst, reinterpret_cast<uint8_t*>(c->h_state[layer]) + off, sh * 4);
+  }
 }
 
 }  // namespace
@@ -511,49 +849,12 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
   *out = nullptr;
   validate_config(*cfg);
   c = new harmony_ctx();
-  c->cfg = *cfg;
-  int ndev = 0;
-  HM_CUDA(cudaGetDeviceCount(&ndev));
-  HM_CHECK(cfg->device >= 0 && cfg->device < ndev, HARMONY_E_INVALID_ARG, "device ordinal out of range");
-  HM_CUDA(cudaSetDevice(cfg->device));
-  cudaDeviceProp prop;
-  HM_CUDA(cudaGetDeviceProperties(&prop, cfg->device));
-  HM_CHECK(prop.major == 10, HARMONY_E_UNSUPPORTED,
-           std::string("libharmony is built for sm_100a (B200); device is ") + prop.name);
-  // Stream priorities: the compute stream carries the step's critical path (the dgrad chain), the
-  // side stream the weight-gradient work that only feeds dW — when SMs free up, the block scheduler
-  // places the compute stream's CTAs first (HARMONY_PRIO=0: all default priority)
-  int prio_lo = 0, prio_hi = 0;
-  HM_CUDA(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
-  {
-    const char* e = getenv("HARMONY_PRIO");
-    if (e && *e == '0') prio_lo = prio_hi = 0;
-  }
-  for (int s = 0; s < S_NUM; ++s) {
-    HM_CUDA(cudaStreamCreateWithPriority(&c->st[s], cudaStreamNonBlocking, s == S_COMPUTE ? prio_hi : 0));
-    HM_CUDA(cudaEventCreate(&c->ev_end[s]));
-  }
-  HM_CUDA(cudaEventCreate(&c->ev_begin));
-  HM_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
-  for (int s = 0; s < S_NUM; ++s) HM_CUDA(cudaEventCreateWithFlags(&c->ev_join[s], cudaEventDisableTiming));
-  c->h_step = static_cast<int*>(alloc_host(sizeof(int)));
-  HM_CUDA(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio_lo));
-  for (auto& e : c->side_ev) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-  {
-    const char* e = getenv("HARMONY_NO_GRAPH");
-    c->use_graph = !(e && *e && *e != '0');
-  }
+  init_rank(c, *cfg, true);
   if (cfg->arena) {
     HM_CHECK(cfg->hbm_cap_bytes > 0, HARMONY_E_INVALID_ARG, "an adopted arena needs hbm_cap_bytes");
     HM_CHECK(is_device_ptr(cfg->arena), HARMONY_E_INVALID_ARG, "cfg.arena is not a device pointer");
     HM_CHECK(reinterpret_cast<uintptr_t>(cfg->arena) % 1024 == 0, HARMONY_E_INVALID_ARG, "cfg.arena must be 1 KiB aligned");
     c->arena = static_cast<uint8_t*>(cfg->arena);
-  }
-  if (cfg->world_size > 1) {
-    HM_CHECK(nccl().load(), HARMONY_E_NCCL, nccl().err);
-    ncclUniqueId id;
-    memcpy(&id, cfg->nccl_id, 128);
-    check_nccl(nccl().CommInitRank(&c->comm, cfg->world_size, id, cfg->rank), "ncclCommInitRank");
   }
   *out = c;
   c = nullptr;
@@ -566,71 +867,87 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
   return HARMONY_OK;
 }
 
+harmony_status harmony_init_group(const harmony_config* cfg, int32_t num_ranks, const int32_t* devices,
+                                  harmony_ctx** out) {
+  harmony_ctx* g = nullptr;
+  HM_API_BEGIN
+  HM_CHECK(cfg && out, HARMONY_E_INVALID_ARG, "NULL argument");
+  *out = nullptr;
+  HM_CHECK(num_ranks >= 1 && num_ranks <= HM_MAX_GROUP, HARMONY_E_INVALID_ARG, "num_ranks must be in 1..16");
+  HM_CHECK(cfg->arena == nullptr, HARMONY_E_INVALID_ARG, "a group allocates its ranks' arenas (cfg.arena must be NULL)");
+  harmony_config gc = *cfg;
+  gc.rank = 0;
+  gc.world_size = num_ranks;
+  gc.device = devices ? devices[0] : 0;
+  validate_config(gc);
+  g = new harmony_ctx();
+  g->cfg = gc;
+  for (int r = 0; r < num_ranks; ++r) {
+    harmony_config rc = gc;
+    rc.rank = r;
+    rc.device = devices ? devices[r] : 0;
+    if (rc.device != gc.device) g->one_device = false;
+    harmony_ctx* m = new harmony_ctx();
+    m->group = g;
+    g->members.push_back(m);
+    init_rank(m, rc, false);
+  }
+  if (!g->one_device) {  // pulls from peers' HBM over NVLink
+    for (int r = 0; r < num_ranks; ++r)
+      for (int q = 0; q < num_ranks; ++q) {
+        const int a = g->members[r]->cfg.device, b = g->members[q]->cfg.device;
+        if (a == b) continue;
+        int can = 0;
+        HM_CUDA(cudaDeviceCanAccessPeer(&can, a, b));
+        HM_CHECK(can, HARMONY_E_UNSUPPORTED, "group ranks on GPUs without peer access");
+        HM_CUDA(cudaSetDevice(a));
+        cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+        else HM_CUDA(e);
+      }
+    HM_CUDA(cudaSetDevice(gc.device));
+  }
+  *out = g;
+  g = nullptr;
+  }
+  catch (const Error& e) {
+    harmony_status st = fail(nullptr, e);
+    destroy(g);
+    return st;
+  }
+  return HARMONY_OK;
+}
+
 harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const harmony_layer_desc* descs,
                                        const float* const* init_params) {
   HM_API_BEGIN
   HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
   HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
   HM_CHECK(!c->registered, HARMONY_E_BAD_STATE, "layers already registered");
+  HM_CHECK(c->group == nullptr, HARMONY_E_BAD_STATE, "a group's rank context is not the caller's");
   HM_CHECK(descs && init_params, HARMONY_E_INVALID_ARG, "NULL argument");
+  for (int l = 0; l < n_layers; ++l) HM_CHECK(init_params[l] != nullptr, HARMONY_E_INVALID_ARG, "init_params[l] is NULL");
+  std::vector<harmony_ctx*> R = ranks_of(c);
+  std::vector<Plan> plans;
+  for (harmony_ctx* r : R) {
+    plans.push_back(make_plan(r->cfg, n_layers, descs));
+    HM_CHECK(plans.back().summary.hazards == 0, HARMONY_E_INVALID_ARG,
+             "internal: planned program has a hazard: " + plans.back().hazard_msg);
+  }
+  // lock-step issue needs the same program shape on every rank (same ops, kinds, streams, edges)
+  for (size_t r = 1; r < plans.size(); ++r) {
+    HM_CHECK(plans[r].ops.size() == plans[0].ops.size(), HARMONY_E_INVALID_ARG, "internal: rank programs differ");
+    for (size_t i = 0; i < plans[0].ops.size(); ++i)
+      HM_CHECK(plans[r].ops[i].kind == plans[0].ops[i].kind && plans[r].ops[i].stream == plans[0].ops[i].stream &&
+                   plans[r].ops[i].waits == plans[0].ops[i].waits && plans[r].ops[i].dev == plans[0].ops[i].dev,
+               HARMONY_E_INVALID_ARG, "internal: rank programs differ");
+  }
+  for (size_t r = 0; r < R.size(); ++r) register_rank(R[r], std::move(plans[r]), init_params);
   HM_CUDA(cudaSetDevice(c->cfg.device));
-  Plan p = make_plan(c->cfg, n_layers, descs);
-  HM_CHECK(p.summary.hazards == 0, HARMONY_E_INVALID_ARG, "internal: planned program has a hazard: " + p.hazard_msg);
-  const int L = n_layers, m = p.m, N = p.N, r = p.rank;
-  const size_t ts = p.dtype ? 2 : 4;
-  for (int l = 0; l < L; ++l) HM_CHECK(init_params[l] != nullptr, HARMONY_E_INVALID_ARG, "init_params[l] is NULL");
-  // arena
-  if (c->arena) {
-    HM_CHECK(p.arena_bytes <= c->cfg.hbm_cap_bytes, HARMONY_E_CAP_TOO_SMALL, "plan exceeds the adopted arena");
-  } else {
-    HM_CUDA(cudaMalloc(&c->arena, p.arena_bytes));
-    c->own_arena = true;
+  if (!c->members.empty()) {
+    c->plan = R[0]->plan;  // the group's view: rank 0's plan (summary, geometry)
+    c->registered = true;
   }
-  // events of the program
-  c->events.resize(p.n_events);
-  for (auto& e : c->events) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-  // pinned host store
-  c->h_wc.assign(L, nullptr);
-  c->h_state.assign(L, nullptr);
-  c->h_stash.assign((size_t)L * m, nullptr);
-  c->h_grad.assign(L, nullptr);
-  c->h_loss = static_cast<double*>(alloc_host((size_t)N * m * 8));
-  std::vector<uint8_t> full;  // staging of a full compute copy for resident layers
-  for (int l = 0; l < L; ++l) {
-    const LayerPlan& lp = p.layers[l];
-    const int64_t sh = lp.shard, P = lp.P;
-    c->h_wc[l] = static_cast<uint8_t*>(alloc_host((size_t)sh * ts));
-    c->h_state[l] = static_cast<float*>(alloc_host((size_t)lp.state_bytes));
-    if (p.retain_grads || p.schedule == HARMONY_SCHED_PER_GPU_VIRT) c->h_grad[l] = static_cast<float*>(alloc_host((size_t)sh * 4));
-    float* master = c->h_state[l];
-    memset(master, 0, lp.state_bytes);  // m = v = 0 (reading c3), padding = 0
-    const int64_t lo = (int64_t)r * sh, hi = std::min<int64_t>(P, lo + sh);
-    if (hi > lo) memcpy(master, init_params[l] + lo, (size_t)(hi - lo) * 4);
-    if (ts == 2) {
-      uint16_t* w = reinterpret_cast<uint16_t*>(c->h_wc[l]);
-      for (int64_t i = 0; i < sh; ++i) w[i] = f32_to_bf16_rne(master[i]);
-    } else {
-      memcpy(c->h_wc[l], master, (size_t)sh * 4);
-    }
-    for (int i = 0; i < m; ++i)
-      if (lp.stash_res[i] < 0) c->h_stash[(size_t)l * m + i] = static_cast<uint8_t*>(alloc_host(lp.g.st.total));
-    // resident tensors go to HBM now
-    if (lp.wc_res >= 0) {
-      full.assign((size_t)lp.Ppad * ts, 0);
-      if (ts == 2) {
-        uint16_t* w = reinterpret_cast<uint16_t*>(full.data());
-        for (int64_t i = 0; i < P; ++i) w[i] = f32_to_bf16_rne(init_params[l][i]);
-      } else {
-        memcpy(full.data(), init_params[l], (size_t)P * 4);
-      }
-      HM_CUDA(cudaMemcpy(c->arena + lp.wc_res, full.data(), full.size(), cudaMemcpyHostToDevice));
-    }
-    if (lp.state_res >= 0)
-      HM_CUDA(cudaMemcpy(c->arena + lp.state_res, c->h_state[l], lp.state_bytes, cudaMemcpyHostToDevice));
-  }
-  HM_CUDA(cudaDeviceSynchronize());
-  c->plan = std::move(p);
-  c->registered = true;
   HM_API_END(c)
 }
 
@@ -640,9 +957,12 @@ harmony_status harmony_step(harmony_ctx* c, const float* x, const float* target,
   HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
   HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
   HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
+  HM_CHECK(c->group == nullptr, HARMONY_E_BAD_STATE, "a group's rank context is not the caller's");
   HM_CHECK(x && target, HARMONY_E_INVALID_ARG, "x/target NULL");
-  HM_CHECK(batch == (int64_t)c->plan.m * c->plan.b, HARMONY_E_INVALID_ARG,
-           "batch must equal microbatches*microbatch_size (this rank's rows)");
+  const int64_t ranks = (int64_t)ranks_of(c).size();
+  HM_CHECK(batch == ranks * c->plan.m * c->plan.b, HARMONY_E_INVALID_ARG,
+           ranks > 1 ? "batch must equal num_ranks*microbatches*microbatch_size (the global batch)"
+                     : "batch must equal microbatches*microbatch_size (this rank's rows)");
   HM_CUDA(cudaSetDevice(c->cfg.device));
   run_step(c, x, target, loss_out, stats);
   HM_API_END(c)
@@ -659,31 +979,27 @@ harmony_status harmony_read_state(harmony_ctx* c, int32_t layer, int32_t which, 
   HM_CHECK(dst && n == (uint64_t)lp.P, HARMONY_E_INVALID_ARG, "n_floats must equal the layer's parameter count");
   HM_CHECK(which >= HARMONY_PARAM && which <= HARMONY_ADAM_V, HARMONY_E_INVALID_ARG, "bad state kind");
   HM_CHECK(which != HARMONY_GRAD || p.retain_grads, HARMONY_E_BAD_STATE, "HARMONY_GRAD needs retain_grads");
-  HM_CUDA(cudaSetDevice(c->cfg.device));
   const uint64_t sh = (uint64_t)lp.shard;
-  std::vector<float> mine(sh);
-  if (which == HARMONY_GRAD) {
-    memcpy(mine.data(), c->h_grad[layer], sh * 4);
-  } else {
-    const uint64_t off = (which == HARMONY_PARAM ? 0 : which == HARMONY_ADAM_M ? 1 : 2) * sh * 4;
-    if (lp.state_res >= 0) HM_CUDA(cudaMemcpy(mine.data(), c->arena + lp.state_res + off, sh * 4, cudaMemcpyDeviceToHost));
-    else memcpy(mine.data(), reinterpret_cast<uint8_t*>(c->h_state[layer]) + off, sh * 4);
-  }
-  if (p.N == 1) {
+  if (!c->members.empty()) {  // a group reads every rank's shard directly
+    std::vector<float> all((size_t)lp.Ppad);
+    for (size_t r = 0; r < c->members.size(); ++r) read_shard(c->members[r], layer, which, all.data() + r * sh);
+    memcpy(dst, all.data(), (size_t)lp.P * 4);
+    HM_CUDA(cudaSetDevice(c->cfg.device));
+  } else if (p.N == 1) {
+    std::vector<float> mine(sh);
+    read_shard(c, layer, which, mine.data());
     memcpy(dst, mine.data(), (size_t)lp.P * 4);
   } else {
-    float* d = nullptr;
-    HM_CUDA(cudaMalloc(&d, (size_t)lp.Ppad * 4));
-    HM_CUDA(cudaMemcpy(d + (uint64_t)p.rank * sh, mine.data(), sh * 4, cudaMemcpyHostToDevice));
-    ncclResult_t rr = nccl().AllGather(d + (uint64_t)p.rank * sh, d, sh, ncclFloat32, c->comm, c->st[S_COMM]);
-    cudaError_t e1 = cudaStreamSynchronize(c->st[S_COMM]);
-    std::vector<float> all((size_t)lp.Ppad);
-    cudaError_t e2 = cudaMemcpy(all.data(), d, (size_t)lp.Ppad * 4, cudaMemcpyDeviceToHost);
-    cudaFree(d);
-    check_nccl(rr, "ncclAllGather(read_state)");
-    HM_CUDA(e1);
-    HM_CUDA(e2);
-    memcpy(dst, all.data(), (size_t)lp.P * 4);
+    // all-gather through the arena: dW buffer 0 (Ppad fp32 elements) is free between steps
+    std::vector<float> mine(sh);
+    read_shard(c, layer, which, mine.data());
+    float* d = reinterpret_cast<float*>(c->arena + p.dw[0]);
+    cudaStream_t cs = c->st[S_COMM];
+    HM_CUDA(cudaMemcpyAsync(d + (uint64_t)p.rank * sh, mine.data(), sh * 4, cudaMemcpyHostToDevice, cs));
+    check_nccl(nccl().AllGather(d + (uint64_t)p.rank * sh, d, sh, ncclFloat32, c->comm, cs), "ncclAllGather(read_state)");
+    HM_CUDA(cudaMemcpyAsync(c->h_gather, d, (size_t)lp.Ppad * 4, cudaMemcpyDeviceToHost, cs));
+    HM_CUDA(cudaStreamSynchronize(cs));
+    memcpy(dst, c->h_gather, (size_t)lp.P * 4);
   }
   HM_API_END(c)
 }
@@ -691,6 +1007,18 @@ harmony_status harmony_read_state(harmony_ctx* c, int32_t layer, int32_t which, 
 harmony_status harmony_read_stats(const harmony_ctx* c, harmony_step_stats* out) {
   if (!c || !out) return HARMONY_E_INVALID_ARG;
   *out = c->last;
+  return HARMONY_OK;
+}
+
+harmony_status harmony_read_rank_stats(const harmony_ctx* c, int32_t rank, harmony_step_stats* out) {
+  if (!c || !out) return HARMONY_E_INVALID_ARG;
+  if (c->members.empty()) {
+    if (rank != 0) return HARMONY_E_INVALID_ARG;
+    *out = c->last;
+    return HARMONY_OK;
+  }
+  if (rank < 0 || rank >= (int32_t)c->members.size()) return HARMONY_E_INVALID_ARG;
+  *out = c->members[rank]->last;
   return HARMONY_OK;
 }
 
@@ -703,6 +1031,10 @@ harmony_status harmony_plan_info(const harmony_ctx* c, harmony_plan_summary* out
 
 harmony_status harmony_set_profiling(harmony_ctx* c, int32_t on) {
   if (!c) return HARMONY_E_INVALID_ARG;
+  if (on && !c->members.empty() && c->members.size() > 1) {
+    c->err = "per-kernel profiling is per rank context (one process per GPU), not for a group";
+    return HARMONY_E_UNSUPPORTED;
+  }
   c->profiling = on != 0;
   c->prof = harmony_kernel_profile{};
   return HARMONY_OK;
@@ -725,6 +1057,7 @@ harmony_status harmony_read_profile(const harmony_ctx* c, harmony_kernel_profile
 
 harmony_status harmony_finalize(harmony_ctx* c) {
   if (!c) return HARMONY_E_INVALID_ARG;
+  if (c->group) return HARMONY_E_BAD_STATE;
   destroy(c);
   return HARMONY_OK;
 }

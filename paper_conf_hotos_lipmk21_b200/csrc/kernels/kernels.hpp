@@ -53,6 +53,11 @@ size_t attention_bwd_scratch_bytes(int64_t b, int S, int H);
 bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, const void* O, const void* dO,
                          const float* lse, void* dQKV, void* scratch, cudaStream_t st);
 
+// The library's own collectives (collective.cu; harmony_init_group): dst = sum of nsrc fp32
+// buffers in source order (sources may live on peer GPUs).
+constexpr int HM_MAX_GROUP = 16;
+void rank_sum(int nsrc, const float* const* src, int64_t n, float* dst, cudaStream_t st);
+
 // Convenience: a GEMM descriptor with defaults (batch 1, alpha 1, no bias/aux).
 inline hk_gemm_args gemm_args(int dtype, int M, int N, int K) {
   hk_gemm_args a{};

@@ -124,6 +124,8 @@ def lib() -> C.CDLL:
         "harmony_last_error": (C.c_char_p, [P]),
         "harmony_get_unique_id": (st, [P]),
         "harmony_init": (st, [C.POINTER(harmony_config), C.POINTER(P)]),
+        "harmony_init_group": (st, [C.POINTER(harmony_config), C.c_int32, P, C.POINTER(P)]),
+        "harmony_read_rank_stats": (st, [P, C.c_int32, C.POINTER(harmony_step_stats)]),
         "harmony_register_layers": (st, [P, C.c_int32, C.POINTER(harmony_layer_desc), C.POINTER(P)]),
         "harmony_step": (st, [P, P, P, C.c_int64, C.POINTER(C.c_double), C.POINTER(harmony_step_stats)]),
         "harmony_read_state": (st, [P, C.c_int32, C.c_int32, P, C.c_uint64]),
@@ -210,6 +212,21 @@ def harmony_init(cfg: harmony_config) -> C.c_void_p:
     ctx = C.c_void_p()
     _check(lib().harmony_init(C.byref(cfg), C.byref(ctx)))
     return ctx
+
+
+def harmony_init_group(cfg: harmony_config, devices) -> C.c_void_p:
+    """One context driving len(devices) data-parallel ranks (rank r on devices[r]; repeats = ranks
+    sharing a GPU, the loopback)."""
+    ctx = C.c_void_p()
+    arr = (C.c_int32 * len(devices))(*devices)
+    _check(lib().harmony_init_group(C.byref(cfg), len(devices), arr, C.byref(ctx)))
+    return ctx
+
+
+def harmony_read_rank_stats(ctx, rank):
+    s = harmony_step_stats()
+    _check(lib().harmony_read_rank_stats(ctx, int(rank), C.byref(s)), ctx)
+    return s
 
 
 def harmony_register_layers(ctx, descs, init_params):
@@ -318,11 +335,13 @@ def hk(name, *args):
 
 
 class Harmony:
-    """Convenience owner of one context (one process = one GPU rank)."""
+    """Convenience owner of one context: one process = one GPU rank, or (group=[dev, ...]) one
+    process driving len(group) ranks as one virtual device (harmony_init_group)."""
 
-    def __init__(self, descs, init_params, **cfg):
+    def __init__(self, descs, init_params, group=None, **cfg):
         self.cfg = make_config(**cfg)
-        self.ctx = harmony_init(self.cfg)
+        self.ranks = len(group) if group else 1
+        self.ctx = harmony_init_group(self.cfg, list(group)) if group else harmony_init(self.cfg)
         self.descs = list(descs)
         try:
             harmony_register_layers(self.ctx, self.descs, init_params)
@@ -333,7 +352,11 @@ class Harmony:
         self.n_params = [int(np.asarray(p).size) for p in init_params]
 
     def step(self, x, target):
-        return harmony_step(self.ctx, x, target, self.cfg.microbatches * self.cfg.microbatch_size)
+        """x, target: this rank's rows (a group: the global batch of ranks*m*b rows)."""
+        return harmony_step(self.ctx, x, target, self.ranks * self.cfg.microbatches * self.cfg.microbatch_size)
+
+    def rank_stats(self, rank):
+        return harmony_read_rank_stats(self.ctx, rank)
 
     def read(self, layer, which=HARMONY_PARAM):
         return harmony_read_state(self.ctx, layer, which, self.n_params[layer])
