@@ -177,6 +177,10 @@ typedef struct {
   uint64_t launches[6];
   double seconds[6];
   double work[6];
+  double busy_seconds[6];  /* union of the class's launch intervals on all streams: launches of one
+                              class that overlap (e.g. a dgrad GEMM on the compute stream beside a
+                              wgrad GEMM on the side stream) count once, so work / busy_seconds is the
+                              class's throughput while it runs, not each launch's stretched share */
 } harmony_kernel_profile;
 
 /* The step timeline of the last profiled step (profiling on): one record per op of the static
@@ -193,6 +197,16 @@ typedef struct {
   double t0, t1;
 } harmony_timeline_rec;
 harmony_status harmony_read_timeline(const harmony_ctx* ctx, harmony_timeline_rec* out, int32_t cap, int32_t* n_out);
+
+/* The kernel launches of the last profiled step: class (as harmony_kernel_profile), stream (0-3 as
+ * above, 4 = the weight-gradient side stream, -1 other), algorithmic work, [t0, t1] seconds from the
+ * step's start (events on the launching stream around the launch). */
+typedef struct {
+  int32_t cat, stream;
+  double work, t0, t1;
+} harmony_kernel_rec;
+harmony_status harmony_read_kernel_timeline(const harmony_ctx* ctx, harmony_kernel_rec* out, int32_t cap,
+                                           int32_t* n_out);
 
 harmony_status harmony_set_profiling(harmony_ctx* ctx, int32_t on);
 harmony_status harmony_read_profile(const harmony_ctx* ctx, harmony_kernel_profile* out);
@@ -273,6 +287,17 @@ harmony_status harmony_split_gemm_init(const harmony_config* cfg, int64_t M, int
 harmony_status harmony_split_gemm_run(harmony_split_gemm* g, const void* X_slice, const void* W_slice,
                                       const void* dY_shard, float* Y_shard, void* dX_slice, float* dW_slice,
                                       double* seconds);
+/* The same decomposition with all ranks in one process (rank r on devices[r]; NULL = device 0;
+ * repeated ordinals = ranks sharing a GPU).  run_group takes per-rank pointer arrays (num_ranks
+ * entries each, rank r's slices/shards as above, DEVICE pointers on rank r's GPU).  The chunk
+ * reduce-scatter is the library's own: rank i's rows of chunk c are the sum of every rank's fp32
+ * partial in rank order 0..N-1 (pulled from the peers' buffers); the dY all-gather is a copy. */
+harmony_status harmony_split_gemm_init_group(int32_t num_ranks, const int32_t* devices, int64_t M, int64_t N,
+                                             int64_t K, int32_t chunks, harmony_split_gemm** out);
+harmony_status harmony_split_gemm_run_group(harmony_split_gemm* g, const void* const* X_slice,
+                                            const void* const* W_slice, const void* const* dY_shard,
+                                            float* const* Y_shard, void* const* dX_slice, float* const* dW_slice,
+                                            double* seconds);
 harmony_status harmony_split_gemm_finalize(harmony_split_gemm* g);
 
 /* Frees every device and pinned allocation and the communicator; ctx is invalid after. */

@@ -47,7 +47,7 @@ struct KProf {
   bool external = false;  // inside a stream capture: record event nodes into the graph
   std::vector<cudaEvent_t> pool;
   size_t used = 0;
-  struct Rec { int cat, e0, e1; double work; };
+  struct Rec { int cat, e0, e1; double work; cudaStream_t st; };
   std::vector<Rec> recs;
   struct OpRec { int op, e0, e1; };  // the step timeline: events around every op of the program
   std::vector<OpRec> oprecs;
@@ -65,7 +65,7 @@ struct KProf {
   void end(int cat, int e0, cudaStream_t st, double work) {
     if (e0 < 0) return;
     int e1 = begin(st);
-    if (e1 >= 0) recs.push_back({cat, e0, e1, work});
+    if (e1 >= 0) recs.push_back({cat, e0, e1, work, st});
   }
 };
 extern thread_local KProf g_prof;

@@ -84,6 +84,7 @@ struct harmony_ctx {
   bool profiling = false;
   harmony_kernel_profile prof{};
   std::vector<harmony_timeline_rec> timeline;  // last profiled step, one record per op
+  std::vector<harmony_kernel_rec> ktimeline;   // last profiled step, one record per kernel launch
   int* h_step = nullptr;  // pinned: Adam's t, copied to the device at the start of every step
   bool use_graph = true;
   StepGraph g_plain, g_prof;  // the step as CUDA graphs: plain, and with per-kernel timing events
@@ -669,12 +670,42 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
   }
   c->t = t_next;
   if (c->profiling) {
+    std::vector<std::pair<float, float>> iv[PROF_NUM];  // launch intervals per class, ms from the step start
+    c->ktimeline.clear();
     for (auto& rc : *recs) {
-      float e = 0.f;
+      float e = 0.f, t0 = 0.f;
       HM_CUDA(cudaEventElapsedTime(&e, g_prof.pool[rc.e0], g_prof.pool[rc.e1]));
+      HM_CUDA(cudaEventElapsedTime(&t0, c0->ev_begin, g_prof.pool[rc.e0]));
       c->prof.launches[rc.cat] += 1;
       c->prof.seconds[rc.cat] += e * 1e-3;
       c->prof.work[rc.cat] += rc.work;
+      iv[rc.cat].push_back({t0, t0 + e});
+      harmony_kernel_rec kr{};
+      kr.cat = rc.cat;
+      kr.stream = -1;
+      for (int k = 0; k < S_NUM; ++k)
+        if (rc.st == c0->st[k]) kr.stream = k;
+      if (rc.st == c0->side) kr.stream = S_NUM;
+      kr.work = rc.work;
+      kr.t0 = t0 * 1e-3;
+      kr.t1 = (t0 + e) * 1e-3;
+      c->ktimeline.push_back(kr);
+    }
+    for (int k = 0; k < PROF_NUM; ++k) {  // union of the class's intervals
+      auto& v = iv[k];
+      std::sort(v.begin(), v.end());
+      double busy = 0.0;
+      float lo = 0.f, hi = -1.f;
+      for (auto& x : v) {
+        if (x.first > hi) {
+          if (hi > lo) busy += hi - lo;
+          lo = x.first; hi = x.second;
+        } else {
+          hi = std::max(hi, x.second);
+        }
+      }
+      if (hi > lo) busy += hi - lo;
+      c->prof.busy_seconds[k] += busy * 1e-3;
     }
     c->timeline.clear();
     for (auto& orc : *oprecs) {
@@ -939,7 +970,9 @@ harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const h
     HM_CHECK(plans[r].ops.size() == plans[0].ops.size(), HARMONY_E_INVALID_ARG, "internal: rank programs differ");
     for (size_t i = 0; i < plans[0].ops.size(); ++i)
       HM_CHECK(plans[r].ops[i].kind == plans[0].ops[i].kind && plans[r].ops[i].stream == plans[0].ops[i].stream &&
-                   plans[r].ops[i].waits == plans[0].ops[i].waits && plans[r].ops[i].dev == plans[0].ops[i].dev,
+                   plans[r].ops[i].waits == plans[0].ops[i].waits &&
+                   (!is_group_collective(plans[0].ops[i].kind) ||
+                    (plans[r].ops[i].dev == plans[0].ops[i].dev && plans[r].ops[i].count == plans[0].ops[i].count)),
                HARMONY_E_INVALID_ARG, "internal: rank programs differ");
   }
   for (size_t r = 0; r < R.size(); ++r) register_rank(R[r], std::move(plans[r]), init_params);
@@ -1046,6 +1079,16 @@ harmony_status harmony_read_timeline(const harmony_ctx* c, harmony_timeline_rec*
   *n_out = n;
   if (out)
     for (int32_t i = 0; i < std::min(n, cap); ++i) out[i] = c->timeline[i];
+  return HARMONY_OK;
+}
+
+harmony_status harmony_read_kernel_timeline(const harmony_ctx* c, harmony_kernel_rec* out, int32_t cap,
+                                           int32_t* n_out) {
+  if (!c || !n_out || cap < 0) return HARMONY_E_INVALID_ARG;
+  const int32_t n = (int32_t)c->ktimeline.size();
+  *n_out = n;
+  if (out)
+    for (int32_t i = 0; i < std::min(n, cap); ++i) out[i] = c->ktimeline[i];
   return HARMONY_OK;
 }
 

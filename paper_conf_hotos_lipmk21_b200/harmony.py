@@ -65,17 +65,26 @@ class harmony_plan_summary(C.Structure):
 
 
 class harmony_kernel_profile(C.Structure):
-    _fields_ = [("launches", C.c_uint64 * 6), ("seconds", C.c_double * 6), ("work", C.c_double * 6)]
+    _fields_ = [("launches", C.c_uint64 * 6), ("seconds", C.c_double * 6), ("work", C.c_double * 6),
+                ("busy_seconds", C.c_double * 6)]
     CLASSES = ("gemm", "adam", "layernorm", "softmax", "other", "attention")
 
     def as_dict(self):
-        return {c: dict(launches=self.launches[i], seconds=self.seconds[i], work=self.work[i])
+        return {c: dict(launches=self.launches[i], seconds=self.seconds[i], work=self.work[i],
+                        busy_seconds=self.busy_seconds[i])
                 for i, c in enumerate(self.CLASSES)}
 
 
 class harmony_timeline_rec(C.Structure):
     _fields_ = [(n, C.c_int32) for n in ("op", "kind", "stream", "cat", "layer", "micro")] + [
         ("bytes", C.c_uint64), ("t0", C.c_double), ("t1", C.c_double)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+class harmony_kernel_rec(C.Structure):
+    _fields_ = [("cat", C.c_int32), ("stream", C.c_int32), ("work", C.c_double), ("t0", C.c_double), ("t1", C.c_double)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -135,6 +144,7 @@ def lib() -> C.CDLL:
                                   C.POINTER(harmony_plan_summary), P, C.c_uint64]),
         "harmony_finalize": (st, [P]),
         "harmony_read_timeline": (st, [P, P, C.c_int32, C.POINTER(C.c_int32)]),
+        "harmony_read_kernel_timeline": (st, [P, P, C.c_int32, C.POINTER(C.c_int32)]),
         "hk_gemm": (st, [C.POINTER(hk_gemm_args), P]),
         "hk_layernorm_fwd": (st, [C.c_int32, C.c_int64, C.c_int32, P, P, P, P, P, P, P]),
         "hk_layernorm_bwd": (st, [C.c_int32, C.c_int64, C.c_int32, P, P, P, P, P, P, P, P, P, C.c_int32, P]),
@@ -154,6 +164,9 @@ def lib() -> C.CDLL:
                                          C.POINTER(P)]),
         "harmony_split_gemm_run": (st, [P, P, P, P, P, P, P, C.POINTER(C.c_double)]),
         "harmony_split_gemm_finalize": (st, [P]),
+        "harmony_split_gemm_init_group": (st, [C.c_int32, P, C.c_int64, C.c_int64, C.c_int64, C.c_int32,
+                                               C.POINTER(P)]),
+        "harmony_split_gemm_run_group": (st, [P, P, P, P, P, P, P, C.POINTER(C.c_double)]),
         "harmony_set_profiling": (st, [P, C.c_int32]),
         "harmony_read_profile": (st, [P, C.POINTER(harmony_kernel_profile)]),
     }
@@ -298,6 +311,15 @@ def harmony_read_timeline(ctx):
     return [arr[i].as_dict() for i in range(n.value)]
 
 
+def harmony_read_kernel_timeline(ctx):
+    """Kernel launches of the last profiled step (list of dicts; see harmony.h)."""
+    n = C.c_int32()
+    _check(lib().harmony_read_kernel_timeline(ctx, None, 0, C.byref(n)), ctx)
+    arr = (harmony_kernel_rec * max(n.value, 1))()
+    _check(lib().harmony_read_kernel_timeline(ctx, arr, n.value, C.byref(n)), ctx)
+    return [arr[i].as_dict() for i in range(n.value)]
+
+
 def harmony_finalize(ctx):
     _check(lib().harmony_finalize(ctx))
 
@@ -314,6 +336,37 @@ class SplitGemm:
         sec = C.c_double()
         _check(lib().harmony_split_gemm_run(self.h, _ptr(X_slice), _ptr(W_slice), _ptr(dY_shard), _ptr(Y_shard),
                                             _ptr(dX_slice), _ptr(dW_slice), C.byref(sec)))
+        return sec.value
+
+    def close(self):
+        if self.h:
+            _check(lib().harmony_split_gemm_finalize(self.h))
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+class SplitGemmGroup:
+    """Operator-split GEMM fwd+bwd with every rank in this process (harmony_split_gemm_init_group):
+    rank r on devices[r]; run() takes per-rank lists of tensors."""
+
+    def __init__(self, M, N, K, devices, chunks=4):
+        self.n = len(devices)
+        self.h = C.c_void_p()
+        arr = (C.c_int32 * self.n)(*devices)
+        _check(lib().harmony_split_gemm_init_group(self.n, arr, M, N, K, chunks, C.byref(self.h)))
+
+    def run(self, X, W, dY, Y, dX, dW):
+        def arr(ts):
+            assert len(ts) == self.n
+            return (C.c_void_p * self.n)(*[_ptr(t) for t in ts])
+        sec = C.c_double()
+        _check(lib().harmony_split_gemm_run_group(self.h, arr(X), arr(W), arr(dY), arr(Y), arr(dX), arr(dW),
+                                                  C.byref(sec)))
         return sec.value
 
     def close(self):

@@ -53,3 +53,30 @@ def test_split_gemm_cfg5_full_size_sampled():
         # path is 2e-2 — the bound here is 2e-3.  dX is additionally rounded to bf16 (2^-9).
         tol = 4e-3 if which == "dX" else 2e-3
         assert rel(got, ref) < tol, which
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_split_gemm_k_split_across_ranks_loopback(world):
+    """Row a15's cross-GPU half: K split over `world` ranks (one process, ranks sharing the GPU),
+    chunked reduce-scatter of the fp32 partials overlapped with the next chunk's GEMM, dY all-gather,
+    local dX / dW slices — against the fp64 oracle's K-split decomposition (= the plain GEMM by the
+    block-matrix identity, self-check ii)."""
+    M, N, K, chunks = 2048, 1024, 8192, 4
+    X, W, dY = synth.gen_gemm_operands(M, N, K)
+    Kr, Mr = K // world, M // world
+    bf = torch.bfloat16
+    Xs = [torch.tensor(X[:, r * Kr:(r + 1) * Kr].copy()).to("cuda", bf) for r in range(world)]
+    Ws = [torch.tensor(W[r * Kr:(r + 1) * Kr].copy()).to("cuda", bf) for r in range(world)]
+    dYs = [torch.tensor(dY[r * Mr:(r + 1) * Mr].copy()).to("cuda", bf) for r in range(world)]
+    Ys = [torch.empty(Mr, N, device="cuda") for _ in range(world)]
+    dXs = [torch.empty(M, Kr, device="cuda", dtype=bf) for _ in range(world)]
+    dWs = [torch.empty(Kr, N, device="cuda") for _ in range(world)]
+    with H.SplitGemmGroup(M, N, K, [0] * world, chunks=chunks) as g:
+        g.run(Xs, Ws, dYs, Ys, dXs, dWs)
+        Y1 = torch.cat(Ys).cpu().numpy()
+        g.run(Xs, Ws, dYs, Ys, dXs, dWs)  # rerun: deterministic (rank-order sums)
+        assert np.array_equal(torch.cat(Ys).cpu().numpy(), Y1)
+    rY, rdX, rdW = oracle.split_gemm_fwd_bwd(X, W, dY, n_k_splits=world, m_tiles=world * chunks)
+    assert rel(Y1, rY) < 1e-5
+    assert rel(torch.cat(dWs).cpu().numpy(), rdW) < 1e-5
+    assert rel(torch.cat(dXs, dim=1).float().cpu().numpy(), rdX) < 4e-3
