@@ -33,6 +33,9 @@ size_t colsum_scratch_bytes(int64_t rows, int n);
 void splitk_sum(int S, int64_t n, const float* ws, float* C, int accumulate, cudaStream_t st);
 void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float* out, int accumulate, float* scratch,
             cudaStream_t st);
+// Xt = (T) X and out (+)= column sums of X, one pass over the fp32 [rows, n] X (n % 4 == 0)
+void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float* out, int accumulate, float* scratch,
+                 cudaStream_t st);
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st);
 void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, const void* P, void* dZ,
                  cudaStream_t st);

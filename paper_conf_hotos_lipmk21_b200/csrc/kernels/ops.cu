@@ -199,6 +199,46 @@ __global__ void __launch_bounds__(128) colsum_partial_vec_kernel(int64_t rows, i
   for (int v = 0; v < VEC; v += 4) *reinterpret_cast<float4*>(p + v) = make_float4(s[v], s[v + 1], s[v + 2], s[v + 3]);
 }
 
+// One pass over an fp32 [rows, n] array: its T copy (the GEMM operand) and the column partials of
+// the column sum (the bias gradient of the branch it feeds), rows in increasing order per chunk.
+template <typename T>
+__global__ void __launch_bounds__(128) cast_colsum_partial_kernel(int64_t rows, int n, const float* __restrict__ X,
+                                                                  T* __restrict__ Xt, float* __restrict__ partial) {
+  const int c0 = (blockIdx.x * blockDim.x + threadIdx.x) * 4;
+  if (c0 >= n) return;
+  const int64_t r0 = (int64_t)blockIdx.y * CS_ROWS, r1 = min(rows, r0 + CS_ROWS);
+  float4 u[CS_ROWS];
+#pragma unroll
+  for (int i = 0; i < CS_ROWS; ++i)
+    u[i] = r0 + i < r1 ? __ldg(reinterpret_cast<const float4*>(X + (r0 + i) * n + c0)) : make_float4(0.f, 0.f, 0.f, 0.f);
+  float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+  for (int i = 0; i < CS_ROWS; ++i) {
+    s.x += u[i].x; s.y += u[i].y; s.z += u[i].z; s.w += u[i].w;
+    if (r0 + i < r1) {
+      T* o = Xt + (r0 + i) * n + c0;
+      o[0] = from_f32<T>(u[i].x); o[1] = from_f32<T>(u[i].y); o[2] = from_f32<T>(u[i].z); o[3] = from_f32<T>(u[i].w);
+    }
+  }
+  *reinterpret_cast<float4*>(partial + (int64_t)blockIdx.y * n + c0) = s;
+}
+
+void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float* out, int accumulate, float* scratch,
+                 cudaStream_t st) {
+  const int nch = (int)ceil_div(rows, CS_ROWS);
+  if (n % 4 || (reinterpret_cast<uintptr_t>(X) & 15) || nch == 0) {  // unaligned: the two separate passes
+    cast(dtype, rows * n, X, Xt, st);
+    colsum(0, rows, n, X, n, out, accumulate, scratch, st);
+    return;
+  }
+  const int e0 = g_prof.begin(st);
+  dim3 grid((unsigned)ceil_div(n / 4, 128), (unsigned)nch);
+  HM_DISPATCH_T(dtype, (cast_colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, X, (T*)Xt, scratch)));
+  check_launch("cast_colsum_partial");
+  colreduce(nch, n, scratch, n, out, accumulate, st);
+  g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (4 + (dtype ? 2 : 4)));
+}
+
 // ------------------------------------------------------------------------------------- softmax
 // P = softmax(scale * Z) over each row; causal rows mask keys j > (row % S) to exactly 0 (c11).
 template <typename T>

@@ -403,9 +403,12 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     HM_CUDA(cudaStreamWaitEvent(t_side, t_side_ev[k], 0));
   };
 
-  // dY as a GEMM operand
+  // dY as a GEMM operand; bf16: its copy and the FC2 bias gradient (column sums) in one pass
   const void* dYop = dY;
-  if (dt == 1) { cast(1, R * D, dY, dYc, st); dYop = dYc; }
+  if (dt == 1) {
+    cast_colsum(1, R, D, dY, dYc, gseg(g, dW, P_BFC2), acc, scratch, st);
+    dYop = dYc;
+  }
   // ---- FC2: dG = dY W_fc2^T, fused with GeLU': dH = dG * gelu'(H)
   {
     hk_gemm_args a = lin_dgrad(g, R, D, 4 * D, dYop, wseg(g, W, P_WFC2));
@@ -416,7 +419,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   if (g.stash_policy == 1) act_fwd_T(dt, HARMONY_ACT_GELU_TANH, R * 4 * D, Hh, rec, st);
   fork(0);
   gemm(lin_wgrad(g, R, D, 4 * D, G, dYop, gseg(g, dW, P_WFC2), first), sw);
-  colsum(0, R, D, dY, D, gseg(g, dW, P_BFC2), acc, wscratch, sw);
+  if (dt == 0) colsum(0, R, D, dY, D, gseg(g, dW, P_BFC2), acc, wscratch, sw);
   // ---- FC1: dU2 = dH W_fc1^T (fp32 for the LN backward); dW_fc1 += U2^T dH
   {
     hk_gemm_args a = lin_dgrad(g, R, 4 * D, D, dHb, wseg(g, W, P_WFC1));
@@ -435,12 +438,11 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), sw);
   colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, wscratch, sw);
   // ---- LN2 backward: dX2 = dY + LN2'(dU2), fused with the bf16 copy of dX2 (the O-projection
-  // GEMM operand); db_o += sum_rows dX2
+  // GEMM operand) and db_o (+)= sum_rows dX2
   const void* dX2op = dt == 1 ? (const void*)dX2c_buf : (const void*)dX2;
   layernorm_bwd_ex(dt, R, D, dUf, X2, mean2, rstd2, wseg(g, W, P_LN2_G), dY, dX2, gseg(g, dW, P_LN2_G),
-                   gseg(g, dW, P_LN2_B), acc, dt == 1 ? dX2c_buf : nullptr, nullptr, 0, scratch, st);
+                   gseg(g, dW, P_LN2_B), acc, dt == 1 ? dX2c_buf : nullptr, gseg(g, dW, P_BO), acc, scratch, st);
   fork(1);
-  colsum(0, R, D, dX2, D, gseg(g, dW, P_BO), acc, wscratch, sw);
   // ---- O projection: dC = dX2 W_o^T; dW_o += C^T dX2
   {
     hk_gemm_args a = lin_dgrad(g, R, D, D, dX2op, wseg(g, W, P_WO));
