@@ -223,22 +223,6 @@ __global__ void __launch_bounds__(128) cast_colsum_partial_kernel(int64_t rows, 
   *reinterpret_cast<float4*>(partial + (int64_t)blockIdx.y * n + c0) = s;
 }
 
-void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float* out, int accumulate, float* scratch,
-                 cudaStream_t st) {
-  const int nch = (int)ceil_div(rows, CS_ROWS);
-  if (n % 4 || (reinterpret_cast<uintptr_t>(X) & 15) || nch == 0) {  // unaligned: the two separate passes
-    cast(dtype, rows * n, X, Xt, st);
-    colsum(0, rows, n, X, n, out, accumulate, scratch, st);
-    return;
-  }
-  const int e0 = g_prof.begin(st);
-  dim3 grid((unsigned)ceil_div(n / 4, 128), (unsigned)nch);
-  HM_DISPATCH_T(dtype, (cast_colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, X, (T*)Xt, scratch)));
-  check_launch("cast_colsum_partial");
-  colreduce(nch, n, scratch, n, out, accumulate, st);
-  g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (4 + (dtype ? 2 : 4)));
-}
-
 // ------------------------------------------------------------------------------------- softmax
 // P = softmax(scale * Z) over each row; causal rows mask keys j > (row % S) to exactly 0 (c11).
 template <typename T>
@@ -475,6 +459,22 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
   check_launch("colsum_partial");
   colreduce(nch, n, scratch, n, out, accumulate, st);
   g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (in_dtype ? 2 : 4));
+}
+
+void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float* out, int accumulate, float* scratch,
+                 cudaStream_t st) {
+  const int nch = (int)ceil_div(rows, CS_ROWS);
+  if (n % 4 || (reinterpret_cast<uintptr_t>(X) & 15) || nch == 0) {  // unaligned: the two separate passes
+    cast(dtype, rows * n, X, Xt, st);
+    colsum(0, rows, n, X, n, out, accumulate, scratch, st);
+    return;
+  }
+  const int e0 = g_prof.begin(st);
+  dim3 grid((unsigned)ceil_div(n / 4, 128), (unsigned)nch);
+  HM_DISPATCH_T(dtype, (cast_colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, X, (T*)Xt, scratch)));
+  check_launch("cast_colsum_partial");
+  colreduce(nch, n, scratch, n, out, accumulate, st);
+  g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (4 + (dtype ? 2 : 4)));
 }
 
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st) {
