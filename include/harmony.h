@@ -86,7 +86,15 @@ typedef enum { HARMONY_PARAM = 0, HARMONY_GRAD = 1, HARMONY_ADAM_M = 2, HARMONY_
  * (per-GPU memory virtualization, Fig. 5(b)): each microbatch swaps
  * the weights in and out for its own forward and backward, and the update runs
  * after the whole backward.  Both compute the identical result. */
-typedef enum { HARMONY_SCHED_HARMONY_DP = 0, HARMONY_SCHED_PER_GPU_VIRT = 1 } harmony_schedule;
+typedef enum { HARMONY_SCHED_HARMONY_DP = 0, HARMONY_SCHED_PER_GPU_VIRT = 1, HARMONY_SCHED_HARMONY_PP = 2 } harmony_schedule;
+/* HARMONY_SCHED_HARMONY_PP (groups only, num_ranks >= 2, layers >= ranks): the paper's virtualized
+ * pipeline (Fig. 4; DESIGN reading c27).  Layer l runs on rank
+ * l % num_ranks; every layer-level task runs its group of m microbatches back to back (input-batch
+ * grouping); activations and gradients go to the next / previous layer's rank peer to peer; each
+ * layer's weights are swapped in once for its forward group, once for its backward group and out
+ * once after its just-in-time update — 3|W| per iteration for the whole box.  The batch is ONE
+ * minibatch of m*b samples (not num_ranks*m*b); the result is bit-identical to the single-rank
+ * Harmony-DP step with the same m and b (same kernels, same accumulation order). */
 
 typedef struct {
   uint32_t struct_size;      /* = sizeof(harmony_config) (ABI versioning)                   */
@@ -232,6 +240,11 @@ harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out);
 harmony_status harmony_init_group(const harmony_config* cfg, int32_t num_ranks, const int32_t* devices,
                                   harmony_ctx** out);
 harmony_status harmony_read_rank_stats(const harmony_ctx* ctx, int32_t rank, harmony_step_stats* out);
+/* Host-only planning of a group of num_ranks ranks (no CUDA call): for HARMONY_SCHED_HARMONY_PP the
+ * group's one program (each op tagged rank=r), else rank 0's data-parallel program. */
+harmony_status harmony_plan_dry_group(const harmony_config* cfg, int32_t num_ranks, int32_t n_layers,
+                                      const harmony_layer_desc* descs, harmony_plan_summary* out, char* program_text,
+                                      uint64_t text_len);
 
 /* Registers the layer stack and its initial fp32 parameters (canonical packing, one
  * host array per layer, identical on every rank).  Decomposes the step into tasks,

@@ -19,6 +19,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <memory>
 #include <stdexcept>
 #include <string>
 #include <vector>
@@ -52,7 +53,7 @@ struct StepGraph {
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
   int sig = -1;                           // (x on device) | (target on device) << 1 at capture
-  struct In { int rank, op; cudaGraphNode_t node; };
+  struct In { int rank; const Op* op; cudaGraphNode_t node; };
   std::vector<In> in_nodes;               // input copies, re-pointed every step
   std::vector<harmony_step_stats> stats;  // per rank
   uint64_t launches = 0;
@@ -96,6 +97,7 @@ struct harmony_ctx {
   harmony_ctx* group = nullptr;
   bool one_device = true;               // group: every rank on the same GPU (loopback)
   cudaEvent_t lb_ready = nullptr, lb_done = nullptr;  // member: rendezvous of a group collective
+  std::unique_ptr<GroupPlan> gplan;     // group under Harmony-PP: the one program of all ranks
 };
 
 namespace {
@@ -302,9 +304,8 @@ void zero_dw_padding(harmony_ctx* c, const Op& o) {
     HM_CUDA(cudaMemsetAsync(c->arena + o.dev + (uint64_t)lp.P * 4, 0, (tot - (uint64_t)lp.P) * 4, c->st[o.stream]));
 }
 
-void op_body(harmony_ctx* c, size_t oi, const RankIn& in, harmony_step_stats& s) {
+void op_body(harmony_ctx* c, const Op& o, const RankIn& in, harmony_step_stats& s) {
   Plan& p = c->plan;
-  const Op& o = p.ops[oi];
   uint8_t* A = c->arena;
   const int dt = p.dtype;
   cudaStream_t st = c->st[o.stream];
@@ -466,8 +467,50 @@ void issue_group_collective(const std::vector<harmony_ctx*>& R, bool one_device,
   }
 }
 
+// Harmony-PP: the group's one program in order; an op's waits may name other ranks' ops (the
+// activation / gradient hand-offs), whose events live in those ranks' contexts.
+void issue_program_pp(harmony_ctx* c, const std::vector<RankIn>& in, std::vector<harmony_step_stats>& s) {
+  const std::vector<harmony_ctx*>& R = c->members;
+  const GroupPlan& gp = *c->gplan;
+  for (harmony_ctx* r : R) {
+    if (!c->one_device) HM_CUDA(cudaSetDevice(r->cfg.device));
+    issue_prologue(r);
+  }
+  for (const GOp& g : gp.ops) {
+    harmony_ctx* rc = R[g.rank];
+    const Op& o = g.op;
+    if (!c->one_device) HM_CUDA(cudaSetDevice(rc->cfg.device));
+    cudaStream_t st = rc->st[o.stream];
+    for (int w : o.waits) HM_CUDA(cudaStreamWaitEvent(st, R[gp.ops[w].rank]->events[gp.ops[w].op.event], 0));
+    if (o.kind == OP_P2P) {  // peer to peer over NVLink (or inside the GPU when the ranks share it)
+      HM_CUDA(cudaMemcpyAsync(rc->arena + o.dev, R[o.peer]->arena + o.peer_off, o.bytes, cudaMemcpyDefault, st));
+      s[g.rank].nvlink_bytes += o.bytes;
+    } else {
+      op_body(rc, o, in[g.rank], s[g.rank]);
+    }
+    if (o.event >= 0) HM_CUDA(cudaEventRecord(rc->events[o.event], st));
+  }
+  if (!c->one_device) HM_CUDA(cudaSetDevice(R[0]->cfg.device));
+}
+
+// The user-input copies of the step: (rank, op).
+std::vector<std::pair<int, const Op*>> input_ops(harmony_ctx* c) {
+  std::vector<std::pair<int, const Op*>> v;
+  if (c->gplan) {
+    for (const GOp& g : c->gplan->ops)
+      if (g.op.kind == OP_INPUT) v.push_back({g.rank, &g.op});
+    return v;
+  }
+  const std::vector<harmony_ctx*> R = ranks_of(c);
+  for (size_t r = 0; r < R.size(); ++r)
+    for (const Op& o : R[r]->plan.ops)
+      if (o.kind == OP_INPUT) v.push_back({(int)r, &o});
+  return v;
+}
+
 // Issue the static program once on every rank's streams (eagerly, or inside a stream capture).
 void issue_program(harmony_ctx* c, const std::vector<RankIn>& in, std::vector<harmony_step_stats>& s) {
+  if (c->gplan) return issue_program_pp(c, in, s);
   const std::vector<harmony_ctx*> R = ranks_of(c);
   const bool group = !c->members.empty();
   const bool one_device = c->one_device;
@@ -484,7 +527,7 @@ void issue_program(harmony_ctx* c, const std::vector<RankIn>& in, std::vector<ha
     for (size_t r = 0; r < R.size(); ++r) {
       if (!one_device) HM_CUDA(cudaSetDevice(R[r]->cfg.device));
       const int e0 = op_pre(R[r], oi);
-      op_body(R[r], oi, in[r], s[r]);
+      op_body(R[r], R[r]->plan.ops[oi], in[r], s[r]);
       op_post(R[r], oi, e0);
     }
   }
@@ -552,9 +595,7 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const std::vector<RankIn>& in, 
   std::vector<cudaGraphNode_t> nodes(n);
   HM_CUDA(cudaGraphGetNodes(G.graph, nodes.data(), &n));
   G.in_nodes.clear();
-  for (size_t r = 0; r < R.size(); ++r)
-    for (size_t i = 0; i < R[r]->plan.ops.size(); ++i)
-      if (R[r]->plan.ops[i].kind == OP_INPUT) G.in_nodes.push_back({(int)r, (int)i, nullptr});
+  for (auto& io : input_ops(c)) G.in_nodes.push_back({io.first, io.second, nullptr});
   for (auto nd : nodes) {
     cudaGraphNodeType ty;
     HM_CUDA(cudaGraphNodeGetType(nd, &ty));
@@ -563,7 +604,7 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const std::vector<RankIn>& in, 
     HM_CUDA(cudaGraphMemcpyNodeGetParams(nd, &mp));
     const uint8_t* dst = static_cast<const uint8_t*>(mp.dstPtr.ptr);
     for (auto& e : G.in_nodes)
-      if (dst == R[e.rank]->arena + R[e.rank]->plan.ops[e.op].dev) e.node = nd;
+      if (dst == R[e.rank]->arena + e.op->dev) e.node = nd;
   }
   for (auto& e : G.in_nodes) HM_CHECK(e.node != nullptr, HARMONY_E_CUDA, "graph capture: input copy node not found");
   G.sig = (in[0].x_dev ? 1 : 0) | (in[0].t_dev ? 2 : 0);
@@ -582,9 +623,10 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
   }
   const PtrKind xk = ptr_kind(x), tk = ptr_kind(tg);
   std::vector<RankIn> in(NR);
+  const bool pp = c->gplan != nullptr;  // Harmony-PP: the whole batch enters at rank 0, targets at the last rank
   for (int r = 0; r < NR; ++r) {
-    in[r].x = x + (size_t)r * p0.m * p0.in_elems_per_mb;
-    in[r].tg = tg + (size_t)r * p0.m * p0.out_elems_per_mb;
+    in[r].x = pp ? x : x + (size_t)r * p0.m * p0.in_elems_per_mb;
+    in[r].tg = pp ? tg : tg + (size_t)r * p0.m * p0.out_elems_per_mb;
     in[r].x_dev = xk == PTR_DEVICE;
     in[r].t_dev = tk == PTR_DEVICE;
   }
@@ -613,7 +655,7 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
       issued = true;
       if (!G.exec || G.sig != sig) capture_graph(c, G, in, c->profiling);
       for (auto& e : G.in_nodes) {
-        const Op& o = R[e.rank]->plan.ops[e.op];
+        const Op& o = *e.op;
         const uint8_t* src = reinterpret_cast<const uint8_t*>(o.hbuf == HB_USER_X ? (const void*)in[e.rank].x
                                                                                   : (const void*)in[e.rank].tg);
         HM_CUDA(cudaGraphExecMemcpyNodeSetParams1D(G.exec, e.node, R[e.rank]->arena + o.dev, src + o.hoff, o.bytes,
@@ -721,8 +763,13 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     g_prof.on = false;
   }
   double loss = 0.0;  // rank partials summed in rank order, microbatches in order (reading c22)
-  for (int r = 0; r < p0.N; ++r)
-    for (int i = 0; i < p0.m; ++i) loss += c0->h_loss[r * p0.m + i];
+  if (pp) {  // the last layer's rank computed the loss of every microbatch
+    const harmony_ctx* cl = R[c->gplan->layer_rank.back()];
+    for (int i = 0; i < p0.m; ++i) loss += cl->h_loss[i];
+  } else {
+    for (int r = 0; r < p0.N; ++r)
+      for (int i = 0; i < p0.m; ++i) loss += c0->h_loss[r * p0.m + i];
+  }
   if (loss_out) *loss_out = loss;
   // a rank's ledger, or a group's box totals (bytes summed over ranks)
   harmony_step_stats tot = s[0];
@@ -736,7 +783,7 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     tot.nvlink_bytes += s[r].nvlink_bytes;
   }
   tot.kernel_launches = launches;
-  tot.n_ops = p0.ops.size() * NR;
+  tot.n_ops = pp ? c->gplan->ops.size() : p0.ops.size() * NR;
   tot.peak_arena_bytes = 0;
   for (harmony_ctx* r : R) tot.peak_arena_bytes = std::max<uint64_t>(tot.peak_arena_bytes, r->plan.arena_bytes);
   tot.graph = use_graph ? 1 : 0;
@@ -873,6 +920,32 @@ harmony_status harmony_plan_dry(const harmony_config* cfg, int32_t n_layers, con
   HM_API_END(nullptr)
 }
 
+harmony_status harmony_plan_dry_group(const harmony_config* cfg, int32_t num_ranks, int32_t n_layers,
+                                      const harmony_layer_desc* descs, harmony_plan_summary* out, char* text,
+                                      uint64_t text_len) {
+  HM_API_BEGIN
+  HM_CHECK(cfg && descs && out, HARMONY_E_INVALID_ARG, "NULL argument");
+  std::string d;
+  if (cfg->schedule == HARMONY_SCHED_HARMONY_PP) {
+    GroupPlan g = make_plan_pp(*cfg, num_ranks, n_layers, descs);
+    *out = g.summary;
+    if (text && text_len > 0) d = dump_group_plan(g);
+  } else {  // data parallel: rank 0's program (every rank's has the same shape)
+    harmony_config c0 = *cfg;
+    c0.rank = 0;
+    c0.world_size = num_ranks;
+    Plan p = make_plan(c0, n_layers, descs);
+    *out = p.summary;
+    if (text && text_len > 0) d = dump_plan(p);
+  }
+  if (text && text_len > 0) {
+    size_t n = std::min<size_t>(d.size(), text_len - 1);
+    memcpy(text, d.data(), n);
+    text[n] = 0;
+  }
+  HM_API_END(nullptr)
+}
+
 harmony_status harmony_init(const harmony_config* cfg, harmony_ctx** out) {
   harmony_ctx* c = nullptr;
   HM_API_BEGIN
@@ -959,6 +1032,26 @@ harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const h
   HM_CHECK(descs && init_params, HARMONY_E_INVALID_ARG, "NULL argument");
   for (int l = 0; l < n_layers; ++l) HM_CHECK(init_params[l] != nullptr, HARMONY_E_INVALID_ARG, "init_params[l] is NULL");
   std::vector<harmony_ctx*> R = ranks_of(c);
+  if (c->cfg.schedule == HARMONY_SCHED_HARMONY_PP) {
+    HM_CHECK(!c->members.empty(), HARMONY_E_UNSUPPORTED, "Harmony-PP runs in a group (harmony_init_group)");
+    auto gp = std::make_unique<GroupPlan>(make_plan_pp(c->cfg, (int)R.size(), n_layers, descs));
+    HM_CHECK(gp->summary.hazards == 0, HARMONY_E_INVALID_ARG, "internal: planned program has a hazard: " + gp->hazard_msg);
+    for (size_t r = 0; r < R.size(); ++r) {
+      std::vector<const float*> mine;
+      for (int l = (int)r; l < n_layers; l += (int)R.size()) mine.push_back(init_params[l]);
+      register_rank(R[r], Plan(gp->ranks[r]), mine.data());
+      HM_CUDA(cudaSetDevice(R[r]->cfg.device));
+      for (auto e : R[r]->events) cudaEventDestroy(e);
+      R[r]->events.assign(gp->n_events, nullptr);  // slots of the group program's events
+      for (auto& e : R[r]->events) HM_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+    HM_CUDA(cudaSetDevice(c->cfg.device));
+    c->plan = R[0]->plan;
+    c->plan.summary = gp->summary;
+    c->gplan = std::move(gp);
+    c->registered = true;
+    return HARMONY_OK;
+  }
   std::vector<Plan> plans;
   for (harmony_ctx* r : R) {
     plans.push_back(make_plan(r->cfg, n_layers, descs));
@@ -992,7 +1085,7 @@ harmony_status harmony_step(harmony_ctx* c, const float* x, const float* target,
   HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
   HM_CHECK(c->group == nullptr, HARMONY_E_BAD_STATE, "a group's rank context is not the caller's");
   HM_CHECK(x && target, HARMONY_E_INVALID_ARG, "x/target NULL");
-  const int64_t ranks = (int64_t)ranks_of(c).size();
+  const int64_t ranks = c->gplan ? 1 : (int64_t)ranks_of(c).size();  // Harmony-PP: one batch flows through the ranks
   HM_CHECK(batch == ranks * c->plan.m * c->plan.b, HARMONY_E_INVALID_ARG,
            ranks > 1 ? "batch must equal num_ranks*microbatches*microbatch_size (the global batch)"
                      : "batch must equal microbatches*microbatch_size (this rank's rows)");
@@ -1006,6 +1099,21 @@ harmony_status harmony_read_state(harmony_ctx* c, int32_t layer, int32_t which, 
   HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
   HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
   HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
+  if (c->gplan) {  // Harmony-PP: the layer lives, unsharded, on rank layer % N
+    const GroupPlan& gp = *c->gplan;
+    HM_CHECK(layer >= 0 && layer < (int)gp.layer_rank.size(), HARMONY_E_INVALID_ARG, "layer out of range");
+    harmony_ctx* m = c->members[gp.layer_rank[layer]];
+    const int k = gp.layer_local[layer];
+    const LayerPlan& lq = m->plan.layers[k];
+    HM_CHECK(dst && n == (uint64_t)lq.P, HARMONY_E_INVALID_ARG, "n_floats must equal the layer's parameter count");
+    HM_CHECK(which >= HARMONY_PARAM && which <= HARMONY_ADAM_V, HARMONY_E_INVALID_ARG, "bad state kind");
+    HM_CHECK(which != HARMONY_GRAD || m->plan.retain_grads, HARMONY_E_BAD_STATE, "HARMONY_GRAD needs retain_grads");
+    std::vector<float> all((size_t)lq.shard);
+    read_shard(m, k, which, all.data());
+    memcpy(dst, all.data(), (size_t)lq.P * 4);
+    HM_CUDA(cudaSetDevice(c->cfg.device));
+    return HARMONY_OK;
+  }
   const Plan& p = c->plan;
   HM_CHECK(layer >= 0 && layer < (int)p.layers.size(), HARMONY_E_INVALID_ARG, "layer out of range");
   const LayerPlan& lp = p.layers[layer];

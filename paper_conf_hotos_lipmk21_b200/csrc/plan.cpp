@@ -24,15 +24,16 @@ void validate_config(const harmony_config& c) {
   HM_CHECK(c.microbatch_size >= 1, HARMONY_E_INVALID_ARG, "microbatch_size must be >= 1");
   HM_CHECK(c.precision == HARMONY_FP32 || c.precision == HARMONY_BF16_FP32MASTER, HARMONY_E_INVALID_ARG,
            "unknown precision");
-  HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP || c.schedule == HARMONY_SCHED_PER_GPU_VIRT, HARMONY_E_INVALID_ARG,
-           "unknown schedule");
+  HM_CHECK(c.schedule == HARMONY_SCHED_HARMONY_DP || c.schedule == HARMONY_SCHED_PER_GPU_VIRT ||
+               c.schedule == HARMONY_SCHED_HARMONY_PP,
+           HARMONY_E_INVALID_ARG, "unknown schedule");
   HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 3, HARMONY_E_INVALID_ARG, "stash_policy must be 0..3");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
 }
 
-static void validate_layers(const harmony_config& c, int n, const harmony_layer_desc* d) {
+static void validate_layers(const harmony_config& c, int n, const harmony_layer_desc* d, bool chain = true) {
   HM_CHECK(n >= 1 && d != nullptr, HARMONY_E_INVALID_ARG, "need >= 1 layer");
   for (int l = 0; l < n; ++l) {
     const harmony_layer_desc& x = d[l];
@@ -52,7 +53,7 @@ static void validate_layers(const harmony_config& c, int n, const harmony_layer_
       HM_CHECK(false, HARMONY_E_INVALID_ARG, "unknown layer kind");
     }
     if (l > 0) {
-      HM_CHECK(d[l - 1].d_out == x.d_in, HARMONY_E_INVALID_ARG, "layer widths do not chain");
+      HM_CHECK(!chain || d[l - 1].d_out == x.d_in, HARMONY_E_INVALID_ARG, "layer widths do not chain");
       HM_CHECK(d[l - 1].kind == x.kind, HARMONY_E_UNSUPPORTED, "mixed layer kinds in one stack");
       if (x.kind == HARMONY_LAYER_TRANSFORMER)
         HM_CHECK(d[l - 1].seq_len == x.seq_len, HARMONY_E_INVALID_ARG, "seq_len must match across layers");
@@ -248,10 +249,14 @@ int validate_program(const Plan& p, std::string* first) {
 }
 
 // ------------------------------------------------------------------------------------ make_plan
-Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs) {
+Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs, bool layout_only,
+               int n_bnd) {
   validate_config(cfg);
-  validate_layers(cfg, n_layers, descs);
+  validate_layers(cfg, n_layers, descs, !layout_only);
+  HM_CHECK(cfg.schedule != HARMONY_SCHED_HARMONY_PP, HARMONY_E_UNSUPPORTED,
+           "Harmony-PP is planned for a group of ranks (harmony_init_group / harmony_plan_dry_group)");
   Plan p;
+  p.n_bnd = n_bnd;
   p.N = cfg.world_size;
   p.rank = cfg.rank;
   p.m = cfg.microbatches;
@@ -295,7 +300,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   const int nDW = N > 1 ? 2 : 1;
   auto fixed_bytes = [&]() {
     uint64_t f = 0;
-    f += 2 * bnd_stride * m;                          // activation / gradient ping-pong
+    f += (uint64_t)p.n_bnd * bnd_stride * m;          // activation / gradient buffers
     f += tgt_stride * m;                              // targets
     f += align_up(ws_need, ALIGN);                    // one task's transients
     f += nDW * align_up(maxP * 4, ALIGN);             // fp32 dW accumulators
@@ -462,8 +467,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   p.bnd_row_stride = bnd_stride;
   p.tgt_row_stride = tgt_stride;
   p.bnd_bytes = bnd_stride * m;
-  p.bnd[0] = a.take(p.bnd_bytes);
-  p.bnd[1] = a.take(p.bnd_bytes);
+  for (int j = 0; j < p.n_bnd; ++j) p.bnd[j] = a.take(p.bnd_bytes);
   p.tgt = a.take(tgt_stride * m);
   p.ws_bytes = ws_need;
   p.ws = a.take(ws_need);
@@ -484,6 +488,14 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
       if (p.layers[l].stash_res[i] >= 0) p.layers[l].stash_res[i] = (int64_t)a.take(p.layers[l].g.st.total);
   p.arena_bytes = a.cur;
   HM_CHECK(uncapped || p.arena_bytes <= p.cap, HARMONY_E_CAP_TOO_SMALL, "internal: arena layout exceeds the cap");
+  if (layout_only) {
+    harmony_plan_summary& s = p.summary;
+    s.arena_bytes = p.arena_bytes;
+    s.min_working_set_bytes = p.min_ws_bytes;
+    s.n_params = p.n_params;
+    s.weight_slots = nW; s.state_slots = nS; s.stash_slots = nG;
+    return p;
+  }
 
   // ---------------------------------------------------------------- program
   Tracker tr;
@@ -858,6 +870,432 @@ std::string dump_plan(const Plan& p) {
     os << i << " " << kn[o.kind] << " " << sn[o.stream] << " cat=" << cn[o.cat] << " l=" << o.layer << " i=" << o.mb
        << " bytes=" << o.bytes;
     if (o.kind == OP_BWD) os << " first=" << o.first;
+    os << " waits=";
+    for (size_t k = 0; k < o.waits.size(); ++k) os << (k ? "," : "") << o.waits[k];
+    os << "\n";
+  }
+  return os.str();
+}
+
+
+// ------------------------------------------------------------------------------------ Harmony-PP
+namespace {
+// resource keys of one rank (bits 48..55 = rank; key() keeps a < 2^20, b < 2^28)
+inline uint64_t rkey(int rank, ResKind k, uint64_t a, uint64_t b = 0) { return key(k, a, b) | ((uint64_t)rank << 48); }
+
+struct GTracker {
+  int N;
+  std::unordered_map<uint64_t, Tracker::Res> res;
+  std::vector<GOp>* ops;
+  int add(int rank, Op op, const std::vector<uint64_t>& reads, const std::vector<uint64_t>& writes) {
+    const int idx = (int)ops->size();
+    std::vector<int> deps;
+    for (uint64_t r : reads) {
+      auto it = res.find(r);
+      if (it != res.end() && it->second.writer >= 0) deps.push_back(it->second.writer);
+    }
+    for (uint64_t w : writes) {
+      auto it = res.find(w);
+      if (it == res.end()) continue;
+      if (it->second.writer >= 0) deps.push_back(it->second.writer);
+      for (int rd : it->second.readers) deps.push_back(rd);
+    }
+    // the latest dependency per other (rank, stream): each stream executes in order
+    std::map<int, int> latest;
+    const int self = rank * S_NUM + op.stream;
+    for (int d : deps) {
+      const int s = (*ops)[d].rank * S_NUM + (*ops)[d].op.stream;
+      if (s != self) latest[s] = std::max(latest.count(s) ? latest[s] : -1, d);
+    }
+    op.waits.clear();
+    for (auto& kv : latest) op.waits.push_back(kv.second);
+    for (uint64_t r : reads) res[r].readers.push_back(idx);
+    for (uint64_t w : writes) {
+      Tracker::Res& x = res[w];
+      x.writer = idx;
+      x.readers.clear();
+    }
+    ops->push_back(GOp{rank, op});
+    return idx;
+  }
+};
+
+// The independent race check of validate_program over the whole group: per-rank arenas and host
+// stores are separate address spaces; happens-before over every (rank, stream).
+int validate_group(const GroupPlan& g, std::string* first) {
+  const size_t n = g.ops.size();
+  const int NS = g.N * S_NUM;
+  std::vector<std::vector<int>> vc(n, std::vector<int>(NS, -1));
+  std::vector<int> pos(n), cnt(NS, 0), last(NS, -1);
+  auto sid = [&](size_t i) { return g.ops[i].rank * S_NUM + g.ops[i].op.stream; };
+  for (size_t i = 0; i < n; ++i) {
+    const int s = sid(i);
+    std::vector<int> c(NS, -1);
+    if (last[s] >= 0) c = vc[last[s]];
+    for (int w : g.ops[i].op.waits)
+      for (int k = 0; k < NS; ++k) c[k] = std::max(c[k], vc[w][k]);
+    pos[i] = cnt[s]++;
+    c[s] = pos[i];
+    vc[i] = c;
+    last[s] = (int)i;
+  }
+  auto hb = [&](size_t a, size_t b) { return vc[b][sid(a)] >= pos[a]; };
+  std::vector<std::vector<Acc>> acc(n);
+  for (size_t i = 0; i < n; ++i) {
+    const GOp& o = g.ops[i];
+    if (o.op.kind == OP_P2P) {
+      acc[i].push_back({16 * o.rank, 0, o.op.dev, o.op.dev + o.op.bytes, true});
+      acc[i].push_back({16 * o.op.peer, 0, o.op.peer_off, o.op.peer_off + o.op.bytes, false});
+      continue;
+    }
+    for (Acc a : accesses(g.ranks[o.rank], o.op)) {
+      a.space += 16 * o.rank;
+      acc[i].push_back(a);
+    }
+  }
+  int hazards = 0;
+  for (size_t j = 0; j < n; ++j)
+    for (size_t i = 0; i < j; ++i) {
+      if (sid(i) == sid(j) || hb(i, j)) continue;
+      for (const Acc& a : acc[i])
+        for (const Acc& b : acc[j])
+          if ((a.write || b.write) && a.space == b.space && a.idx == b.idx && a.lo < b.hi && b.lo < a.hi) {
+            if (hazards == 0 && first)
+              *first = "ops " + std::to_string(i) + " and " + std::to_string(j) + " race on space " +
+                       std::to_string(a.space) + "[" + std::to_string(a.idx) + "]";
+            ++hazards;
+            goto next_pair;
+          }
+    next_pair:;
+    }
+  return hazards;
+}
+}  // namespace
+
+GroupPlan make_plan_pp(const harmony_config& cfg, int N, int L, const harmony_layer_desc* descs) {
+  validate_config(cfg);
+  validate_layers(cfg, L, descs);
+  HM_CHECK(N >= 2 && N <= 16, HARMONY_E_INVALID_ARG, "Harmony-PP needs a group of 2..16 ranks");
+  HM_CHECK(L >= N, HARMONY_E_INVALID_ARG, "Harmony-PP needs at least as many layers as ranks");
+  GroupPlan G;
+  G.N = N;
+  G.layer_rank.resize(L);
+  G.layer_local.resize(L);
+  for (int l = 0; l < L; ++l) { G.layer_rank[l] = l % N; G.layer_local[l] = l / N; }
+  // per-rank layout: the rank's layers as one stack of one rank (the update is not sharded: each layer
+  // lives on one GPU), four activation buffers (A_in, A_out, G_in, G_out)
+  harmony_config rc = cfg;
+  rc.world_size = 1; rc.rank = 0; rc.schedule = HARMONY_SCHED_HARMONY_DP;
+  for (int r = 0; r < N; ++r) {
+    std::vector<harmony_layer_desc> sub;
+    for (int l = r; l < L; l += N) sub.push_back(descs[l]);
+    G.ranks.push_back(make_plan(rc, (int)sub.size(), sub.data(), /*layout_only=*/true, /*n_bnd=*/4));
+  }
+  const int m = cfg.microbatches;
+  const uint64_t ts = cfg.precision == HARMONY_BF16_FP32MASTER ? 2 : 4;
+  GTracker tr{N, {}, &G.ops};
+  auto row = [&](int r, int buf, int i) { return G.ranks[r].bnd[buf] + (uint64_t)i * G.ranks[r].bnd_row_stride; };
+  enum { A_IN = 0, A_OUT = 1, G_IN = 2, G_OUT = 3 };
+
+  struct Rec { int rank; Op op; std::vector<uint64_t> rd, wr; };
+  struct Item { int need = 0, release = -1; std::vector<Rec> ops; };
+  struct Task { Rec t; std::vector<Rec> post; };
+  std::vector<Task> tasks;
+  std::vector<Item> items;
+  struct Slots { std::vector<int> wlast, slast, glast; int wn = 0, sn = 0, gn = 0; };
+  std::vector<Slots> sl(N);
+  for (int r = 0; r < N; ++r) {
+    sl[r].wlast.assign(G.ranks[r].wslot.size(), -1);
+    sl[r].slast.assign(G.ranks[r].sslot.size(), -1);
+    sl[r].glast.assign(G.ranks[r].stage.size(), -1);
+  }
+  auto weight_use = [&](int r, int k, int need, int& slot) -> uint64_t {
+    Plan& P = G.ranks[r];
+    LayerPlan& lp = P.layers[k];
+    if (lp.wc_res >= 0) { slot = -1; return (uint64_t)lp.wc_res; }
+    Slots& S = sl[r];
+    slot = S.wn;
+    S.wn = (S.wn + 1) % (int)P.wslot.size();
+    Item it;
+    it.need = need;
+    it.release = S.wlast[slot];
+    Op h;
+    h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_WEIGHT; h.layer = k;
+    h.hbuf = HB_WC; h.hidx = k; h.dev = P.wslot[slot]; h.bytes = (uint64_t)lp.shard * ts;
+    it.ops.push_back({r, h, {rkey(r, H_WC, k)}, {rkey(r, R_WSLOT, slot)}});
+    items.push_back(it);
+    return P.wslot[slot];
+  };
+  auto wkey = [&](int r, int k, int slot) { return slot >= 0 ? rkey(r, R_WSLOT, slot) : rkey(r, R_WRES, k); };
+
+  // ---- forward: layer by layer, each layer's m microbatches back to back on its rank (grouping)
+  std::vector<int> fwd_slot(L, -1), spill_task((size_t)L * m, -1);
+  for (int l = 0; l < L; ++l) {
+    const int r = G.layer_rank[l], k = G.layer_local[l];
+    Plan& P = G.ranks[r];
+    LayerPlan& lp = P.layers[k];
+    for (int i = 0; i < m; ++i) {
+      int slot = fwd_slot[l];
+      uint64_t w;
+      if (i == 0) { w = weight_use(r, k, (int)tasks.size(), slot); fwd_slot[l] = slot; }
+      else w = slot >= 0 ? P.wslot[slot] : (uint64_t)lp.wc_res;
+      Task t;
+      t.t.rank = r;
+      Op& o = t.t.op;
+      o.kind = OP_FWD; o.stream = S_COMPUTE; o.layer = k; o.mb = i;
+      o.w = w; o.in = row(r, A_IN, i); o.out = row(r, A_OUT, i); o.ws = P.ws;
+      t.t.rd = {wkey(r, k, slot), rkey(r, R_BND, A_IN, i)};
+      t.t.wr = {rkey(r, R_BND, A_OUT, i)};
+      if (lp.stash_res[i] >= 0) {
+        o.stash = (uint64_t)lp.stash_res[i];
+        t.t.wr.push_back(rkey(r, R_STASHRES, k, i));
+      } else {
+        Slots& S = sl[r];
+        const int gq = S.gn;
+        S.gn = (S.gn + 1) % (int)P.stage.size();
+        o.stash = P.stage[gq];
+        t.t.wr.push_back(rkey(r, R_STAGE, gq));
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = k; d.mb = i;
+        d.hbuf = HB_STASH; d.hidx = (int64_t)k * m + i; d.dev = P.stage[gq]; d.bytes = lp.g.st.total;
+        t.post.push_back({r, d, {rkey(r, R_STAGE, gq)}, {rkey(r, H_STASH, k, i)}});
+        S.glast[gq] = (int)tasks.size();
+        spill_task[(size_t)l * m + i] = (int)tasks.size();
+      }
+      if (slot >= 0) sl[r].wlast[slot] = (int)tasks.size();
+      if (l + 1 < L) {  // hand the activation rows to the next layer's rank, peer to peer
+        const int r2 = G.layer_rank[l + 1];
+        Op x;
+        x.kind = OP_P2P; x.stream = S_COMM; x.cat = CAT_NONE; x.layer = G.layer_local[l + 1]; x.mb = i;
+        x.dev = row(r2, A_IN, i); x.peer = r; x.peer_off = row(r, A_OUT, i);
+        x.bytes = (uint64_t)lp.g.rows * lp.g.desc.d_out * 4;
+        t.post.push_back({r2, x, {rkey(r, R_BND, A_OUT, i)}, {rkey(r2, R_BND, A_IN, i)}});
+      }
+      tasks.push_back(t);
+    }
+  }
+  // ---- loss on the last layer's rank: dY of the last layer into its incoming-gradient rows
+  const int rl = G.layer_rank[L - 1];
+  {
+    Plan& P = G.ranks[rl];
+    for (int i = 0; i < m; ++i) {
+      Task t;
+      t.t.rank = rl;
+      Op& o = t.t.op;
+      o.kind = OP_LOSS; o.stream = S_COMPUTE; o.mb = i;
+      o.in = row(rl, A_OUT, i); o.tgt = P.tgt + (uint64_t)i * P.tgt_row_stride; o.out = row(rl, G_IN, i);
+      o.loss = P.loss + (uint64_t)i * 8;
+      t.t.rd = {rkey(rl, R_BND, A_OUT, i), rkey(rl, R_TGT, i)};
+      t.t.wr = {rkey(rl, R_BND, G_IN, i), rkey(rl, R_LOSS, i)};
+      if (i == m - 1) {
+        Op d;
+        d.kind = OP_LOSS_OUT; d.stream = S_D2H; d.cat = CAT_OUTPUT; d.dev = P.loss; d.bytes = (uint64_t)m * 8;
+        std::vector<uint64_t> rds;
+        for (int j = 0; j < m; ++j) rds.push_back(rkey(rl, R_LOSS, j));
+        t.post.push_back({rl, d, rds, {}});
+      }
+      tasks.push_back(t);
+    }
+  }
+  // ---- backward (reverse layers, grouped) + JIT update of each layer right after its group
+  std::vector<int> bwd_slot(L, -1);
+  for (int l = L - 1; l >= 0; --l) {
+    const int r = G.layer_rank[l], k = G.layer_local[l];
+    Plan& P = G.ranks[r];
+    LayerPlan& lp = P.layers[k];
+    for (int i = 0; i < m; ++i) {
+      int slot = bwd_slot[l];
+      uint64_t w;
+      if (i == 0) { w = weight_use(r, k, (int)tasks.size(), slot); bwd_slot[l] = slot; }
+      else w = slot >= 0 ? P.wslot[slot] : (uint64_t)lp.wc_res;
+      Task t;
+      t.t.rank = r;
+      Op& o = t.t.op;
+      o.kind = OP_BWD; o.stream = S_COMPUTE; o.layer = k; o.mb = i; o.first = i == 0;
+      o.w = w; o.in = row(r, G_IN, i); o.out = row(r, G_OUT, i); o.ws = P.ws; o.dw = P.dw[0];
+      t.t.rd = {wkey(r, k, slot), rkey(r, R_BND, G_IN, i)};
+      t.t.wr = {rkey(r, R_BND, G_OUT, i), rkey(r, R_DW, 0)};
+      if (i > 0) t.t.rd.push_back(rkey(r, R_DW, 0));
+      if (lp.stash_res[i] >= 0) {
+        o.stash = (uint64_t)lp.stash_res[i];
+        t.t.rd.push_back(rkey(r, R_STASHRES, k, i));
+      } else {
+        Slots& S = sl[r];
+        const int gq = S.gn;
+        S.gn = (S.gn + 1) % (int)P.stage.size();
+        Item it;
+        it.need = (int)tasks.size();
+        it.release = std::max(S.glast[gq], spill_task[(size_t)l * m + i]);
+        Op h;
+        h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STASH; h.layer = k; h.mb = i;
+        h.hbuf = HB_STASH; h.hidx = (int64_t)k * m + i; h.dev = P.stage[gq]; h.bytes = lp.g.st.total;
+        it.ops.push_back({r, h, {rkey(r, H_STASH, k, i)}, {rkey(r, R_STAGE, gq)}});
+        items.push_back(it);
+        o.stash = P.stage[gq];
+        t.t.rd.push_back(rkey(r, R_STAGE, gq));
+        S.glast[gq] = (int)tasks.size();
+      }
+      if (slot >= 0) sl[r].wlast[slot] = (int)tasks.size();
+      if (l > 0) {  // the input gradient to the previous layer's rank
+        const int r2 = G.layer_rank[l - 1];
+        Op x;
+        x.kind = OP_P2P; x.stream = S_COMM; x.cat = CAT_NONE; x.layer = G.layer_local[l - 1]; x.mb = i;
+        x.dev = row(r2, G_IN, i); x.peer = r; x.peer_off = row(r, G_OUT, i);
+        x.bytes = (uint64_t)lp.g.rows * lp.g.desc.d_in * 4;
+        t.post.push_back({r2, x, {rkey(r, R_BND, G_OUT, i)}, {rkey(r2, R_BND, G_IN, i)}});
+      }
+      tasks.push_back(t);
+    }
+    // UPD(l) just in time: dW is this rank's whole (unsharded) accumulator
+    Task t;
+    t.t.rank = r;
+    Op& o = t.t.op;
+    o.kind = OP_UPD; o.stream = S_COMPUTE; o.layer = k; o.grad = P.dw[0];
+    t.t.rd = {rkey(r, R_DW, 0)};
+    if (lp.state_res >= 0) {
+      o.state = (uint64_t)lp.state_res;
+      t.t.rd.push_back(rkey(r, R_SRES, k));
+      t.t.wr.push_back(rkey(r, R_SRES, k));
+    } else {
+      Slots& S = sl[r];
+      const int ss = S.sn;
+      S.sn = (S.sn + 1) % (int)P.sslot.size();
+      Item it;
+      it.need = (int)tasks.size();
+      it.release = S.slast[ss];
+      Op h;
+      h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STATE; h.layer = k;
+      h.hbuf = HB_STATE; h.hidx = k; h.dev = P.sslot[ss]; h.bytes = lp.state_bytes;
+      it.ops.push_back({r, h, {rkey(r, H_STATE, k)}, {rkey(r, R_SSLOT, ss)}});
+      items.push_back(it);
+      o.state = P.sslot[ss];
+      t.t.rd.push_back(rkey(r, R_SSLOT, ss));
+      t.t.wr.push_back(rkey(r, R_SSLOT, ss));
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STATE; d.layer = k;
+      d.hbuf = HB_STATE; d.hidx = k; d.dev = P.sslot[ss]; d.bytes = lp.state_bytes;
+      t.post.push_back({r, d, {rkey(r, R_SSLOT, ss)}, {rkey(r, H_STATE, k)}});
+      S.slast[ss] = (int)tasks.size();
+    }
+    const int ws = bwd_slot[l];
+    if (lp.wc_res >= 0) {
+      o.w = (uint64_t)lp.wc_res;
+      t.t.wr.push_back(rkey(r, R_WRES, k));
+    } else {
+      o.w = P.wslot[ws];
+      t.t.wr.push_back(rkey(r, R_WSLOT, ws));
+      Op d;  // the updated compute copy out once (the third |W| of P:773-775)
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = k;
+      d.hbuf = HB_WC; d.hidx = k; d.dev = P.wslot[ws]; d.bytes = (uint64_t)lp.shard * ts;
+      t.post.push_back({r, d, {rkey(r, R_WSLOT, ws)}, {rkey(r, H_WC, k)}});
+      sl[r].wlast[ws] = (int)tasks.size();
+    }
+    if (P.retain_grads) {
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_GRAD; d.layer = k;
+      d.hbuf = HB_GRAD; d.hidx = k; d.dev = P.dw[0]; d.bytes = (uint64_t)lp.shard * 4;
+      t.post.push_back({r, d, {rkey(r, R_DW, 0)}, {rkey(r, H_GRAD, k)}});
+    }
+    tasks.push_back(t);
+  }
+
+  // ---- one program: inputs, then tasks with their prefetch items merged by need
+  {
+    Plan& P0 = G.ranks[0];
+    for (int i = 0; i < m; ++i) {
+      Op x;
+      x.kind = OP_INPUT; x.stream = S_H2D; x.cat = CAT_INPUT; x.hbuf = HB_USER_X; x.mb = i;
+      x.dev = row(0, A_IN, i); x.hoff = (uint64_t)i * P0.in_elems_per_mb * 4; x.bytes = (uint64_t)P0.in_elems_per_mb * 4;
+      tr.add(0, x, {}, {rkey(0, R_BND, A_IN, i)});
+    }
+    Plan& PL = G.ranks[rl];
+    for (int i = 0; i < m; ++i) {
+      Op x;
+      x.kind = OP_INPUT; x.stream = S_H2D; x.cat = CAT_INPUT; x.hbuf = HB_USER_T; x.mb = i;
+      x.dev = PL.tgt + (uint64_t)i * PL.tgt_row_stride; x.hoff = (uint64_t)i * PL.out_elems_per_mb * 4;
+      x.bytes = (uint64_t)PL.out_elems_per_mb * 4;
+      tr.add(rl, x, {}, {rkey(rl, R_TGT, i)});
+    }
+    std::stable_sort(items.begin(), items.end(), [](const Item& a, const Item& b) { return a.need < b.need; });
+    size_t next = 0;
+    auto emit = [&](Item& it) {
+      for (auto& x : it.ops) tr.add(x.rank, x.op, x.rd, x.wr);
+    };
+    for (int k = 0; k < (int)tasks.size(); ++k) {
+      while (next < items.size() && items[next].need <= k) emit(items[next++]);
+      Task& t = tasks[k];
+      tr.add(t.t.rank, t.t.op, t.t.rd, t.t.wr);
+      for (auto& x : t.post) tr.add(x.rank, x.op, x.rd, x.wr);
+      while (next < items.size() && items[next].release <= k) emit(items[next++]);
+    }
+    while (next < items.size()) emit(items[next++]);
+  }
+  {  // events: one per op another stream waits on (owned by the op's rank)
+    std::vector<int> ev(G.ops.size(), -1);
+    int ne = 0;
+    for (auto& o : G.ops)
+      for (int w : o.op.waits)
+        if (ev[w] < 0) ev[w] = ne++;
+    for (size_t i = 0; i < G.ops.size(); ++i) G.ops[i].op.event = ev[i];
+    G.n_events = ne;
+  }
+  // ---- box summary
+  harmony_plan_summary& s = G.summary;
+  double fl = 0;
+  for (auto& P : G.ranks) {
+    s.arena_bytes = std::max(s.arena_bytes, P.arena_bytes);
+    s.min_working_set_bytes = std::max(s.min_working_set_bytes, P.min_ws_bytes);
+    s.weight_slots = std::max(s.weight_slots, (int32_t)P.wslot.size());
+    s.state_slots = std::max(s.state_slots, (int32_t)P.sslot.size());
+    s.stash_slots = std::max(s.stash_slots, (int32_t)P.stage.size());
+    s.n_params += P.n_params;
+    for (auto& lp : P.layers) {
+      s.total_weight_bytes += lp.wc_bytes;
+      s.total_state_bytes += lp.state_bytes;
+      s.total_stash_bytes += (uint64_t)m * lp.g.st.total;
+      if (lp.wc_res >= 0) s.resident_weight_bytes += lp.wc_bytes;
+      if (lp.state_res >= 0) s.resident_state_bytes += lp.state_bytes;
+      for (int i = 0; i < m; ++i)
+        if (lp.stash_res[i] >= 0) s.resident_stash_bytes += lp.g.st.total;
+      fl += 3.0 * lp.g.flops_fwd * m;
+    }
+  }
+  s.flops_per_step = (uint64_t)fl;
+  for (auto& g : G.ops) {
+    const Op& o = g.op;
+    const bool in = o.kind == OP_H2D || o.kind == OP_INPUT, out = o.kind == OP_D2H || o.kind == OP_LOSS_OUT;
+    if (in) s.pred_h2d_bytes += o.bytes;
+    if (out) s.pred_d2h_bytes += o.bytes;
+    if (in && o.cat == CAT_WEIGHT) s.pred_h2d_weight_bytes += o.bytes;
+    if (out && o.cat == CAT_WEIGHT) s.pred_d2h_weight_bytes += o.bytes;
+    if (o.stream == S_COMPUTE) s.n_compute_ops++;
+    else if (o.stream == S_COMM) s.n_comm_ops++;
+    else s.n_copy_ops++;
+  }
+  s.n_ops = (int32_t)G.ops.size();
+  std::string why;
+  s.hazards = validate_group(G, &why);
+  G.hazard_msg = why;
+  return G;
+}
+
+std::string dump_group_plan(const GroupPlan& g) {
+  static const char* kn[] = {"INPUT", "H2D", "D2H", "FWD", "LOSS", "BWD", "UPD", "ALLGATHER", "REDUCESCATTER",
+                             "LOSS_GATHER", "LOSS_OUT", "P2P"};
+  static const char* sn[] = {"compute", "h2d", "d2h", "comm"};
+  static const char* cn[] = {"weight", "state", "stash", "input", "output", "grad", "-"};
+  std::ostringstream os;
+  os << "# group plan N=" << g.N << " ops=" << g.ops.size() << " events=" << g.n_events << "\n";
+  std::vector<std::vector<int>> glob(g.N);  // local layer -> global layer
+  for (size_t l = 0; l < g.layer_rank.size(); ++l) glob[g.layer_rank[l]].push_back((int)l);
+  for (size_t i = 0; i < g.ops.size(); ++i) {
+    const GOp& x = g.ops[i];
+    const Op& o = x.op;
+    const int gl = o.layer >= 0 && o.kind != OP_P2P ? glob[x.rank][o.layer]
+                   : o.kind == OP_P2P ? glob[x.rank][o.layer] : -1;
+    os << i << " " << kn[o.kind] << " " << sn[o.stream] << " rank=" << x.rank << " cat=" << cn[o.cat]
+       << " l=" << gl << " i=" << o.mb << " bytes=" << o.bytes;
+    if (o.kind == OP_P2P) os << " peer=" << o.peer;
     os << " waits=";
     for (size_t k = 0; k < o.waits.size(); ++k) os << (k ? "," : "") << o.waits[k];
     os << "\n";

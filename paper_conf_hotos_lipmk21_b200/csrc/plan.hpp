@@ -31,7 +31,8 @@ enum OpKind {
   OP_ALLGATHER = 7,      // in-place all-gather of a layer's shards (weights)
   OP_REDUCESCATTER = 8,  // dW -> this rank's summed shard
   OP_LOSS_GATHER = 9,    // all-gather of every rank's per-microbatch loss partials
-  OP_LOSS_OUT = 10       // loss partials -> host
+  OP_LOSS_OUT = 10,      // loss partials -> host
+  OP_P2P = 11            // Harmony-PP: a peer rank's arena -> this rank's arena (activation / gradient hand-off)
 };
 enum Cat { CAT_WEIGHT = 0, CAT_STATE = 1, CAT_STASH = 2, CAT_INPUT = 3, CAT_OUTPUT = 4, CAT_GRAD = 5, CAT_NONE = 6 };
 enum HostBuf { HB_NONE = -1, HB_WC = 0, HB_STATE = 1, HB_STASH = 2, HB_USER_X = 3, HB_USER_T = 4, HB_GRAD = 5 };
@@ -47,6 +48,8 @@ struct Op {
   // compute operands: arena byte offsets
   uint64_t w = 0, in = 0, out = 0, stash = 0, ws = 0, dw = 0, state = 0, grad = 0, tgt = 0, loss = 0;
   uint64_t count = 0;  // collectives: elements per rank
+  int peer = -1;       // OP_P2P: source rank; peer_off: byte offset in its arena
+  uint64_t peer_off = 0;
   std::vector<int> waits;  // ops on other streams this op waits for
   int event = -1;          // event slot recorded after this op
 };
@@ -67,7 +70,10 @@ struct Plan {
   std::vector<LayerPlan> layers;
   // arena layout
   uint64_t arena_bytes = 0, min_ws_bytes = 0;
-  uint64_t bnd[2] = {0, 0}, bnd_bytes = 0, bnd_row_stride = 0;  // fp32 activation ping-pong; per-microbatch stride
+  // fp32 activation / gradient buffers of m microbatch rows each: [0], [1] the ping-pong of the DP step;
+  // Harmony-PP uses four (layer input, layer output, incoming gradient, outgoing gradient)
+  uint64_t bnd[4] = {0, 0, 0, 0}, bnd_bytes = 0, bnd_row_stride = 0;
+  int n_bnd = 2;
   uint64_t tgt = 0, tgt_row_stride = 0;
   uint64_t ws = 0, ws_bytes = 0;
   uint64_t dw[2] = {0, 0};
@@ -86,7 +92,31 @@ struct Plan {
 };
 
 // Throws hm::Error (HARMONY_E_INVALID_ARG / UNSUPPORTED / CAP_TOO_SMALL).
-Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs);
+// layout_only: residency, slots and arena layout for a sub-stack (Harmony-PP: one rank's layers,
+// which need not chain), with n_bnd activation buffers, and no program.
+Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs, bool layout_only = false,
+               int n_bnd = 2);
+
+// ---- Harmony-PP (Fig. 4; reading c27): layer l runs on rank l % N;
+// every layer-level task runs its group of m microbatches back to back; activations (forward) and
+// gradients (backward) are handed to the next rank peer to peer; each layer's weights are swapped in
+// once for its forward group and once for its backward group and out once after its JIT update.
+// One program for the whole group: ops tagged with their rank, waits are global op indices.
+struct GOp {
+  int rank = 0;
+  Op op;  // op.waits: indices into GroupPlan::ops; op.event: event slot of op.rank's context
+};
+struct GroupPlan {
+  int N = 1;
+  std::vector<Plan> ranks;                  // per-rank layout (local layers; their own ops unused)
+  std::vector<int> layer_rank, layer_local;  // global layer -> (rank, local index)
+  std::vector<GOp> ops;
+  int n_events = 0;
+  harmony_plan_summary summary{};           // box totals (bytes summed over ranks, arena = max)
+  std::string hazard_msg;
+};
+GroupPlan make_plan_pp(const harmony_config& cfg, int num_ranks, int n_layers, const harmony_layer_desc* descs);
+std::string dump_group_plan(const GroupPlan& g);
 std::string dump_plan(const Plan& p);
 void validate_config(const harmony_config& cfg);
 int validate_program(const Plan& p, std::string* first);

@@ -22,7 +22,7 @@ HARMONY_FP32, HARMONY_BF16_FP32MASTER = 0, 1
 HARMONY_LAYER_MLP, HARMONY_LAYER_TRANSFORMER = 0, 1
 HARMONY_ACT_NONE, HARMONY_ACT_RELU, HARMONY_ACT_GELU_TANH = 0, 1, 2
 HARMONY_PARAM, HARMONY_GRAD, HARMONY_ADAM_M, HARMONY_ADAM_V = 0, 1, 2, 3
-HARMONY_SCHED_HARMONY_DP, HARMONY_SCHED_PER_GPU_VIRT = 0, 1
+HARMONY_SCHED_HARMONY_DP, HARMONY_SCHED_PER_GPU_VIRT, HARMONY_SCHED_HARMONY_PP = 0, 1, 2
 HK_EPI_STORE_T, HK_EPI_STORE_F32, HK_EPI_RESID_F32, HK_EPI_ACC_F32 = 0, 1, 2, 3
 HK_EPI_BIAS_ACT, HK_EPI_ACT_BWD, HK_EPI_BIAS_ACT_F32, HK_EPI_ACT_T = 4, 5, 6, 7
 
@@ -135,6 +135,8 @@ def lib() -> C.CDLL:
         "harmony_init": (st, [C.POINTER(harmony_config), C.POINTER(P)]),
         "harmony_init_group": (st, [C.POINTER(harmony_config), C.c_int32, P, C.POINTER(P)]),
         "harmony_read_rank_stats": (st, [P, C.c_int32, C.POINTER(harmony_step_stats)]),
+        "harmony_plan_dry_group": (st, [C.POINTER(harmony_config), C.c_int32, C.c_int32, C.POINTER(harmony_layer_desc),
+                                        C.POINTER(harmony_plan_summary), P, C.c_uint64]),
         "harmony_register_layers": (st, [P, C.c_int32, C.POINTER(harmony_layer_desc), C.POINTER(P)]),
         "harmony_step": (st, [P, P, P, C.c_int64, C.POINTER(C.c_double), C.POINTER(harmony_step_stats)]),
         "harmony_read_state": (st, [P, C.c_int32, C.c_int32, P, C.c_uint64]),
@@ -292,6 +294,14 @@ def harmony_plan_dry(cfg, descs, text_len=1 << 22):
     return s, (buf.value.decode() if buf is not None else "")
 
 
+def harmony_plan_dry_group(cfg, num_ranks, descs, text_len=1 << 22):
+    s = harmony_plan_summary()
+    buf = C.create_string_buffer(text_len) if text_len else None
+    _check(lib().harmony_plan_dry_group(C.byref(cfg), int(num_ranks), len(descs), make_descs(descs), C.byref(s), buf,
+                                        text_len))
+    return s, (buf.value.decode() if buf is not None else "")
+
+
 def harmony_set_profiling(ctx, on):
     _check(lib().harmony_set_profiling(ctx, int(on)), ctx)
 
@@ -405,8 +415,10 @@ class Harmony:
         self.n_params = [int(np.asarray(p).size) for p in init_params]
 
     def step(self, x, target):
-        """x, target: this rank's rows (a group: the global batch of ranks*m*b rows)."""
-        return harmony_step(self.ctx, x, target, self.ranks * self.cfg.microbatches * self.cfg.microbatch_size)
+        """x, target: this rank's rows (a data-parallel group: the global batch of ranks*m*b rows; Harmony-PP:
+        the one minibatch of m*b rows that flows through the ranks)."""
+        mult = 1 if self.cfg.schedule == HARMONY_SCHED_HARMONY_PP else self.ranks
+        return harmony_step(self.ctx, x, target, mult * self.cfg.microbatches * self.cfg.microbatch_size)
 
     def rank_stats(self, rank):
         return harmony_read_rank_stats(self.ctx, rank)
