@@ -6,7 +6,7 @@ import numpy as np
 import pytest
 
 import synth
-from test_gpu_step import CFG1, batches_for, bitwise_equal, compare, run_gpu, run_oracle, tiny_transformer
+from test_gpu_step import batches_for, bitwise_equal, compare, run_gpu, run_oracle, tiny_transformer
 
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
@@ -22,7 +22,7 @@ def pp_cap(descs, N, **kw):
 
 @pytest.mark.parametrize("N", [2, 4])
 def test_pp_mlp_fp32_matches_oracle_and_is_bitwise_the_single_rank_step(N):
-    descs = synth.mlp_stack(4, 256)
+    descs = synth.mlp_stack(8, 256)  # two or more layers per rank, so a capped rank must stream
     params = synth.gen_params(descs)
     m, b = 4, 8
     batches = batches_for(descs, m * b, 3, 0)
@@ -32,7 +32,7 @@ def test_pp_mlp_fp32_matches_oracle_and_is_bitwise_the_single_rank_step(N):
     st = pp[-1]["stats"]
     assert st["nvlink_bytes"] > 0 and st["h2d_weight_bytes"] > 0
     compare(pp, run_oracle(descs, params, batches), 1e-5)
-    dp, _ = run_gpu(descs, params, batches, hbm_cap_bytes=CFG1["cap"], **kw)
+    dp, _ = run_gpu(descs, params, batches, hbm_cap_bytes=0, **kw)
     bitwise_equal(pp, dp)
     unc, _ = run_gpu(descs, params, batches, group=[0] * N, schedule=PP, hbm_cap_bytes=0, **kw)
     bitwise_equal(pp, unc)
