@@ -191,6 +191,9 @@ struct TcParams {
   int M, N, K, nz0, nz, a_mn, b_mn;
   int tma_epi;  // 1: epilogue through shared-memory staging + TMA stores (maps tmC / tmIn / tmO2)
   int group_m;  // tile raster: GROUP_M consecutive m-tiles per n sweep (order only; results unchanged)
+  int diag;     // experiments only (HARMONY_GEMM_DIAG): bit 0 = epilogue warps drain nothing (timing of the
+                // mainloop alone; the output is not written); bit 1 = no TMEM loads (zeros stored);
+                // bit 2 = no TMA stores of the (first) output
   EpiParams e;
 };
 
@@ -204,8 +207,12 @@ struct TcParams {
 // mainloop), each next one while the current one is processed.  BIAS_ACT writes its two bf16
 // outputs through both boxes.  (BIAS_ACT_F32, an fp32 second output, keeps the register path.)
 constexpr int EPI_BUF = 4096;
-constexpr int EPI_BIAS = 128 * 4;  // fp32 bias of a warp's (at most 128) columns
-constexpr int EPI_SMEM = EPI_WARPS * (2 * EPI_BUF + EPI_BIAS) + EPI_WARPS * 2 * 8;
+// fp32 bias of a warp's (at most 128) columns, staged once per (accumulator buffer, column half): the
+// four row-quadrant warps of a half write the same values, and a warp is never more than one tile
+// ahead of another (the accumulator hand-off), so the tile-parity double buffer is race-free
+constexpr int EPI_BIAS_SET = 128 * 4;  // fp32
+constexpr int EPI_BIAS = 4 * EPI_BIAS_SET;  // [2 accumulators][2 halves]
+constexpr int EPI_SMEM = EPI_WARPS * 2 * EPI_BUF + EPI_BIAS + EPI_WARPS * 2 * 8;
 
 struct EpiWarp {
   uint32_t buf;   // shared address of the two staging boxes
@@ -227,6 +234,14 @@ __device__ __forceinline__ uint4 lds128(uint32_t a) {
 __device__ __forceinline__ float4 lds128f(uint32_t a) {
   uint4 v = lds128(a);
   return make_float4(__uint_as_float(v.x), __uint_as_float(v.y), __uint_as_float(v.z), __uint_as_float(v.w));
+}
+// four bf16 at a shared address (8-byte aligned) as fp32
+__device__ __forceinline__ float4 lds_bf16x4(uint32_t a) {
+  uint32_t x, y;
+  asm volatile("ld.shared.v2.b32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(a) : "memory");
+  const float2 lo = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&x));
+  const float2 hi = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&y));
+  return make_float4(lo.x, lo.y, hi.x, hi.y);
 }
 __device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
@@ -299,7 +314,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       bulk_wait_read<1>();
     }
     float v[CPB];
-    if (have_acc) {
+    if (have_acc && !(p.diag & 2)) {
 #pragma unroll
       for (int h = 0; h < CPB / 32; ++h) tmem_ld32(tacc + CPB * bi + 32 * h, v + 32 * h);
     } else {
@@ -379,7 +394,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
     }
     fence_proxy_async_smem();
     __syncwarp();
-    if (lane == 0) {
+    if (lane == 0 && !(p.diag & 4)) {
       tma_store_box(mC, sb, n, row0, z0, z1);
       bulk_commit();
     }
@@ -429,6 +444,13 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // Persistent tile walk shared by the three roles: tile t -> (z, m_blk, n_blk), grouped along M
 // (GROUP_M row-blocks share their B column panels in L2).
 // HARMONY_GEMM_GROUP_M (default 8): raster width of the persistent tile order, an A/B knob
+static int gemm_diag() {
+  static const int v = [] {
+    const char* e = getenv("HARMONY_GEMM_DIAG");
+    return e ? atoi(e) : 0;
+  }();
+  return v;
+}
 static int gemm_group_m() {
   static const int g = [] {
     const char* v = getenv("HARMONY_GEMM_GROUP_M");
@@ -463,7 +485,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
   uint8_t* sE = smem + STAGES * Cfg::STAGE_BYTES;  // epilogue staging boxes
-  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * (2 * EPI_BUF + EPI_BIAS));
+  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * 2 * EPI_BUF + EPI_BIAS);
   uint64_t* full = ebar + EPI_WARPS * 2;
   uint64_t* empty = full + STAGES;
   uint64_t* tmem_full = empty + STAGES;   // [2]
@@ -567,8 +589,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int half = (warp - 2) >> 2;  // which half of the tile's columns this warp drains
     const EpiParams& e = p.e;
-    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF + (warp - 2) * EPI_BIAS,
-               ebar + (warp - 2) * 2, 0u, 0u};
+    const uint32_t bias_base = smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF;
+    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, bias_base, ebar + (warp - 2) * 2, 0u, 0u};
     const bool out_f32 = e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32 || e.epi == HK_EPI_ACC_F32;
     int it = 0;
     for (int t = blockIdx.x; t < tm.total; t += gridDim.x, ++it) {
@@ -580,6 +602,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int ncols = min(BN, p.N - n0);
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
       const uint32_t tacc = tmem_base + acc * Cfg::ACC_COLS + ((uint32_t)(q * 32) << 16);
+      ew.bias = bias_base + (uint32_t)((acc << 1) | half) * EPI_BIAS_SET;
       if (p.tma_epi) {
         if (out_f32)
           tma_epi_tile<4>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, m0 + q * 32, n0 + c_beg, n0 + c_end,
@@ -650,6 +673,7 @@ static void launch_tc(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
   p.group_m = gemm_group_m();
+  p.diag = gemm_diag();
   p.e = e;
   CUtensorMap mc, mi, mo;
   make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
@@ -757,7 +781,9 @@ struct Tc2Cfg {
   static constexpr int A_BYTES = 128 * BK * 2; // 16 KB
   static constexpr int B_BYTES = HB * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_SMEM + 1024 + 256;
+  // no alignment slack: dynamic shared memory starts right after the 1 KB the system reserves, i.e.
+  // 1024-aligned (checked in the kernel, which traps otherwise)
+  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_SMEM + 256;
   static_assert(SMEM <= 232448, "shared memory per CTA");
   static constexpr int TMEM_COLS = 2 * BN;     // double-buffered accumulator (BN fp32 columns each)
 };
@@ -768,12 +794,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
                     const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmIn,
                     const __grid_constant__ CUtensorMap tmO2, TcParams p) {
   using Cfg = Tc2Cfg<BN, STAGES>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  if (smem_u32(smem_raw) & 1023) __trap();  // the layout below assumes a 1024-aligned base (128B-swizzle atoms)
+  uint8_t* smem = smem_raw;
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * Cfg::A_BYTES;
   uint8_t* sE = smem + STAGES * Cfg::STAGE_BYTES;  // epilogue staging boxes
-  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * (2 * EPI_BUF + EPI_BIAS));
+  uint64_t* ebar = reinterpret_cast<uint64_t*>(sE + EPI_WARPS * 2 * EPI_BUF + EPI_BIAS);
   uint64_t* full = ebar + EPI_WARPS * 2;
   uint64_t* empty = full + STAGES;
   uint64_t* tmem_full = empty + STAGES;  // [2]
@@ -884,8 +911,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const int half = (warp - 2) >> 2;
     const EpiParams& e = p.e;
     const uint32_t te = mapa_leader(&tmem_empty[0]);
-    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF + (warp - 2) * EPI_BIAS,
-               ebar + (warp - 2) * 2, 0u, 0u};
+    const uint32_t bias_base = smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF;
+    EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, bias_base, ebar + (warp - 2) * 2, 0u, 0u};
     const bool out_f32 = e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32 || e.epi == HK_EPI_ACC_F32;
     int it = 0;
     for (int t = pair; t < tm.total; t += npairs, ++it) {
@@ -898,7 +925,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       const int c_beg = half * (BN / 2), c_end = min(ncols, c_beg + BN / 2);
       const int row0 = mb * 256 + (int)rank * 128 + q * 32;
       const uint32_t tacc = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
-      if (p.tma_epi) {
+      ew.bias = bias_base + (uint32_t)((acc << 1) | half) * EPI_BIAS_SET;
+      if (p.diag & 1) {
+        mbar_wait(&tmem_full[acc], (it >> 1) & 1);
+        tc_fence_after();
+      } else if (p.tma_epi) {
         if (out_f32)
           tma_epi_tile<4>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0, z1,
                           &tmem_full[acc], (it >> 1) & 1);
@@ -935,6 +966,7 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   TcParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.nz0 = a.nz0; p.nz = a.nz0 * a.nz1; p.a_mn = a.a_mn_major; p.b_mn = a.b_mn_major;
   p.group_m = gemm_group_m();
+  p.diag = gemm_diag();
   p.e = e;
   CUtensorMap mc, mi, mo;
   make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
@@ -992,7 +1024,16 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
   if (mode && a.M >= 256 && a.N >= 256 && pair_tiles >= 37) {
     // CTA-pair 256 x 256 tiles (measured best for every cfg2 shape, tools/gemm_bench.py);
     // HARMONY_GEMM_2SM=3 selects 256 x 128 pair tiles, 0 the single-CTA kernel
+    // five 32 KB stages for plain products, four for batched ones (split-K weight gradients:
+    // measured 2-6% faster / 4% slower, profiles/r02_gemm_stages_cfg2.txt); HARMONY_GEMM_STAGES
+    // forces one (the stage count only paces the loads: results are bitwise the same)
+    static const int force = [] {
+      const char* v = getenv("HARMONY_GEMM_STAGES");
+      return v ? atoi(v) : 0;
+    }();
+    const int stages = force ? force : (nz == 1 ? 5 : 4);
     if (mode == 3) tc::launch_tc2<128, 6>(a, e, st);
+    else if (stages == 5) tc::launch_tc2<256, 5>(a, e, st);
     else tc::launch_tc2<256, 4>(a, e, st);
     return;
   }
