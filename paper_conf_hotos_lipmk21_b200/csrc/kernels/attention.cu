@@ -1006,6 +1006,13 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
                          cudaStream_t st) {
   using namespace attn;
   if (S % BQ != 0 || (dh != 64 && dh != 128)) return false;
+  {  // HARMONY_ATTN_FWD=2: the two-query-tile kernel for dh = 64 (an A/B alternative, attention_fwd2.cu)
+    static const int which = [] {
+      const char* v = getenv("HARMONY_ATTN_FWD");
+      return v ? atoi(v) : 1;
+    }();
+    if (which == 2 && attention_fwd2_fused(b, S, H, dh, causal, QKV, C, lse, st)) return true;
+  }
   const int d = H * dh;
   CUtensorMap mq, mk, mv, mc;
   // Q, K: K-major operands (inner = dh, rows = S, z0 = head, z1 = sequence); V: MN-major (inner = dh)

@@ -262,6 +262,19 @@ __device__ __forceinline__ void tma_store_box(const CUtensorMap* map, uint32_t s
                "r"(src), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
                : "memory");
 }
+// the same with an L2 eviction-priority policy (createpolicy) for the written lines
+__device__ __forceinline__ void tma_store_box_hint(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2, int c3,
+                                                   uint64_t pol) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4, %5}], [%1], %6;" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(src), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 
 // Is the TMA epilogue usable for this epilogue kind / tile width (host and device agree)?
 __host__ __device__ __forceinline__ bool tma_epi_kind_ok(int epi) { return epi != HK_EPI_BIAS_ACT_F32; }
@@ -395,7 +408,8 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
     fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0 && !(p.diag & 4)) {
-      tma_store_box(mC, sb, n, row0, z0, z1);
+      if (p.diag & 8) tma_store_box_hint(mC, sb, n, row0, z0, z1, policy_evict_first());
+      else tma_store_box(mC, sb, n, row0, z0, z1);
       bulk_commit();
     }
     if (ESZ == 2 && two) {
@@ -418,7 +432,8 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       fence_proxy_async_smem();
       __syncwarp();
       if (lane == 0) {
-        tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
+        if (p.diag & 8) tma_store_box_hint(mO2, w.buf + EPI_BUF, n, row0, z0, z1, policy_evict_first());
+        else tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
         bulk_commit();
       }
     }

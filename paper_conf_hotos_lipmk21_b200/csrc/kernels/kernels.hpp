@@ -51,6 +51,9 @@ void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st);
 // fused attention forward (attention.cu); false when the shape does not qualify
 bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, void* C, float* lse,
                          cudaStream_t st);
+// two-query-tile forward (attention_fwd2.cu): dh = 64, S % 256 == 0; false otherwise
+bool attention_fwd2_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, void* C, float* lse,
+                          cudaStream_t st);
 // fused attention backward: dQKV from QKV, O, dO, lse (scratch: attention_bwd_scratch_bytes)
 size_t attention_bwd_scratch_bytes(int64_t b, int S, int H);
 bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void* QKV, const void* O, const void* dO,
