@@ -51,7 +51,9 @@ typedef struct {
   void* C; int64_t ldc, c_sz0, c_sz1;
   int32_t epilogue;    /* hk_epilogue */
   int32_t act;         /* harmony_act for BIAS_ACT / ACT_BWD */
-  int32_t accumulate;  /* HK_EPI_ACC_F32: 1 = add into C */
+  int32_t accumulate;  /* HK_EPI_ACC_F32: 1 = add into C; 2 = CONTINUE C's reduction: the K sum starts
+                          from C instead of 0 (alpha 1; fp32 SIMT GEMM only), so a K-split into
+                          slices run in order is bit-identical to one GEMM over the whole K */
   float alpha;
   const void* bias;    /* [N] of T, nullable */
   const void* aux;     /* RESID_F32: f32 residual; ACT_BWD: T pre-activation */

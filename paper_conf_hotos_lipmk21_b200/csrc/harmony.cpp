@@ -1068,7 +1068,33 @@ harmony_status harmony_register_layers(harmony_ctx* c, int32_t n_layers, const h
                     (plans[r].ops[i].dev == plans[0].ops[i].dev && plans[r].ops[i].count == plans[0].ops[i].count)),
                HARMONY_E_INVALID_ARG, "internal: rank programs differ");
   }
-  for (size_t r = 0; r < R.size(); ++r) register_rank(R[r], std::move(plans[r]), init_params);
+  // parameters per task layer: a column panel gets its W[:, panel] and b[panel] (every rank plans the
+  // same panels: the split depends on the layer shapes and the cap only)
+  std::vector<std::vector<float>> panel_store;
+  std::vector<const float*> tparams;
+  {
+    const Plan& p0 = plans[0];
+    for (int u = 0; u < n_layers; ++u) {
+      const int cnt = p0.user_count[u];
+      if (cnt == 1) { tparams.push_back(init_params[u]); continue; }
+      const int din = descs[u].d_in, dout = descs[u].d_out, dp = dout / cnt;
+      for (int k = 0; k < cnt; ++k) {
+        std::vector<float> w((size_t)din * dp + dp);
+        for (int i = 0; i < din; ++i)
+          memcpy(w.data() + (size_t)i * dp, init_params[u] + (size_t)i * dout + (size_t)k * dp, (size_t)dp * 4);
+        memcpy(w.data() + (size_t)din * dp, init_params[u] + (size_t)din * dout + (size_t)k * dp, (size_t)dp * 4);
+        panel_store.push_back(std::move(w));
+      }
+    }
+    size_t q = 0;
+    tparams.clear();
+    for (int u = 0; u < n_layers; ++u) {
+      if (p0.user_count[u] == 1) tparams.push_back(init_params[u]);
+      else
+        for (int k = 0; k < p0.user_count[u]; ++k) tparams.push_back(panel_store[q++].data());
+    }
+  }
+  for (size_t r = 0; r < R.size(); ++r) register_rank(R[r], std::move(plans[r]), tparams.data());
   HM_CUDA(cudaSetDevice(c->cfg.device));
   if (!c->members.empty()) {
     c->plan = R[0]->plan;  // the group's view: rank 0's plan (summary, geometry)
@@ -1094,11 +1120,39 @@ harmony_status harmony_step(harmony_ctx* c, const float* x, const float* target,
   HM_API_END(c)
 }
 
+static harmony_status read_task_layer(harmony_ctx* c, int32_t layer, int32_t which, float* dst, uint64_t n);
+
 harmony_status harmony_read_state(harmony_ctx* c, int32_t layer, int32_t which, float* dst, uint64_t n) {
   HM_API_BEGIN
   HM_CHECK(c != nullptr, HARMONY_E_INVALID_ARG, "ctx is NULL");
   HM_CHECK(!c->broken, HARMONY_E_BAD_STATE, "context has a sticky CUDA/NCCL error: " + c->err);
   HM_CHECK(c->registered, HARMONY_E_BAD_STATE, "harmony_register_layers first");
+  const Plan& p = c->plan;
+  if (!c->gplan && !p.user_first.empty() && p.user_count.size() == (size_t)p.n_user &&
+      (size_t)p.n_user != p.layers.size()) {  // some layer runs as column panels: reassemble W, b
+    HM_CHECK(layer >= 0 && layer < p.n_user, HARMONY_E_INVALID_ARG, "layer out of range");
+    const int first = p.user_first[layer], cnt = p.user_count[layer];
+    if (cnt == 1) return read_task_layer(c, first, which, dst, n);
+    const LayerGeom& g0 = p.layers[first].g;
+    const int din = g0.desc.d_in, dp = g0.desc.d_out, dout = g0.ld_out;
+    HM_CHECK(dst && n == (uint64_t)din * dout + dout, HARMONY_E_INVALID_ARG,
+             "n_floats must equal the layer's parameter count");
+    std::vector<float> part((size_t)din * dp + dp);
+    for (int k = 0; k < cnt; ++k) {
+      const harmony_status st = read_task_layer(c, first + k, which, part.data(), part.size());
+      if (st != HARMONY_OK) return st;
+      for (int i = 0; i < din; ++i)
+        memcpy(dst + (size_t)i * dout + (size_t)k * dp, part.data() + (size_t)i * dp, (size_t)dp * 4);
+      memcpy(dst + (size_t)din * dout + (size_t)k * dp, part.data() + (size_t)din * dp, (size_t)dp * 4);
+    }
+    return HARMONY_OK;
+  }
+  return read_task_layer(c, layer, which, dst, n);
+  HM_API_END(c)
+}
+
+static harmony_status read_task_layer(harmony_ctx* c, int32_t layer, int32_t which, float* dst, uint64_t n) {
+  HM_API_BEGIN
   if (c->gplan) {  // Harmony-PP: the layer lives, unsharded, on rank layer % N
     const GroupPlan& gp = *c->gplan;
     HM_CHECK(layer >= 0 && layer < (int)gp.layer_rank.size(), HARMONY_E_INVALID_ARG, "layer out of range");

@@ -42,6 +42,17 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(SimtParams p) {
   const float* B = p.B + z0 * p.b_sz0 + z1 * p.b_sz1;
   const int tx = tid % 16, ty = tid / 16;
   float acc[4][4] = {};
+  const bool cont = p.e.epi == HK_EPI_ACC_F32 && p.e.accumulate == 2;  // continue C's K reduction
+  if (cont) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int m = m0 + ty + 16 * i, n = n0 + tx + 16 * j;
+        if (m < p.M && n < p.N)
+          acc[i][j] = reinterpret_cast<const float*>(p.e.C)[z0 * p.e.c_sz0 + z1 * p.e.c_sz1 + (int64_t)m * p.e.ldc + n];
+      }
+  }
   for (int k0 = 0; k0 < p.K; k0 += SBK) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
@@ -78,7 +89,8 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(SimtParams p) {
       int n = n0 + tx + 16 * j;
       if (n >= p.N) continue;
       int64_t off = z0 * e.c_sz0 + z1 * e.c_sz1 + (int64_t)m * e.ldc + n;
-      epi_scalar<float>(e, off, n, acc[i][j]);
+      if (cont) reinterpret_cast<float*>(e.C)[off] = acc[i][j];
+      else epi_scalar<float>(e, off, n, acc[i][j]);
     }
   }
 }
@@ -1013,6 +1025,8 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
   e.C = a.C; e.ldc = a.ldc; e.c_sz0 = a.c_sz0; e.c_sz1 = a.c_sz1;
   e.epi = a.epilogue; e.act = a.act; e.accumulate = a.accumulate; e.alpha = a.alpha;
   e.bias = a.bias; e.aux = a.aux; e.aux_out = a.aux_out; e.M = a.M; e.N = a.N;
+  HM_CHECK(a.accumulate != 2 || (a.dtype == 0 && a.epilogue == HK_EPI_ACC_F32 && a.alpha == 1.f),
+           HARMONY_E_UNSUPPORTED, "gemm: accumulate = 2 (continue C's reduction) is the fp32 ACC_F32 path only");
   if (a.dtype == 0) {
     const int e0 = g_prof.begin(st);
     const double flops = 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1;

@@ -45,6 +45,24 @@ static uint64_t wgrad_split_ws_bytes(const LayerGeom& g, int64_t rows, int n, in
   const int S = wgrad_splits(g, rows, n, k);
   return S > 1 ? (uint64_t)S * k * n * 4 : 0;
 }
+LayerGeom make_panel_geom(const harmony_layer_desc& full, int b, int dtype, int stash_policy, int panel, int npanel) {
+  HM_CHECK(full.kind == HARMONY_LAYER_MLP && npanel >= 1 && full.d_out % (16 * npanel) == 0, HARMONY_E_INVALID_ARG,
+           "column panels: MLP layers with d_out a multiple of 16 * panels");
+  harmony_layer_desc d = full;
+  d.d_out = full.d_out / npanel;
+  LayerGeom g = make_geom(d, b, dtype, stash_policy);
+  g.npanel = npanel;
+  g.panel = panel;
+  g.col0 = panel * d.d_out;
+  g.ld_out = full.d_out;
+  if (npanel > 1) {  // contiguous copies of the panel's output / output-gradient columns
+    const uint64_t tmp = align_up((uint64_t)g.rows * d.d_out * 4, 256);
+    g.ws_fwd += tmp;
+    g.ws_bwd += tmp;
+  }
+  return g;
+}
+
 LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_policy) {
   if ((stash_policy == 2 || stash_policy == 3) && desc.kind == HARMONY_LAYER_TRANSFORMER) {
     // Block recompute ([7] P:881): the stash is the block input X; the forward and the
@@ -79,6 +97,7 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   g.stash_policy = stash_policy;
   g.b = b;
   g.n_params = layer_n_params(desc);
+  g.ld_out = desc.d_out;
   if (desc.kind == HARMONY_LAYER_MLP) {
     g.S = 1;
     g.rows = b;
@@ -352,6 +371,9 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     if (dX) {
       hk_gemm_args a = lin_dgrad(g, g.rows, d.d_out, d.d_in, dZ, wseg(g, W, P_MLP_W));
       a.C = dX; a.epilogue = HK_EPI_STORE_F32;
+      // a later column panel continues the K reduction of dX where the previous panel left it: the
+      // panels, run in order, reproduce the unsplit dgrad bit for bit (fp32 path)
+      if (g.panel > 0) { a.epilogue = HK_EPI_ACC_F32; a.accumulate = 2; }
       gemm(a, st);
     }
     return;
@@ -533,6 +555,14 @@ static LayerGeom core_geom(const LayerGeom& g) {
 }
 
 void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* st) {
+  if (g.npanel > 1) {  // column panel: its output columns into Y[:, col0 ..] (row stride ld_out)
+    float* Yt = reinterpret_cast<float*>(ws);
+    const uint64_t tmp = align_up((uint64_t)g.rows * g.desc.d_out * 4, 256);
+    fwd_core(g, W, X, Yt, stash, ws + tmp, st);
+    HM_CUDA(cudaMemcpy2DAsync(Y + g.col0, (size_t)g.ld_out * 4, Yt, (size_t)g.desc.d_out * 4, (size_t)g.desc.d_out * 4,
+                              (size_t)g.rows, cudaMemcpyDeviceToDevice, static_cast<cudaStream_t>(st)));
+    return;
+  }
   if (g.stash_policy < 2) return fwd_core(g, W, X, Y, stash, ws, st);
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;
@@ -545,6 +575,13 @@ void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint
 
 void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,
                int first, uint8_t* ws, void* st) {
+  if (g.npanel > 1) {  // column panel: its columns of dY; dX written (panel 0) or continued (later panels)
+    float* dYt = reinterpret_cast<float*>(ws);
+    const uint64_t tmp = align_up((uint64_t)g.rows * g.desc.d_out * 4, 256);
+    HM_CUDA(cudaMemcpy2DAsync(dYt, (size_t)g.desc.d_out * 4, dY + g.col0, (size_t)g.ld_out * 4, (size_t)g.desc.d_out * 4,
+                              (size_t)g.rows, cudaMemcpyDeviceToDevice, static_cast<cudaStream_t>(st)));
+    return bwd_core(g, W, stash, dYt, dX, dW, first, ws + tmp, st);
+  }
   if (g.stash_policy < 2) return bwd_core(g, W, stash, dY, dX, dW, first, ws, st);
   const LayerGeom c = core_geom(g);
   uint8_t* full = ws + g.core_off;

@@ -40,7 +40,12 @@ struct LayerGeom {
   double flops_fwd = 0;             // algorithmic GEMM FLOPs of one forward task
   StashLayout core_st;              // policy 2: the policy-0 layout the recompute materialises
   uint64_t core_ws_fwd = 0, core_ws_bwd = 0;
+  // operator split (row a15): this task is column panel `panel` of `npanel` of an fp32 MLP layer whose
+  // full output width is ld_out; it writes / reads output columns [col0, col0 + desc.d_out)
+  int npanel = 1, panel = 0, col0 = 0, ld_out = 0;
 };
+// A layer's geometry as column panel `panel` of `npanel` (MLP, d_out % (16 npanel) == 0).
+LayerGeom make_panel_geom(const harmony_layer_desc& full, int b, int dtype, int stash_policy, int panel, int npanel);
 
 enum { P_LN1_G = 0, P_LN1_B, P_WQKV, P_BQKV, P_WO, P_BO, P_LN2_G, P_LN2_B, P_WFC1, P_BFC1, P_WFC2, P_BFC2 };
 enum { P_MLP_W = 0, P_MLP_B = 1 };

@@ -152,7 +152,7 @@ static std::vector<Acc> accesses(const Plan& p, const Op& o) {
       const LayerPlan& lp = p.layers[o.layer];
       ar(o.w, (uint64_t)lp.P * ts, false);
       ar(o.in, (uint64_t)lp.g.rows * lp.g.desc.d_in * 4, false);
-      ar(o.out, (uint64_t)lp.g.rows * lp.g.desc.d_out * 4, true);
+      ar(o.out, (uint64_t)lp.g.rows * lp.g.ld_out * 4, true);  // (a column panel: within these rows)
       ar(o.stash, lp.g.st.total, true);
       ar(o.ws, lp.g.ws_fwd, true);
       break;
@@ -161,7 +161,7 @@ static std::vector<Acc> accesses(const Plan& p, const Op& o) {
       const LayerPlan& lp = p.layers[o.layer];
       ar(o.w, (uint64_t)lp.P * ts, false);
       ar(o.stash, lp.g.st.total, false);
-      ar(o.in, (uint64_t)lp.g.rows * lp.g.desc.d_out * 4, false);
+      ar(o.in, (uint64_t)lp.g.rows * lp.g.ld_out * 4, false);
       ar(o.out, (uint64_t)lp.g.rows * lp.g.desc.d_in * 4, true);
       ar(o.dw, (uint64_t)lp.P * 4, true);
       ar(o.ws, lp.g.ws_bwd, true);
@@ -249,8 +249,45 @@ int validate_program(const Plan& p, std::string* first) {
 }
 
 // ------------------------------------------------------------------------------------ make_plan
+static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs, bool layout_only,
+                           int n_bnd, const std::vector<int>& npanel);
+
+// Operator split inside the step (row a15): when the cap cannot hold a registered layer's
+// working set, fp32 MLP layers are decomposed into column panels — sub-tasks that each need only their
+// W[:, panel] columns (compute copy, master / m / v, dW) — the widest layer halved first, until the
+// plan fits.  Panels in order reproduce the unsplit layer bit for bit (the forward and the weight
+// gradient split along N; dX continues one K reduction across the panels), so capped == uncapped
+// stays exact (reading c21).
 Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs, bool layout_only,
                int n_bnd) {
+  std::vector<int> np(n_layers > 0 ? n_layers : 0, 1);
+  try {
+    return make_plan_impl(cfg, n_layers, descs, layout_only, n_bnd, np);
+  } catch (const Error& e) {
+    if (e.code != HARMONY_E_CAP_TOO_SMALL || cfg.precision != HARMONY_FP32 || layout_only) throw;
+    for (int round = 0; round < 16; ++round) {
+      int best = -1;
+      int64_t best_p = 0;
+      for (int l = 0; l < n_layers; ++l) {
+        const harmony_layer_desc& d = descs[l];
+        if (d.kind != HARMONY_LAYER_MLP || d.d_out % (16 * 2 * np[l]) != 0) continue;
+        const int64_t per = ((int64_t)d.d_in + 1) * d.d_out / np[l];
+        if (per > best_p) { best_p = per; best = l; }
+      }
+      if (best < 0) throw;
+      np[best] *= 2;
+      try {
+        return make_plan_impl(cfg, n_layers, descs, layout_only, n_bnd, np);
+      } catch (const Error& e2) {
+        if (e2.code != HARMONY_E_CAP_TOO_SMALL) throw;
+      }
+    }
+    throw;
+  }
+}
+
+static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmony_layer_desc* descs, bool layout_only,
+                           int n_bnd, const std::vector<int>& npanel) {
   validate_config(cfg);
   validate_layers(cfg, n_layers, descs, !layout_only);
   HM_CHECK(cfg.schedule != HARMONY_SCHED_HARMONY_PP, HARMONY_E_UNSUPPORTED,
@@ -267,22 +304,35 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   p.retain_grads = cfg.retain_grads;
   p.cap = cfg.hbm_cap_bytes;
   p.upd_lag = (p.N > 1 && p.schedule == HARMONY_SCHED_HARMONY_DP) ? 1 : 0;
-  const int L = n_layers, m = p.m, N = p.N, r = p.rank;
+  const int m = p.m, N = p.N, r = p.rank;
   const uint64_t ts = p.dtype ? 2 : 4;
+  // task layers: each registered layer, or its column panels
+  p.n_user = n_layers;
+  std::vector<std::pair<int, int>> tl;  // (registered layer, panel)
+  for (int u = 0; u < n_layers; ++u) {
+    p.user_first.push_back((int)tl.size());
+    p.user_count.push_back(npanel[u]);
+    for (int k = 0; k < npanel[u]; ++k) tl.push_back({u, k});
+  }
+  const int L = (int)tl.size();
+  const int LU = n_layers;
 
   p.layers.resize(L);
   int dmax = 0;
+  for (int u = 0; u < LU; ++u) dmax = std::max({dmax, descs[u].d_in, descs[u].d_out});
   uint64_t ws_need = 256, maxP = 0, max_shard = 0;
   for (int l = 0; l < L; ++l) {
     LayerPlan& lp = p.layers[l];
-    lp.g = make_geom(descs[l], p.b, p.dtype, p.stash_policy);
+    const int u = tl[l].first;
+    lp.user = u;
+    lp.g = npanel[u] > 1 ? make_panel_geom(descs[u], p.b, p.dtype, p.stash_policy, tl[l].second, npanel[u])
+                         : make_geom(descs[u], p.b, p.dtype, p.stash_policy);
     lp.P = lp.g.n_params;
     lp.Ppad = (int64_t)align_up((uint64_t)lp.P, (uint64_t)N * 1024);
     lp.shard = lp.Ppad / N;
     lp.wc_bytes = (uint64_t)lp.Ppad * ts;
     lp.state_bytes = 3 * (uint64_t)lp.shard * 4;
     lp.stash_res.assign(m, -1);
-    dmax = std::max({dmax, descs[l].d_in, descs[l].d_out});
     ws_need = std::max({ws_need, lp.g.ws_fwd, lp.g.ws_bwd});
     maxP = std::max<uint64_t>(maxP, (uint64_t)lp.Ppad);
     max_shard = std::max<uint64_t>(max_shard, (uint64_t)lp.shard);
@@ -290,9 +340,9 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   }
   const int64_t rows = p.layers[0].g.rows;
   p.d_in0 = descs[0].d_in;
-  p.d_out_last = descs[L - 1].d_out;
+  p.d_out_last = descs[LU - 1].d_out;
   p.in_elems_per_mb = rows * descs[0].d_in;
-  p.out_elems_per_mb = rows * descs[L - 1].d_out;
+  p.out_elems_per_mb = rows * descs[LU - 1].d_out;
 
   // ---------------------------------------------------------------- fixed working set
   const uint64_t bnd_stride = align_up((uint64_t)rows * dmax * 4, ALIGN);
@@ -556,7 +606,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
   }
   for (int l = 0; l < L; ++l) {
     LayerPlan& lp = p.layers[l];
-    const int in_buf = l % 2, out_buf = (l + 1) % 2;
+    const int in_buf = lp.user % 2, out_buf = (lp.user + 1) % 2;  // a registered layer's panels share its buffers
     for (int i = 0; i < m; ++i) {
       int slot = -1;
       uint64_t wdev;
@@ -594,7 +644,7 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     }
   }
   // ---- loss
-  const int Lb = L % 2, dYb = (L + 1) % 2;
+  const int Lb = LU % 2, dYb = (LU + 1) % 2;
   for (int i = 0; i < m; ++i) {
     Task t;
     t.op.kind = OP_LOSS; t.op.stream = S_COMPUTE; t.op.mb = i;
@@ -702,9 +752,13 @@ Plan make_plan(const harmony_config& cfg, int n_layers, const harmony_layer_desc
     tasks.push_back(t);
   };
 
-  for (int l = L - 1; l >= 0; --l) {
+  // registered layers in reverse; a layer's column panels in order (the dX reduction runs through them)
+  std::vector<int> bwd_order;
+  for (int u = LU - 1; u >= 0; --u)
+    for (int k = 0; k < p.user_count[u]; ++k) bwd_order.push_back(p.user_first[u] + k);
+  for (int l : bwd_order) {
     LayerPlan& lp = p.layers[l];
-    const int in_buf = l % 2, out_buf = (l + 1) % 2;
+    const int in_buf = lp.user % 2, out_buf = (lp.user + 1) % 2;
     const int j = l % nDW;
     for (int i = 0; i < m; ++i) {
       int slot = -1;

@@ -61,13 +61,16 @@ struct LayerPlan {
   uint64_t state_bytes = 0;            // master|m|v shard (fp32)
   int64_t wc_res = -1, state_res = -1; // resident offsets (-1 = streamed)
   std::vector<int64_t> stash_res;      // per microbatch: resident offset or -1 (spilled)
+  int user = 0;                        // the registered layer this task layer belongs to (column panels)
 };
 
 struct Plan {
   int N = 1, rank = 0, m = 1, b = 1, dtype = 0, stash_policy = 0, schedule = 0, retain_grads = 0;
   uint64_t cap = 0;
   int upd_lag = 0;
-  std::vector<LayerPlan> layers;
+  std::vector<LayerPlan> layers;   // task layers: a registered layer, or its column panels (operator split)
+  int n_user = 0;                  // registered layers
+  std::vector<int> user_first, user_count;  // registered layer -> its task layers
   // arena layout
   uint64_t arena_bytes = 0, min_ws_bytes = 0;
   // fp32 activation / gradient buffers of m microbatch rows each: [0], [1] the ping-pong of the DP step;

@@ -267,3 +267,24 @@ def test_plan_scales_to_paper_configs():
                     hbm_cap_bytes=c["cap"])
         assert s.hazards == 0 and s.arena_bytes <= c["cap"]
         assert s.pred_h2d_bytes > 10e9  # op-input stash spills: host-link bound
+
+
+def test_operator_split_column_panels_only_when_the_cap_forces_them():
+    """Row a15 inside the step: an fp32 MLP layer whose working set does not fit the cap is
+    decomposed into column-panel sub-tasks (each needs only W[:, panel]); the plan stays race-free and
+    moves each panel's weights as the unsplit layer would (same total bytes per pass)."""
+    from synth import LayerDesc, LAYER_MLP, ACT_GELU, ACT_NONE
+    descs = [LayerDesc(LAYER_MLP, 256, 2048, act=ACT_GELU), LayerDesc(LAYER_MLP, 2048, 256, act=ACT_GELU),
+             LayerDesc(LAYER_MLP, 256, 256, act=ACT_NONE)]
+    kw = dict(microbatches=2, microbatch_size=8)
+    base, _ = plan(descs, hbm_cap_bytes=1 << 40, **kw)
+    counts = []
+    for f in (2.0, 0.9, 0.4, 0.25):
+        s, ops = plan(descs, hbm_cap_bytes=int(base.min_working_set_bytes * f), **kw)
+        assert s.hazards == 0 and s.arena_bytes <= int(base.min_working_set_bytes * f)
+        counts.append(sum(1 for o in ops if o["kind"] == "FWD"))
+    assert counts[0] == 3 * 2  # fits: no split
+    assert counts[1] > counts[0] and counts[3] > counts[2] > counts[1]  # more panels as the cap shrinks
+    with pytest.raises(H.HarmonyError) as e:  # bf16 layers are not split: the cap is simply too small
+        plan(descs, hbm_cap_bytes=int(base.min_working_set_bytes * 0.4), precision=1, **kw)
+    assert e.value.code == H.HARMONY_E_CAP_TOO_SMALL

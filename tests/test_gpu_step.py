@@ -275,3 +275,23 @@ def test_graph_replay_equals_eager_and_tracks_input_pointers():
                             m=[h.read(l, H.HARMONY_ADAM_M) for l in range(len(descs))],
                             v=[h.read(l, H.HARMONY_ADAM_V) for l in range(len(descs))]))
     bitwise_equal(eager, res)
+
+
+@pytest.mark.parametrize("frac", [0.9, 0.25])
+def test_operator_split_panels_match_oracle_and_are_bitwise_the_unsplit_step(frac):
+    """Row a15 inside the step: under a cap smaller than the wide layers' working set the planner runs
+    them as column-panel sub-tasks (forward and weight gradient split along N, dX one K reduction
+    continued panel to panel); the result is the oracle's full-batch step (1e-5, fp32) and bit for bit
+    the uncapped, unsplit run (reading c21)."""
+    descs = [LayerDesc(LAYER_MLP, 256, 2048, act=synth.ACT_GELU), LayerDesc(LAYER_MLP, 2048, 256, act=synth.ACT_GELU),
+             LayerDesc(LAYER_MLP, 256, 256, act=ACT_NONE)]
+    params = synth.gen_params(descs)
+    batches = batches_for(descs, 16, 3, 0)
+    kw = dict(microbatches=2, microbatch_size=8)
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, **kw), descs, text_len=0)
+    cap = int(s.min_working_set_bytes * frac)
+    split, plan = run_gpu(descs, params, batches, hbm_cap_bytes=cap, **kw)
+    assert plan["arena_bytes"] <= cap and plan["n_ops"] > 40
+    compare(split, run_oracle(descs, params, batches), 1e-5)
+    whole, _ = run_gpu(descs, params, batches, hbm_cap_bytes=0, **kw)
+    bitwise_equal(split, whole)
