@@ -123,6 +123,13 @@ typedef struct {
                                 the kernel uses fp32 b and (1-b) each rounded once from these */
   uint8_t nccl_id[128];      /* ncclUniqueId from harmony_get_unique_id() on rank 0, broadcast
                                 to all ranks by the caller (ignored when world_size == 1)    */
+  int32_t groups;            /* G microbatch groups (0 or 1 = one group; m % G == 0; Harmony-DP):
+                                group 0's forward, then each group's backward interleaved layer by
+                                layer with the next group's forward, so stash swap-ins and spills
+                                use both directions of the host link (SURVEY §8(d) direction
+                                balance).  Every layer's fp32 dW stays in HBM across the groups.
+                                The microbatches keep their canonical order in every accumulation:
+                                results are bit-identical for every G (reading c21).             */
 } harmony_config;
 
 typedef struct {

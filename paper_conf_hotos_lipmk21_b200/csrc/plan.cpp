@@ -28,6 +28,7 @@ void validate_config(const harmony_config& c) {
                c.schedule == HARMONY_SCHED_HARMONY_PP,
            HARMONY_E_INVALID_ARG, "unknown schedule");
   HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 3, HARMONY_E_INVALID_ARG, "stash_policy must be 0..3");
+  HM_CHECK(c.groups >= 0 && c.groups <= 64, HARMONY_E_INVALID_ARG, "groups must be in 0..64");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
@@ -347,7 +348,15 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
   // ---------------------------------------------------------------- fixed working set
   const uint64_t bnd_stride = align_up((uint64_t)rows * dmax * 4, ALIGN);
   const uint64_t tgt_stride = align_up((uint64_t)p.out_elems_per_mb * 4, ALIGN);
-  const int nDW = N > 1 ? 2 : 1;
+  // microbatch groups (direction balance): G > 1 keeps every layer's fp32 dW accumulator from its
+  // first group's backward to its last
+  const int G = cfg.groups > 1 ? cfg.groups : 1;
+  HM_CHECK(m % G == 0, HARMONY_E_INVALID_ARG, "microbatches must be a multiple of groups");
+  HM_CHECK(G == 1 || p.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
+           "microbatch groups are a Harmony-DP schedule");
+  const int mg = m / G;
+  const int nDW = G > 1 ? L : (N > 1 ? 2 : 1);
+  auto dwi = [&](int l) { return G > 1 ? l : l % nDW; };
   auto fixed_bytes = [&]() {
     uint64_t f = 0;
     f += (uint64_t)p.n_bnd * bnd_stride * m;          // activation / gradient buffers
@@ -521,6 +530,7 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
   p.tgt = a.take(tgt_stride * m);
   p.ws_bytes = ws_need;
   p.ws = a.take(ws_need);
+  p.dw.assign(nDW, 0);
   for (int j = 0; j < nDW; ++j) p.dw[j] = a.take(maxP * 4);
   if (N > 1) for (int j = 0; j < 2; ++j) p.gsh[j] = a.take(max_shard * 4);
   p.loss = a.take((uint64_t)N * m * 8);
@@ -604,48 +614,46 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
     Task t;  // inputs are issued as the first ops (not prefetch items)
     (void)t;
   }
-  for (int l = 0; l < L; ++l) {
+  auto fwd_task = [&](int l, int i, bool gfirst) {
     LayerPlan& lp = p.layers[l];
     const int in_buf = lp.user % 2, out_buf = (lp.user + 1) % 2;  // a registered layer's panels share its buffers
-    for (int i = 0; i < m; ++i) {
-      int slot = -1;
-      uint64_t wdev;
-      if (baseline || i == 0) wdev = weight_use(l, (int)tasks.size(), slot);  // grouping: one swap-in per layer
-      else { slot = fwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
-      fwd_wslot[l] = slot;
-      Task t;
-      t.op.kind = OP_FWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i;
-      t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws;
-      t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
-      t.wr = {key(R_BND, out_buf, i)};
-      if (lp.stash_res[i] >= 0) {
-        t.op.stash = (uint64_t)lp.stash_res[i];
-        t.wr.push_back(key(R_STASHRES, l, i));
-      } else {
-        int g = gnext;
-        gnext = (gnext + 1) % nG;
-        t.op.stash = p.stage[g];
-        t.wr.push_back(key(R_STAGE, g));
-        Op d;
-        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = l; d.mb = i;
-        d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + i; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
-        t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, i)}}});
-        stage_last[g] = (int)tasks.size();
-        spill_task[(size_t)l * m + i] = (int)tasks.size();
-      }
-      if (slot >= 0) wslot_last[slot] = (int)tasks.size();
-      if (baseline && slot >= 0) {  // per-GPU virtualization: weights out again after each forward
-        Op d;
-        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
-        d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
-        t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
-      }
-      tasks.push_back(t);
+    int slot = -1;
+    uint64_t wdev;
+    if (baseline || gfirst) wdev = weight_use(l, (int)tasks.size(), slot);  // grouping: one swap-in per layer and group
+    else { slot = fwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
+    fwd_wslot[l] = slot;
+    Task t;
+    t.op.kind = OP_FWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i;
+    t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws;
+    t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
+    t.wr = {key(R_BND, out_buf, i)};
+    if (lp.stash_res[i] >= 0) {
+      t.op.stash = (uint64_t)lp.stash_res[i];
+      t.wr.push_back(key(R_STASHRES, l, i));
+    } else {
+      int g = gnext;
+      gnext = (gnext + 1) % nG;
+      t.op.stash = p.stage[g];
+      t.wr.push_back(key(R_STAGE, g));
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = l; d.mb = i;
+      d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + i; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
+      t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, i)}}});
+      stage_last[g] = (int)tasks.size();
+      spill_task[(size_t)l * m + i] = (int)tasks.size();
     }
-  }
+    if (slot >= 0) wslot_last[slot] = (int)tasks.size();
+    if (baseline && slot >= 0) {  // per-GPU virtualization: weights out again after each forward
+      Op d;
+      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
+      d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
+      t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
+    }
+    tasks.push_back(t);
+  };
   // ---- loss
   const int Lb = LU % 2, dYb = (LU + 1) % 2;
-  for (int i = 0; i < m; ++i) {
+  auto loss_task = [&](int i) {
     Task t;
     t.op.kind = OP_LOSS; t.op.stream = S_COMPUTE; t.op.mb = i;
     t.op.in = bnd_row(Lb, i); t.op.tgt = p.tgt + (uint64_t)i * tgt_stride; t.op.out = bnd_row(dYb, i);
@@ -670,7 +678,7 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
       }
     }
     tasks.push_back(t);
-  }
+  };
   // ---- backward + JIT update
   std::vector<int> bwd_wslot(L, -1);
   std::vector<int> pending_upd;
@@ -678,7 +686,7 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
     LayerPlan& lp = p.layers[l];
     Task t;
     t.op.kind = OP_UPD; t.op.stream = S_COMPUTE; t.op.layer = l;
-    const int j = l % nDW;
+    const int j = dwi(l);
     uint64_t gkey = key(R_DW, j);
     if (N > 1) { t.op.grad = p.gsh[l % 2]; gkey = key(R_GSH, l % 2); }
     else t.op.grad = p.dw[j];
@@ -756,78 +764,99 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
   std::vector<int> bwd_order;
   for (int u = LU - 1; u >= 0; --u)
     for (int k = 0; k < p.user_count[u]; ++k) bwd_order.push_back(p.user_first[u] + k);
-  for (int l : bwd_order) {
+  auto bwd_task = [&](int l, int i, bool gfirst) {
     LayerPlan& lp = p.layers[l];
     const int in_buf = lp.user % 2, out_buf = (lp.user + 1) % 2;
-    const int j = l % nDW;
-    for (int i = 0; i < m; ++i) {
-      int slot = -1;
-      uint64_t wdev;
-      if (baseline || i == 0) wdev = weight_use(l, (int)tasks.size(), slot);
-      else { slot = bwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
-      bwd_wslot[l] = slot;
-      Task t;
-      t.op.kind = OP_BWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i; t.op.first = i == 0;
-      t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws; t.op.dw = p.dw[j];
-      t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
-      t.wr = {key(R_BND, out_buf, i), key(R_DW, j)};
-      if (i > 0) t.rd.push_back(key(R_DW, j));
-      if (lp.stash_res[i] >= 0) {
-        t.op.stash = (uint64_t)lp.stash_res[i];
-        t.rd.push_back(key(R_STASHRES, l, i));
-      } else {
-        int g = gnext;
-        gnext = (gnext + 1) % nG;
-        Item it;
-        it.need = (int)tasks.size();
-        // free staging slot AND the spill of this very stash already issued (read after write)
-        it.release = std::max(stage_last[g], spill_task[(size_t)l * m + i]);
-        Op h;
-        h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STASH; h.layer = l; h.mb = i;
-        h.hbuf = HB_STASH; h.hidx = (int64_t)l * m + i; h.dev = p.stage[g]; h.bytes = lp.g.st.total;
-        it.ops.push_back({h, {{key(H_STASH, l, i)}, {key(R_STAGE, g)}}});
-        items.push_back(it);
-        t.op.stash = p.stage[g];
-        t.rd.push_back(key(R_STAGE, g));
-        stage_last[g] = (int)tasks.size();
-      }
-      if (slot >= 0) wslot_last[slot] = (int)tasks.size();
-      if (i == m - 1 && N > 1) {
-        Op rs;
-        rs.kind = OP_REDUCESCATTER; rs.stream = S_COMM; rs.cat = CAT_GRAD; rs.layer = l;
-        rs.dev = p.dw[j]; rs.grad = p.gsh[l % 2]; rs.count = (uint64_t)lp.shard;
-        rs.bytes = (uint64_t)lp.shard * 4 * (N - 1);
-        t.post.push_back({rs, {{key(R_DW, j)}, {key(R_GSH, l % 2)}}});
-      }
-      if (baseline) {
-        // per-GPU virtualization swaps the layer's weights out again after every microbatch's
-        // backward (Fig. 5(b); clean, so the bytes are those already on the host), and
-        // parks the finished gradient on the host until the update at the end of the backward
-        if (slot >= 0) {
-          Op d;
-          d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
-          d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
-          t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
-        }
-        if (i == m - 1) {
-          const uint64_t gk = N > 1 ? key(R_GSH, l % 2) : key(R_DW, j);
-          Op d;
-          d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_GRAD; d.layer = l;
-          d.hbuf = HB_GRAD; d.hidx = l; d.dev = N > 1 ? p.gsh[l % 2] : p.dw[j]; d.bytes = (uint64_t)lp.shard * 4;
-          t.post.push_back({d, {{gk}, {key(H_GRAD, l)}}});
-        }
-      }
-      tasks.push_back(t);
-    }
-    if (!baseline) {
-      pending_upd.push_back(l);
-      while ((int)pending_upd.size() > p.upd_lag) {
-        emit_upd(pending_upd.front());
-        pending_upd.erase(pending_upd.begin());
-      }
+    const int j = dwi(l);
+    int slot = -1;
+    uint64_t wdev;
+    if (baseline || gfirst) wdev = weight_use(l, (int)tasks.size(), slot);
+    else { slot = bwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
+    bwd_wslot[l] = slot;
+    Task t;
+    t.op.kind = OP_BWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i; t.op.first = i == 0;
+    t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws; t.op.dw = p.dw[j];
+    t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
+    t.wr = {key(R_BND, out_buf, i), key(R_DW, j)};
+    if (i > 0) t.rd.push_back(key(R_DW, j));
+    if (lp.stash_res[i] >= 0) {
+      t.op.stash = (uint64_t)lp.stash_res[i];
+      t.rd.push_back(key(R_STASHRES, l, i));
     } else {
-      pending_upd.push_back(l);  // baseline: every update after the whole backward
+      int g = gnext;
+      gnext = (gnext + 1) % nG;
+      Item it;
+      it.need = (int)tasks.size();
+      // free staging slot AND the spill of this very stash already issued (read after write)
+      it.release = std::max(stage_last[g], spill_task[(size_t)l * m + i]);
+      Op h;
+      h.kind = OP_H2D; h.stream = S_H2D; h.cat = CAT_STASH; h.layer = l; h.mb = i;
+      h.hbuf = HB_STASH; h.hidx = (int64_t)l * m + i; h.dev = p.stage[g]; h.bytes = lp.g.st.total;
+      it.ops.push_back({h, {{key(H_STASH, l, i)}, {key(R_STAGE, g)}}});
+      items.push_back(it);
+      t.op.stash = p.stage[g];
+      t.rd.push_back(key(R_STAGE, g));
+      stage_last[g] = (int)tasks.size();
     }
+    if (slot >= 0) wslot_last[slot] = (int)tasks.size();
+    if (i == m - 1 && N > 1) {
+      Op rs;
+      rs.kind = OP_REDUCESCATTER; rs.stream = S_COMM; rs.cat = CAT_GRAD; rs.layer = l;
+      rs.dev = p.dw[j]; rs.grad = p.gsh[l % 2]; rs.count = (uint64_t)lp.shard;
+      rs.bytes = (uint64_t)lp.shard * 4 * (N - 1);
+      t.post.push_back({rs, {{key(R_DW, j)}, {key(R_GSH, l % 2)}}});
+    }
+    if (baseline) {
+      // per-GPU virtualization swaps the layer's weights out again after every microbatch's
+      // backward (Fig. 5(b); clean, so the bytes are those already on the host), and
+      // parks the finished gradient on the host until the update at the end of the backward
+      if (slot >= 0) {
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_WEIGHT; d.layer = l; d.mb = i;
+        d.hbuf = HB_WC; d.hidx = l; d.dev = wdev + (uint64_t)r * lp.shard * ts; d.bytes = (uint64_t)lp.shard * ts;
+        t.post.push_back({d, {{key(R_WSLOT, slot)}, {key(H_WC, l)}}});
+      }
+      if (i == m - 1) {
+        const uint64_t gk = N > 1 ? key(R_GSH, l % 2) : key(R_DW, j);
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_GRAD; d.layer = l;
+        d.hbuf = HB_GRAD; d.hidx = l; d.dev = N > 1 ? p.gsh[l % 2] : p.dw[j]; d.bytes = (uint64_t)lp.shard * 4;
+        t.post.push_back({d, {{gk}, {key(H_GRAD, l)}}});
+      }
+    }
+    tasks.push_back(t);
+  };
+  auto bwd_layer_done = [&](int l) {  // after the layer's last microbatch: its update, just in time
+  if (!baseline) {
+    pending_upd.push_back(l);
+    while ((int)pending_upd.size() > p.upd_lag) {
+      emit_upd(pending_upd.front());
+      pending_upd.erase(pending_upd.begin());
+    }
+  } else {
+    pending_upd.push_back(l);  // baseline: every update after the whole backward
+  }
+  };
+  // Microbatch groups (direction balance): group 0's forward, then each group's
+  // backward interleaved layer by layer with the next group's forward, so stash swap-ins (backward)
+  // and spills (forward) use both directions of the host link at once.  The microbatches stay in
+  // canonical order in every dW accumulation: the result is bit-identical for every G (reading c21).
+  auto fwd_group = [&](int g, int l) {
+    for (int i = g * mg; i < (g + 1) * mg; ++i) fwd_task(l, i, i == g * mg);
+  };
+  auto loss_group = [&](int g) {
+    for (int i = g * mg; i < (g + 1) * mg; ++i) loss_task(i);
+  };
+  for (int l = 0; l < L; ++l) fwd_group(0, l);
+  loss_group(0);
+  for (int g = 0; g < G; ++g) {
+    for (int k = 0; k < (int)bwd_order.size(); ++k) {
+      const int l = bwd_order[k];
+      for (int i = g * mg; i < (g + 1) * mg; ++i) bwd_task(l, i, i == g * mg);
+      if (g == G - 1) bwd_layer_done(l);
+      if (g + 1 < G) fwd_group(g + 1, k);
+    }
+    if (g + 1 < G) loss_group(g + 1);
   }
   for (int l : pending_upd) emit_upd(l);
 
@@ -1038,8 +1067,9 @@ GroupPlan make_plan_pp(const harmony_config& cfg, int N, int L, const harmony_la
   for (int l = 0; l < L; ++l) { G.layer_rank[l] = l % N; G.layer_local[l] = l / N; }
   // per-rank layout: the rank's layers as one stack of one rank (the update is not sharded: each layer
   // lives on one GPU), four activation buffers (A_in, A_out, G_in, G_out)
+  HM_CHECK(cfg.groups <= 1, HARMONY_E_UNSUPPORTED, "microbatch groups are a Harmony-DP schedule");
   harmony_config rc = cfg;
-  rc.world_size = 1; rc.rank = 0; rc.schedule = HARMONY_SCHED_HARMONY_DP;
+  rc.world_size = 1; rc.rank = 0; rc.schedule = HARMONY_SCHED_HARMONY_DP; rc.groups = 1;
   for (int r = 0; r < N; ++r) {
     std::vector<harmony_layer_desc> sub;
     for (int l = r; l < L; l += N) sub.push_back(descs[l]);

@@ -79,7 +79,7 @@ struct Plan {
   int n_bnd = 2;
   uint64_t tgt = 0, tgt_row_stride = 0;
   uint64_t ws = 0, ws_bytes = 0;
-  uint64_t dw[2] = {0, 0};
+  std::vector<uint64_t> dw;  // fp32 dW accumulators (two alternating when N > 1; one per layer with groups)
   uint64_t gsh[2] = {0, 0};
   uint64_t loss = 0, loss_scratch = 0, tstep = 0;  // tstep: device int holding Adam's t
   std::vector<uint64_t> wslot, sslot, stage;  // slot offsets

@@ -97,11 +97,15 @@ def test_transformer_plans_hazard_free_over_caps(policy, S, L, m):
 
 def test_cap_too_small_is_reported():
     cap = min_cap(MLP, **dict(CFG1))
+    s, ops = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap))
+    assert s.hazards == 0 and sum(o["kind"] == "FWD" for o in ops) == 4 * 4
+    # below the unsplit minimum the fp32 layers run as column panels (operator split, row a15) ...
+    s, ops = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap - 1))
+    assert s.hazards == 0 and sum(o["kind"] == "FWD" for o in ops) > 4 * 4
+    # ... until not even the activations and one panel fit
     with pytest.raises(H.HarmonyError) as e:
-        plan(MLP, **dict(CFG1, hbm_cap_bytes=cap - 1))
+        plan(MLP, **dict(CFG1, hbm_cap_bytes=cap // 8))
     assert e.value.code == H.HARMONY_E_CAP_TOO_SMALL
-    s, _ = plan(MLP, **dict(CFG1, hbm_cap_bytes=cap))
-    assert s.hazards == 0
 
 
 def test_harmony_dp_weight_swap_volume_is_3W():
@@ -288,3 +292,27 @@ def test_operator_split_column_panels_only_when_the_cap_forces_them():
     with pytest.raises(H.HarmonyError) as e:  # bf16 layers are not split: the cap is simply too small
         plan(descs, hbm_cap_bytes=int(base.min_working_set_bytes * 0.4), precision=1, **kw)
     assert e.value.code == H.HARMONY_E_CAP_TOO_SMALL
+
+
+@pytest.mark.parametrize("G", [2, 4])
+def test_microbatch_groups_interleave_backward_with_the_next_forward(G):
+    """SURVEY §8(d) direction balance: G microbatch groups; group g's backward is interleaved layer by
+    layer with group g+1's forward (stash fetches and spills on both host-link directions at once);
+    each layer's update follows the LAST group's backward; the plan stays race-free."""
+    descs = synth.transformer_stack(4, 128, 2, 128, True)
+    kw = dict(microbatches=4, microbatch_size=2, precision=1, stash_policy=0)
+    base, _ = plan(descs, hbm_cap_bytes=1 << 40, **kw)
+    s, ops = plan(descs, hbm_cap_bytes=int(base.min_working_set_bytes * 1.5), groups=G, **kw)
+    assert s.hazards == 0
+    comp = [(o["kind"], o["l"], o["i"]) for o in ops if o["stream"] == "compute"]
+    mg = 4 // G
+    first_bwd = next(k for k, c in enumerate(comp) if c[0] == "BWD")
+    assert all(c[2] < mg for c in comp[:first_bwd] if c[0] in ("FWD", "LOSS"))  # only group 0 before
+    # after the first backward, the next group's forward tasks appear between backward tasks
+    later_fwd = [k for k, c in enumerate(comp) if c[0] == "FWD" and c[2] >= mg]
+    assert later_fwd and later_fwd[0] > first_bwd and later_fwd[0] < max(k for k, c in enumerate(comp) if c[0] == "BWD")
+    for l in range(4):  # UPD(l) after every microbatch's backward of layer l
+        upd = next(k for k, c in enumerate(comp) if c[0] == "UPD" and c[1] == l)
+        assert all(k < upd for k, c in enumerate(comp) if c[0] == "BWD" and c[1] == l)
+    with pytest.raises(H.HarmonyError):
+        plan(descs, hbm_cap_bytes=0, groups=3, **kw)  # m % G != 0

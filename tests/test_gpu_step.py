@@ -295,3 +295,17 @@ def test_operator_split_panels_match_oracle_and_are_bitwise_the_unsplit_step(fra
     compare(split, run_oracle(descs, params, batches), 1e-5)
     whole, _ = run_gpu(descs, params, batches, hbm_cap_bytes=0, **kw)
     bitwise_equal(split, whole)
+
+
+@pytest.mark.parametrize("G", [2, 4])
+def test_microbatch_groups_are_bitwise_identical_to_one_group(G):
+    """Direction-balancing microbatch groups only reorder tasks: the microbatches keep their canonical
+    order in every dW accumulation, so any G gives the one-group step bit for bit (reading c21),
+    capped with stash spills (op-input stash policy) included."""
+    descs, params, batches, kw = tiny_transformer(True, 1, L=3, d=128, h=2, S=128, B=8, m=4)
+    s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, groups=G, **kw), descs, text_len=0)
+    cap = int(s.min_working_set_bytes * 1.3)
+    one, _ = run_gpu(descs, params, batches, hbm_cap_bytes=cap, **kw)
+    grouped, plan = run_gpu(descs, params, batches, hbm_cap_bytes=cap, groups=G, **kw)
+    assert grouped[0]["stats"]["h2d_stash_bytes"] > 0
+    bitwise_equal(one, grouped)
