@@ -328,7 +328,8 @@ def main():
     ap.add_argument("--schedule", default="harmony", choices=["harmony", "baseline"],
                     help="harmony: Harmony-DP; baseline: the paper's per-GPU-virtualization comparison (Fig. 5(b))")
     ap.add_argument("--tune", action="store_true",
-                    help="pick the microbatch count by the tuner (plan feasibility + 2 timed steps per candidate)")
+                    help="pick microbatches, groups and stash policy by the tuner (planner feasibility, a cost model, "
+                         "then 2 timed steps of the best-ranked candidates)")
     ap.add_argument("--microbatches", type=int, default=0,
                     help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--groups", type=int, default=1,
@@ -393,11 +394,15 @@ def main():
         from paper_conf_hotos_lipmk21_b200 import tuner
         Xt, Tt = synth.gen_batch(descs, B, 1, precision)
         Xt, Tt = torch.tensor(Xt, device=device), torch.tensor(Tt, device=device)
-        tcfg = dict(hbm_cap_bytes=wl["cap"], precision=precision, stash_policy=args.stash_policy if precision else 0,
-                    lr=1e-4)
-        res = tuner.tune_microbatches(descs, B, tcfg, tuner.measure_on_device(descs, params, Xt, Tt, tcfg))
-        m = res.best
-        tuning = res.as_dict()
+        tcfg = dict(hbm_cap_bytes=wl["cap"], precision=precision, lr=1e-4)
+        run = tuner.measure_on_device(descs, params, Xt, Tt, tcfg)
+        best, cands = tuner.tune(descs, B, tcfg, lambda mm, G, pol: run(mm, B // mm, groups=G, stash_policy=pol),
+                                 link_gbs=55.0)
+        m, args.groups, args.stash_policy = best.microbatches, best.groups, best.stash_policy
+        tuning = {"best": dict(microbatches=m, groups=best.groups, stash_policy=best.stash_policy),
+                  "candidates": [dict(m=c.microbatches, G=c.groups, policy=c.stash_policy, feasible=c.feasible,
+                                      pred_ms=None if c.pred_seconds is None else c.pred_seconds * 1e3,
+                                      ms=None if c.step_seconds is None else c.step_seconds * 1e3) for c in cands]}
         del Xt, Tt
         torch.cuda.empty_cache()
     cfg = dict(rank=rank, world_size=world, device=local, hbm_cap_bytes=wl["cap"], microbatches=m,

@@ -1,5 +1,5 @@
-"""Microbatch-size tuner (the paper's "task packing" knob: pack size and microbatch
-size per pass).
+"""Performance tuner (the paper's "memory-performance tango" and task-packing knobs,
+P:749-757, 783-810): microbatch count, microbatch groups (direction balance) and stash policy.
 
 The same global batch per GPU can be run as m microbatches of b = batch / m sequences.  Larger
 microbatches amortise every kernel's launch and tail cost; a wider microbatch also widens the
@@ -71,10 +71,71 @@ def tune_microbatches(descs, batch: int, cfg: dict, measure, cands=None) -> Tune
     return TuneResult(best.microbatches, trials)
 
 
+# ------------------------------------------------------------------------------------------------ (m, G, policy)
+@dataclass
+class Candidate:
+    microbatches: int
+    groups: int
+    stash_policy: int
+    feasible: bool = True
+    reason: str = ""
+    pred_seconds: float | None = None   # cost model (host-only plan + link / tensor rates)
+    step_seconds: float | None = None   # measured (top candidates only)
+
+    def key(self):
+        return (self.microbatches, self.groups, self.stash_policy)
+
+
+# executed GEMM FLOPs per algorithmic FLOP: block recompute re-runs the forward (without its last
+# projection, ~2/3 of it); policy 3 also skips the attention forward — the same to this model
+EXEC = {0: 1.0, 1: 1.0, 2: 1.0 + 1.0 / 3.0 * 0.67 + 0.1, 3: 1.0 + 1.0 / 3.0 * 0.67}
+
+
+def predict_seconds(summary, policy, groups, tflops=1000.0, link_gbs=55.0):
+    """The step time the plan implies: the slower of its GEMM work at `tflops` and its host traffic at
+    `link_gbs` per direction, where one group moves the forward's spills and the backward's fetches in
+    two phases (the sum) and G groups overlap all but 1/G of them (SURVEY §8(d) direction balance)."""
+    compute = summary.flops_per_step * EXEC.get(policy, 1.0) / (tflops * 1e12)
+    h2d, d2h = summary.pred_h2d_bytes / 1e9, summary.pred_d2h_bytes / 1e9
+    overlapped = max(h2d, d2h) + min(h2d, d2h) / groups
+    return max(compute, overlapped / link_gbs)
+
+
+def tune(descs, batch: int, cfg: dict, measure, ms=None, groups=(1, 2, 4), policies=(0, 2, 3), top=4,
+         **model) -> "tuple[Candidate, list]":
+    """The memory-performance tango: over microbatch count m, microbatch groups G and stash
+    policy, the planner says what fits the cap, a cost model ranks what fits, and the `top` best are
+    measured (`measure(m, G, policy)` -> seconds per step); the fastest measured wins.  The fp32 path
+    has no recompute policies (0 only)."""
+    if cfg.get("precision", 0) == 0:
+        policies = (0,)
+    cands = []
+    for m in (ms or candidates(batch)):
+        for G in groups:
+            if m % G:
+                continue
+            for pol in policies:
+                c = Candidate(m, G, pol)
+                try:
+                    s, _ = H.harmony_plan_dry(H.make_config(microbatches=m, microbatch_size=batch // m, groups=G,
+                                                            stash_policy=pol, **cfg), descs, text_len=0)
+                    c.pred_seconds = predict_seconds(s, pol, G, **model)
+                except H.HarmonyError as e:
+                    c.feasible, c.reason = False, str(e)
+                cands.append(c)
+    ok = sorted((c for c in cands if c.feasible), key=lambda c: (c.pred_seconds, -c.microbatches * 0 + c.groups))
+    if not ok:
+        raise H.HarmonyError(H.HARMONY_E_CAP_TOO_SMALL, "no (microbatches, groups, policy) fits the cap")
+    for c in ok[:top]:
+        c.step_seconds = float(measure(c.microbatches, c.groups, c.stash_policy))
+    best = min((c for c in ok if c.step_seconds is not None), key=lambda c: (c.step_seconds, c.groups))
+    return best, cands
+
+
 def measure_on_device(descs, params, X, T, cfg: dict, steps=2, warmup=1):
     """A `measure` callable: builds a context per candidate and returns its mean device step time."""
-    def run(m, b):
-        with H.Harmony(descs, params, microbatches=m, microbatch_size=b, **cfg) as h:
+    def run(m, b, **extra):
+        with H.Harmony(descs, params, microbatches=m, microbatch_size=b, **dict(cfg, **extra)) as h:
             for _ in range(warmup):
                 h.step(X, T)
             tot = 0.0

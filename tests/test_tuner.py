@@ -43,3 +43,29 @@ def test_tuner_breaks_ties_toward_larger_microbatches_and_raises_when_nothing_fi
     assert r.best == 1
     with pytest.raises(H.HarmonyError):
         tuner.tune_microbatches(descs, 32, dict(hbm_cap_bytes=1024), lambda m, b: 1.0)
+
+
+def test_tango_ranks_by_the_cost_model_and_measures_only_the_top():
+    """(m, G, policy): infeasible points are recorded, the feasible ones ranked by the plan-implied
+    time (GEMM work vs host traffic with direction balance), only the top few are measured."""
+    descs = synth.transformer_stack(4, 128, 2, 128, True)
+    cfg = dict(precision=1)
+    s, _ = H.harmony_plan_dry(H.make_config(microbatches=4, microbatch_size=2, stash_policy=2,
+                                            hbm_cap_bytes=1 << 40), descs, text_len=0)
+    cap = int(s.min_working_set_bytes * 1.6)
+    seen = []
+
+    def measure(m, G, pol):
+        seen.append((m, G, pol))
+        return 1.0 / m + 0.01 * G + 0.001 * pol
+
+    best, cands = tuner.tune(descs, 8, dict(cfg, hbm_cap_bytes=cap), measure, top=3)
+    feas = [c for c in cands if c.feasible]
+    assert len(seen) == min(3, len(feas)) and best.key() in seen
+    ranked = sorted(feas, key=lambda c: c.pred_seconds)
+    assert set(seen) == {c.key() for c in ranked[:3]}
+    assert all(c.pred_seconds > 0 for c in feas)
+    # more groups overlap the two host-link directions: never a worse prediction for the same plan bytes
+    s0, _ = H.harmony_plan_dry(H.make_config(microbatches=4, microbatch_size=2, stash_policy=0, hbm_cap_bytes=cap,
+                                             **cfg), descs, text_len=0)
+    assert tuner.predict_seconds(s0, 0, 4) <= tuner.predict_seconds(s0, 0, 1)
