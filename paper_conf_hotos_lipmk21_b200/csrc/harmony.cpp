@@ -22,6 +22,7 @@
 #include <memory>
 #include <stdexcept>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "comm.hpp"
@@ -98,6 +99,9 @@ struct harmony_ctx {
   bool one_device = true;               // group: every rank on the same GPU (loopback)
   cudaEvent_t lb_ready = nullptr, lb_done = nullptr;  // member: rendezvous of a group collective
   std::unique_ptr<GroupPlan> gplan;     // group under Harmony-PP: the one program of all ranks
+  // pageable inputs are copied here first (pinned), so the step still replays its CUDA graph
+  uint8_t* h_stage[2] = {nullptr, nullptr};
+  size_t h_stage_bytes[2] = {0, 0};
 };
 
 namespace {
@@ -190,6 +194,8 @@ void destroy(harmony_ctx* c) {
   for (auto p : c->h_grad) free_host(p);
   free_host(c->h_loss);
   free_host(c->h_gather);
+  free_host(c->h_stage[0]);
+  free_host(c->h_stage[1]);
   delete c;
 }
 
@@ -258,6 +264,21 @@ PtrKind ptr_kind(const void* p) {
   if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return PTR_DEVICE;
   if (a.type == cudaMemoryTypeHost) return PTR_PINNED;
   return PTR_PAGEABLE;
+}
+
+// Host copy on a few threads (pageable -> pinned staging of the step's inputs).
+void parallel_memcpy(void* dst, const void* src, size_t n) {
+  const size_t chunk = 16u << 20;
+  const int nt = (int)std::min<size_t>(8, (n + chunk - 1) / chunk);
+  if (nt <= 1) { memcpy(dst, src, n); return; }
+  std::vector<std::thread> th;
+  const size_t per = (n + nt - 1) / nt;
+  for (int i = 0; i < nt; ++i) {
+    const size_t lo = (size_t)i * per, hi = std::min(n, lo + per);
+    if (lo >= hi) break;
+    th.emplace_back([=] { memcpy(static_cast<char*>(dst) + lo, static_cast<const char*>(src) + lo, hi - lo); });
+  }
+  for (auto& t : th) t.join();
 }
 
 // This rank's view of the step's user inputs.
@@ -621,9 +642,34 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     r->t = t_next;  // the value the update kernels of this step read (reverted below on failure)
     *r->h_step = t_next;
   }
-  const PtrKind xk = ptr_kind(x), tk = ptr_kind(tg);
-  std::vector<RankIn> in(NR);
+  PtrKind xk = ptr_kind(x), tk = ptr_kind(tg);
   const bool pp = c->gplan != nullptr;  // Harmony-PP: the whole batch enters at rank 0, targets at the last rank
+  {  // pageable host inputs: staged into pinned buffers (parallel host copy), then the graph replays
+    static const bool stage = [] {
+      const char* e = getenv("HARMONY_PAGEABLE_STAGE");
+      return !(e && *e == '0');
+    }();
+    const size_t rows = (size_t)(pp ? 1 : NR) * p0.m;
+    const size_t nb[2] = {rows * p0.in_elems_per_mb * 4, rows * p0.out_elems_per_mb * 4};
+    const float* src[2] = {x, tg};
+    PtrKind* kinds[2] = {&xk, &tk};
+    bool staged[2] = {false, false};
+    for (int q = 0; q < 2 && stage; ++q) {
+      if (*kinds[q] != PTR_PAGEABLE) continue;
+      staged[q] = true;
+      if (c->h_stage_bytes[q] < nb[q]) {
+        free_host(c->h_stage[q]);
+        c->h_stage[q] = nullptr;
+        c->h_stage[q] = static_cast<uint8_t*>(alloc_host(nb[q]));
+        c->h_stage_bytes[q] = nb[q];
+      }
+      parallel_memcpy(c->h_stage[q], src[q], nb[q]);
+      *kinds[q] = PTR_PINNED;
+    }
+    if (staged[0]) x = reinterpret_cast<const float*>(c->h_stage[0]);
+    if (staged[1]) tg = reinterpret_cast<const float*>(c->h_stage[1]);
+  }
+  std::vector<RankIn> in(NR);
   for (int r = 0; r < NR; ++r) {
     in[r].x = pp ? x : x + (size_t)r * p0.m * p0.in_elems_per_mb;
     in[r].tg = pp ? tg : tg + (size_t)r * p0.m * p0.out_elems_per_mb;

@@ -288,6 +288,29 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
   return p;
 }
 
+// One warp writes a staged 32-row x 128-byte box (128B-swizzled) to global memory with coalesced
+// 16-byte stores (8 lanes per 128-byte row) — the LSU path instead of a TMA store, which leaves the
+// TMA unit to the mainloop's loads.  Rows / columns past M / N are not written.
+template <int ESZ>
+__device__ __forceinline__ void warp_store_box(void* base, int64_t ld, uint32_t sb, int row0, int n, int M, int N,
+                                               int lane) {
+  constexpr int EPC = 16 / ESZ;  // elements per 16-byte chunk
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int idx = it * 32 + lane, r = idx >> 3, k = idx & 7;
+    const int grow = row0 + r, gcol = n + k * EPC;
+    if (grow >= M || gcol >= N) continue;
+    const uint4 v = lds128(sb + swz128(r, k));
+    char* dst = static_cast<char*>(base) + ((int64_t)grow * ld + gcol) * ESZ;
+    if (gcol + EPC <= N) {
+      *reinterpret_cast<uint4*>(dst) = v;
+    } else {
+      const char* src = reinterpret_cast<const char*>(&v);
+      for (int q = 0; q < (N - gcol) * ESZ; ++q) dst[q] = src[q];
+    }
+  }
+}
+
 // Is the TMA epilogue usable for this epilogue kind / tile width (host and device agree)?
 __host__ __device__ __forceinline__ bool tma_epi_kind_ok(int epi) { return epi != HK_EPI_BIAS_ACT_F32; }
 
@@ -417,9 +440,18 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
         sts128(ad, o[0], o[1], o[2], o[3]);
       }
     }
-    fence_proxy_async_smem();
-    __syncwarp();
-    if (lane == 0 && !(p.diag & 4)) {
+    const bool lsu = p.diag & 16;  // experiment: LSU stores instead of TMA stores
+    const int64_t zoff_c = (int64_t)z0 * e.c_sz0 + (int64_t)z1 * e.c_sz1;
+    if (lsu) {
+      __syncwarp();
+      warp_store_box<ESZ>(static_cast<char*>(e.C) + zoff_c * ESZ, e.ldc, sb, row0, n, e.M, e.N, lane);
+      fence_proxy_async_smem();  // these generic reads before a later TMA load into the buffer
+      __syncwarp();
+    } else {
+      fence_proxy_async_smem();
+      __syncwarp();
+    }
+    if (!lsu && lane == 0 && !(p.diag & 4)) {
       if (p.diag & 8) tma_store_box_hint(mC, sb, n, row0, z0, z1, policy_evict_first());
       else tma_store_box(mC, sb, n, row0, z0, z1);
       bulk_commit();
@@ -440,6 +472,15 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
           g[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
         }
         sts128(w.buf + EPI_BUF + swz128(r, k), g[0], g[1], g[2], g[3]);
+      }
+      if (lsu) {
+        __syncwarp();
+        warp_store_box<ESZ>(static_cast<char*>(e.aux_out) + zoff_c * ESZ, e.ldc, w.buf + EPI_BUF, row0, n, e.M, e.N,
+                            lane);
+        fence_proxy_async_smem();
+        __syncwarp();
+        ++w.j;
+        continue;
       }
       fence_proxy_async_smem();
       __syncwarp();

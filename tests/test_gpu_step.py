@@ -259,11 +259,20 @@ def test_step_errors():
 
 def test_graph_replay_equals_eager_and_tracks_input_pointers():
     """Pinned or device inputs replay the captured CUDA graph (input copy nodes re-pointed every
-    step); pageable inputs run the same program eagerly.  Both are bit-identical."""
+    step); pageable inputs are staged into pinned buffers and replay it too; HARMONY_NO_GRAPH=1 issues
+    the same program eagerly.  All bit-identical."""
     descs, params, batches, kw = tiny_transformer(True, 1, L=2, d=64, h=2, S=64, B=4, m=2)
     s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, **kw), descs, text_len=0)
     kw["hbm_cap_bytes"] = int(s.min_working_set_bytes * 1.3)
-    eager, _ = run_gpu(descs, params, batches, **kw)
+    os.environ["HARMONY_NO_GRAPH"] = "1"
+    try:
+        eager, _ = run_gpu(descs, params, batches, **kw)
+    finally:
+        del os.environ["HARMONY_NO_GRAPH"]
+    assert eager[0]["stats"]["graph"] == 0
+    staged, _ = run_gpu(descs, params, batches, **kw)  # pageable numpy inputs
+    assert staged[0]["stats"]["graph"] == 1
+    bitwise_equal(eager, staged)
     pinned = [(torch.tensor(X).pin_memory(), torch.tensor(T).pin_memory()) for X, T in batches]
     res = []
     with H.Harmony(descs, params, retain_grads=1, **kw) as h:

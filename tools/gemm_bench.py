@@ -74,6 +74,11 @@ def shapes():
     lin_wgrad("fc1_wgrad", 4 * D, D)
     lin_wgrad("out_wgrad", D, D)
     lin_wgrad("qkv_wgrad", 3 * D, D)
+    # the d x d weight gradient as the step runs it: S token slices (batched) into fp32 partials
+    for S_ in (2, 4, 8):
+        ks = T // S_
+        g(f"out_wgrad_split{S_}", D, D, ks, X, 1, D, X, 1, D, C32, D, H.HK_EPI_STORE_F32, nz0=S_,
+          a_sz0=ks * D, b_sz0=ks * D, c_sz0=D * D)
     return out, (x, w, qkv, p, c32, c16, keep)
 
 
