@@ -624,8 +624,13 @@ void capture_graph(harmony_ctx* c, StepGraph& G, const std::vector<RankIn>& in, 
     cudaMemcpy3DParms mp;
     HM_CUDA(cudaGraphMemcpyNodeGetParams(nd, &mp));
     const uint8_t* dst = static_cast<const uint8_t*>(mp.dstPtr.ptr);
-    for (auto& e : G.in_nodes)
-      if (dst == R[e.rank]->arena + e.op->dev) e.node = nd;
+    const uint8_t* srcp = static_cast<const uint8_t*>(mp.srcPtr.ptr);
+    for (auto& e : G.in_nodes) {  // destination AND source: other copies may land in the same rows
+      const uint8_t* want = reinterpret_cast<const uint8_t*>(e.op->hbuf == HB_USER_X ? (const void*)in[e.rank].x
+                                                                                    : (const void*)in[e.rank].tg) +
+                            e.op->hoff;
+      if (dst == R[e.rank]->arena + e.op->dev && srcp == want) e.node = nd;
+    }
   }
   for (auto& e : G.in_nodes) HM_CHECK(e.node != nullptr, HARMONY_E_CUDA, "graph capture: input copy node not found");
   G.sig = (in[0].x_dev ? 1 : 0) | (in[0].t_dev ? 2 : 0);
