@@ -495,6 +495,30 @@ def main():
     t_strict = max(h2d / (bw["h2d"] * 1e9), d2h / (bw["d2h"] * 1e9), (h2d + d2h) / (bw["duplex"] * 1e9))
     t_lenient = (h2d + d2h) / (max(bw["h2d"], bw["d2h"]) * 1e9)
     t_roof = max(t_gemm, t_strict)
+    # the roofline GIVEN THE CAP: the cap decides how much must be stashed, swapped or recomputed, so
+    # take the best stash policy's max(executed GEMM FLOPs at peak, its planned swap bytes at the link)
+    cap_aware = None
+    if precision == 1 and descs[0].kind == synth.LAYER_TRANSFORMER and world == 1:
+        d0, S0, L0 = descs[0].d_in, descs[0].seq_len, len(descs)
+        Tm = (B // m) * S0
+        recomp = {2: 16.0 * Tm * d0 * d0 + 4.0 * (B // m) * S0 * S0 * d0, 3: 16.0 * Tm * d0 * d0}
+        per = {}
+        for pol in (0, 1, 2, 3):
+            try:
+                sp, _ = H.harmony_plan_dry(H.make_config(**dict(cfg, stash_policy=pol, arena=None)), descs, text_len=0)
+            except H.HarmonyError:
+                continue
+            fx = F + recomp.get(pol, 0.0) * m * L0
+            tg = fx / (peaks["bf16_tflops"] * 1e12)
+            hh, dd = sp.pred_h2d_bytes, sp.pred_d2h_bytes
+            ts = max(hh / (bw["h2d"] * 1e9), dd / (bw["d2h"] * 1e9), (hh + dd) / (bw["duplex"] * 1e9))
+            per[pol] = {"t_ms": max(tg, ts) * 1e3, "t_gemm_ms": tg * 1e3, "t_swap_ms": ts * 1e3, "exec_flops": fx}
+        if per:
+            best = min(per, key=lambda k: per[k]["t_ms"])
+            cap_aware = {"t_roof_ms": per[best]["t_ms"], "policy": best, "frac": per[best]["t_ms"] / ms,
+                         "per_policy": per,
+                         "note": "min over stash policies of max(executed GEMM FLOPs / burst peak, planned swap bytes "
+                                 "at the measured host link) under this cap"}
     g = prof["gemm"]
     gemm_tflops = g["work"] / g["seconds"] / 1e12 if g["seconds"] else 0.0
     gemm_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
@@ -537,7 +561,7 @@ def main():
                           "frac_lenient": max(t_gemm, t_lenient) / (dev_s / args.steps),
                           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                           "swap_gbs": (h2d + d2h) / (dev_s / args.steps) / 1e9,
-                          "host_link_gbs_measured": bw, "flops_per_step": F},
+                          "host_link_gbs_measured": bw, "flops_per_step": F, "cap_aware": cap_aware},
         "kernels": {k: dict(v, per_launch_us=(v["seconds"] / v["launches"] * 1e6 if v["launches"] else None))
                     for k, v in prof.items()},
         "attention": {"achieved_tflops": (prof["attention"]["work"] / prof["attention"]["seconds"] / 1e12
