@@ -143,6 +143,38 @@ def host_link_bandwidth(torch, device):
     return out
 
 
+def nvlink_probe(torch, dist, device, layer_params, world, reps=10):
+    """Phase 0 of SURVEY §8(d) at N > 1: NCCL reduce-scatter (fp32) and all-gather (bf16) bus bandwidth at
+    the step's per-layer message sizes, all ranks at once (a separate NCCL group; max time over ranks)."""
+    g = dist.new_group(backend="nccl")
+    n = (layer_params + world * 1024 - 1) // (world * 1024) * (world * 1024)
+    out = {}
+    for name, dt, op in (("reduce_scatter_f32", torch.float32, "rs"), ("all_gather_bf16", torch.bfloat16, "ag")):
+        full = torch.ones(n, dtype=dt, device=device)
+        shard = torch.empty(n // world, dtype=dt, device=device)
+        def run():
+            if op == "rs":
+                dist.reduce_scatter_tensor(shard, full, group=g)
+            else:
+                dist.all_gather_into_tensor(full, shard, group=g)
+        for _ in range(3):
+            run()
+        torch.cuda.synchronize(device)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        dist.barrier(group=g)
+        e0.record()
+        for _ in range(reps):
+            run()
+        e1.record()
+        torch.cuda.synchronize(device)
+        t = torch.tensor([e0.elapsed_time(e1) / reps / 1e3], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        sec = t.item()
+        nbytes = n * full.element_size()
+        out[name] = {"bytes": nbytes, "us": sec * 1e6, "busbw_gbs": nbytes * (world - 1) / world / sec / 1e9}
+    return out
+
+
 def oracle_step_work(wl, batch=1):
     """One complete oracle training step of the workload's full stack (every layer: forward, the
     loss, backward, Adam) on `batch` sequences, as a list of work items in the step's order (the
@@ -429,10 +461,15 @@ def main():
     # the slowest rank's figures bound the step
     barrier()
     bw = host_link_bandwidth(torch, device)
+    nvlink = None
     if dist is not None:
         t = torch.tensor([-bw["h2d"], -bw["d2h"], -bw["duplex"]], dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         bw = {"h2d": -t[0].item(), "d2h": -t[1].item(), "duplex": -t[2].item(), "ranks": world}
+        try:
+            nvlink = nvlink_probe(torch, dist, device, descs[0].n_params(), world)
+        except Exception as e:  # the probe is informative only
+            nvlink = {"error": str(e)[:200]}
     for _ in range(args.warmup):
         h.step(Xd, Td)
     # ---- timed region: device-resident inputs, CUDA-graph replay of the step program
@@ -561,7 +598,8 @@ def main():
                           "frac_lenient": max(t_gemm, t_lenient) / (dev_s / args.steps),
                           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                           "swap_gbs": (h2d + d2h) / (dev_s / args.steps) / 1e9,
-                          "host_link_gbs_measured": bw, "flops_per_step": F, "cap_aware": cap_aware},
+                          "host_link_gbs_measured": bw, "flops_per_step": F, "cap_aware": cap_aware,
+                          "nvlink_phase0": nvlink},
         "kernels": {k: dict(v, per_launch_us=(v["seconds"] / v["launches"] * 1e6 if v["launches"] else None))
                     for k, v in prof.items()},
         "attention": {"achieved_tflops": (prof["attention"]["work"] / prof["attention"]["seconds"] / 1e12

@@ -128,3 +128,15 @@ def test_group_errors():
         with pytest.raises(H.HarmonyError) as e:
             H.harmony_set_profiling(h.ctx, 1)
         assert e.value.code == H.HARMONY_E_UNSUPPORTED
+
+
+def test_group_with_microbatch_groups_is_bitwise_one_group():
+    """N = 2 ranks sharing the GPU, each with G = 2 microbatch groups: bit-identical to G = 1 (the
+    groups only reorder tasks; the reduce-scatter still follows each layer's last microbatch)."""
+    descs = CFG1["descs"]()
+    params = synth.gen_params(descs)
+    batches = batches_for(descs, 2 * 32, 2, 0)
+    kw = dict(microbatches=4, microbatch_size=8, group=[0, 0], hbm_cap_bytes=CFG1["cap"])
+    a, _ = run_gpu(descs, params, batches, **kw)
+    b, _ = run_gpu(descs, params, batches, groups=2, **kw)
+    bitwise_equal(a, b)
