@@ -85,12 +85,19 @@ def test_group_of_one_is_bitwise_the_single_rank_context():
 
 def test_group_graph_replay_equals_eager():
     """Pinned inputs: the N ranks' programs are captured as ONE CUDA graph (every rank's streams and
-    the collectives' rendezvous events) and replayed; pageable inputs issue the same program eagerly."""
+    the collectives' rendezvous events) and replayed; HARMONY_NO_GRAPH=1 issues the same program
+    eagerly.  Bit-identical."""
+    import os
     N = 2
     descs, params, _, kw = tiny_transformer(True, 1, L=2, d=64, h=2, S=64, B=4, m=2)
     batches = batches_for(descs, N * 4, 3, 1)
     kw["group"] = [0] * N
-    eager, _ = run_gpu(descs, params, batches, **kw)
+    os.environ["HARMONY_NO_GRAPH"] = "1"
+    try:
+        eager, _ = run_gpu(descs, params, batches, **kw)
+    finally:
+        del os.environ["HARMONY_NO_GRAPH"]
+    assert eager[0]["stats"]["graph"] == 0
     res = []
     with H.Harmony(descs, params, retain_grads=1, **kw) as h:
         for X, T in batches:
