@@ -37,7 +37,7 @@ import synth  # noqa: E402
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 # per-launch DRAM traffic of the roofline kernel class, from the committed ncu launch list of the
 # same step (tools/traffic_summary.py); ncu replays cold, so this is the no-L2-reuse upper end
-TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r01_traffic_cfg2_m2.json")}
+TRAFFIC_FILES = {"cfg2": os.path.join(ROOT, "profiles", "r02_traffic_cfg2_m2.json")}
 FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
 
 WORKLOADS = {
@@ -427,9 +427,9 @@ def main():
         Xt, Tt = synth.gen_batch(descs, B, 1, precision)
         Xt, Tt = torch.tensor(Xt, device=device), torch.tensor(Tt, device=device)
         tcfg = dict(hbm_cap_bytes=wl["cap"], precision=precision, lr=1e-4)
-        run = tuner.measure_on_device(descs, params, Xt, Tt, tcfg)
+        run = tuner.measure_on_device(descs, params, Xt, Tt, tcfg, steps=3, warmup=2)
         best, cands = tuner.tune(descs, B, tcfg, lambda mm, G, pol: run(mm, B // mm, groups=G, stash_policy=pol),
-                                 link_gbs=55.0)
+                                 incumbent=(m, args.groups, args.stash_policy if precision else 0), link_gbs=55.0)
         m, args.groups, args.stash_policy = best.microbatches, best.groups, best.stash_policy
         tuning = {"best": dict(microbatches=m, groups=best.groups, stash_policy=best.stash_policy),
                   "candidates": [dict(m=c.microbatches, G=c.groups, policy=c.stash_policy, feasible=c.feasible,

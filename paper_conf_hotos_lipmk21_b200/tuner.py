@@ -102,11 +102,13 @@ def predict_seconds(summary, policy, groups, tflops=1000.0, link_gbs=55.0):
 
 
 def tune(descs, batch: int, cfg: dict, measure, ms=None, groups=(1, 2, 4), policies=(0, 2, 3), top=4,
-         **model) -> "tuple[Candidate, list]":
+         per_policy=2, incumbent=None, **model) -> "tuple[Candidate, list]":
     """The memory-performance tango: over microbatch count m, microbatch groups G and stash
-    policy, the planner says what fits the cap, a cost model ranks what fits, and the `top` best are
-    measured (`measure(m, G, policy)` -> seconds per step); the fastest measured wins.  The fp32 path
-    has no recompute policies (0 only)."""
+    policy, the planner says what fits the cap, a cost model ranks what fits, and the best-ranked are
+    measured (`measure(m, G, policy)` -> seconds per step); the fastest measured wins.  The model only
+    ranks (it knows GEMM work and host traffic, not kernel efficiency), so the measured set takes at
+    most `per_policy` candidates of each stash policy (up to `top` in all) plus the `incumbent`
+    (m, G, policy) when given.  The fp32 path has no recompute policies (0 only)."""
     if cfg.get("precision", 0) == 0:
         policies = (0,)
     cands = []
@@ -123,10 +125,21 @@ def tune(descs, batch: int, cfg: dict, measure, ms=None, groups=(1, 2, 4), polic
                 except H.HarmonyError as e:
                     c.feasible, c.reason = False, str(e)
                 cands.append(c)
-    ok = sorted((c for c in cands if c.feasible), key=lambda c: (c.pred_seconds, -c.microbatches * 0 + c.groups))
+    ok = sorted((c for c in cands if c.feasible), key=lambda c: (c.pred_seconds, c.groups))
     if not ok:
         raise H.HarmonyError(H.HARMONY_E_CAP_TOO_SMALL, "no (microbatches, groups, policy) fits the cap")
-    for c in ok[:top]:
+    chosen, taken = [], {}
+    for c in ok:
+        if len(chosen) >= top:
+            break
+        if taken.get(c.stash_policy, 0) < per_policy:
+            chosen.append(c)
+            taken[c.stash_policy] = taken.get(c.stash_policy, 0) + 1
+    if incumbent is not None:
+        inc = next((c for c in ok if c.key() == tuple(incumbent)), None)
+        if inc is not None and inc not in chosen:
+            chosen.append(inc)
+    for c in chosen:
         c.step_seconds = float(measure(c.microbatches, c.groups, c.stash_policy))
     best = min((c for c in ok if c.step_seconds is not None), key=lambda c: (c.step_seconds, c.groups))
     return best, cands

@@ -59,11 +59,17 @@ def test_tango_ranks_by_the_cost_model_and_measures_only_the_top():
         seen.append((m, G, pol))
         return 1.0 / m + 0.01 * G + 0.001 * pol
 
-    best, cands = tuner.tune(descs, 8, dict(cfg, hbm_cap_bytes=cap), measure, top=3)
+    best, cands = tuner.tune(descs, 8, dict(cfg, hbm_cap_bytes=cap), measure, top=3, per_policy=1,
+                             incumbent=(2, 1, 2))
     feas = [c for c in cands if c.feasible]
-    assert len(seen) == min(3, len(feas)) and best.key() in seen
-    ranked = sorted(feas, key=lambda c: c.pred_seconds)
-    assert set(seen) == {c.key() for c in ranked[:3]}
+    assert best.key() in seen and (2, 1, 2) in seen  # the incumbent is always measured
+    pols = [k[2] for k in seen if k != (2, 1, 2)]
+    assert len(pols) == len(set(pols)) <= 3  # at most one per stash policy (per_policy=1)
+    for k in seen:  # each measured non-incumbent candidate is its policy's best prediction
+        if k == (2, 1, 2):
+            continue
+        c = next(c for c in feas if c.key() == k)
+        assert c.pred_seconds == min(x.pred_seconds for x in feas if x.stash_policy == k[2])
     assert all(c.pred_seconds > 0 for c in feas)
     # more groups overlap the two host-link directions: never a worse prediction for the same plan bytes
     s0, _ = H.harmony_plan_dry(H.make_config(microbatches=4, microbatch_size=2, stash_policy=0, hbm_cap_bytes=cap,

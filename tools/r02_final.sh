@@ -12,7 +12,7 @@ timeout 1200 python bench.py --workload cfg4s --no-cpu-baseline --steps 3 > gpur
 timeout 600 python bench.py --workload cfg1 --no-cpu-baseline > gpurun_out/r02_final_cfg1.json 2> gpurun_out/r02_final_cfg1.err; echo "cfg1 $?"
 timeout 900 python bench.py --workload cfg5 --steps 3 > gpurun_out/r02_final_cfg5.json 2> gpurun_out/r02_final_cfg5.err; echo "cfg5 $?"
 timeout 1500 python bench.py --tune --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/r02_final_cfg2_tuned.json 2> gpurun_out/r02_final_cfg2_tuned.err; echo "tune $?"
-/usr/bin/time -f "ref wall %e s" timeout 1500 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/r02_final_ref.json 2> gpurun_out/r02_final_ref.err; echo "ref $?"; tail -1 gpurun_out/r02_final_ref.err
+SECONDS=0; timeout 1500 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/r02_final_ref.json 2> gpurun_out/r02_final_ref.err; echo "ref $? wall ${SECONDS}s"; tail -1 gpurun_out/r02_final_ref.err
 for f in cfg2 cfg3 cfg4s cfg1 cfg5 cfg2_tuned ref; do python -c "
 import json
 d=json.loads(open('gpurun_out/r02_final_$f.json').read().strip().splitlines()[-1])
