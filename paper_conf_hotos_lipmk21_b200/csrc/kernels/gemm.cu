@@ -109,12 +109,13 @@ __device__ __forceinline__ uint32_t make_idesc(int bn, int a_mn, int b_mn) { ret
 
 // Epilogue inputs read from global memory: 1 = fp32 residual (aux), 2 = old fp32 C (dW accumulate),
 // 3 = bf16 stored pre-activation (aux of ACT_BWD), 0 = none.
-__device__ __forceinline__ int epi_in_kind(const EpiParams& e) {
-  if (e.epi == HK_EPI_RESID_F32) return 1;
-  if (e.epi == HK_EPI_ACC_F32 && e.accumulate) return 2;
-  if (e.epi == HK_EPI_ACT_BWD) return 3;
+__device__ __forceinline__ int epi_in_kind(const EpiParams& e, int epi) {
+  if (epi == HK_EPI_RESID_F32) return 1;
+  if (epi == HK_EPI_ACC_F32 && e.accumulate) return 2;
+  if (epi == HK_EPI_ACT_BWD) return 3;
   return 0;
 }
+__device__ __forceinline__ int epi_in_kind(const EpiParams& e) { return epi_in_kind(e, e.epi); }
 
 // L2 prefetch of this thread's row segment [n_beg, n_end) of the epilogue input, issued before the
 // accumulator wait so the (cold, HBM) residual / dW / pre-activation read overlaps the mainloop.
@@ -315,20 +316,24 @@ __device__ __forceinline__ void warp_store_box(void* base, int64_t ld, uint32_t 
 __host__ __device__ __forceinline__ bool tma_epi_kind_ok(int epi) { return epi != HK_EPI_BIAS_ACT_F32; }
 
 // One warp's share of one tile: 32 rows (row0..) x columns [n_beg, n_end) (n_end - n_beg <= 128),
-// TMEM columns from tacc.  ESZ = output element size (4: fp32 outputs, 2: bf16 outputs).
-template <int ESZ>
+// TMEM columns from tacc.  ESZ = output element size (4: fp32 outputs, 2: bf16 outputs).  EK >= 0:
+// the epilogue kind fixed at compile time (only its code is emitted, no diagnostics); -1: read
+// from the parameters (every kind and the HARMONY_GEMM_DIAG experiments in one body).
+template <int ESZ, int EK = -1>
 __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMap* mC, const CUtensorMap* mIn,
                                              const CUtensorMap* mO2, EpiWarp& w, uint32_t tacc, bool have_acc,
                                              int lane, int row0, int n_beg, int n_end, int z0, int z1,
                                              uint64_t* full_bar, uint32_t full_par) {
   constexpr int CPB = 128 / ESZ;  // columns per box
   const EpiParams& e = p.e;
-  const int kind = epi_in_kind(e);
-  const bool two = e.epi == HK_EPI_BIAS_ACT;
+  const int epi = EK >= 0 ? EK : e.epi;
+  const int diag = EK >= 0 ? 0 : p.diag;
+  const int kind = epi_in_kind(e, epi);
+  const bool two = epi == HK_EPI_BIAS_ACT;
   const int nbox = n_end > n_beg ? (n_end - n_beg + CPB - 1) / CPB : 0;
-  const bool has_bias = e.bias != nullptr && (e.epi == HK_EPI_STORE_T || e.epi == HK_EPI_BIAS_ACT ||
-                                              e.epi == HK_EPI_ACT_T || e.epi == HK_EPI_STORE_F32 ||
-                                              e.epi == HK_EPI_RESID_F32);
+  const bool has_bias = e.bias != nullptr && (epi == HK_EPI_STORE_T || epi == HK_EPI_BIAS_ACT ||
+                                              epi == HK_EPI_ACT_T || epi == HK_EPI_STORE_F32 ||
+                                              epi == HK_EPI_RESID_F32);
   if (kind && nbox > 0 && lane == 0) {
     const int b = w.j & 1;
     bulk_wait_read<1>();  // the store two boxes back has left this box
@@ -362,7 +367,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       bulk_wait_read<1>();
     }
     float v[CPB];
-    if (have_acc && !(p.diag & 2)) {
+    if (have_acc && !(diag & 2)) {
 #pragma unroll
       for (int h = 0; h < CPB / 32; ++h) tmem_ld32(tacc + CPB * bi + 32 * h, v + 32 * h);
     } else {
@@ -382,12 +387,12 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
         const uint32_t ad = sb + swz128(r, k);
         float o0 = e.alpha * v[4 * k], o1 = e.alpha * v[4 * k + 1], o2 = e.alpha * v[4 * k + 2],
               o3 = e.alpha * v[4 * k + 3];
-        if (e.epi == HK_EPI_RESID_F32) {  // C = aux + (acc + b)
+        if (epi == HK_EPI_RESID_F32) {  // C = aux + (acc + b)
           float4 bb = has_bias ? lds128f(bias_row + 16 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
           const float4 in = lds128f(ad);
           o0 = in.x + (v[4 * k] + bb.x); o1 = in.y + (v[4 * k + 1] + bb.y);
           o2 = in.z + (v[4 * k + 2] + bb.z); o3 = in.w + (v[4 * k + 3] + bb.w);
-        } else if (e.epi == HK_EPI_ACC_F32) {  // C (+)= alpha * acc
+        } else if (epi == HK_EPI_ACC_F32) {  // C (+)= alpha * acc
           if (kind) {
             const float4 in = lds128f(ad);
             o0 = in.x + o0; o1 = in.y + o1; o2 = in.z + o2; o3 = in.w + o3;
@@ -404,7 +409,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
         const uint32_t ad = sb + swz128(r, k);
         const float* x = v + 8 * k;
         uint32_t o[4];
-        if (e.epi == HK_EPI_ACT_BWD) {  // dH = dG * act'(H)
+        if (epi == HK_EPI_ACT_BWD) {  // dH = dG * act'(H)
           const uint4 in = lds128(ad);
           const uint32_t hw[4] = {in.x, in.y, in.z, in.w};
 #pragma unroll
@@ -421,11 +426,11 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
 #pragma unroll
             for (int t = 0; t < 8; ++t) bb[t] = 0.f;
           }
-          if (e.epi == HK_EPI_STORE_T) {
+          if (epi == HK_EPI_STORE_T) {
 #pragma unroll
             for (int t = 0; t < 4; ++t)
               o[t] = pack_bf16(e.alpha * x[2 * t] + bb[2 * t], e.alpha * x[2 * t + 1] + bb[2 * t + 1]);
-          } else if (e.epi == HK_EPI_ACT_T) {  // G = act(H as it would be stored), H not written
+          } else if (epi == HK_EPI_ACT_T) {  // G = act(H as it would be stored), H not written
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
               const uint32_t hz = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
@@ -440,7 +445,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
         sts128(ad, o[0], o[1], o[2], o[3]);
       }
     }
-    const bool lsu = p.diag & 16;  // experiment: LSU stores instead of TMA stores
+    const bool lsu = diag & 16;  // experiment: LSU stores instead of TMA stores
     const int64_t zoff_c = (int64_t)z0 * e.c_sz0 + (int64_t)z1 * e.c_sz1;
     if (lsu) {
       __syncwarp();
@@ -451,8 +456,8 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       fence_proxy_async_smem();
       __syncwarp();
     }
-    if (!lsu && lane == 0 && !(p.diag & 4)) {
-      if (p.diag & 8) tma_store_box_hint(mC, sb, n, row0, z0, z1, policy_evict_first());
+    if (!lsu && lane == 0 && !(diag & 4)) {
+      if (diag & 8) tma_store_box_hint(mC, sb, n, row0, z0, z1, policy_evict_first());
       else tma_store_box(mC, sb, n, row0, z0, z1);
       bulk_commit();
     }
@@ -485,7 +490,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       fence_proxy_async_smem();
       __syncwarp();
       if (lane == 0) {
-        if (p.diag & 8) tma_store_box_hint(mO2, w.buf + EPI_BUF, n, row0, z0, z1, policy_evict_first());
+        if (diag & 8) tma_store_box_hint(mO2, w.buf + EPI_BUF, n, row0, z0, z1, policy_evict_first());
         else tma_store_box(mO2, w.buf + EPI_BUF, n, row0, z0, z1);
         bulk_commit();
       }
@@ -856,7 +861,11 @@ struct Tc2Cfg {
   static constexpr int TMEM_COLS = 2 * BN;     // double-buffered accumulator (BN fp32 columns each)
 };
 
-template <int BN, int STAGES>
+// EK: the epilogue kind compiled in (>= 0: that kind through the TMA-store epilogue only, a kernel a
+// fraction of the generic one's size — the generic body, every kind plus the register epilogue and
+// the diagnostics, overflowed the instruction cache: its epilogue warps stalled on instruction
+// fetch); -1: the generic kernel
+template <int BN, int STAGES, int EK = -1>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmIn,
@@ -893,7 +902,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 2); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tmem_full[a], 1); mbar_init(&tmem_empty[a], 2 * 32 * EPI_WARPS); }
     for (int i = 0; i < EPI_WARPS * 2; ++i) mbar_init(&ebar[i], 1);
-    if (p.tma_epi) { prefetch_tmap(&tmC); prefetch_tmap(&tmIn); prefetch_tmap(&tmO2); }
+    if (EK >= 0 || p.tma_epi) { prefetch_tmap(&tmC); prefetch_tmap(&tmIn); prefetch_tmap(&tmO2); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -981,7 +990,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     const uint32_t te = mapa_leader(&tmem_empty[0]);
     const uint32_t bias_base = smem_u32(sE) + EPI_WARPS * 2 * EPI_BUF;
     EpiWarp ew{smem_u32(sE) + (warp - 2) * 2 * EPI_BUF, bias_base, ebar + (warp - 2) * 2, 0u, 0u};
-    const bool out_f32 = e.epi == HK_EPI_STORE_F32 || e.epi == HK_EPI_RESID_F32 || e.epi == HK_EPI_ACC_F32;
+    const int epi = EK >= 0 ? EK : e.epi;
+    const bool tma_epi = EK >= 0 || p.tma_epi;
+    const bool out_f32 = epi == HK_EPI_STORE_F32 || epi == HK_EPI_RESID_F32 || epi == HK_EPI_ACC_F32;
     int it = 0;
     for (int t = pair; t < tm.total; t += npairs, ++it) {
       int z, mb, nb;
@@ -994,17 +1005,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       const int row0 = mb * 256 + (int)rank * 128 + q * 32;
       const uint32_t tacc = tmem_base + acc * BN + ((uint32_t)(q * 32) << 16);
       ew.bias = bias_base + (uint32_t)((acc << 1) | half) * EPI_BIAS_SET;
-      if (p.diag & 1) {
+      if (EK < 0 && (p.diag & 1)) {
         mbar_wait(&tmem_full[acc], (it >> 1) & 1);
         tc_fence_after();
-      } else if (p.tma_epi) {
+      } else if (tma_epi) {
         if (out_f32)
-          tma_epi_tile<4>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0, z1,
-                          &tmem_full[acc], (it >> 1) & 1);
+          tma_epi_tile<4, EK>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0,
+                              z1, &tmem_full[acc], (it >> 1) & 1);
         else
-          tma_epi_tile<2>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0, z1,
-                          &tmem_full[acc], (it >> 1) & 1);
-      } else {
+          tma_epi_tile<2, EK>(p, &tmC, &tmIn, &tmO2, ew, tacc + c_beg, nkb > 0, lane, row0, n0 + c_beg, n0 + c_end, z0,
+                              z1, &tmem_full[acc], (it >> 1) & 1);
+      } else if (EK < 0) {
         epi_prefetch(e, row0 + lane, n0 + c_beg, n0 + c_end, zoff);
         mbar_wait(&tmem_full[acc], (it >> 1) & 1);
         tc_fence_after();
@@ -1014,7 +1025,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       tc_fence_before();
       mbar_arrive_cluster(te + acc * 8);
     }
-    if (p.tma_epi && lane == 0) bulk_wait_all();
+    if (tma_epi && lane == 0) bulk_wait_all();
   }
   tc_fence_before();
   cluster_sync_all();
@@ -1023,6 +1034,28 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(Cfg::TMEM_COLS)
                  : "memory");
   }
+}
+
+template <int BN, int STAGES, int EK>
+static void launch_tc2_k(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc, const CUtensorMap& mi,
+                         const CUtensorMap& mo, const TcParams& p, dim3 grid, cudaStream_t st) {
+  using Cfg = Tc2Cfg<BN, STAGES>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    HM_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel<BN, STAGES, EK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 Cfg::SMEM));
+    attr_set = true;
+  }
+  gemm_tc2_kernel<BN, STAGES, EK><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
+}
+
+// HARMONY_GEMM_SPECIALIZE=0: always the generic kernel (A/B of the per-kind specialisation)
+static bool gemm_specialize() {
+  static const bool v = [] {
+    const char* e = getenv("HARMONY_GEMM_SPECIALIZE");
+    return !(e && *e == '0');
+  }();
+  return v;
 }
 
 template <int BN, int STAGES>
@@ -1038,11 +1071,6 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   p.e = e;
   CUtensorMap mc, mi, mo;
   make_epi_maps(a, e, BN, &mc, &mi, &mo, p);
-  static bool attr_set = false;
-  if (!attr_set) {
-    HM_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel<BN, STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
-    attr_set = true;
-  }
   static int num_sms = 0;
   if (!num_sms) {
     int dev = 0;
@@ -1052,7 +1080,21 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   const int64_t tiles = ceil_div(a.M, 256) * ceil_div(a.N, BN) * (int64_t)a.nz0 * a.nz1;
   dim3 grid((unsigned)(2 * std::min<int64_t>(tiles, num_sms / 2)));  // persistent pairs
   const int e0 = g_prof.begin(st);
-  gemm_tc2_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
+  // the per-kind kernels for the TMA-store epilogue (same code path as the generic one for that kind,
+  // so the results are bit-identical); the generic kernel for the register epilogue and diagnostics
+  const bool spec = BN == 256 && p.tma_epi && p.diag == 0 && gemm_specialize();
+  if constexpr (BN != 256) {
+    launch_tc2_k<BN, STAGES, -1>(ma, mb, mc, mi, mo, p, grid, st);
+  } else switch (spec ? e.epi : -1) {
+    case HK_EPI_STORE_T: launch_tc2_k<BN, STAGES, HK_EPI_STORE_T>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_STORE_F32: launch_tc2_k<BN, STAGES, HK_EPI_STORE_F32>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_RESID_F32: launch_tc2_k<BN, STAGES, HK_EPI_RESID_F32>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_ACC_F32: launch_tc2_k<BN, STAGES, HK_EPI_ACC_F32>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_BIAS_ACT: launch_tc2_k<BN, STAGES, HK_EPI_BIAS_ACT>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_ACT_BWD: launch_tc2_k<BN, STAGES, HK_EPI_ACT_BWD>(ma, mb, mc, mi, mo, p, grid, st); break;
+    case HK_EPI_ACT_T: launch_tc2_k<BN, STAGES, HK_EPI_ACT_T>(ma, mb, mc, mi, mo, p, grid, st); break;
+    default: launch_tc2_k<BN, STAGES, -1>(ma, mb, mc, mi, mo, p, grid, st); break;
+  }
   check_launch("gemm_tc2_kernel");
   g_prof.end(PROF_GEMM, e0, st, 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1);
 }
