@@ -367,6 +367,7 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       bulk_wait_read<1>();
     }
     float v[CPB];
+    uint32_t hkeep[ESZ == 2 ? 32 : 1];  // BIAS_ACT: this box's packed H, the input of G
     if (have_acc && !(diag & 2)) {
 #pragma unroll
       for (int h = 0; h < CPB / 32; ++h) tmem_ld32(tacc + CPB * bi + 32 * h, v + 32 * h);
@@ -439,7 +440,10 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
             }
           } else {  // BIAS_ACT: H = acc + b (bf16) now; G = act(H as stored) after H's store is issued
 #pragma unroll
-            for (int t = 0; t < 4; ++t) o[t] = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
+            for (int t = 0; t < 4; ++t) {
+              o[t] = pack_bf16(x[2 * t] + bb[2 * t], x[2 * t + 1] + bb[2 * t + 1]);
+              hkeep[ESZ == 2 ? 4 * k + t : 0] = o[t];
+            }
           }
         }
         sts128(ad, o[0], o[1], o[2], o[3]);
@@ -462,18 +466,16 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
       bulk_commit();
     }
     if (ESZ == 2 && two) {
-      // G = act(H as stored): H is read back from buffer A (which the H store only reads) and G
-      // goes into buffer B once the previous box's G store has left it
+      // G = act(H as stored), from the packed H kept in registers; G goes into buffer B once the
+      // previous box's G store has left it
       if (lane == 0) bulk_wait_read<1>();
       __syncwarp();
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
-        const uint4 hq = lds128(sb + swz128(r, k));
-        const uint32_t hw[4] = {hq.x, hq.y, hq.z, hq.w};
         uint32_t g[4];
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
-          const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hw[t]));
+          const float2 zr = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hkeep[ESZ == 2 ? 4 * k + t : 0]));
           g[t] = pack_bf16(act_f<true>(e.act, zr.x), act_f<true>(e.act, zr.y));
         }
         sts128(w.buf + EPI_BUF + swz128(r, k), g[0], g[1], g[2], g[3]);

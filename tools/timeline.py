@@ -80,6 +80,17 @@ def summarise(recs, step_s):
         if r["t0"] - prev > 2e-6:
             gaps.append((r["t0"] - prev, KIND[r["kind"]], r["layer"], r["micro"]))
         prev = max(prev, r["t1"])
+    # direction balance over the step: the busy fraction of each stream in 20 equal windows
+    t_end = max(r["t1"] for r in recs)
+    nb = 20
+    s["windows"] = []
+    for k in range(nb):
+        w = [[k * t_end / nb, (k + 1) * t_end / nb]]
+        row = {}
+        for nm, st in (("compute", 0), ("h2d", 1), ("d2h", 2)):
+            iv = union([(r["t0"], r["t1"]) for r in recs if r["stream"] == st])
+            row[nm] = round(total(intersect(iv, w)) / (t_end / nb), 2)
+        s["windows"].append(row)
     s["compute_idle_ms"] = sum(g[0] for g in gaps) * 1e3
     s["compute_idle_top"] = [{"ms": round(g[0] * 1e3, 3), "before": f"{g[1]}(l={g[2]}, i={g[3]})"}
                              for g in sorted(gaps, reverse=True)[:12]]
