@@ -15,6 +15,7 @@ struct EpiParams {
   const void* aux;
   void* aux_out;
   int M, N;
+  float* colsum = nullptr;  // optional: per-32-row-block column sums of the bf16 output (gemm_colsum)
 };
 
 // Apply the epilogue to one accumulator element.  T = activation type.

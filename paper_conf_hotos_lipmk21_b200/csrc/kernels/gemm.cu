@@ -18,6 +18,7 @@
 #include <mutex>
 
 #include "epilogue.cuh"
+#include "kernels.hpp"
 #include "tc_common.cuh"
 
 namespace hm {
@@ -447,6 +448,27 @@ __device__ __forceinline__ void tma_epi_tile(const TcParams& p, const CUtensorMa
           }
         }
         sts128(ad, o[0], o[1], o[2], o[3]);
+      }
+      if (EK == HK_EPI_ACT_BWD && e.colsum != nullptr && row0 < e.M) {
+        // gemm_colsum: this box's column sums over its 32 rows, from the staged (stored) bf16 values;
+        // lane = a column pair, rows in increasing order
+        __syncwarp();
+        const int c = n + 2 * lane;
+        float s0 = 0.f, s1 = 0.f;
+        const uint32_t col_off = (uint32_t)((lane & 3) * 4);
+#pragma unroll 8
+        for (int rr = 0; rr < 32; ++rr) {
+          if (row0 + rr < e.M) {
+            uint32_t wv;
+            asm volatile("ld.shared.b32 %0, [%1];" : "=r"(wv) : "r"(sb + swz128(rr, lane >> 2) + col_off) : "memory");
+            const float2 f = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&wv));
+            s0 += f.x;
+            s1 += f.y;
+          }
+        }
+        float* dst = e.colsum + (int64_t)(row0 / 32) * e.N + c;
+        if (c + 1 < e.N) *reinterpret_cast<float2*>(dst) = make_float2(s0, s1);
+        else if (c < e.N) dst[0] = s0;
       }
     }
     const bool lsu = diag & 16;  // experiment: LSU stores instead of TMA stores
@@ -1061,7 +1083,7 @@ static bool gemm_specialize() {
 }
 
 template <int BN, int STAGES>
-static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st) {
+static bool launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st) {
   using Cfg = Tc2Cfg<BN, STAGES>;
   CUtensorMap ma, mb;
   make_operand_map(&ma, a.A, a.a_mn_major, a.M, a.K, a.lda, a.nz0, a.a_sz0, a.nz1, a.a_sz1, 128);
@@ -1085,6 +1107,10 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   // the per-kind kernels for the TMA-store epilogue (same code path as the generic one for that kind,
   // so the results are bit-identical); the generic kernel for the register epilogue and diagnostics
   const bool spec = BN == 256 && p.tma_epi && p.diag == 0 && gemm_specialize();
+  // the ACT_BWD kernel sums its output boxes for gemm_colsum (plain products, 8-column-aligned rows)
+  const bool fused_colsum = spec && e.epi == HK_EPI_ACT_BWD && e.colsum != nullptr && p.nz == 1 && a.N % 2 == 0 &&
+                            (reinterpret_cast<uintptr_t>(e.colsum) & 7) == 0;
+  if (!fused_colsum) p.e.colsum = nullptr;
   if constexpr (BN != 256) {
     launch_tc2_k<BN, STAGES, -1>(ma, mb, mc, mi, mo, p, grid, st);
   } else switch (spec ? e.epi : -1) {
@@ -1099,17 +1125,20 @@ static void launch_tc2(const hk_gemm_args& a, const EpiParams& e, cudaStream_t s
   }
   check_launch("gemm_tc2_kernel");
   g_prof.end(PROF_GEMM, e0, st, 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1);
+  return fused_colsum;
 }
 
 }  // namespace tc
 
-void gemm(const hk_gemm_args& a, cudaStream_t st) {
+// returns true when the GEMM itself produced the gemm_colsum partials
+static bool gemm_impl(const hk_gemm_args& a, float* colsum, cudaStream_t st) {
   HM_CHECK(a.M >= 0 && a.N >= 0 && a.K >= 0 && a.nz0 >= 1 && a.nz1 >= 1, HARMONY_E_INVALID_ARG, "gemm: bad shape");
-  if (a.M == 0 || a.N == 0) return;
+  if (a.M == 0 || a.N == 0) return false;
   EpiParams e;
   e.C = a.C; e.ldc = a.ldc; e.c_sz0 = a.c_sz0; e.c_sz1 = a.c_sz1;
   e.epi = a.epilogue; e.act = a.act; e.accumulate = a.accumulate; e.alpha = a.alpha;
   e.bias = a.bias; e.aux = a.aux; e.aux_out = a.aux_out; e.M = a.M; e.N = a.N;
+  e.colsum = colsum;
   HM_CHECK(a.accumulate != 2 || (a.dtype == 0 && a.epilogue == HK_EPI_ACC_F32 && a.alpha == 1.f),
            HARMONY_E_UNSUPPORTED, "gemm: accumulate = 2 (continue C's reduction) is the fp32 ACC_F32 path only");
   if (a.dtype == 0) {
@@ -1124,7 +1153,7 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
     gemm_simt_kernel<<<grid, 256, 0, st>>>(p);
     check_launch("gemm_simt_kernel");
     g_prof.end(PROF_GEMM, e0, st, flops);
-    return;
+    return false;
   }
   // Tile shape from the problem shape only (never from the memory cap): bit-exact capped == uncapped.
   static const int mode = [] {
@@ -1146,17 +1175,26 @@ void gemm(const hk_gemm_args& a, cudaStream_t st) {
       return v ? atoi(v) : 0;
     }();
     const int stages = force ? force : (nz == 1 ? 5 : 4);
-    if (mode == 3) tc::launch_tc2<128, 6>(a, e, st);
-    else if (stages == 5) tc::launch_tc2<256, 5>(a, e, st);
-    else tc::launch_tc2<256, 4>(a, e, st);
-    return;
+    if (mode == 3) return tc::launch_tc2<128, 6>(a, e, st);
+    if (stages == 5) return tc::launch_tc2<256, 5>(a, e, st);
+    return tc::launch_tc2<256, 4>(a, e, st);
   }
+  e.colsum = nullptr;
   if (a.N <= 64)
     tc::launch_tc<64, 6>(a, e, st);
   else if (a.N <= 128 || (int64_t)ceil_div(a.M, 128) * ceil_div(a.N, 256) * nz < 148)
     tc::launch_tc<128, 4>(a, e, st);
   else
     tc::launch_tc<256, 3>(a, e, st);
+  return false;
+}
+
+void gemm(const hk_gemm_args& a, cudaStream_t st) { gemm_impl(a, nullptr, st); }
+
+void gemm_colsum(const hk_gemm_args& a, float* partial, cudaStream_t st) {
+  HM_CHECK(a.dtype == 1 && a.nz0 == 1 && a.nz1 == 1 && partial != nullptr, HARMONY_E_INVALID_ARG,
+           "gemm_colsum: a plain bf16 product and a partial buffer");
+  if (!gemm_impl(a, partial, st)) colsum32_partial(a.M, a.N, a.C, a.ldc, partial, st);
 }
 
 }  // namespace hm

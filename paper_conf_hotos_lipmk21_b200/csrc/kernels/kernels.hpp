@@ -9,6 +9,15 @@
 namespace hm {
 
 void gemm(const hk_gemm_args& a, cudaStream_t st);
+// gemm() with a bf16 output C (nz0 = nz1 = 1) that also writes partial[rb][c] = sum of the STORED
+// (bf16-rounded) C[r][c] over the rows r of block rb = r / 32, rows in increasing order (fp32);
+// partial is [ceil(M/32)][N].  The ACT_BWD CTA-pair kernel sums its staged output boxes in its
+// epilogue; any other path runs a separate pass with the same order (identical partials).
+void gemm_colsum(const hk_gemm_args& a, float* partial, cudaStream_t st);
+inline size_t colsum32_partial_bytes(int64_t rows, int n) { return (size_t)((rows + 31) / 32) * n * sizeof(float); }
+void colsum32_partial(int64_t rows, int n, const void* X, int64_t ld, float* partial, cudaStream_t st);
+// out[c] (+)= sum over the ceil(rows/32) partials of gemm_colsum, in a fixed tree (deterministic)
+void colsum32_reduce(int64_t rows, int n, const float* partial, float* out, int accumulate, cudaStream_t st);
 
 void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g, const void* b, void* U, float* mean,
                    float* rstd, cudaStream_t st, float* Xcopy = nullptr);

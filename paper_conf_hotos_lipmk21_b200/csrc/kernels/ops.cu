@@ -160,6 +160,34 @@ static void colreduce(int nchunks, int n, const float* partial, int64_t stride, 
   check_launch("colreduce");
 }
 
+// gemm_colsum's 32-row-block partials when the GEMM did not produce them: one thread per column, the
+// block's rows in increasing order — the order of the fused epilogue, so the partials are identical
+__global__ void colsum32_partial_kernel(int64_t rows, int n, const __nv_bfloat16* __restrict__ X, int64_t ld,
+                                        float* __restrict__ partial) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t rb = blockIdx.y;
+  if (c >= n) return;
+  float s = 0.f;
+  for (int r = 0; r < 32 && rb * 32 + r < rows; ++r) s += __bfloat162float(X[(rb * 32 + r) * ld + c]);
+  partial[rb * n + c] = s;
+}
+void colsum32_partial(int64_t rows, int n, const void* X, int64_t ld, float* partial, cudaStream_t st) {
+  if (rows <= 0 || n <= 0) return;
+  dim3 grid((unsigned)ceil_div(n, 128), (unsigned)ceil_div(rows, 32));
+  colsum32_partial_kernel<<<grid, 128, 0, st>>>(rows, n, static_cast<const __nv_bfloat16*>(X), ld, partial);
+  check_launch("colsum32_partial");
+}
+void colsum32_reduce(int64_t rows, int n, const float* partial, float* out, int accumulate, cudaStream_t st) {
+  const int nch = (int)ceil_div(rows, 32);
+  if (nch == 0) {
+    if (!accumulate) HM_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * n, st));
+    return;
+  }
+  const int e0 = g_prof.begin(st);
+  colreduce(nch, n, partial, n, out, accumulate, st);
+  g_prof.end(PROF_OTHER, e0, st, (double)nch * n * 4);
+}
+
 // ------------------------------------------------------------------------------------- column sums
 // partial[chunk][c] = sum of rows [chunk*CS_ROWS, ...) of column c, rows in increasing order; each
 // thread owns VEC adjacent columns (16-byte loads) and keeps CS_ROWS independent loads in flight.

@@ -171,6 +171,7 @@ LayerGeom make_geom(const harmony_layer_desc& desc, int b, int dtype, int stash_
   bump(wb, R * 3 * D * ts);  // dQKV
   bump(wb, colsum_scratch_bytes(g.rows, (int)(4 * D)));  // side-stream column-sum scratch
   bump(wb, std::max<uint64_t>(wgrad_split_ws_bytes(g, g.rows, (int)D, (int)D), 256));  // split-K dW_o partials
+  if (dtype == 1) bump(wb, colsum32_partial_bytes(g.rows, (int)(4 * D)));  // db_fc1 partials (FC2 dgrad epilogue)
   g.ws_bwd = wb;
   g.flops_fwd = 24.0 * (double)R * D * D + 4.0 * (double)b * g.S * g.S * D;
   return g;
@@ -415,6 +416,7 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   uint8_t* dQKV_buf = ws + bump(wc, R * 3 * D * ts);
   float* side_scratch = reinterpret_cast<float*>(ws + bump(wc, colsum_scratch_bytes(R, 4 * D)));
   float* split_ws = reinterpret_cast<float*>(ws + bump(wc, std::max<uint64_t>(wgrad_split_ws_bytes(g, R, D, D), 256)));
+  float* bfc1_part = dt == 1 ? reinterpret_cast<float*>(ws + bump(wc, colsum32_partial_bytes(R, (int)(4 * D)))) : nullptr;
   // weight gradients on the side stream (not with policy 1: its recompute buffer is reused in place)
   const bool overlap = t_side != nullptr && g.stash_policy != 1;
   cudaStream_t sw = overlap ? t_side : st;     // stream of the weight-gradient work
@@ -431,11 +433,13 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     cast_colsum(1, R, D, dY, dYc, gseg(g, dW, P_BFC2), acc, scratch, st);
     dYop = dYc;
   }
-  // ---- FC2: dG = dY W_fc2^T, fused with GeLU': dH = dG * gelu'(H)
+  // ---- FC2: dG = dY W_fc2^T, fused with GeLU': dH = dG * gelu'(H); bf16: the same epilogue also
+  // column-sums dH per 32-row block (the FC1 bias gradient's partials)
   {
     hk_gemm_args a = lin_dgrad(g, R, D, 4 * D, dYop, wseg(g, W, P_WFC2));
     a.C = dHb; a.epilogue = HK_EPI_ACT_BWD; a.act = HARMONY_ACT_GELU_TANH; a.aux = Hh;
-    gemm(a, st);
+    if (dt == 1) gemm_colsum(a, bfc1_part, st);
+    else gemm(a, st);
   }
   const uint8_t* G = g.stash_policy == 0 ? stash + g.st.G : rec;
   if (g.stash_policy == 1) act_fwd_T(dt, HARMONY_ACT_GELU_TANH, R * 4 * D, Hh, rec, st);
@@ -458,7 +462,8 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
   }
   if (g.stash_policy == 1) fork(0);
   gemm(lin_wgrad(g, R, 4 * D, D, U2, dHb, gseg(g, dW, P_WFC1), first), sw);
-  colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, wscratch, sw);
+  if (dt == 1) colsum32_reduce(R, (int)(4 * D), bfc1_part, gseg(g, dW, P_BFC1), acc, sw);
+  else colsum(dt, R, 4 * D, dHb, 4 * D, gseg(g, dW, P_BFC1), acc, wscratch, sw);
   // ---- LN2 backward: dX2 = dY + LN2'(dU2), fused with the bf16 copy of dX2 (the O-projection
   // GEMM operand) and db_o (+)= sum_rows dX2
   const void* dX2op = dt == 1 ? (const void*)dX2c_buf : (const void*)dX2;

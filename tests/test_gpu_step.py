@@ -318,3 +318,41 @@ def test_microbatch_groups_are_bitwise_identical_to_one_group(G):
     grouped, plan = run_gpu(descs, params, batches, hbm_cap_bytes=cap, groups=G, **kw)
     assert grouped[0]["stats"]["h2d_stash_bytes"] > 0
     bitwise_equal(one, grouped)
+
+
+def _step_in_subprocess(env, L, d, h, S, B, m):
+    """Run tiny_transformer steps in a fresh process (library knobs are read once per process)."""
+    import os
+    import pickle
+    import subprocess
+    import sys
+    import tempfile
+    code = f"""
+import pickle, sys
+sys.path.insert(0, {repr(os.path.dirname(os.path.abspath(__file__)))})
+sys.path.insert(0, {repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))})
+from test_gpu_step import tiny_transformer, run_gpu
+descs, params, batches, kw = tiny_transformer(False, 1, L={L}, d={d}, h={h}, S={S}, B={B}, m={m})
+res, _ = run_gpu(descs, params, batches, **kw)
+pickle.dump([{{k: r[k] for k in ('loss', 'g', 'W', 'm', 'v')}} for r in res], open(sys.argv[1], 'wb'))
+"""
+    with tempfile.NamedTemporaryFile(suffix=".pkl", delete=False) as f:
+        path = f.name
+    try:
+        subprocess.run([sys.executable, "-c", code, path], check=True, env=dict(os.environ, **env), timeout=600)
+        return pickle.load(open(path, "rb"))
+    finally:
+        os.unlink(path)
+
+
+def test_per_kind_gemm_kernels_are_bitwise_the_generic_kernel():
+    """The CTA-pair GEMM compiled per epilogue kind (default; the ACT_BWD one also column-sums its
+    output for the FC1 bias gradient) vs the generic kernel + the separate 32-row-block column-sum
+    pass (HARMONY_GEMM_SPECIALIZE=0): bit-identical steps.  d = 256, 3072 tokens per microbatch, so
+    the FC2 dgrad runs on 48 CTA-pair tiles (the fused path)."""
+    shape = dict(L=2, d=256, h=4, S=512, B=12, m=2)
+    spec = _step_in_subprocess({}, **shape)
+    generic = _step_in_subprocess({"HARMONY_GEMM_SPECIALIZE": "0"}, **shape)
+    bitwise_equal(spec, generic)
+    descs, params, batches, kw = tiny_transformer(False, 1, **shape)
+    compare(spec, run_oracle(descs, params, batches), 2e-2)
