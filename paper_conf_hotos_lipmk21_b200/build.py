@@ -63,6 +63,10 @@ def build(force: bool = False, jobs: int = 0, verbose: bool = False) -> str:
                     "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
                     "-I", nccl_include(), "-DNDEBUG"] + os.environ.get("HARMONY_NVCC_EXTRA", "").split()
     hdr_mtime = max([os.path.getmtime(h) for h in headers()] + [os.path.getmtime(__file__)])
+    # objects built with other flags (e.g. a HARMONY_NVCC_EXTRA diagnostic build) are rebuilt
+    stamp = os.path.join(BUILD, "flags.txt")
+    if not os.path.exists(stamp) or open(stamp).read() != " ".join(flags):
+        force = True
     srcs = sources()
     objs, todo = [], []
     for s in srcs:
@@ -94,6 +98,8 @@ def build(force: bool = False, jobs: int = 0, verbose: bool = False) -> str:
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")
         os.replace(LIB + ".tmp", LIB)
+    with open(stamp, "w") as f:
+        f.write(" ".join(flags))
     return LIB
 
 

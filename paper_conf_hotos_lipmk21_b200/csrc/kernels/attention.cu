@@ -31,6 +31,53 @@ __device__ __forceinline__ float fast_exp2(float x) {
   return y;
 }
 
+// HM_ATTN_TRACE builds (diagnostics only): CTA 0 of the forward records clock64 stamps of its
+// pipeline events — row 0: softmax warp 2 lane 0, row 1: the MMA issuer, row 2: the TMA producer —
+// read back with hm_attn_trace_read()
+#ifdef HM_ATTN_TRACE
+__device__ unsigned long long g_attn_trace[3][2048];
+__device__ int g_attn_trace_n[3];
+// the event index lives in a register of the recording thread (tr_cnt, declared at kernel entry):
+// a stamp is one fire-and-forget global store
+#define TR(row, code)                                                                                   \
+  do {                                                                                                  \
+    if (blockIdx.x == 0 && threadIdx.x == (row == 0 ? 64 : row == 1 ? 32 : 0)) {                         \
+      if (tr_cnt < 2048) g_attn_trace[row][tr_cnt] = ((unsigned long long)(code) << 56) | (clock64() & 0xffffffffffffffull); \
+      ++tr_cnt;                                                                                         \
+    }                                                                                                   \
+  } while (0)
+#define TR_END()                                                                                        \
+  do {                                                                                                  \
+    if (blockIdx.x == 0 && (threadIdx.x == 64 || threadIdx.x == 32 || threadIdx.x == 0))                 \
+      g_attn_trace_n[threadIdx.x == 64 ? 0 : threadIdx.x == 32 ? 1 : 2] = tr_cnt;                       \
+  } while (0)
+#else
+#define TR(row, code) do { } while (0)
+#define TR_END() do { } while (0)
+#endif
+
+// 2^x for a pair on the FMA pipe: x = j + f with j = rint(x) (the 1.5 * 2^23 rounding trick, whose
+// low mantissa bits are j), f in [-0.5, 0.5]; 2^f by a degree-5 polynomial fitted for relative error
+// (max 2.3e-7 in fp32 Horner, the accuracy of ex2.approx), and 2^j added to the exponent field.
+// x is clamped to [-125, 126]: below that 2^x is < 2^-125 (ex2.approx.ftz gives 0 there), which no
+// caller can tell from 0 after the bf16 rounding and the row sum.
+__device__ __forceinline__ float2 exp2_poly2(float2 x) {
+  x.x = fminf(fmaxf(x.x, -125.f), 126.f);
+  x.y = fminf(fmaxf(x.y, -125.f), 126.f);
+  const float2 one = make_float2(1.f, 1.f), magic = make_float2(12582912.f, 12582912.f);
+  const float2 t = tcx::ffma2(x, one, magic);                                    // 1.5 * 2^23 + rint(x)
+  const float2 r = tcx::ffma2(t, one, make_float2(-12582912.f, -12582912.f));    // rint(x)
+  const float2 f = tcx::ffma2(r, make_float2(-1.f, -1.f), x);                    // x - rint(x)
+  float2 q = tcx::ffma2(make_float2(1.32764e-3f, 1.32764e-3f), f, make_float2(9.67552e-3f, 9.67552e-3f));
+  q = tcx::ffma2(q, f, make_float2(5.550713e-2f, 5.550713e-2f));
+  q = tcx::ffma2(q, f, make_float2(2.402212e-1f, 2.402212e-1f));
+  q = tcx::ffma2(q, f, make_float2(6.9314697e-1f, 6.9314697e-1f));
+  q = tcx::ffma2(q, f, make_float2(1.00000007f, 1.00000007f));
+  // low 9 bits of the magic's bit pattern are 0: (bits(t) << 23) == rint(x) << 23 (mod 2^32)
+  return make_float2(__int_as_float(__float_as_int(q.x) + (__float_as_int(t.x) << 23)),
+                     __int_as_float(__float_as_int(q.y) + (__float_as_int(t.y) << 23)));
+}
+
 constexpr int BQ = 128;   // query rows per CTA
 constexpr int BKV = 128;  // keys per tile
 constexpr int THREADS = 320;  // warp 0: TMA, warp 1: MMA + TMEM, warps 2-9: softmax (2 per row quadrant)
@@ -41,11 +88,18 @@ struct FwdCfg {
   static constexpr int K_BYTES = BKV * DH * 2;
   static constexpr int V_BYTES = BKV * DH * 2;          // 2 key-atoms x DH/64 MN-chunks of 8 KB
   static constexpr int O_BYTES = BQ * DH * 2;           // output staging (DH/64 boxes of 64 columns)
-  static constexpr int QST = DH == 64 ? 2 : 1, KST = DH == 64 ? 4 : 2, VST = DH == 64 ? 4 : 2;
-  static constexpr int SMEM = QST * Q_BYTES + KST * K_BYTES + VST * V_BYTES + O_BYTES + 1024 + 256 + 2 * BQ * 4 + 4 * BQ * 4;
+  static constexpr int QST = DH == 64 ? 3 : 1, KST = DH == 64 ? 4 : 2, VST = DH == 64 ? 4 : 2;
+  static constexpr int BAR_BYTES = 512;                 // mbarriers + the TMEM base
+  static constexpr int SMEM = QST * Q_BYTES + KST * K_BYTES + VST * V_BYTES + O_BYTES + 1024 + BAR_BYTES + 2 * BQ * 4 + 4 * BQ * 4;
   static constexpr int S_COLS = BKV;                    // fp32 accumulator columns per S buffer
-  static constexpr int O_COL = 2 * BKV;                 // O after the two S buffers
-  static constexpr int P_COL = 2 * BKV + DH;            // two P buffers (bf16 pairs: BKV/2 columns each)
+  // SPLIT (an A/B variant, off): the two warps of a lane quadrant run independent online softmaxes
+  // over the two 64-key halves of every tile, each with its own O accumulator (combined in the
+  // epilogue), so they never meet at a per-tile barrier.  Measured at dh = 64, b = 32, S = 512:
+  // 80.6 vs 77.3 us — the exponential phase shrinks (1270 -> 880 cycles per tile) but the softmax
+  // then waits on the scores: the MMA issue (about 145 cycles per tcgen05.mma here) paces the tile.
+  static constexpr bool SPLIT = false;
+  static constexpr int O_COL = 2 * BKV;                 // O (SPLIT: O_0, O_1) after the two S buffers
+  static constexpr int P_COL = 2 * BKV + (SPLIT ? 2 : 1) * DH;  // two P buffers (bf16 pairs: BKV/2 columns each)
   static constexpr int TMEM_COLS = 512;
   static_assert(P_COL + BKV <= TMEM_COLS, "TMEM columns");
   static_assert(SMEM <= 232448, "shared memory per CTA");
@@ -82,11 +136,13 @@ __device__ __forceinline__ void fwd_item(int item, int nq, int H, int B, int& b,
 // empty barriers), and the output leaves through shared memory with TMA stores.  P never touches
 // shared memory: the softmax warps store it (bf16 pairs) into TMEM and O += P V takes its A
 // operand from there.
-template <int DH>
+template <int DH, int NPOLY>
 __global__ void __launch_bounds__(THREADS, 1)
     attn_fwd_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                     const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmC, FwdParams p) {
   using Cfg = FwdCfg<DH>;
+  int tr_cnt = 0;  // HM_ATTN_TRACE event index (unused otherwise)
+  (void)tr_cnt;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
@@ -94,22 +150,22 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint8_t* sV = sK + Cfg::KST * Cfg::K_BYTES;
   uint8_t* sO = sV + Cfg::VST * Cfg::V_BYTES;  // output staging
   uint64_t* bars = reinterpret_cast<uint64_t*>(sO + Cfg::O_BYTES);
-  uint64_t* q_full = bars;                      // [2]
-  uint64_t* q_empty = q_full + 2;               // [2]
-  uint64_t* k_full = q_empty + 2;               // [KST]
+  uint64_t* q_full = bars;                      // [QST]
+  uint64_t* q_empty = q_full + Cfg::QST;        // [QST]
+  uint64_t* k_full = q_empty + Cfg::QST;        // [KST]
   uint64_t* k_empty = k_full + Cfg::KST;        // [KST]
   uint64_t* v_full = k_empty + Cfg::KST;        // [VST]
   uint64_t* v_empty = v_full + Cfg::VST;        // [VST]
   uint64_t* s_full = v_empty + Cfg::VST;        // [2]
   uint64_t* s_empty = s_full + 2;               // [2]
-  uint64_t* p_full = s_empty + 2;               // [2]
-  uint64_t* p_empty = p_full + 2;               // [2]
-  uint64_t* o_full = p_empty + 2;
+  uint64_t* p_full = s_empty + 2;               // [2 buffers][2 key halves] (non-SPLIT: [b][0] only)
+  uint64_t* p_empty = p_full + 4;               // [2][2]
+  uint64_t* o_full = p_empty + 4;
   uint64_t* o_empty = o_full + 1;
   uint32_t* tmem_base_s = reinterpret_cast<uint32_t*>(o_empty + 1);
-  static_assert((14 + 2 * Cfg::KST + 2 * Cfg::VST) * 8 + 4 <= 256, "barrier area");
-  float(*sm_x)[BQ] = reinterpret_cast<float(*)[BQ]>(reinterpret_cast<uint8_t*>(bars) + 256);  // [2][BQ] row stats
-  float(*sm_t)[2][BQ] = reinterpret_cast<float(*)[2][BQ]>(reinterpret_cast<uint8_t*>(bars) + 256 + 2 * BQ * 4);  // [2][2][BQ]
+  static_assert((14 + 2 * Cfg::QST + 2 * Cfg::KST + 2 * Cfg::VST) * 8 + 4 <= Cfg::BAR_BYTES, "barrier area");
+  float(*sm_x)[BQ] = reinterpret_cast<float(*)[BQ]>(reinterpret_cast<uint8_t*>(bars) + Cfg::BAR_BYTES);  // [2][BQ] row stats
+  float(*sm_t)[2][BQ] = reinterpret_cast<float(*)[2][BQ]>(reinterpret_cast<uint8_t*>(bars) + Cfg::BAR_BYTES + 2 * BQ * 4);  // [2][2][BQ]
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int nq = p.S / BQ;
@@ -117,11 +173,9 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); prefetch_tmap(&tmC);
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1);
-      mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 256);
-      mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1);
-    }
+    for (int i = 0; i < Cfg::QST; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 256); }
+    for (int i = 0; i < 4; ++i) { mbar_init(&p_full[i], Cfg::SPLIT ? 128 : 256); mbar_init(&p_empty[i], 1); }
     for (int i = 0; i < Cfg::KST; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
     for (int i = 0; i < Cfg::VST; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
     mbar_init(o_full, 1); mbar_init(o_empty, 256);
@@ -149,18 +203,21 @@ __global__ void __launch_bounds__(THREADS, 1)
         const int ntiles = p.causal ? qt + 1 : nq;
         const int qs = n % Cfg::QST;
         mbar_wait(&q_empty[qs], ((n / Cfg::QST) & 1) ^ 1);
+        TR(2, 1);
         mbar_expect_tx(&q_full[qs], Cfg::Q_BYTES);
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a)
           tma_load_4d(sQ + qs * Cfg::Q_BYTES + a * (BQ * 128), &tmQ, &q_full[qs], a * 64, qt * BQ, h, b);
         for (int j = 0; j < ntiles; ++j) {
           mbar_wait(&k_empty[ks], kph ^ 1);
+          TR(2, 2);
           mbar_expect_tx(&k_full[ks], Cfg::K_BYTES);
 #pragma unroll
           for (int a = 0; a < DH / 64; ++a)
             tma_load_4d(sK + ks * Cfg::K_BYTES + a * (BKV * 128), &tmK, &k_full[ks], a * 64, j * BKV, h, b);
           if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
           mbar_wait(&v_empty[vs], vph ^ 1);
+          TR(2, 3);
           mbar_expect_tx(&v_full[vs], Cfg::V_BYTES);
 #pragma unroll
           for (int ka = 0; ka < 2; ++ka)
@@ -183,55 +240,96 @@ __global__ void __launch_bounds__(THREADS, 1)
       int vs = 0; uint32_t vph = 0;
       int it = 0;  // S-buffer uses
       int pc = 0;  // P-buffer uses
+      // Q of item n_ (waits for its TMA load)
+      auto q_addr = [&](int n_) {
+        const int qs_ = n_ % Cfg::QST;
+        mbar_wait(&q_full[qs_], (n_ / Cfg::QST) & 1);
+        return smem_u32(sQ + qs_ * Cfg::Q_BYTES);
+      };
+      auto issue_s = [&](uint32_t qa) {
+        const int sb = it & 1;
+        mbar_wait(&k_full[ks], kph);
+        mbar_wait(&s_empty[sb], ((it >> 1) & 1) ^ 1);
+        TR(1, 10);
+        tc_fence_after();
+        const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
+        if constexpr (DH == 64) {  // one swizzle atom: the four K=16 steps from one asm block
+          mma4_bf16(tmem + sb * Cfg::S_COLS, make_sdesc(qa, 16, 1024), make_sdesc(ka, 16, 1024), 2, 2, idesc_s, 0u);
+        } else {
+#pragma unroll
+          for (int kk = 0; kk < DH / 16; ++kk) {
+            const int atom = kk / 4, sub = kk % 4;
+            uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
+            uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
+            mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
+          }
+        }
+        mma_commit(&k_empty[ks]);
+        mma_commit(&s_full[sb]);
+        TR(1, 15);
+        if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
+        ++it;
+      };
+      // score cursor: S is issued two key tiles ahead of O += P V, across item boundaries, as soon
+      // as the softmax has read the S buffer it reuses — so when the softmax finishes a tile the
+      // scores of the one after next are already in TMEM, and a PV never delays the next scores
+      // (the cursor may enter item n + QST - 1 at most: its Q slot is free once item n - 1 is done)
+      int s_n = 0, s_item = snake(0), s_j = 0, s_nt = 0, s_cnt = 0;
+      uint32_t s_qa = 0;
+      auto issue_s_upto = [&](int target, int n_pv) {
+        while (s_cnt < target && s_item < items && s_n <= n_pv + Cfg::QST - 1) {
+          if (s_j == 0) {
+            int b_, h_, qt_;
+            fwd_item(s_item, nq, p.H, p.B, b_, h_, qt_);
+            s_nt = p.causal ? qt_ + 1 : nq;
+            s_qa = q_addr(s_n);
+          }
+          issue_s(s_qa);
+          ++s_cnt;
+          if (++s_j == s_nt) { s_j = 0; ++s_n; s_item = snake(s_n); }
+        }
+      };
       int n = 0;
       for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
         int b, h, qt;
         fwd_item(item, nq, p.H, p.B, b, h, qt);
         const int ntiles = p.causal ? qt + 1 : nq;
         const int qs = n % Cfg::QST;
-        mbar_wait(&q_full[qs], (n / Cfg::QST) & 1);
-        const uint32_t qa = smem_u32(sQ + qs * Cfg::Q_BYTES);
-        auto issue_s = [&]() {
-          const int sb = it & 1;
-          mbar_wait(&k_full[ks], kph);
-          mbar_wait(&s_empty[sb], ((it >> 1) & 1) ^ 1);
-          tc_fence_after();
-          const uint32_t ka = smem_u32(sK + ks * Cfg::K_BYTES);
-          if constexpr (DH == 64) {  // one swizzle atom: the four K=16 steps from one asm block
-            mma4_bf16(tmem + sb * Cfg::S_COLS, make_sdesc(qa, 16, 1024), make_sdesc(ka, 16, 1024), 2, 2, idesc_s, 0u);
-          } else {
-#pragma unroll
-            for (int kk = 0; kk < DH / 16; ++kk) {
-              const int atom = kk / 4, sub = kk % 4;
-              uint64_t ad = make_sdesc(qa + atom * (BQ * 128) + sub * 32, 16, 1024);
-              uint64_t bd = make_sdesc(ka + atom * (BKV * 128) + sub * 32, 16, 1024);
-              mma_bf16(tmem + sb * Cfg::S_COLS, ad, bd, idesc_s, kk ? 1u : 0u);
-            }
-          }
-          mma_commit(&k_empty[ks]);
-          mma_commit(&s_full[sb]);
-          if (++ks == Cfg::KST) { ks = 0; kph ^= 1; }
-          ++it;
-        };
-        // S_{j+1} is issued before PV_j so the softmax of j+1 overlaps PV_j
-        issue_s();
         for (int j = 0; j < ntiles; ++j) {
-          if (j + 1 < ntiles) issue_s();
+          issue_s_upto(pc + 3, n);  // scores up to two tiles past this PV's
           const int pb = pc & 1;
-          mbar_wait(&p_full[pb], (pc >> 1) & 1);
           mbar_wait(&v_full[vs], vph);
           if (j == 0) mbar_wait(o_empty, (n & 1) ^ 1);  // the previous item's O has been drained
-          tc_fence_after();
           const uint32_t pa = tmem + Cfg::P_COL + pb * (BKV / 2);
           const uint32_t va = smem_u32(sV + vs * Cfg::V_BYTES);
+          if constexpr (Cfg::SPLIT) {
+            // O_h += P[:, 64h .. 64h+63] V[64h .. 64h+63, :], each half as soon as its P is stored
 #pragma unroll
-          for (int kk = 0; kk < BKV / 16; ++kk) {
-            const int atom = kk / 4, sub = kk % 4;
-            uint64_t bd = make_sdesc(va + atom * (DH / 64) * 8192 + sub * 2048, 8192, 1024);
-            mma_bf16_ts(tmem + Cfg::O_COL, pa + kk * 8, bd, idesc_o, (j | kk) ? 1u : 0u);
+            for (int hh = 0; hh < 2; ++hh) {
+              mbar_wait(&p_full[pb * 2 + hh], (pc >> 1) & 1);
+              if (hh == 0) TR(1, 11);
+              tc_fence_after();
+#pragma unroll
+              for (int sub = 0; sub < 4; ++sub) {
+                uint64_t bd = make_sdesc(va + hh * 8192 + sub * 2048, 8192, 1024);
+                mma_bf16_ts(tmem + Cfg::O_COL + hh * DH, pa + hh * 32 + sub * 8, bd, idesc_o, (j | sub) ? 1u : 0u);
+              }
+              mma_commit(&p_empty[pb * 2 + hh]);
+            }
+          } else {
+            mbar_wait(&p_full[pb * 2], (pc >> 1) & 1);
+            TR(1, 11);
+            tc_fence_after();
+#pragma unroll
+            for (int kk = 0; kk < BKV / 16; ++kk) {
+              const int atom = kk / 4, sub = kk % 4;
+              uint64_t bd = make_sdesc(va + atom * (DH / 64) * 8192 + sub * 2048, 8192, 1024);
+              mma_bf16_ts(tmem + Cfg::O_COL, pa + kk * 8, bd, idesc_o, (j | kk) ? 1u : 0u);
+            }
+            mma_commit(&p_empty[pb * 2]);
           }
           mma_commit(&v_empty[vs]);
-          mma_commit(&p_empty[pb]);
+          TR(1, 14);
           if (++vs == Cfg::VST) { vs = 0; vph ^= 1; }
           ++pc;
         }
@@ -250,6 +348,79 @@ __global__ void __launch_bounds__(THREADS, 1)
     const uint32_t trow = (uint32_t)(qd * 32) << 16;
     const bool issuer = qd == 0 && lane == 0;  // of this half's TMA store of O
     int it = 0, pc = 0, n = 0, tp = 0;
+    // deferred epilogue state: the item whose O is still in TMEM
+    bool pend = false;
+    int e_n = 0, e_b = 0, e_h = 0, e_qt = 0;
+    float e_m = 0.f, e_l = 0.f;
+    auto epilogue = [&]() {
+      float l = e_l;
+      if (issuer) bulk_wait_read<0>();  // the previous item's O store has left the staging boxes
+      asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
+      sm_x[half][r] = l;
+      if constexpr (Cfg::SPLIT) sm_t[0][half][r] = e_m;
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      float f0 = 1.f, f1 = 1.f, mrow = e_m;
+      if constexpr (Cfg::SPLIT) {
+        // combine the two key halves' softmaxes: shift both to the row max (a half with no visible
+        // key has m = -inf and l = 0: factor 0)
+        const float m0 = sm_t[0][0][r], m1 = sm_t[0][1][r];
+        mrow = fmaxf(m0, m1);
+        f0 = fast_exp2((m0 - mrow) * p.scale_log2);
+        f1 = fast_exp2((m1 - mrow) * p.scale_log2);
+        l = sm_x[0][r] * f0 + sm_x[1][r] * f1;
+      } else {
+        l = sm_x[0][r] + sm_x[1][r];
+      }
+      const float inv_l = 1.f / l;
+      // ---- epilogue: O row (normalised, bf16) -> this half's DH/2 columns in a swizzled staging
+      // box (P buffer `half`, free once O is complete) -> TMA store to C; then the LSE
+      mbar_wait(o_full, e_n & 1);
+      TR(0, 26);
+      tc_fence_after();
+      float v[DH / 2];
+#pragma unroll
+      for (int c = 0; c < DH / 2; c += 32) tmem_ld32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, v + c);
+      if constexpr (Cfg::SPLIT) {
+        float w[DH / 2];
+#pragma unroll
+        for (int c = 0; c < DH / 2; c += 32) tmem_ld32(tmem + trow + Cfg::O_COL + DH + half * (DH / 2) + c, w + c);
+#pragma unroll
+        for (int i = 0; i < DH / 2; ++i) v[i] = v[i] * f0 + w[i] * f1;
+      }
+      tc_fence_before();
+      mbar_arrive_local(o_empty);  // O is in registers: the next item's PV may start
+      TR(0, 27);
+      // staging: boxes of 64 bf16 columns (128 B rows, 128B swizzle); DH=64: half h -> 32 columns
+      // of box 0 (chunks 4h..4h+3); DH=128: half h -> box h
+      uint8_t* box = sO + (DH == 64 ? 0 : half * (BQ * 128)) + r * 128;
+      const int ch0 = DH == 64 ? half * 4 : 0;
+#pragma unroll
+      for (int u = 0; u < DH / 16; ++u) {
+        uint32_t pk[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          __nv_bfloat162 h2 = __floats2bfloat162_rn(v[8 * u + 2 * t] * inv_l, v[8 * u + 2 * t + 1] * inv_l);
+          pk[t] = *reinterpret_cast<uint32_t*>(&h2);
+        }
+        *reinterpret_cast<uint4*>(box + (((ch0 + u) ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      if (DH == 64) {
+        asm volatile("bar.sync 1, 256;" ::: "memory");  // both halves wrote the box
+        if (half == 0 && issuer) {
+          tma_store_4d(&tmC, sO, 0, e_qt * BQ, e_h, e_b);
+          bulk_commit();
+        }
+      } else {
+        asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");
+        if (issuer) {
+          tma_store_4d(&tmC, sO + half * (BQ * 128), half * 64, e_qt * BQ, e_h, e_b);
+          bulk_commit();
+        }
+      }
+      // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
+      if (half == 0) p.lse[((int64_t)e_b * p.H + e_h) * p.S + e_qt * BQ + r] = mrow * p.scale + logf(l);
+    };
     for (int item = snake(0); item < items; item = snake(n + 1), ++n) {
       int b, h, qt;
       fwd_item(item, nq, p.H, p.B, b, h, qt);
@@ -269,11 +440,13 @@ __global__ void __launch_bounds__(THREADS, 1)
         constexpr bool DIAG = decltype(diag_tag)::value;
         const int sb = it & 1, pb = pc & 1;
         mbar_wait(&s_full[sb], (it >> 1) & 1);
+        TR(0, 20);
         tc_fence_after();
         float v[64];
         tmem_ld64(tmem + trow + sb * Cfg::S_COLS + cb, v);
         tc_fence_before();
         mbar_arrive_local(&s_empty[sb]);  // S is in registers: the MMA may overwrite the buffer
+        TR(0, 21);
         if constexpr (DIAG) {
           const int lim = qrow - (j * BKV + cb);  // keys cb + i with i <= lim are visible
 #pragma unroll
@@ -284,11 +457,14 @@ __global__ void __launch_bounds__(THREADS, 1)
 #pragma unroll
         for (int i = 0; i < 64; ++i) m4[i & 3] = fmaxf(m4[i & 3], v[i]);
         float tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
-        // the other half of the row (the partner warp of this lane quadrant)
-        sm_t[tp][half][r] = tm;
-        asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
-        tm = fmaxf(tm, sm_t[tp][half ^ 1][r]);
-        tp ^= 1;
+        if constexpr (!Cfg::SPLIT) {
+          // the other half of the row (the partner warp of this lane quadrant)
+          sm_t[tp][half][r] = tm;
+          asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
+          tm = fmaxf(tm, sm_t[tp][half ^ 1][r]);
+          tp ^= 1;
+        }
+        TR(0, 22);
         const bool raise = (tm - m) * p.scale_log2 > 8.f;  // true on the first tile (m = -inf)
         float f = 1.f;
         if (raise) {
@@ -298,95 +474,72 @@ __global__ void __launch_bounds__(THREADS, 1)
           l2b = make_float2(l2b.x * f, l2b.y * f);
         }
         if (__any_sync(0xffffffffu, raise && j > 0)) {
-          // rescale this warp's rows of O (its DH/2 columns) once PV_{j-1} has landed
+          // rescale this warp's rows of O once PV_{j-1} has landed: its DH/2 columns of O, or
+          // (SPLIT) all of O_half
           const int u = pc - 1;
-          mbar_wait(&p_empty[u & 1], (u >> 1) & 1);
+          mbar_wait(&p_empty[(u & 1) * 2 + (Cfg::SPLIT ? half : 0)], (u >> 1) & 1);
           tc_fence_after();
+          constexpr int OC = Cfg::SPLIT ? DH : DH / 2;
+          const uint32_t o_base = tmem + trow + Cfg::O_COL + half * OC;
 #pragma unroll
-          for (int c = 0; c < DH / 2; c += 32) {
+          for (int c = 0; c < OC; c += 32) {
             float o[32];
-            tmem_ld32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, o);
+            tmem_ld32(o_base + c, o);
             uint32_t ou[32];
 #pragma unroll
             for (int i = 0; i < 32; ++i) ou[i] = __float_as_uint(o[i] * f);
-            tmem_st32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, ou);
+            tmem_st32(o_base + c, ou);
           }
           tmem_wait_st();
         }
-        const float ms = m * p.scale_log2;
+        // (SPLIT: a key half with no visible key yet keeps m = -inf; its probabilities are 0)
+        const float ms = (Cfg::SPLIT && m == -INFINITY) ? 0.f : m * p.scale_log2;
         uint32_t pk[32];
         const float2 sl2 = make_float2(p.scale_log2, p.scale_log2), nms2 = make_float2(-ms, -ms);
         const float2 one2 = make_float2(1.f, 1.f);
 #pragma unroll
         for (int i = 0; i < 32; ++i) {
           const float2 x = ffma2(make_float2(v[2 * i], v[2 * i + 1]), sl2, nms2);
-          const float2 e2 = make_float2(fast_exp2(x.x), fast_exp2(x.y));
+          // NPOLY of the 32 pairs take 2^x on the FMA pipe instead of the SFU (A/B variant);
+          // the causal diagonal tile keeps ex2 for all, so masked scores give exactly 0
+          const bool poly = !DIAG && (i * NPOLY) % 32 < NPOLY;
+          const float2 e2 = poly ? exp2_poly2(x) : make_float2(fast_exp2(x.x), fast_exp2(x.y));
           if (i & 1) l2b = ffma2(e2, one2, l2b);
           else l2a = ffma2(e2, one2, l2a);
           __nv_bfloat162 h2 = __floats2bfloat162_rn(e2.x, e2.y);
           pk[i] = *reinterpret_cast<uint32_t*>(&h2);
         }
-        mbar_wait(&p_empty[pb], ((pc >> 1) & 1) ^ 1);
+        TR(0, 23);
+        mbar_wait(&p_empty[pb * 2 + (Cfg::SPLIT ? half : 0)], ((pc >> 1) & 1) ^ 1);
+        TR(0, 24);
         tc_fence_after();
         // this thread's 64 keys -> 32 TMEM columns (bf16 pairs) of P buffer pb, row = its lane
         tmem_st32(tmem + trow + Cfg::P_COL + pb * (BKV / 2) + half * 32, pk);
         tmem_wait_st();
         tc_fence_before();
-        mbar_arrive_local(&p_full[pb]);
+        mbar_arrive_local(&p_full[pb * 2 + (Cfg::SPLIT ? half : 0)]);
+        TR(0, 25);
         ++it; ++pc;
       };
+      // the previous item's epilogue runs after this item's first tile: by then its last PV has
+      // landed in O (no wait), and the scores of this tile were computed while that PV ran
       const int nfull = p.causal ? ntiles - 1 : ntiles;
-      for (int j = 0; j < nfull; ++j) tile(j, std::false_type{});
-      if (p.causal) tile(ntiles - 1, std::true_type{});
-      float l = (l2a.x + l2a.y) + (l2b.x + l2b.y);
-      if (issuer) bulk_wait_read<0>();  // the previous item's O store has left the staging boxes
-      asm volatile("bar.sync 1, 256;" ::: "memory");  // every thread has read sm_x before it is reused
-      sm_x[half][r] = l;
-      asm volatile("bar.sync 1, 256;" ::: "memory");
-      l = sm_x[0][r] + sm_x[1][r];
-      const float inv_l = 1.f / l;
-      // ---- epilogue: O row (normalised, bf16) -> this half's DH/2 columns in a swizzled staging
-      // box (P buffer `half`, free once O is complete) -> TMA store to C; then the LSE
-      mbar_wait(o_full, n & 1);
-      tc_fence_after();
-      float v[DH / 2];
-#pragma unroll
-      for (int c = 0; c < DH / 2; c += 32) tmem_ld32(tmem + trow + Cfg::O_COL + half * (DH / 2) + c, v + c);
-      tc_fence_before();
-      mbar_arrive_local(o_empty);  // O is in registers: the next item's PV may start
-      // staging: boxes of 64 bf16 columns (128 B rows, 128B swizzle); DH=64: half h -> 32 columns
-      // of box 0 (chunks 4h..4h+3); DH=128: half h -> box h
-      uint8_t* box = sO + (DH == 64 ? 0 : half * (BQ * 128)) + r * 128;
-      const int ch0 = DH == 64 ? half * 4 : 0;
-#pragma unroll
-      for (int u = 0; u < DH / 16; ++u) {
-        uint32_t pk[4];
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          __nv_bfloat162 h2 = __floats2bfloat162_rn(v[8 * u + 2 * t] * inv_l, v[8 * u + 2 * t + 1] * inv_l);
-          pk[t] = *reinterpret_cast<uint32_t*>(&h2);
-        }
-        *reinterpret_cast<uint4*>(box + (((ch0 + u) ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+      for (int j = 0; j < nfull; ++j) {
+        tile(j, std::false_type{});
+        if (j == 0 && pend) { epilogue(); pend = false; }
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      if (DH == 64) {
-        asm volatile("bar.sync 1, 256;" ::: "memory");  // both halves wrote the box
-        if (half == 0 && issuer) {
-          tma_store_4d(&tmC, sO, 0, qt * BQ, h, b);
-          bulk_commit();
-        }
-      } else {
-        asm volatile("bar.sync %0, 128;" ::"r"(2 + half) : "memory");
-        if (issuer) {
-          tma_store_4d(&tmC, sO + half * (BQ * 128), half * 64, qt * BQ, h, b);
-          bulk_commit();
-        }
+      if (p.causal) {
+        tile(ntiles - 1, std::true_type{});
+        if (ntiles == 1 && pend) { epilogue(); pend = false; }
       }
-      // natural-log LSE of the scaled scores: lse = scale*m + ln(l)
-      if (half == 0) p.lse[((int64_t)b * p.H + h) * p.S + qrow] = m * p.scale + logf(l);
+      pend = true;
+      e_n = n; e_b = b; e_h = h; e_qt = qt; e_m = m;
+      e_l = (l2a.x + l2a.y) + (l2b.x + l2b.y);
     }
+    if (pend) epilogue();
     if (issuer) bulk_wait_all();
   }
+  TR_END();
   tc_fence_before();
   __syncthreads();
   if (warp == 1) {
@@ -691,6 +844,7 @@ __device__ __forceinline__ void bwd_item(int item, int nk, int H, int B, int& b,
   b = rem / H;
 }
 
+template <bool ALT>
 __global__ void __launch_bounds__(THREADS, 1)
     attn_bwd_persistent(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
                         const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmdO,
@@ -724,7 +878,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     for (int i = 0; i < 2; ++i) {
       mbar_init(&kv_full[i], 1); mbar_init(&kv_empty[i], 1);
       mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 256); mbar_init(&p_empty[i], 1);
+      mbar_init(&p_full[i], ALT ? 128 : 256); mbar_init(&p_empty[i], 1);
     }
     for (int i = 0; i < Cfg::QST; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
     mbar_init(kd_full, 1); mbar_init(kd_empty, 256);
@@ -857,19 +1011,29 @@ __global__ void __launch_bounds__(THREADS, 1)
       const int nt = nqs - i0;
       const int key = kt * BKV + r;
       for (int t = 0; t < nt; ++t, ++g) {
-        const float* sl2 = sStat + qsl * (2 * BQS) + half * 32;
-        const float* ssd = sl2 + BQS;
-        mbar_wait(&q_full[qsl], qslph);  // the TMA-written statistics are visible to this thread
+        const int cur = qsl;  // this sub-tile's (Q, dO, statistics) ring slot
+        const uint32_t curph = qslph;
         if (++qsl == Cfg::QST) { qsl = 0; qslph ^= 1; }
-        const int q0 = (i0 + t) * BQS;
         const int buf = g & 1;
+        // ALT: the two warps of a lane quadrant take alternate sub-tiles (half h: buffer pair h), all 64
+        // queries each, so on every SM sub-partition one warp reads scores from TMEM while the other
+        // exponentiates; otherwise both take the same sub-tile, 32 queries each
+        if (ALT && buf != half) continue;
+        mbar_wait(&q_full[cur], curph);  // the TMA-written statistics are visible to this thread
+        const int q0 = (i0 + t) * BQS;
         mbar_wait(&s_full[buf], (g >> 1) & 1);
         tc_fence_after();
         const bool diag = p.causal && q0 < kt * BKV + BKV;  // the sub-tile overlaps the key range
-        const int qc = q0 + half * 32;  // first query of this thread's 32 columns
+        if (ALT && lane == 0) bulk_wait_read<0>();  // this warp's store of sub-tile g-2 left the dS^T buffer
+        bool waited_empty = false;
+#pragma unroll 1
+        for (int c = ALT ? 0 : half * 32; c < (ALT ? 64 : half * 32 + 32); c += 32) {
+        const float* sl2 = sStat + cur * (2 * BQS) + c;
+        const float* ssd = sl2 + BQS;
+        const int qc = q0 + c;  // first query of this thread's 32 columns
         uint32_t rs[32], rd[32];
-        tmem_ld32_nw(tmem + trow + Cfg::ST_COL + buf * BQS + half * 32, rs);
-        tmem_ld32_nw(tmem + trow + Cfg::DP_COL + buf * BQS + half * 32, rd);
+        tmem_ld32_nw(tmem + trow + Cfg::ST_COL + buf * BQS + c, rs);
+        tmem_ld32_nw(tmem + trow + Cfg::DP_COL + buf * BQS + c, rd);
         float2 l2[16], sd[16];  // broadcast reads of the staged statistics (-lse2, -sD), in pairs
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
@@ -903,35 +1067,49 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
         // the P^T / dS^T buffers are free once the dV / dK MMAs of sub-tile g-2 are done (waited only
         // now, so the score loads and the exponentials above overlap those MMAs)
-        mbar_wait(&p_empty[buf], ((g >> 1) & 1) ^ 1);
-        tc_fence_after();
+        if (!waited_empty) {
+          mbar_wait(&p_empty[buf], ((g >> 1) & 1) ^ 1);
+          tc_fence_after();
+          waited_empty = true;
+        }
         // P^T: this thread's 32 queries -> 16 TMEM columns (bf16 pairs) of P buffer `buf`
         asm volatile(
             "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
-                tmem + trow + Cfg::PT_COL + buf * (BQS / 2) + half * 16),
+                tmem + trow + Cfg::PT_COL + buf * (BQS / 2) + c / 2),
             "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]), "r"(pk[8]),
             "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]), "r"(pk[15])
             : "memory");
-        // dS^T: the row's 16-byte chunks 4*half .. 4*half+3 of the 128-byte (64-query) row, swizzled
+        // dS^T: the row's 16-byte chunks c/8 .. c/8+3 of the 128-byte (64-query) row, swizzled
+        if (ALT && c == 0) __syncwarp();  // lane 0's wait for the buffer's previous store precedes every write
         const uint32_t drow = smem_u32(sDS + buf * Cfg::DS_BYTES + r * 128);
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(drow + (((4 * half + u) ^ (r & 7)) << 4)),
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(drow + (((c / 8 + u) ^ (r & 7)) << 4)),
                        "r"(dk[4 * u]), "r"(dk[4 * u + 1]), "r"(dk[4 * u + 2]), "r"(dk[4 * u + 3])
                        : "memory");
+        }
         tmem_wait_st();
         tc_fence_before();
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_arrive_local(&p_full[buf]);
-        // this lane quadrant's 32 keys x 64 queries are written (both halves): one TMA store per
-        // quadrant, synchronised by the quadrant's two warps only.  The quadrant's store of the
-        // sub-tile two back (same buffer) was waited for before the previous instance of this
-        // barrier, so its rows were free when they were written above.
-        if (issuer) bulk_wait_read<0>();
-        asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
-        if (issuer) {
-          tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES + qd * 32 * 128, q0, kt * BKV + qd * 32, h, b);
-          bulk_commit();
+        if (ALT) {
+          // the warp wrote its quadrant's 32 keys x 64 queries: one TMA store from lane 0
+          __syncwarp();
+          if (lane == 0) {
+            tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES + qd * 32 * 128, q0, kt * BKV + qd * 32, h, b);
+            bulk_commit();
+          }
+        } else {
+          // this lane quadrant's 32 keys x 64 queries are written (both halves): one TMA store per
+          // quadrant, synchronised by the quadrant's two warps only.  The quadrant's store of the
+          // sub-tile two back (same buffer) was waited for before the previous instance of this
+          // barrier, so its rows were free when they were written above.
+          if (issuer) bulk_wait_read<0>();
+          asm volatile("bar.sync %0, 64;" ::"r"(4 + qd) : "memory");
+          if (issuer) {
+            tma_store_4d(&tmdS, sDS + buf * Cfg::DS_BYTES + qd * 32 * 128, q0, kt * BKV + qd * 32, h, b);
+            bulk_commit();
+          }
         }
       }
       // epilogue: dV_j (half 0) / dK_j (half 1) rows -> dQKV (bf16)
@@ -953,7 +1131,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         *reinterpret_cast<uint4*>(out + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
       }
     }
-    if (issuer) bulk_wait_all();
+    if (ALT ? lane == 0 : issuer) bulk_wait_all();
   }
   tc_fence_before();
   __syncthreads();
@@ -1036,14 +1214,29 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   const int64_t items = (int64_t)(S / BQ) * H * b;
   dim3 grid((unsigned)std::min<int64_t>(items, num_sms));  // persistent
   const int e0 = g_prof.begin(st);
+  // pairs of exponentials (of 32 per thread and tile) computed on the FMA pipe instead of the SFU;
+  // HARMONY_ATTN_POLY = 8 / 12 / 16 for A/B runs (measured 78.7 / 79.1 / 82.3 us against 77.9 with
+  // none: the exponentials are not what paces the tile)
+  static const int npoly = [] {
+    const char* v = getenv("HARMONY_ATTN_POLY");
+    const int k = v ? atoi(v) : 0;
+    return (k == 8 || k == 12 || k == 16) ? k : 0;
+  }();
+  static bool attr_set[5] = {false, false, false, false, false};  // per kernel variant
+  auto launch = [&](int variant, auto kern, int smem) {
+    if (!attr_set[variant]) {
+      HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+      attr_set[variant] = true;
+    }
+    kern<<<grid, THREADS, smem, st>>>(mq, mk, mv, mc, p);
+  };
   if (dh == 64) {
-    static bool set = false;
-    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<64>::SMEM)); set = true; }
-    attn_fwd_kernel<64><<<grid, THREADS, FwdCfg<64>::SMEM, st>>>(mq, mk, mv, mc, p);
+    if (npoly == 8) launch(1, attn_fwd_kernel<64, 8>, FwdCfg<64>::SMEM);
+    else if (npoly == 12) launch(3, attn_fwd_kernel<64, 12>, FwdCfg<64>::SMEM);
+    else if (npoly == 16) launch(2, attn_fwd_kernel<64, 16>, FwdCfg<64>::SMEM);
+    else launch(0, attn_fwd_kernel<64, 0>, FwdCfg<64>::SMEM);
   } else {
-    static bool set = false;
-    if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_fwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdCfg<128>::SMEM)); set = true; }
-    attn_fwd_kernel<128><<<grid, THREADS, FwdCfg<128>::SMEM, st>>>(mq, mk, mv, mc, p);
+    launch(4, attn_fwd_kernel<128, 0>, FwdCfg<128>::SMEM);
   }
   check_launch("attn_fwd_kernel");
   // algorithmic FLOPs of the attention contractions (QK^T and PV, causal or not)
@@ -1090,9 +1283,17 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   p.d = d;
   dim3 grid((unsigned)(S / BKV), (unsigned)H, (unsigned)b);
   if (dh == 64) {
+    // HARMONY_ATTN_BWD_ALT=1 alternates sub-tiles between the two warps of a lane quadrant (each
+    // takes all 64 queries of its sub-tiles) instead of splitting every sub-tile between them: an
+    // A/B variant, measured 169.6 vs 164.8 us at b = 32, S = 512 (the softmax is not the bound)
+    static const bool alt = [] {
+      const char* v = getenv("HARMONY_ATTN_BWD_ALT");
+      return v && v[0] == '1';
+    }();
     static bool set = false;
     if (!set) {
-      HM_CUDA(cudaFuncSetAttribute(attn_bwd_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdPCfg::SMEM));
+      HM_CUDA(cudaFuncSetAttribute(attn_bwd_persistent<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdPCfg::SMEM));
+      HM_CUDA(cudaFuncSetAttribute(attn_bwd_persistent<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdPCfg::SMEM));
       set = true;
     }
     static int num_sms = 0;
@@ -1107,8 +1308,8 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
     tcx::make_map_4d(&mds32, dst, S, S, H, b, S, (int64_t)S * S, (int64_t)H * S * S, 64, 32);  // per-quadrant boxes
     tcx::make_map_4d(&mq64, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BwdPCfg::BQS);
     tcx::make_map_4d(&mo64, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BwdPCfg::BQS);
-    attn_bwd_persistent<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq64, mk, mv, mo64,
-                                                                                                    mds32, p, (int)b);
+    auto kern = alt ? attn_bwd_persistent<true> : attn_bwd_persistent<false>;
+    kern<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq64, mk, mv, mo64, mds32, p, (int)b);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }
@@ -1126,5 +1327,16 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   gemm(a, st);
   return true;
 }
+
+#ifdef HM_ATTN_TRACE
+extern "C" int hm_attn_trace_read(unsigned long long* out, int* counts) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, attn::g_attn_trace, sizeof(attn::g_attn_trace));
+  cudaMemcpyFromSymbol(counts, attn::g_attn_trace_n, sizeof(attn::g_attn_trace_n));
+  int z[3] = {0, 0, 0};
+  cudaMemcpyToSymbol(attn::g_attn_trace_n, z, sizeof(z));
+  return 0;
+}
+#endif
 
 }  // namespace hm

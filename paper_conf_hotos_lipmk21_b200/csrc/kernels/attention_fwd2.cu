@@ -30,6 +30,22 @@
 namespace hm {
 namespace attn2 {
 
+// HM_ATTN_TRACE builds (diagnostics only): CTA 0 records clock64 stamps — row 0: softmax warp 4
+// lane 0 (tile A), row 1: the MMA issuer, row 2: softmax warp 8 lane 0 (tile B)
+#ifdef HM_ATTN_TRACE
+__device__ unsigned long long g_attn2_trace[3][2048];
+__device__ int g_attn2_trace_n[3];
+#define TR(row, code)                                                                                   \
+  do {                                                                                                  \
+    if (blockIdx.x == 0 && (row == 1 || (threadIdx.x == 128 || threadIdx.x == 256))) {                 \
+      const int i_ = g_attn2_trace_n[row]++;                                                            \
+      if (i_ < 2048) g_attn2_trace[row][i_] = ((unsigned long long)(code) << 56) | (clock64() & 0xffffffffffffffull); \
+    }                                                                                                   \
+  } while (0)
+#else
+#define TR(row, code) do { } while (0)
+#endif
+
 using namespace tcx;
 
 __device__ __forceinline__ float fast_exp2(float x) {
@@ -212,6 +228,7 @@ __global__ void __launch_bounds__(THREADS, 1)
             // the item's first tile: B's scores only once A has read its own, so the two softmax groups
             // start half a phase apart (one reads scores from TMEM while the other exponentiates)
             if (x == 1 && j == 0 && nt[0] > 0) mbar_wait(&s_empty[0], (su[0] & 1) ^ 1);
+            TR(1, x ? 12 : 10);
             tc_fence_after();
             mma4_bf16(tmem + S_COL + x * BKV, make_sdesc(qa[x], 16, 1024), make_sdesc(ka, 16, 1024), 2, 2, idesc_s, 0u);
             mma_commit(&s_full[x]);
@@ -229,6 +246,7 @@ __global__ void __launch_bounds__(THREADS, 1)
             if (j >= nt[x]) continue;
             mbar_wait(&p_full[x], pu[x] & 1);
             if (j == 0) mbar_wait(&o_empty[x], (n & 1) ^ 1);  // the previous item's O_X has been drained
+            TR(1, x ? 13 : 11);
             tc_fence_after();
             const uint32_t pa = tmem + P_COL + x * (BKV / 2);
 #pragma unroll
@@ -278,11 +296,13 @@ __global__ void __launch_bounds__(THREADS, 1)
       auto tile = [&](int j, auto diag_tag) {
         constexpr bool DIAG = decltype(diag_tag)::value;
         mbar_wait(&s_full[x], su & 1);
+        TR(x ? 2 : 0, 20);
         tc_fence_after();
         uint32_t raw[128];
         tmem_ld128_sync(tS, raw);
         tc_fence_before();
         mbar_arrive_local(&s_empty[x]);  // S is in registers: the next tile's scores may land
+        TR(x ? 2 : 0, 21);
         ++su;
         float* v = reinterpret_cast<float*>(raw);
         if constexpr (DIAG) {
@@ -317,7 +337,9 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
         // P_X is single-buffered: the PV of the previous key tile must have consumed it (and, for a
         // rescale, must have landed in O_X) — waited for only now, so the exponentials overlap it
+        TR(x ? 2 : 0, 23);
         mbar_wait(&p_empty[x], (pu & 1) ^ 1);
+        TR(x ? 2 : 0, 24);
         tc_fence_after();
         tmem_st32(tP, pk);
         tmem_st32(tP + 32, pk + 32);
@@ -346,6 +368,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         tmem_wait_st();
         tc_fence_before();
         mbar_arrive_local(&p_full[x]);
+        TR(x ? 2 : 0, 25);
         ++pu;
       };
       const int nfull = p.causal ? ntiles - 1 : ntiles;
@@ -355,11 +378,13 @@ __global__ void __launch_bounds__(THREADS, 1)
       const float inv_l = 1.f / l;
       // ---- epilogue: O_X (normalised, bf16) -> swizzled staging -> TMA store to C; then the LSE
       mbar_wait(&o_full[x], n & 1);
+      TR(x ? 2 : 0, 26);
       tc_fence_after();
       uint32_t o[DH];
       tmem_ld64_sync(tO, o);
       tc_fence_before();
       mbar_arrive_local(&o_empty[x]);  // O_X is in registers: the next item's PV may start
+      TR(x ? 2 : 0, 27);
       if (issuer) bulk_wait_read<0>();  // the previous item's store has left the staging box
       asm volatile("bar.sync %0, 128;" ::"r"(2 + x) : "memory");
       uint8_t* row = stage + r * 128;
@@ -439,5 +464,16 @@ bool attention_fwd2_fused(int64_t b, int S, int H, int dh, int causal, const voi
   g_prof.end(PROF_ATTN, e0, st, 4.0 * b * H * (double)S * S * dh);
   return true;
 }
+
+#ifdef HM_ATTN_TRACE
+extern "C" int hm_attn2_trace_read(unsigned long long* out, int* counts) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, attn2::g_attn2_trace, sizeof(attn2::g_attn2_trace));
+  cudaMemcpyFromSymbol(counts, attn2::g_attn2_trace_n, sizeof(attn2::g_attn2_trace_n));
+  int z[3] = {0, 0, 0};
+  cudaMemcpyToSymbol(attn2::g_attn2_trace_n, z, sizeof(z));
+  return 0;
+}
+#endif
 
 }  // namespace hm
