@@ -19,7 +19,8 @@ import torch  # noqa: E402
 
 from paper_conf_hotos_lipmk21_b200 import harmony as H  # noqa: E402
 
-NAMES = {1: "tma:Q", 2: "tma:K", 3: "tma:V", 10: "mma:S", 11: "mma:PV", 12: "mma:S_B", 13: "mma:PV_B", 14: "mma:PV_issued", 15: "mma:S_issued", 20: "sm:s_full", 21: "sm:ld", 22: "sm:max_bar",
+NAMES = {1: "tma:Q", 2: "tma:K", 3: "tma:V", 10: "mma:S", 11: "mma:PV", 12: "mma:S_B", 13: "mma:PV_B", 14: "mma:PV_issued", 15: "mma:S_issued", 30: "b:s_full", 31: "b:ld", 33: "b:p_empty", 34: "b:p_full",
+         40: "bm:p_full", 41: "bm:dVdK_issued", 42: "bm:S_start", 43: "bm:S_issued", 20: "sm:s_full", 21: "sm:ld", 22: "sm:max_bar",
          23: "sm:exps", 24: "sm:p_empty", 25: "sm:p_full", 26: "sm:o_full", 27: "sm:o_read"}
 
 
@@ -29,6 +30,7 @@ def main():
     ap.add_argument("--causal", type=int, default=0)
     ap.add_argument("--show", type=int, default=60)
     ap.add_argument("--fwd2", type=int, default=0, help="trace the two-query-tile kernel (HARMONY_ATTN_FWD=2)")
+    ap.add_argument("--bwd", type=int, default=0, help="trace the persistent backward (its first CTA)")
     a = ap.parse_args()
     b, S, h, dh = a.b, 512, 16, 64
     d = h * dh
@@ -39,9 +41,15 @@ def main():
     fn = lib.hm_attn2_trace_read if a.fwd2 else lib.hm_attn_trace_read
     out = np.zeros((3, 2048), np.uint64)
     cnt = np.zeros(3, np.int32)
+    dC = torch.randn(b * S, d, device="cuda").to(torch.bfloat16)
+    dQKV = torch.zeros(b * S, 3 * d, device="cuda", dtype=torch.bfloat16)
     for _ in range(2):
         H.hk("hk_attention_fwd", b, S, h, dh, a.causal, qkv.data_ptr(), C_.data_ptr(), lse.data_ptr(), None)
         fn(out.ctypes.data_as(C.c_void_p), cnt.ctypes.data_as(C.c_void_p))
+        if a.bwd:
+            H.hk("hk_attention_bwd", b, S, h, dh, a.causal, qkv.data_ptr(), C_.data_ptr(), dC.data_ptr(),
+                 lse.data_ptr(), dQKV.data_ptr(), None)
+            fn(out.ctypes.data_as(C.c_void_p), cnt.ctypes.data_as(C.c_void_p))
     t0 = None
     roles = ["softmax warp 4 (tile A)", "MMA", "softmax warp 8 (tile B)"] if a.fwd2 else ["softmax warp 2", "MMA", "TMA"]
     for row, name in enumerate(roles):
