@@ -47,6 +47,13 @@ WORKLOADS = {
     "cfg3": dict(name="cfg3: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=2 x b=4), bf16/fp32-master Adam, "
                       "HBM cap 16 GiB/GPU", model="gpt2-xl-like-preLN", descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True),
                  per_gpu_batch=8, m=2, cap=16 << 30, S=1024),
+    # north_star's ">= 4x the capped HBM": full cfg3 (18 B/param: 26.6 GB of model and
+    # optimizer state) under a 6 GiB cap, 4.1x; nearly every weight, state shard and stash crosses the
+    # host link each step, so the strict swap roofline is the bound
+    "cfg3s": dict(name="cfg3s: GPT-2 XL 48L d1600 h25 S1024 causal, 8 seq/GPU (m=2 x b=4), bf16/fp32-master Adam, "
+                       "HBM cap 6 GiB/GPU (model + Adam state 4.1x the cap)", model="gpt2-xl-like-preLN",
+                  descs=lambda: synth.transformer_stack(48, 1600, 25, 1024, True), per_gpu_batch=8, m=2, cap=6 << 30,
+                  S=1024),
     "cfg4s": dict(name="cfg4s: 8 of cfg4's 36 GPT blocks (d5120 h40 S1024 causal, 2.5B params), 8 seq/GPU (m=4 x b=2), "
                        "bf16/fp32-master Adam, weights + Adam state streamed from pinned host (HBM cap 12 GiB/GPU)",
                   model="gpt-11b-like-preLN-8-of-36", descs=lambda: synth.transformer_stack(8, 5120, 40, 1024, True),

@@ -273,6 +273,20 @@ def test_plan_scales_to_paper_configs():
         assert s.pred_h2d_bytes > 10e9  # op-input stash spills: host-link bound
 
 
+def test_plan_cfg3_at_a_quarter_of_its_state():
+    """north_star's >= 4x claim as a plan: full cfg3 (48 blocks, d = 1600; 18 B/param of
+    model + Adam state = 26.6 GB) under a 6 GiB cap is race-free, inside the cap, and streams nearly
+    all of its state and stash each step (bench.py --workload cfg3s runs it)."""
+    c = synth.CONFIGS["cfg3"]
+    descs = c["descs"]()
+    cap = 6 << 30
+    n_params = sum(12 * d.d_in * d.d_in + 13 * d.d_in for d in descs)
+    assert 18 * n_params > 4 * cap
+    s, _ = plan(descs, microbatches=2, microbatch_size=4, precision=1, hbm_cap_bytes=cap, stash_policy=2)
+    assert s.hazards == 0 and s.arena_bytes <= cap
+    assert s.pred_h2d_bytes > 15e9 and s.pred_d2h_bytes > 15e9
+
+
 def test_operator_split_column_panels_only_when_the_cap_forces_them():
     """Row a15 inside the step: an fp32 MLP layer whose working set does not fit the cap is
     decomposed into column-panel sub-tasks (each needs only W[:, panel]); the plan stays race-free and
