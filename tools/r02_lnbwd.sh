@@ -1,0 +1,14 @@
+# register-only LN backward (co-resident with the side stream's GEMM) vs the 8-warp shared-memory kernel
+mkdir -p gpurun_out
+python -m paper_conf_hotos_lipmk21_b200.build > gpurun_out/build.log 2>&1; echo "build $?"
+timeout 600 python -m pytest tests/test_gpu_kernels.py -m gpu -x -q -p no:cacheprovider -k "layernorm" 2>&1 | tail -1
+for v in 0 1; do HARMONY_LN_BWD_SMEM=$v timeout 300 python tools/ln_bench.py 2>&1 | tail -3 | sed "s/^/smem$v /"; done
+for v in 0 1; do
+  HARMONY_LN_BWD_SMEM=$v timeout 600 python bench.py --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/ab.json 2>gpurun_out/ab.err
+  python -c "
+import json
+d=json.loads(open('gpurun_out/ab.json').read().strip().splitlines()[-1])
+k=d['kernels']
+print('bench smem=$v', round(d['value'],1), round(d['ms_per_step'],2), d['clocks']['sm_mhz'], {c: round(x['seconds']/d['steps']*1e3,2) for c,x in k.items() if x['seconds']})"
+done
+timeout 900 python -m pytest tests/test_gpu_step.py -m gpu -x -q -p no:cacheprovider 2>&1 | tail -1
