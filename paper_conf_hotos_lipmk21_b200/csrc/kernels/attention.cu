@@ -190,6 +190,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   if (warp == 0) {
     if (lane == 0) {
@@ -629,6 +630,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   if (warp == 0) {
     if (lane == 0) {
@@ -893,6 +895,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   if (warp == 0) {
     if (lane == 0) {
@@ -1150,6 +1153,7 @@ __global__ void __launch_bounds__(256) attn_bwd_prep(int64_t ntok, int S, int H,
                                                      const __nv_bfloat16* __restrict__ dO,
                                                      const __nv_bfloat16* __restrict__ O, const float* __restrict__ lse,
                                                      float* __restrict__ sD, float* __restrict__ lse2) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int d = H * dh, lph = dh / 8;  // lanes per head (8 or 16: a head never straddles a warp)
   const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;  // 8-element vector index
   const int64_t nvec = ntok * (d / 8);
@@ -1228,7 +1232,7 @@ bool attention_fwd_fused(int64_t b, int S, int H, int dh, int causal, const void
       HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       attr_set[variant] = true;
     }
-    kern<<<grid, THREADS, smem, st>>>(mq, mk, mv, mc, p);
+    launch_k(kern, dim3(grid), dim3(THREADS), smem, st, mq, mk, mv, mc, p);
   };
   if (dh == 64) {
     if (npoly == 8) launch(1, attn_fwd_kernel<64, 8>, FwdCfg<64>::SMEM);
@@ -1261,7 +1265,7 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
   float* lse2 = sD + align_up((uint64_t)b * H * S * 4, 256) / 4;
   const float scale = 1.0f / std::sqrt((float)dh);
   const int e0 = g_prof.begin(st);
-  attn_bwd_prep<<<(unsigned)ceil_div(b * S * (d / 8), 256), 256, 0, st>>>(b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
+  launch_k(attn_bwd_prep, dim3((unsigned)ceil_div(b * S * (d / 8), 256)), dim3(256), 0, st, b * S, S, H, dh, scale, static_cast<const __nv_bfloat16*>(dO),
                                                              static_cast<const __nv_bfloat16*>(O), lse, sD, lse2);
   check_launch("attn_bwd_prep");
   if (causal) HM_CUDA(cudaMemsetAsync(dst, 0, (size_t)b * H * S * S * 2, st));  // key tiles never visited by a query tile
@@ -1309,11 +1313,11 @@ bool attention_bwd_fused(int64_t b, int S, int H, int dh, int causal, const void
     tcx::make_map_4d(&mq64, q, dh, S, H, b, 3LL * d, dh, (int64_t)S * 3 * d, 64, BwdPCfg::BQS);
     tcx::make_map_4d(&mo64, dO, dh, S, H, b, d, dh, (int64_t)S * d, 64, BwdPCfg::BQS);
     auto kern = alt ? attn_bwd_persistent<true> : attn_bwd_persistent<false>;
-    kern<<<(unsigned)std::min<int64_t>(items, num_sms), THREADS, BwdPCfg::SMEM, st>>>(mq64, mk, mv, mo64, mds32, p, (int)b);
+    launch_k(kern, dim3((unsigned)std::min<int64_t>(items, num_sms)), dim3(THREADS), BwdPCfg::SMEM, st, mq64, mk, mv, mo64, mds32, p, (int)b);
   } else {
     static bool set = false;
     if (!set) { HM_CUDA(cudaFuncSetAttribute(attn_bwd_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, BwdCfg<128>::SMEM)); set = true; }
-    attn_bwd_kernel<128><<<grid, THREADS, BwdCfg<128>::SMEM, st>>>(mq, mk, mv, mo, mds, p);
+    launch_k(attn_bwd_kernel<128>, dim3(grid), dim3(THREADS), BwdCfg<128>::SMEM, st, mq, mk, mv, mo, mds, p);
   }
   check_launch("attn_bwd_kernel");
   g_prof.end(PROF_ATTN, e0, st, 8.0 * b * H * (double)S * S * dh);  // S^T, dP^T, dV, dK contractions

@@ -167,6 +167,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   // registers move to the softmax warpgroups (the per-SM-subpartition file holds one warp of each
   // CTA: 4 x 80 + 8 x 208 <= 12 x 168 registers per lane, the launch allocation)
@@ -459,7 +460,7 @@ bool attention_fwd2_fused(int64_t b, int S, int H, int dh, int causal, const voi
     set = true;
   }
   const int e0 = g_prof.begin(st);
-  attn_fwd2_kernel<<<grid, THREADS, SMEM, st>>>(mq, mk, mv, mc, p);
+  launch_k(attn_fwd2_kernel, dim3(grid), dim3(THREADS), SMEM, st, mq, mk, mv, mc, p);
   check_launch("attn_fwd2_kernel");
   g_prof.end(PROF_ATTN, e0, st, 4.0 * b * H * (double)S * S * dh);
   return true;

@@ -21,6 +21,7 @@ struct RankPtrs {
 
 // dst[k] = (((src_0[k] + src_1[k]) + src_2[k]) + ...) for k < n, float4-vectorised (n4 = n / 4)
 __global__ void __launch_bounds__(256) rank_sum_kernel(int nsrc, int64_t n4, RankPtrs src, float4* __restrict__ dst) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
     float4 a = reinterpret_cast<const float4*>(src.p[0])[i];
     for (int q = 1; q < nsrc; ++q) {
@@ -32,6 +33,7 @@ __global__ void __launch_bounds__(256) rank_sum_kernel(int nsrc, int64_t n4, Ran
 }
 
 __global__ void rank_sum_tail_kernel(int nsrc, int64_t lo, int64_t n, RankPtrs src, float* __restrict__ dst) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t i = lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   float a = src.p[0][i];
@@ -50,12 +52,12 @@ void rank_sum(int nsrc, const float* const* src, int64_t n, float* dst, cudaStre
   int64_t n4 = aligned ? n / 4 : 0;
   if (n4 > 0) {
     const int grid = (int)std::min<int64_t>(ceil_div(n4, 256), 148 * 8);
-    rank_sum_kernel<<<grid, 256, 0, st>>>(nsrc, n4, rp, reinterpret_cast<float4*>(dst));
+    launch_k(rank_sum_kernel, dim3(grid), dim3(256), 0, st, nsrc, n4, rp, reinterpret_cast<float4*>(dst));
     check_launch("rank_sum_kernel");
   }
   const int64_t lo = n4 * 4;
   if (lo < n) {
-    rank_sum_tail_kernel<<<(int)ceil_div(n - lo, 256), 256, 0, st>>>(nsrc, lo, n, rp, dst);
+    launch_k(rank_sum_tail_kernel, dim3((int)ceil_div(n - lo, 256)), dim3(256), 0, st, nsrc, lo, n, rp, dst);
     check_launch("rank_sum_tail_kernel");
   }
 }

@@ -34,6 +34,7 @@ struct SimtParams {
 constexpr int SBM = 64, SBN = 64, SBK = 16;
 
 __global__ void __launch_bounds__(256) gemm_simt_kernel(SimtParams p) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   __shared__ float As[SBK][SBM + 4];
   __shared__ float Bs[SBK][SBN + 4];
   const int tid = threadIdx.x;
@@ -617,6 +618,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   if (warp == 0) {
     if (lane == 0) {
@@ -789,7 +791,7 @@ static void launch_tc(const hk_gemm_args& a, const EpiParams& e, cudaStream_t st
   dim3 grid((unsigned)std::min<int64_t>(tiles, num_sms));  // persistent: at most one CTA per SM
   // profiling events bracket only the device work (tensor maps are encoded before)
   const int e0 = g_prof.begin(st);
-  gemm_tc_kernel<BN, STAGES><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
+  launch_k(gemm_tc_kernel<BN, STAGES>, dim3(grid), dim3(NUM_THREADS), Cfg::SMEM, st, ma, mb, mc, mi, mo, p);
   check_launch("gemm_tc_kernel");
   g_prof.end(PROF_GEMM, e0, st, 2.0 * a.M * a.N * (double)a.K * a.nz0 * a.nz1);
 }
@@ -939,6 +941,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   cluster_sync_all();  // barriers of both CTAs initialised, TMEM allocated in both
   tc_fence_after();
   const uint32_t tmem_base = *tmem_base_s;
+  pdl_wait();  // (after the setup, which touches no global data: it overlaps the previous kernel's tail)
 
   if (warp == 0) {
     if (lane == 0) {
@@ -1070,7 +1073,7 @@ static void launch_tc2_k(const CUtensorMap& ma, const CUtensorMap& mb, const CUt
                                  Cfg::SMEM));
     attr_set = true;
   }
-  gemm_tc2_kernel<BN, STAGES, EK><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(ma, mb, mc, mi, mo, p);
+  launch_k(gemm_tc2_kernel<BN, STAGES, EK>, dim3(grid), dim3(NUM_THREADS), Cfg::SMEM, st, ma, mb, mc, mi, mo, p);
 }
 
 // HARMONY_GEMM_SPECIALIZE=0: always the generic kernel (A/B of the per-kind specialisation)
@@ -1150,7 +1153,7 @@ static bool gemm_impl(const hk_gemm_args& a, float* colsum, cudaStream_t st) {
     p.B = static_cast<const float*>(a.B); p.b_mn = a.b_mn_major; p.ldb = a.ldb; p.b_sz0 = a.b_sz0; p.b_sz1 = a.b_sz1;
     p.e = e;
     dim3 grid((unsigned)ceil_div(a.N, SBN), (unsigned)ceil_div(a.M, SBM), (unsigned)(a.nz0 * a.nz1));
-    gemm_simt_kernel<<<grid, 256, 0, st>>>(p);
+    launch_k(gemm_simt_kernel, dim3(grid), dim3(256), 0, st, p);
     check_launch("gemm_simt_kernel");
     g_prof.end(PROF_GEMM, e0, st, flops);
     return false;

@@ -2,11 +2,37 @@
 #pragma once
 #include <cmath>
 #include <algorithm>
+#include <utility>
 
 #include "../common.hpp"
 #include "harmony_kernels.h"
 
 namespace hm {
+
+// Programmatic dependent launch: every kernel of the step is launched with programmatic stream
+// serialisation, so the next kernel on the stream is launched (and, for the persistent tcgen05
+// kernels, runs its setup: barriers, tensor-map prefetch, TMEM allocation) while the previous one
+// drains; each kernel executes griddepcontrol.wait (pdl_wait) before it touches global memory, which
+// returns once the previous grid has completed and its writes are visible — the results are the
+// same as with plain stream order.  HARMONY_PDL=0 launches without the attribute (A/B).
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+inline void launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  HM_CUDA(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
+}
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+#endif
 
 void gemm(const hk_gemm_args& a, cudaStream_t st);
 // gemm() with a bf16 output C (nz0 = nz1 = 1) that also writes partial[rb][c] = sum of the STORED

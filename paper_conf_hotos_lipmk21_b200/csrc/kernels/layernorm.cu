@@ -49,6 +49,7 @@ __global__ void __launch_bounds__(256) ln_fwd_v(int64_t rows, int d, const float
                                                const T* __restrict__ g, const T* __restrict__ b, T* __restrict__ U,
                                                float* __restrict__ mean, float* __restrict__ rstd,
                                                float* __restrict__ Xcopy) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int lane = threadIdx.x & 31;
   const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (row >= rows) return;
@@ -99,6 +100,7 @@ __global__ void __launch_bounds__(256, 2) ln_bwd_v(int64_t rows, int d, const fl
                                                const float* __restrict__ rstd, const T* __restrict__ g,
                                                const float* __restrict__ dres, float* __restrict__ dX,
                                                T* __restrict__ dXt, int np, float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   // per-warp column partials of dgamma / dbeta (/ sum dX when np == 3) live in shared memory
   // ([8][np][d]); each lane owns
   // fixed columns, so a warp accumulates its rows without races; the 8 warps are then summed in
@@ -196,6 +198,7 @@ struct ColOuts {
 };
 __global__ void __launch_bounds__(1024) colreduce2_kernel(int nchunks, int n, const float* __restrict__ partial,
                                                           int64_t stride, ColOuts outs) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   __shared__ float sh[32][33];
   const int cl = threadIdx.x & 31, g = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
@@ -233,7 +236,7 @@ bool layernorm_fwd_vec(int dtype, int64_t rows, int d, const float* X, const voi
   const int v = ln_vpt(d);
   if (!v) return false;
   const unsigned grid = (unsigned)ceil_div(rows, 8);
-#define HM_LNF(T, V) ln_fwd_v<T, V><<<grid, 256, 0, st>>>(rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd, Xcopy)
+#define HM_LNF(T, V) launch_k(ln_fwd_v<T, V>, dim3(grid), dim3(256), 0, st, rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd, Xcopy)
 #define HM_LNF_ALL(T)                   \
   switch (v) {                          \
     case 1: HM_LNF(T, 1); break;        \
@@ -267,7 +270,7 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
   do {                                                                                                 \
     if (smem > 48 * 1024)                                                                              \
       HM_CUDA(cudaFuncSetAttribute(ln_bwd_v<T, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-    ln_bwd_v<T, V><<<nblk, 256, smem, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres, dX, (T*)dXt, np, scratch); \
+    launch_k(ln_bwd_v<T, V>, dim3(nblk), dim3(256), smem, st, rows, d, dU, X, mean, rstd, (const T*)g, dres, dX, (T*)dXt, np, scratch); \
   } while (0)
 #define HM_LNB_ALL(T)                   \
   switch (v) {                          \
@@ -283,7 +286,7 @@ bool layernorm_bwd_vec(int dtype, int64_t rows, int d, const float* dU, const fl
 #undef HM_LNB
   check_launch("layernorm_bwd_vec");
   ColOuts outs{{dg, db, dsum}, {accumulate, accumulate, dsum_acc}};
-  colreduce2_kernel<<<dim3((unsigned)ceil_div(d, 32), (unsigned)np), 1024, 0, st>>>(nblk, d, scratch, np * (int64_t)d,
+  launch_k(colreduce2_kernel, dim3(dim3((unsigned)ceil_div(d, 32), (unsigned)np)), dim3(1024), 0, st, nblk, d, scratch, np * (int64_t)d,
                                                                                  outs);
   check_launch("colreduce(dgamma, dbeta[, sum dX])");
   return true;

@@ -10,6 +10,14 @@
 
 namespace hm {
 
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* v = getenv("HARMONY_PDL");
+    return !(v && *v == '0');
+  }();
+  return on;
+}
+
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -34,6 +42,7 @@ __global__ void __launch_bounds__(256) layernorm_fwd_kernel(int64_t rows, int d,
                                                             const T* __restrict__ g, const T* __restrict__ b,
                                                             T* __restrict__ U, float* __restrict__ mean,
                                                             float* __restrict__ rstd) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int lane = threadIdx.x & 31;
   const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (row >= rows) return;
@@ -62,6 +71,7 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(int64_t rows, int d,
                                                             const float* __restrict__ rstd, const T* __restrict__ g,
                                                             const float* __restrict__ dres, float* __restrict__ dX,
                                                             float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t r0 = (int64_t)blockIdx.x * LN_ROWS_PER_BLOCK;
   // phase 1: dX per row (one warp per row)
@@ -109,6 +119,7 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(int64_t rows, int d,
 // coalesced along the columns, every load of a warp in flight at once.
 __global__ void __launch_bounds__(1024) colreduce_kernel(int nchunks, int n, const float* __restrict__ partial,
                                                          int64_t stride, float* __restrict__ out, int accumulate) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   // 32 columns x 32 warps per block: warp g sums chunks g, g+32, ... in order (a handful of loads,
   // all in flight at once), then the 32 warp sums are added in warp order — a fixed tree
   __shared__ float sh[32][33];
@@ -132,6 +143,7 @@ __global__ void __launch_bounds__(1024) colreduce_kernel(int nchunks, int n, con
 // (a fixed order: deterministic), four elements per thread with 16-byte loads.
 __global__ void __launch_bounds__(256) splitk_sum_kernel(int S, int64_t n4, const float4* __restrict__ ws,
                                                         float4* __restrict__ C, int accumulate) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n4) return;
   float4 t = ws[i];
@@ -148,7 +160,7 @@ __global__ void __launch_bounds__(256) splitk_sum_kernel(int S, int64_t n4, cons
 void splitk_sum(int S, int64_t n, const float* ws, float* C, int accumulate, cudaStream_t st) {
   HM_CHECK(n % 4 == 0, HARMONY_E_INVALID_ARG, "splitk_sum: n % 4 != 0");
   const int e0 = g_prof.begin(st);
-  splitk_sum_kernel<<<(unsigned)ceil_div(n / 4, 256), 256, 0, st>>>(S, n / 4, reinterpret_cast<const float4*>(ws),
+  launch_k(splitk_sum_kernel, dim3((unsigned)ceil_div(n / 4, 256)), dim3(256), 0, st, S, n / 4, reinterpret_cast<const float4*>(ws),
                                                                    reinterpret_cast<float4*>(C), accumulate);
   check_launch("splitk_sum");
   g_prof.end(PROF_OTHER, e0, st, (double)n * 4 * (S + 1 + (accumulate ? 1 : 0)));
@@ -156,7 +168,7 @@ void splitk_sum(int S, int64_t n, const float* ws, float* C, int accumulate, cud
 
 static void colreduce(int nchunks, int n, const float* partial, int64_t stride, float* out, int accumulate,
                       cudaStream_t st) {
-  colreduce_kernel<<<(unsigned)ceil_div(n, 32), 1024, 0, st>>>(nchunks, n, partial, stride, out, accumulate);
+  launch_k(colreduce_kernel, dim3((unsigned)ceil_div(n, 32)), dim3(1024), 0, st, nchunks, n, partial, stride, out, accumulate);
   check_launch("colreduce");
 }
 
@@ -164,6 +176,7 @@ static void colreduce(int nchunks, int n, const float* partial, int64_t stride, 
 // block's rows in increasing order — the order of the fused epilogue, so the partials are identical
 __global__ void colsum32_partial_kernel(int64_t rows, int n, const __nv_bfloat16* __restrict__ X, int64_t ld,
                                         float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t rb = blockIdx.y;
   if (c >= n) return;
@@ -174,7 +187,7 @@ __global__ void colsum32_partial_kernel(int64_t rows, int n, const __nv_bfloat16
 void colsum32_partial(int64_t rows, int n, const void* X, int64_t ld, float* partial, cudaStream_t st) {
   if (rows <= 0 || n <= 0) return;
   dim3 grid((unsigned)ceil_div(n, 128), (unsigned)ceil_div(rows, 32));
-  colsum32_partial_kernel<<<grid, 128, 0, st>>>(rows, n, static_cast<const __nv_bfloat16*>(X), ld, partial);
+  launch_k(colsum32_partial_kernel, dim3(grid), dim3(128), 0, st, rows, n, static_cast<const __nv_bfloat16*>(X), ld, partial);
   check_launch("colsum32_partial");
 }
 void colsum32_reduce(int64_t rows, int n, const float* partial, float* out, int accumulate, cudaStream_t st) {
@@ -195,6 +208,7 @@ constexpr int CS_ROWS = 16;
 template <typename Tin>
 __global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict__ X, int64_t ld,
                                       float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= n) return;
   int64_t r0 = (int64_t)blockIdx.y * CS_ROWS, r1 = min(rows, r0 + CS_ROWS);
@@ -205,6 +219,7 @@ __global__ void colsum_partial_kernel(int64_t rows, int n, const Tin* __restrict
 template <typename Tin>
 __global__ void __launch_bounds__(128) colsum_partial_vec_kernel(int64_t rows, int n, const Tin* __restrict__ X,
                                                                  int64_t ld, float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   constexpr int VEC = 16 / sizeof(Tin);
   const int c0 = (blockIdx.x * blockDim.x + threadIdx.x) * VEC;
   if (c0 >= n) return;
@@ -232,6 +247,7 @@ __global__ void __launch_bounds__(128) colsum_partial_vec_kernel(int64_t rows, i
 template <typename T>
 __global__ void __launch_bounds__(128) cast_colsum_partial_kernel(int64_t rows, int n, const float* __restrict__ X,
                                                                   T* __restrict__ Xt, float* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int c0 = (blockIdx.x * blockDim.x + threadIdx.x) * 4;
   if (c0 >= n) return;
   const int64_t r0 = (int64_t)blockIdx.y * CS_ROWS, r1 = min(rows, r0 + CS_ROWS);
@@ -256,6 +272,7 @@ __global__ void __launch_bounds__(128) cast_colsum_partial_kernel(int64_t rows, 
 template <typename T>
 __global__ void __launch_bounds__(256) softmax_fwd_kernel(int64_t rows, int S, int causal, float scale,
                                                           const float* __restrict__ Z, T* __restrict__ P) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int lane = threadIdx.x & 31;
   const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (row >= rows) return;
@@ -276,6 +293,7 @@ template <typename T>
 __global__ void __launch_bounds__(256) softmax_bwd_kernel(int64_t rows, int S, float alpha,
                                                           const float* __restrict__ dP, const T* __restrict__ P,
                                                           T* __restrict__ dZ) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int lane = threadIdx.x & 31;
   const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (row >= rows) return;
@@ -294,6 +312,7 @@ template <typename T>
 __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict__ m, float* __restrict__ v,
                             const float* __restrict__ g, T* __restrict__ Wc, float lr, float b1, float omb1, float b2,
                             float omb2, float eps, double b1d, double b2d, const int* __restrict__ t_dev, int t_host) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   // bias corrections 1/(1-b^t) in double, once per block; t from device memory when given
   // (a CUDA-graph replay updates it without re-launching)
   __shared__ float s_bc[2];
@@ -347,6 +366,7 @@ __global__ void adam_kernel(int64_t n, float* __restrict__ W, float* __restrict_
 constexpr int MSE_BLOCK = 256;
 __global__ void mse_kernel(int64_t n, const float* __restrict__ Y, const float* __restrict__ Tg, float inv_batch,
                            float* __restrict__ dY, double* __restrict__ partial) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   __shared__ double sh[MSE_BLOCK / 32];
   double acc = 0.0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -368,6 +388,7 @@ __global__ void mse_kernel(int64_t n, const float* __restrict__ Y, const float* 
 // fixed-order tree over the block partials: thread t sums t, t+256, ...; then a smem tree
 __global__ void __launch_bounds__(256) mse_final_kernel(int nblk, const double* __restrict__ partial,
                                                         double half_inv_batch, double* __restrict__ out) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   __shared__ double sh[256];
   double s = 0.0;
   for (int j = threadIdx.x; j < nblk; j += 256) s += partial[j];
@@ -383,23 +404,27 @@ __global__ void __launch_bounds__(256) mse_final_kernel(int nblk, const double* 
 // ------------------------------------------------------------------------------------- elementwise
 template <typename T>
 __global__ void cast_kernel(int64_t n, const float* __restrict__ in, T* __restrict__ out) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = from_f32<T>(in[i]);
 }
 template <typename T>
 __global__ void act_bwd_kernel(int act, int64_t n, const float* __restrict__ dY, const T* __restrict__ Z,
                                T* __restrict__ dZ) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
     dZ[i] = from_f32<T>(dY[i] * act_grad_T<T>(act, to_f32(Z[i])));
 }
 template <typename T>
 __global__ void act_fwd_kernel(int act, int64_t n, const T* __restrict__ Z, T* __restrict__ out) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
     out[i] = from_f32<T>(act_T<T>(act, to_f32(Z[i])));
 }
 __global__ void copy_rows_kernel(int64_t n4, const float4* __restrict__ src, float4* __restrict__ dst) {
+  pdl_wait();  // programmatic dependent launch: the previous kernel's results are visible
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) dst[i] = src[i];
 }
@@ -425,7 +450,7 @@ void layernorm_fwd(int dtype, int64_t rows, int d, const float* X, const void* g
     return;
   }
   if (Xcopy) copy_f32(rows * d, X, Xcopy, st);
-  HM_DISPATCH_T(dtype, (layernorm_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(
+  HM_DISPATCH_T(dtype, (launch_k(layernorm_fwd_kernel<T>, dim3((unsigned)ceil_div(rows, 8)), dim3(256), 0, st, 
                            rows, d, X, (const T*)g, (const T*)b, (T*)U, mean, rstd)));
   check_launch("layernorm_fwd");
   g_prof.end(PROF_LN, e0, st, (double)rows * d * (4 + (dtype ? 2 : 4)) + rows * 8.0);
@@ -455,7 +480,7 @@ void layernorm_bwd_ex(int dtype, int64_t rows, int d, const float* dU, const flo
     return;
   }
   int nblk = (int)ceil_div(rows, LN_ROWS_PER_BLOCK);
-  HM_DISPATCH_T(dtype, (layernorm_bwd_kernel<T><<<nblk, 256, 0, st>>>(rows, d, dU, X, mean, rstd, (const T*)g, dres,
+  HM_DISPATCH_T(dtype, (launch_k(layernorm_bwd_kernel<T>, dim3(nblk), dim3(256), 0, st, rows, d, dU, X, mean, rstd, (const T*)g, dres,
                                                                       dX, scratch)));
   check_launch("layernorm_bwd");
   colreduce(nblk, d, scratch, 2 * (int64_t)d, dg, accumulate, st);
@@ -479,10 +504,10 @@ void colsum(int in_dtype, int64_t rows, int n, const void* X, int64_t ld, float*
   const int e0 = g_prof.begin(st);
   if (vok) {
     dim3 grid((unsigned)ceil_div(n / vec, 128), (unsigned)nch);
-    HM_DISPATCH_T(in_dtype, (colsum_partial_vec_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+    HM_DISPATCH_T(in_dtype, (launch_k(colsum_partial_vec_kernel<T>, dim3(grid), dim3(128), 0, st, rows, n, (const T*)X, ld, scratch)));
   } else {
     dim3 grid((unsigned)ceil_div(n, 128), (unsigned)nch);
-    HM_DISPATCH_T(in_dtype, (colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, (const T*)X, ld, scratch)));
+    HM_DISPATCH_T(in_dtype, (launch_k(colsum_partial_kernel<T>, dim3(grid), dim3(128), 0, st, rows, n, (const T*)X, ld, scratch)));
   }
   check_launch("colsum_partial");
   colreduce(nch, n, scratch, n, out, accumulate, st);
@@ -499,7 +524,7 @@ void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float
   }
   const int e0 = g_prof.begin(st);
   dim3 grid((unsigned)ceil_div(n / 4, 128), (unsigned)nch);
-  HM_DISPATCH_T(dtype, (cast_colsum_partial_kernel<T><<<grid, 128, 0, st>>>(rows, n, X, (T*)Xt, scratch)));
+  HM_DISPATCH_T(dtype, (launch_k(cast_colsum_partial_kernel<T>, dim3(grid), dim3(128), 0, st, rows, n, X, (T*)Xt, scratch)));
   check_launch("cast_colsum_partial");
   colreduce(nch, n, scratch, n, out, accumulate, st);
   g_prof.end(PROF_OTHER, e0, st, (double)rows * n * (4 + (dtype ? 2 : 4)));
@@ -508,7 +533,7 @@ void cast_colsum(int dtype, int64_t rows, int n, const float* X, void* Xt, float
 void softmax_fwd(int dtype, int64_t rows, int S, int causal, float scale, const float* Z, void* P, cudaStream_t st) {
   if (rows == 0) return;
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(dtype, (softmax_fwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, causal, scale, Z,
+  HM_DISPATCH_T(dtype, (launch_k(softmax_fwd_kernel<T>, dim3((unsigned)ceil_div(rows, 8)), dim3(256), 0, st, rows, S, causal, scale, Z,
                                                                                           (T*)P)));
   check_launch("softmax_fwd");
   g_prof.end(PROF_SOFTMAX, e0, st, (double)rows * S * (4 + (dtype ? 2 : 4)));
@@ -518,7 +543,7 @@ void softmax_bwd(int dtype, int64_t rows, int S, float alpha, const float* dP, c
                  cudaStream_t st) {
   if (rows == 0) return;
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(dtype, (softmax_bwd_kernel<T><<<(unsigned)ceil_div(rows, 8), 256, 0, st>>>(rows, S, alpha, dP,
+  HM_DISPATCH_T(dtype, (launch_k(softmax_bwd_kernel<T>, dim3((unsigned)ceil_div(rows, 8)), dim3(256), 0, st, rows, S, alpha, dP,
                                                                                           (const T*)P, (T*)dZ)));
   check_launch("softmax_bwd");
   g_prof.end(PROF_SOFTMAX, e0, st, (double)rows * S * (4 + 2 * (dtype ? 2 : 4)));
@@ -530,7 +555,7 @@ void adam(int dtype, int64_t n, float* W, float* m, float* v, const float* g, vo
   HM_CHECK(((uintptr_t)W | (uintptr_t)m | (uintptr_t)v | (uintptr_t)g) % 16 == 0, HARMONY_E_INVALID_ARG,
            "adam: fp32 state must be 16-byte aligned");
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(dtype, (adam_kernel<T><<<grid_for(ceil_div(n, 4), 256), 256, 0, st>>>(
+  HM_DISPATCH_T(dtype, (launch_k(adam_kernel<T>, dim3(grid_for(ceil_div(n, 4), 256)), dim3(256), 0, st, 
                            n, W, m, v, g, (T*)Wc, (float)lr, (float)b1, (float)(1.0 - b1), (float)b2, (float)(1.0 - b2), (float)eps,
                            b1, b2, t_dev, t)));
   check_launch("adam");
@@ -542,16 +567,16 @@ size_t mse_scratch_bytes() { return 1024 * sizeof(double); }
 void mse(int64_t n, const float* Y, const float* Tg, float inv_batch, float* dY, double* loss_out, double* scratch,
          cudaStream_t st) {
   int nblk = (int)std::min<int64_t>(1024, std::max<int64_t>(1, ceil_div(n, MSE_BLOCK * 8)));
-  mse_kernel<<<nblk, MSE_BLOCK, 0, st>>>(n, Y, Tg, inv_batch, dY, scratch);
+  launch_k(mse_kernel, dim3(nblk), dim3(MSE_BLOCK), 0, st, n, Y, Tg, inv_batch, dY, scratch);
   check_launch("mse");
-  mse_final_kernel<<<1, 256, 0, st>>>(nblk, scratch, 0.5 * (double)inv_batch, loss_out);
+  launch_k(mse_final_kernel, dim3(1), dim3(256), 0, st, nblk, scratch, 0.5 * (double)inv_batch, loss_out);
   check_launch("mse_final");
 }
 
 void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st) {
   if (n == 0) return;
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(dtype, (cast_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(n, in, (T*)out)));
+  HM_DISPATCH_T(dtype, (launch_k(cast_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, n, in, (T*)out)));
   check_launch("cast");
   g_prof.end(PROF_OTHER, e0, st, (double)n * (4 + (dtype ? 2 : 4)));
 }
@@ -559,14 +584,14 @@ void cast(int dtype, int64_t n, const float* in, void* out, cudaStream_t st) {
 void act_bwd(int dtype, int act, int64_t n, const float* dY, const void* Z, void* dZ, cudaStream_t st) {
   if (n == 0) return;
   const int e0 = g_prof.begin(st);
-  HM_DISPATCH_T(dtype, (act_bwd_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(act, n, dY, (const T*)Z, (T*)dZ)));
+  HM_DISPATCH_T(dtype, (launch_k(act_bwd_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, act, n, dY, (const T*)Z, (T*)dZ)));
   check_launch("act_bwd");
   g_prof.end(PROF_OTHER, e0, st, (double)n * (4 + 2 * (dtype ? 2 : 4)));
 }
 
 void act_fwd_T(int dtype, int act, int64_t n, const void* Z, void* out, cudaStream_t st) {
   if (n == 0) return;
-  HM_DISPATCH_T(dtype, (act_fwd_kernel<T><<<grid_for(n, 256), 256, 0, st>>>(act, n, (const T*)Z, (T*)out)));
+  HM_DISPATCH_T(dtype, (launch_k(act_fwd_kernel<T>, dim3(grid_for(n, 256)), dim3(256), 0, st, act, n, (const T*)Z, (T*)out)));
   check_launch("act_fwd");
 }
 
@@ -574,7 +599,7 @@ void copy_f32(int64_t n, const float* src, float* dst, cudaStream_t st) {
   if (n == 0) return;
   if (n % 4 == 0 && ((uintptr_t)src | (uintptr_t)dst) % 16 == 0) {
     const int e0 = g_prof.begin(st);
-    copy_rows_kernel<<<grid_for(n / 4, 256), 256, 0, st>>>(n / 4, (const float4*)src, (float4*)dst);
+    launch_k(copy_rows_kernel, dim3(grid_for(n / 4, 256)), dim3(256), 0, st, n / 4, (const float4*)src, (float4*)dst);
     check_launch("copy_f32");
     g_prof.end(PROF_OTHER, e0, st, (double)n * 8);
   } else {
