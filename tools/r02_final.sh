@@ -7,7 +7,7 @@ python tools/traffic_summary.py gpurun_out/r02_traffic_launches.csv --last 158 >
 python tools/launch_shares.py gpurun_out/r02_traffic_launches.csv --last 158 > gpurun_out/r02_launch_shares_cfg2_m2.txt 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:gemm_tc2 -c 1 -s 3 -o gpurun_out/r02_ncu_full_gemm_qkv -f python tools/gemm_bench.py --only qkv_fwd --reps 3 > /dev/null 2>&1; echo "ncu full $?"
 timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/r02_final_cfg2.json 2> gpurun_out/r02_final_cfg2.err; echo "cfg2 $?"
-timeout 900 python bench.py --workload cfg3 --no-cpu-baseline > gpurun_out/r02_final_cfg3.json 2> gpurun_out/r02_final_cfg3.err; echo "cfg3 $?"
+timeout 900 python bench.py --workload cfg3 --no-cpu-baseline --steps 5 > gpurun_out/r02_final_cfg3.json 2> gpurun_out/r02_final_cfg3.err; echo "cfg3 $?"
 timeout 1500 python bench.py --workload cfg3s --no-cpu-baseline --steps 3 > gpurun_out/r02_final_cfg3s.json 2> gpurun_out/r02_final_cfg3s.err; echo "cfg3s $?"
 timeout 1200 python bench.py --workload cfg4s --no-cpu-baseline --steps 3 > gpurun_out/r02_final_cfg4s.json 2> gpurun_out/r02_final_cfg4s.err; echo "cfg4s $?"
 timeout 600 python bench.py --workload cfg1 --no-cpu-baseline > gpurun_out/r02_final_cfg1.json 2> gpurun_out/r02_final_cfg1.err; echo "cfg1 $?"
