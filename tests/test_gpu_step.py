@@ -356,3 +356,13 @@ def test_per_kind_gemm_kernels_are_bitwise_the_generic_kernel():
     bitwise_equal(spec, generic)
     descs, params, batches, kw = tiny_transformer(False, 1, **shape)
     compare(spec, run_oracle(descs, params, batches), 2e-2)
+
+
+def test_programmatic_dependent_launch_is_bitwise_plain_stream_order():
+    """Every kernel is launched with programmatic stream serialisation and waits (griddepcontrol.wait)
+    before touching global memory; the step must equal the one launched in plain stream order
+    (HARMONY_PDL=0) bit for bit — a kernel reading its predecessor's output early would show here."""
+    shape = dict(L=2, d=256, h=4, S=512, B=12, m=2)
+    pdl = _step_in_subprocess({}, **shape)
+    plain = _step_in_subprocess({"HARMONY_PDL": "0"}, **shape)
+    bitwise_equal(pdl, plain)
