@@ -373,6 +373,8 @@ def main():
                     help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--groups", type=int, default=1,
                     help="G microbatch groups (direction balance: group g's backward interleaved with g+1's forward)")
+    ap.add_argument("--fwd-pack", type=int, default=1,
+                    help="forward pack size (2: each layer's forward on two microbatches at once; NEXT-4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
@@ -446,7 +448,7 @@ def main():
         torch.cuda.empty_cache()
     cfg = dict(rank=rank, world_size=world, device=local, hbm_cap_bytes=wl["cap"], microbatches=m,
                microbatch_size=B // m, precision=precision, stash_policy=args.stash_policy if precision else 0,
-               lr=1e-4, nccl_id=nccl_id, groups=args.groups,
+               lr=1e-4, nccl_id=nccl_id, groups=args.groups, fwd_pack=args.fwd_pack,
                schedule=H.HARMONY_SCHED_PER_GPU_VIRT if args.schedule == "baseline" else H.HARMONY_SCHED_HARMONY_DP)
     h = H.Harmony(descs, params, **cfg)
     del params
@@ -583,6 +585,7 @@ def main():
         "vs_baseline": None, "dtype": "bf16" if precision else "f32", "data": "synthetic (seeded, paper-shaped)",
         "config": {"workload": wl["name"], "global_batch": B * world, "seq_len": wl["S"],
                    "microbatches": m, "microbatch_size": B // m, "schedule": args.schedule, "groups": args.groups,
+                   "fwd_pack": args.fwd_pack,
                    **({"tuning": tuning} if tuning else {}),
                    "parallelism": f"dp{world}", "hbm_cap_bytes_per_gpu": wl["cap"],
                    "arena_bytes": plan["arena_bytes"], "stash_policy": cfg["stash_policy"],

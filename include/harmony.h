@@ -130,6 +130,14 @@ typedef struct {
                                 balance).  Every layer's fp32 dW stays in HBM across the groups.
                                 The microbatches keep their canonical order in every accumulation:
                                 results are bit-identical for every G (reading c21).             */
+  int32_t fwd_pack;          /* forward pack size ("pack size per pass", P:749-757,
+                                783-801): 0 or 1 = one forward task per microbatch; 2 = the forward
+                                pass runs each layer on two consecutive microbatches at once (GEMMs
+                                of 2*b*S rows), while the backward stays per microbatch (its working
+                                set is the larger one).  Harmony-DP, block recompute (stash_policy
+                                2), transformer layers of one width, m % (2*G) == 0; anything else
+                                is HARMONY_E_UNSUPPORTED.  Every per-row and per-element result is
+                                computed in the same order, so the step is bit-identical.        */
 } harmony_config;
 
 typedef struct {

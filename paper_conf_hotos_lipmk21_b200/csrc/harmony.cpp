@@ -368,8 +368,12 @@ void op_body(harmony_ctx* c, const Op& o, const RankIn& in, harmony_step_stats& 
     }
     case OP_FWD: {
       const LayerPlan& lp = p.layers[o.layer];
-      layer_fwd(lp.g, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
-                A + o.stash, A + o.ws, st);
+      if (o.pack == 2)
+        layer_fwd_pack2(lp.gp, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
+                        A + o.stash, A + o.stash2, A + o.ws, st);
+      else
+        layer_fwd(lp.g, A + o.w, reinterpret_cast<const float*>(A + o.in), reinterpret_cast<float*>(A + o.out),
+                  A + o.stash, A + o.ws, st);
       break;
     }
     case OP_LOSS: {

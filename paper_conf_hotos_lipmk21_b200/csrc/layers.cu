@@ -249,7 +249,8 @@ struct AttnStash {
 };
 
 static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws,
-                     void* stv, bool stash_x = true, const AttnStash* as = nullptr, float* x_copy = nullptr) {
+                     void* stv, bool stash_x = true, const AttnStash* as = nullptr, float* x_copy = nullptr,
+                     float* x_copy2 = nullptr) {
   cudaStream_t st = static_cast<cudaStream_t>(stv);
   const harmony_layer_desc& d = g.desc;
   if (d.kind == HARMONY_LAYER_MLP) {
@@ -287,7 +288,16 @@ static void fwd_core(const LayerGeom& g, const void* W, const float* X, float* Y
   if (stash_x) copy_f32(R * D, X, Xs, st);
   // U = LN1(X)
   // (block recompute: the LN reads X once and also writes the stashed copy of the block input)
-  layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st, x_copy);
+  if (x_copy2) {
+    // a forward pack of two microbatches: each half of the rows stashes its block input in its own
+    // microbatch's stash (LayerNorm is per row: the same bits as one launch)
+    const int64_t h = R / 2;
+    layernorm_fwd(g.dtype, h, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st, x_copy);
+    layernorm_fwd(g.dtype, h, D, X + h * D, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U + (size_t)h * D * ts,
+                  mean1 + h, rstd1 + h, st, x_copy2);
+  } else {
+    layernorm_fwd(g.dtype, R, D, X, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), U, mean1, rstd1, st, x_copy);
+  }
   // QKV = U W_qkv + b_qkv
   {
     hk_gemm_args a = lin_fwd(g, R, 3 * D, D, U, wseg(g, W, P_WQKV));
@@ -576,6 +586,19 @@ void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint
   const AttnStash as{stash + g.st.C, reinterpret_cast<float*>(stash + g.st.P), false};
   fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false, g.stash_policy == 3 ? &as : nullptr,
            reinterpret_cast<float*>(stash + g.st.X));
+}
+
+// A forward pack (fwd_pack = 2): gp is the layer's geometry at two microbatches (block recompute);
+// X / Y span both microbatches' rows, and each writes its block input into its own stash.
+void layer_fwd_pack2(const LayerGeom& gp, const void* W, const float* X, float* Y, uint8_t* stash0, uint8_t* stash1,
+                     uint8_t* ws, void* st) {
+  HM_CHECK(gp.stash_policy == 2 && gp.desc.kind == HARMONY_LAYER_TRANSFORMER, HARMONY_E_UNSUPPORTED,
+           "forward packs: block-recompute transformer layers");
+  const LayerGeom c = core_geom(gp);
+  uint8_t* full = ws + gp.core_off;
+  uint8_t* rest = ws + align_up(c.st.total, 256);
+  fwd_core(c, W, X, Y, full, rest, st, /*stash_x=*/false, nullptr, reinterpret_cast<float*>(stash0 + gp.st.X),
+           reinterpret_cast<float*>(stash1 + gp.st.X));
 }
 
 void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,

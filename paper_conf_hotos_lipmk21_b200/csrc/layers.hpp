@@ -55,6 +55,8 @@ int64_t layer_n_params(const harmony_layer_desc& desc);
 
 // Task bodies (launch kernels on st).  W: compute copy of the layer (T elements, canonical packing).
 void layer_fwd(const LayerGeom& g, const void* W, const float* X, float* Y, uint8_t* stash, uint8_t* ws, void* st);
+void layer_fwd_pack2(const LayerGeom& gp, const void* W, const float* X, float* Y, uint8_t* stash0, uint8_t* stash1,
+                     uint8_t* ws, void* st);
 // Lend the backward tasks a second stream (and 4 events) for weight-gradient work; nullptr = none.
 void set_side_stream(void* st, void* const* events);
 void layer_bwd(const LayerGeom& g, const void* W, const uint8_t* stash, const float* dY, float* dX, float* dW,

@@ -29,6 +29,7 @@ void validate_config(const harmony_config& c) {
            HARMONY_E_INVALID_ARG, "unknown schedule");
   HM_CHECK(c.stash_policy >= 0 && c.stash_policy <= 3, HARMONY_E_INVALID_ARG, "stash_policy must be 0..3");
   HM_CHECK(c.groups >= 0 && c.groups <= 64, HARMONY_E_INVALID_ARG, "groups must be in 0..64");
+  HM_CHECK(c.fwd_pack >= 0 && c.fwd_pack <= 2, HARMONY_E_INVALID_ARG, "fwd_pack must be 0, 1 or 2");
   HM_CHECK(c.weight_decay == 0.0, HARMONY_E_UNSUPPORTED, "weight_decay must be 0 (reading c3)");
   HM_CHECK(c.lr > 0 && c.beta1 >= 0 && c.beta1 < 1 && c.beta2 >= 0 && c.beta2 < 1 && c.eps > 0,
            HARMONY_E_INVALID_ARG, "bad Adam hyper-parameters");
@@ -151,11 +152,13 @@ static std::vector<Acc> accesses(const Plan& p, const Op& o) {
     case OP_D2H: ar(o.dev, o.bytes, false); hb(o.hbuf, o.hidx, o.hoff, o.bytes, true); break;
     case OP_FWD: {
       const LayerPlan& lp = p.layers[o.layer];
+      const uint64_t pk = (uint64_t)o.pack;  // a pack spans its microbatches' contiguous rows
       ar(o.w, (uint64_t)lp.P * ts, false);
-      ar(o.in, (uint64_t)lp.g.rows * lp.g.desc.d_in * 4, false);
-      ar(o.out, (uint64_t)lp.g.rows * lp.g.ld_out * 4, true);  // (a column panel: within these rows)
+      ar(o.in, pk * lp.g.rows * lp.g.desc.d_in * 4, false);
+      ar(o.out, pk * lp.g.rows * lp.g.ld_out * 4, true);  // (a column panel: within these rows)
       ar(o.stash, lp.g.st.total, true);
-      ar(o.ws, lp.g.ws_fwd, true);
+      if (o.pack == 2) ar(o.stash2, lp.g.st.total, true);
+      ar(o.ws, o.pack == 2 ? lp.gp.ws_fwd : lp.g.ws_fwd, true);
       break;
     }
     case OP_BWD: {
@@ -335,6 +338,10 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
     lp.state_bytes = 3 * (uint64_t)lp.shard * 4;
     lp.stash_res.assign(m, -1);
     ws_need = std::max({ws_need, lp.g.ws_fwd, lp.g.ws_bwd});
+    if (cfg.fwd_pack == 2) {  // the forward pass on two microbatches at once (NEXT-4 pack size)
+      lp.gp = make_geom(descs[u], 2 * p.b, p.dtype, p.stash_policy);
+      ws_need = std::max(ws_need, lp.gp.ws_fwd);
+    }
     maxP = std::max<uint64_t>(maxP, (uint64_t)lp.Ppad);
     max_shard = std::max<uint64_t>(max_shard, (uint64_t)lp.shard);
     p.n_params += lp.P;
@@ -355,6 +362,16 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
   HM_CHECK(G == 1 || p.schedule == HARMONY_SCHED_HARMONY_DP, HARMONY_E_UNSUPPORTED,
            "microbatch groups are a Harmony-DP schedule");
   const int mg = m / G;
+  p.fwd_pack = cfg.fwd_pack == 2 ? 2 : 1;
+  if (p.fwd_pack == 2) {
+    bool ok = p.schedule == HARMONY_SCHED_HARMONY_DP && p.stash_policy == 2 && mg % 2 == 0 && L == LU;
+    for (int l = 0; l < L && ok; ++l)
+      ok = descs[l].kind == HARMONY_LAYER_TRANSFORMER && descs[l].d_in == dmax &&
+           bnd_stride == (uint64_t)rows * dmax * 4;  // consecutive microbatches' rows are contiguous
+    HM_CHECK(ok, HARMONY_E_UNSUPPORTED,
+             "fwd_pack = 2 needs Harmony-DP, stash_policy 2, uniform transformer layers and "
+             "microbatches per group a multiple of 2");
+  }
   const int nDW = G > 1 ? L : (N > 1 ? 2 : 1);
   auto dwi = [&](int l) { return G > 1 ? l : l % nDW; };
   auto fixed_bytes = [&]() {
@@ -614,7 +631,7 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
     Task t;  // inputs are issued as the first ops (not prefetch items)
     (void)t;
   }
-  auto fwd_task = [&](int l, int i, bool gfirst) {
+  auto fwd_task = [&](int l, int i, bool gfirst, int pack) {
     LayerPlan& lp = p.layers[l];
     const int in_buf = lp.user % 2, out_buf = (lp.user + 1) % 2;  // a registered layer's panels share its buffers
     int slot = -1;
@@ -623,25 +640,33 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
     else { slot = fwd_wslot[l]; wdev = slot >= 0 ? p.wslot[slot] : (uint64_t)lp.wc_res; }
     fwd_wslot[l] = slot;
     Task t;
-    t.op.kind = OP_FWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i;
+    t.op.kind = OP_FWD; t.op.stream = S_COMPUTE; t.op.layer = l; t.op.mb = i; t.op.pack = pack;
     t.op.w = wdev; t.op.in = bnd_row(in_buf, i); t.op.out = bnd_row(out_buf, i); t.op.ws = p.ws;
-    t.rd = {wkey(l, slot), key(R_BND, in_buf, i)};
-    t.wr = {key(R_BND, out_buf, i)};
-    if (lp.stash_res[i] >= 0) {
-      t.op.stash = (uint64_t)lp.stash_res[i];
-      t.wr.push_back(key(R_STASHRES, l, i));
-    } else {
-      int g = gnext;
-      gnext = (gnext + 1) % nG;
-      t.op.stash = p.stage[g];
-      t.wr.push_back(key(R_STAGE, g));
-      Op d;
-      d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = l; d.mb = i;
-      d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + i; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
-      t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, i)}}});
-      stage_last[g] = (int)tasks.size();
-      spill_task[(size_t)l * m + i] = (int)tasks.size();
+    t.rd = {wkey(l, slot)};
+    // a pack reads / writes the consecutive (contiguous) rows of its microbatches and writes each one's stash
+    for (int k = 0; k < pack; ++k) {
+      const int ik = i + k;
+      t.rd.push_back(key(R_BND, in_buf, ik));
+      t.wr.push_back(key(R_BND, out_buf, ik));
+      uint64_t& dst = k == 0 ? t.op.stash : t.op.stash2;
+      if (lp.stash_res[ik] >= 0) {
+        dst = (uint64_t)lp.stash_res[ik];
+        t.wr.push_back(key(R_STASHRES, l, ik));
+      } else {
+        int g = gnext;
+        gnext = (gnext + 1) % nG;
+        dst = p.stage[g];
+        t.wr.push_back(key(R_STAGE, g));
+        Op d;
+        d.kind = OP_D2H; d.stream = S_D2H; d.cat = CAT_STASH; d.layer = l; d.mb = ik;
+        d.hbuf = HB_STASH; d.hidx = (int64_t)l * m + ik; d.dev = p.stage[g]; d.bytes = lp.g.st.total;
+        t.post.push_back({d, {{key(R_STAGE, g)}, {key(H_STASH, l, ik)}}});
+        stage_last[g] = (int)tasks.size();
+        spill_task[(size_t)l * m + ik] = (int)tasks.size();
+      }
     }
+    HM_CHECK(pack == 1 || t.op.stash != t.op.stash2, HARMONY_E_CAP_TOO_SMALL,
+             "fwd_pack = 2 needs two staging slots for two spilled stashes");
     if (slot >= 0) wslot_last[slot] = (int)tasks.size();
     if (baseline && slot >= 0) {  // per-GPU virtualization: weights out again after each forward
       Op d;
@@ -842,7 +867,7 @@ static Plan make_plan_impl(const harmony_config& cfg, int n_layers, const harmon
   // and spills (forward) use both directions of the host link at once.  The microbatches stay in
   // canonical order in every dW accumulation: the result is bit-identical for every G (reading c21).
   auto fwd_group = [&](int g, int l) {
-    for (int i = g * mg; i < (g + 1) * mg; ++i) fwd_task(l, i, i == g * mg);
+    for (int i = g * mg; i < (g + 1) * mg; i += p.fwd_pack) fwd_task(l, i, i == g * mg, p.fwd_pack);
   };
   auto loss_group = [&](int g) {
     for (int i = g * mg; i < (g + 1) * mg; ++i) loss_task(i);

@@ -41,12 +41,14 @@ struct Op {
   int kind = 0, stream = 0, cat = CAT_NONE;
   int layer = -1, mb = -1;
   int first = 0;  // BWD: first microbatch of the group (dW written, not accumulated)
+  int pack = 1;   // FWD: microbatches mb .. mb+pack-1 in one task (rows contiguous in the activation buffers)
   // copies: host side (buffer kind, index = layer or layer*m+mb, byte offset), device side arena offset
   int hbuf = HB_NONE;
   int64_t hidx = -1;
   uint64_t hoff = 0, dev = 0, bytes = 0;
   // compute operands: arena byte offsets
   uint64_t w = 0, in = 0, out = 0, stash = 0, ws = 0, dw = 0, state = 0, grad = 0, tgt = 0, loss = 0;
+  uint64_t stash2 = 0;  // FWD with pack = 2: the second microbatch's stash
   uint64_t count = 0;  // collectives: elements per rank
   int peer = -1;       // OP_P2P: source rank; peer_off: byte offset in its arena
   uint64_t peer_off = 0;
@@ -56,6 +58,7 @@ struct Op {
 
 struct LayerPlan {
   LayerGeom g;
+  LayerGeom gp;                        // fwd_pack = 2: the same layer on two microbatches (2*b rows)
   int64_t P = 0, Ppad = 0, shard = 0;  // params, padded to N*1024, per-rank shard (elements)
   uint64_t wc_bytes = 0;               // full compute copy on device
   uint64_t state_bytes = 0;            // master|m|v shard (fp32)
@@ -66,6 +69,7 @@ struct LayerPlan {
 
 struct Plan {
   int N = 1, rank = 0, m = 1, b = 1, dtype = 0, stash_policy = 0, schedule = 0, retain_grads = 0;
+  int fwd_pack = 1;
   uint64_t cap = 0;
   int upd_lag = 0;
   std::vector<LayerPlan> layers;   // task layers: a registered layer, or its column panels (operator split)

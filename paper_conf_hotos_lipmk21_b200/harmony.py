@@ -33,7 +33,7 @@ class harmony_config(C.Structure):
                 ("microbatch_size", C.c_int32), ("precision", C.c_int32), ("schedule", C.c_int32),
                 ("retain_grads", C.c_int32), ("stash_policy", C.c_int32), ("lr", C.c_double), ("beta1", C.c_double),
                 ("beta2", C.c_double), ("eps", C.c_double), ("weight_decay", C.c_double), ("nccl_id", C.c_uint8 * 128),
-                ("groups", C.c_int32)]
+                ("groups", C.c_int32), ("fwd_pack", C.c_int32)]
 
 
 class harmony_layer_desc(C.Structure):
@@ -196,7 +196,8 @@ def _check(code, ctx=None):
 # ------------------------------------------------------------------------------- C-ABI wrappers
 def make_config(*, rank=0, world_size=1, device=0, hbm_cap_bytes=0, arena=None, microbatches=1, microbatch_size=1,
                 precision=HARMONY_FP32, schedule=HARMONY_SCHED_HARMONY_DP, retain_grads=0, stash_policy=0, lr=1e-3,
-                beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=0.0, nccl_id=None, groups=1) -> harmony_config:
+                beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=0.0, nccl_id=None, groups=1,
+                fwd_pack=1) -> harmony_config:
     c = harmony_config()
     c.struct_size = C.sizeof(harmony_config)
     c.rank, c.world_size, c.device = rank, world_size, device
@@ -208,6 +209,7 @@ def make_config(*, rank=0, world_size=1, device=0, hbm_cap_bytes=0, arena=None, 
     if nccl_id is not None:
         C.memmove(c.nccl_id, bytes(nccl_id), 128)
     c.groups = groups
+    c.fwd_pack = fwd_pack
     return c
 
 

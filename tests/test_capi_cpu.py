@@ -330,3 +330,23 @@ def test_microbatch_groups_interleave_backward_with_the_next_forward(G):
         assert all(k < upd for k, c in enumerate(comp) if c[0] == "BWD" and c[1] == l)
     with pytest.raises(H.HarmonyError):
         plan(descs, hbm_cap_bytes=0, groups=3, **kw)  # m % G != 0
+
+
+def test_forward_pack_halves_the_forward_tasks_and_keeps_the_traffic():
+    """SURVEY NEXT-4's pack size per pass: fwd_pack = 2 runs each layer's forward on
+    two consecutive microbatches in one task (the backward stays per microbatch).  The plan stays
+    race-free and inside the cap, has half the forward tasks, and moves exactly the same bytes."""
+    c = synth.CONFIGS["cfg2"]
+    kw = dict(microbatches=4, microbatch_size=16, precision=1, hbm_cap_bytes=c["cap"], stash_policy=2)
+    one, ops1 = plan(c["descs"](), **kw)
+    two, ops2 = plan(c["descs"](), fwd_pack=2, **kw)
+    assert two.hazards == 0 and two.arena_bytes <= c["cap"]
+    n1 = sum(o["kind"] == "FWD" for o in ops1)
+    n2 = sum(o["kind"] == "FWD" for o in ops2)
+    assert n1 == 24 * 4 and n2 == n1 // 2
+    assert sum(o["kind"] == "BWD" for o in ops1) == sum(o["kind"] == "BWD" for o in ops2)
+    assert (two.pred_h2d_bytes, two.pred_d2h_bytes) == (one.pred_h2d_bytes, one.pred_d2h_bytes)
+    # outside its domain the pack is refused
+    with pytest.raises(H.HarmonyError) as e:
+        plan(c["descs"](), fwd_pack=2, **dict(kw, stash_policy=0))
+    assert e.value.code == H.HARMONY_E_UNSUPPORTED

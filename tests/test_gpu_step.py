@@ -366,3 +366,25 @@ def test_programmatic_dependent_launch_is_bitwise_plain_stream_order():
     pdl = _step_in_subprocess({}, **shape)
     plain = _step_in_subprocess({"HARMONY_PDL": "0"}, **shape)
     bitwise_equal(pdl, plain)
+
+
+@pytest.mark.parametrize("capped", [False, True])
+def test_forward_pack_is_bitwise_the_per_microbatch_forward(capped):
+    """fwd_pack = 2 (pack size per pass): each layer's forward runs on two consecutive
+    microbatches in one task — GEMMs of 2*b*S rows, attention over 2*b sequences, LayerNorm per row —
+    while the backward stays per microbatch.  Every output element keeps its reduction order, so the
+    step is bit-identical to one forward task per microbatch, with stash spills (capped) or without,
+    and matches the oracle."""
+    descs, params, batches, kw = tiny_transformer(False, 1, L=3, d=128, h=2, S=128, B=8, m=4)
+    kw["stash_policy"] = 2
+    cap = 0
+    if capped:
+        s, _ = H.harmony_plan_dry(H.make_config(hbm_cap_bytes=1 << 40, fwd_pack=2, **kw), descs, text_len=0)
+        cap = int(s.min_working_set_bytes * 1.2)
+    one, plan1 = run_gpu(descs, params, batches, hbm_cap_bytes=cap, **kw)
+    two, plan2 = run_gpu(descs, params, batches, hbm_cap_bytes=cap, fwd_pack=2, **kw)
+    assert plan2["n_ops"] < plan1["n_ops"]
+    if capped:
+        assert two[0]["stats"]["d2h_stash_bytes"] > 0
+    bitwise_equal(one, two)
+    compare(two, run_oracle(descs, params, batches), 2e-2)
