@@ -437,11 +437,15 @@ def main():
         Xt, Tt = torch.tensor(Xt, device=device), torch.tensor(Tt, device=device)
         tcfg = dict(hbm_cap_bytes=wl["cap"], precision=precision, lr=1e-4)
         run = tuner.measure_on_device(descs, params, Xt, Tt, tcfg, steps=3, warmup=2)
-        best, cands = tuner.tune(descs, B, tcfg, lambda mm, G, pol: run(mm, B // mm, groups=G, stash_policy=pol),
+        best, cands = tuner.tune(descs, B, tcfg, lambda mm, G, pol, pk=1: run(mm, B // mm, groups=G, stash_policy=pol,
+                                                                              fwd_pack=pk),
                                  incumbent=(m, args.groups, args.stash_policy if precision else 0), link_gbs=55.0)
         m, args.groups, args.stash_policy = best.microbatches, best.groups, best.stash_policy
-        tuning = {"best": dict(microbatches=m, groups=best.groups, stash_policy=best.stash_policy),
-                  "candidates": [dict(m=c.microbatches, G=c.groups, policy=c.stash_policy, feasible=c.feasible,
+        args.fwd_pack = best.fwd_pack
+        tuning = {"best": dict(microbatches=m, groups=best.groups, stash_policy=best.stash_policy,
+                               fwd_pack=best.fwd_pack),
+                  "candidates": [dict(m=c.microbatches, G=c.groups, policy=c.stash_policy, fwd_pack=c.fwd_pack,
+                                      feasible=c.feasible,
                                       pred_ms=None if c.pred_seconds is None else c.pred_seconds * 1e3,
                                       ms=None if c.step_seconds is None else c.step_seconds * 1e3) for c in cands]}
         del Xt, Tt

@@ -1,5 +1,6 @@
 """Performance tuner (the paper's "memory-performance tango" and task-packing knobs,
-P:749-757, 783-810): microbatch count, microbatch groups (direction balance) and stash policy.
+P:749-757, 783-810): microbatch count, microbatch groups (direction balance), stash policy and the
+forward pack size (microbatches per forward task).
 
 The same global batch per GPU can be run as m microbatches of b = batch / m sequences.  Larger
 microbatches amortise every kernel's launch and tail cost; a wider microbatch also widens the
@@ -77,13 +78,14 @@ class Candidate:
     microbatches: int
     groups: int
     stash_policy: int
+    fwd_pack: int = 1                   # microbatches per forward task (the backward's pack is 1)
     feasible: bool = True
     reason: str = ""
     pred_seconds: float | None = None   # cost model (host-only plan + link / tensor rates)
     step_seconds: float | None = None   # measured (top candidates only)
 
     def key(self):
-        return (self.microbatches, self.groups, self.stash_policy)
+        return (self.microbatches, self.groups, self.stash_policy, self.fwd_pack)
 
 
 # executed GEMM FLOPs per algorithmic FLOP: block recompute re-runs the forward (without its last
@@ -102,13 +104,15 @@ def predict_seconds(summary, policy, groups, tflops=1000.0, link_gbs=55.0):
 
 
 def tune(descs, batch: int, cfg: dict, measure, ms=None, groups=(1, 2, 4), policies=(0, 2, 3), top=4,
-         per_policy=2, incumbent=None, **model) -> "tuple[Candidate, list]":
+         per_policy=2, incumbent=None, packs=(1, 2), **model) -> "tuple[Candidate, list]":
     """The memory-performance tango: over microbatch count m, microbatch groups G and stash
     policy, the planner says what fits the cap, a cost model ranks what fits, and the best-ranked are
     measured (`measure(m, G, policy)` -> seconds per step); the fastest measured wins.  The model only
     ranks (it knows GEMM work and host traffic, not kernel efficiency), so the measured set takes at
     most `per_policy` candidates of each stash policy (up to `top` in all) plus the `incumbent`
-    (m, G, policy) when given.  The fp32 path has no recompute policies (0 only)."""
+    (m, G, policy) when given.  The fp32 path has no recompute policies (0 only).  Forward packs of 2
+    (where the planner accepts them) move the same bytes and FLOPs, so the model cannot rank them:
+    each measured candidate's pack-2 twin is measured beside it.  `measure(m, G, policy, pack)`."""
     if cfg.get("precision", 0) == 0:
         policies = (0,)
     cands = []
@@ -117,30 +121,37 @@ def tune(descs, batch: int, cfg: dict, measure, ms=None, groups=(1, 2, 4), polic
             if m % G:
                 continue
             for pol in policies:
-                c = Candidate(m, G, pol)
-                try:
-                    s, _ = H.harmony_plan_dry(H.make_config(microbatches=m, microbatch_size=batch // m, groups=G,
-                                                            stash_policy=pol, **cfg), descs, text_len=0)
-                    c.pred_seconds = predict_seconds(s, pol, G, **model)
-                except H.HarmonyError as e:
-                    c.feasible, c.reason = False, str(e)
-                cands.append(c)
-    ok = sorted((c for c in cands if c.feasible), key=lambda c: (c.pred_seconds, c.groups))
+                for pack in packs:
+                    c = Candidate(m, G, pol, pack)
+                    try:
+                        s, _ = H.harmony_plan_dry(H.make_config(microbatches=m, microbatch_size=batch // m, groups=G,
+                                                                stash_policy=pol, fwd_pack=pack, **cfg), descs,
+                                                  text_len=0)
+                        c.pred_seconds = predict_seconds(s, pol, G, **model)
+                    except H.HarmonyError as e:
+                        c.feasible, c.reason = False, str(e)
+                        if pack > 1:
+                            continue  # outside the pack's domain: not a candidate
+                    cands.append(c)
+    ok = sorted((c for c in cands if c.feasible), key=lambda c: (c.pred_seconds, c.groups, c.fwd_pack))
     if not ok:
         raise H.HarmonyError(H.HARMONY_E_CAP_TOO_SMALL, "no (microbatches, groups, policy) fits the cap")
     chosen, taken = [], {}
     for c in ok:
         if len(chosen) >= top:
             break
-        if taken.get(c.stash_policy, 0) < per_policy:
+        if c.fwd_pack == 1 and taken.get(c.stash_policy, 0) < per_policy:
             chosen.append(c)
             taken[c.stash_policy] = taken.get(c.stash_policy, 0) + 1
     if incumbent is not None:
-        inc = next((c for c in ok if c.key() == tuple(incumbent)), None)
+        inc_key = tuple(incumbent) + ((1,) if len(incumbent) == 3 else ())
+        inc = next((c for c in ok if c.key() == inc_key), None)
         if inc is not None and inc not in chosen:
             chosen.append(inc)
-    for c in chosen:
-        c.step_seconds = float(measure(c.microbatches, c.groups, c.stash_policy))
+    twins = [t for c in chosen for t in ok
+             if t.fwd_pack > 1 and t.key()[:3] == c.key()[:3] and t not in chosen]
+    for c in chosen + twins:
+        c.step_seconds = float(measure(c.microbatches, c.groups, c.stash_policy, c.fwd_pack))
     best = min((c for c in ok if c.step_seconds is not None), key=lambda c: (c.step_seconds, c.groups))
     return best, cands
 

@@ -46,8 +46,10 @@ def test_tuner_breaks_ties_toward_larger_microbatches_and_raises_when_nothing_fi
 
 
 def test_tango_ranks_by_the_cost_model_and_measures_only_the_top():
-    """(m, G, policy): infeasible points are recorded, the feasible ones ranked by the plan-implied
-    time (GEMM work vs host traffic with direction balance), only the top few are measured."""
+    """(m, G, policy, forward pack): infeasible points are recorded, the feasible ones ranked by the
+    plan-implied time (GEMM work vs host traffic with direction balance), only the top few are
+    measured — plus, for each, its forward-pack-2 twin where the planner accepts one (same bytes and
+    FLOPs: the model cannot rank it, so it is measured beside it)."""
     descs = synth.transformer_stack(4, 128, 2, 128, True)
     cfg = dict(precision=1)
     s, _ = H.harmony_plan_dry(H.make_config(microbatches=4, microbatch_size=2, stash_policy=2,
@@ -55,21 +57,25 @@ def test_tango_ranks_by_the_cost_model_and_measures_only_the_top():
     cap = int(s.min_working_set_bytes * 1.6)
     seen = []
 
-    def measure(m, G, pol):
-        seen.append((m, G, pol))
-        return 1.0 / m + 0.01 * G + 0.001 * pol
+    def measure(m, G, pol, pack):
+        seen.append((m, G, pol, pack))
+        return 1.0 / m + 0.01 * G + 0.001 * pol - 0.0001 * pack
 
     best, cands = tuner.tune(descs, 8, dict(cfg, hbm_cap_bytes=cap), measure, top=3, per_policy=1,
                              incumbent=(2, 1, 2))
     feas = [c for c in cands if c.feasible]
-    assert best.key() in seen and (2, 1, 2) in seen  # the incumbent is always measured
-    pols = [k[2] for k in seen if k != (2, 1, 2)]
+    inc = (2, 1, 2, 1)
+    assert best.key() in seen and inc in seen  # the incumbent is always measured
+    singles = [k for k in seen if k[3] == 1 and k != inc]
+    pols = [k[2] for k in singles]
     assert len(pols) == len(set(pols)) <= 3  # at most one per stash policy (per_policy=1)
-    for k in seen:  # each measured non-incumbent candidate is its policy's best prediction
-        if k == (2, 1, 2):
-            continue
+    for k in singles:  # each measured non-incumbent candidate is its policy's best prediction
         c = next(c for c in feas if c.key() == k)
         assert c.pred_seconds == min(x.pred_seconds for x in feas if x.stash_policy == k[2])
+    for k in seen:  # pack-2 twins: only for block recompute (the pack's domain), beside their pack-1 point
+        if k[3] == 2:
+            assert k[2] == 2 and k[:3] + (1,) in seen
+    assert any(k[3] == 2 for k in seen)
     assert all(c.pred_seconds > 0 for c in feas)
     # more groups overlap the two host-link directions: never a worse prediction for the same plan bytes
     s0, _ = H.harmony_plan_dry(H.make_config(microbatches=4, microbatch_size=2, stash_policy=0, hbm_cap_bytes=cap,
