@@ -534,12 +534,11 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     gemm(a, st);
   }
   }
-  // ---- QKV projection: dU = dQKV W_qkv^T; dW_qkv += U^T dQKV; db_qkv += sum dQKV
-  {
-    hk_gemm_args a = lin_dgrad(g, R, 3 * D, D, dQKV, wseg(g, W, P_WQKV));
-    a.C = dUf; a.epilogue = HK_EPI_STORE_F32;
-    gemm(a, st);
-  }
+  // ---- QKV projection: dU = dQKV W_qkv^T; dW_qkv += U^T dQKV; db_qkv += sum dQKV.  The weight
+  // gradient (and db) go to the side stream FIRST: both products only read dQKV, and with the data
+  // gradient and the LN1 backward after the fork this stream has ~150 us of work beside the weight
+  // gradient's ~150 instead of ~70 — the task's closing join no longer idles this stream (measured:
+  // ~125 us per task, profiles/r02_kernel_timeline_join.txt)
   const uint8_t* U = stash + g.st.U;
   if (g.stash_policy == 1) {
     float* tmp_mean = reinterpret_cast<float*>(scratch);
@@ -547,9 +546,20 @@ static void bwd_core(const LayerGeom& g, const void* W, const uint8_t* stash, co
     layernorm_fwd(dt, R, D, Xs, wseg(g, W, P_LN1_G), wseg(g, W, P_LN1_B), rec, tmp_mean, tmp_rstd, st);
     U = rec;
   }
+  static const bool wgrad_first = [] {  // HARMONY_QKV_WGRAD_FIRST=0: the dgrad first (A/B)
+    const char* e = getenv("HARMONY_QKV_WGRAD_FIRST");
+    return !(e && *e == '0');
+  }();
+  auto qkv_dgrad = [&]() {
+    hk_gemm_args a = lin_dgrad(g, R, 3 * D, D, dQKV, wseg(g, W, P_WQKV));
+    a.C = dUf; a.epilogue = HK_EPI_STORE_F32;
+    gemm(a, st);
+  };
+  if (!wgrad_first) qkv_dgrad();
   fork(2);
   gemm(lin_wgrad(g, R, 3 * D, D, U, dQKV, gseg(g, dW, P_WQKV), first), sw);
   colsum(dt, R, 3 * D, dQKV, 3 * D, gseg(g, dW, P_BQKV), acc, wscratch, sw);
+  if (wgrad_first) qkv_dgrad();
   // ---- LN1 backward: dX = dX2 + LN1'(dU)
   layernorm_bwd(dt, R, D, dUf, Xs, mean1, rstd1, wseg(g, W, P_LN1_G), dX2, dX, gseg(g, dW, P_LN1_G),
                 gseg(g, dW, P_LN1_B), acc, scratch, st);
