@@ -373,12 +373,17 @@ def main():
                     help="m per GPU (0 = the workload's default); the microbatch size is per_gpu_batch / m")
     ap.add_argument("--groups", type=int, default=1,
                     help="G microbatch groups (direction balance: group g's backward interleaved with g+1's forward)")
+    ap.add_argument("--cap-gib", type=float, default=0,
+                    help="override the workload's per-GPU HBM cap (GiB; A/B runs, reported in config)")
     ap.add_argument("--fwd-pack", type=int, default=1,
                     help="forward pack size (2: each layer's forward on two microbatches at once; NEXT-4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
-    wl = WORKLOADS[args.workload]
+    wl = dict(WORKLOADS[args.workload])
+    if args.cap_gib:
+        wl["cap"] = int(args.cap_gib * (1 << 30))
+        wl["name"] = wl["name"] + f" [cap overridden: {args.cap_gib:g} GiB]"
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         # one process per GPU: launch this script under torchrun with args.gpus ranks
         import socket
