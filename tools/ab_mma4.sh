@@ -1,3 +1,4 @@
+# round 1: kernel tests + GEMM set after the four-UMMA issue change
 timeout 600 python -m pytest tests/test_gpu_kernels.py -m gpu -x -q > gpurun_out/t_kernels.log 2>&1; echo "kernel tests $?"; tail -2 gpurun_out/t_kernels.log
 timeout 300 python tools/gemm_bench.py --reps 20 --graph > gpurun_out/gb_mma4.jsonl 2>&1
 python -c "

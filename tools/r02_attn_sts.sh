@@ -1,3 +1,4 @@
+# attention forward with the row-max exchange in shared state space (A/B)
 mkdir -p gpurun_out
 python -m paper_conf_hotos_lipmk21_b200.build > gpurun_out/build.log 2>&1; echo "build $?"
 timeout 600 python -m pytest tests/test_gpu_kernels.py -m gpu -x -q -p no:cacheprovider -k "fused_attention" 2>&1 | tail -1

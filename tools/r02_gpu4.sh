@@ -1,3 +1,4 @@
+# Harmony-PP, step and group test suites
 mkdir -p gpurun_out
 python -m paper_conf_hotos_lipmk21_b200.build > gpurun_out/build.log 2>&1
 timeout 900 python -m pytest tests/test_gpu_pp.py -m gpu -x -q -s > gpurun_out/t_pp.log 2>&1; echo "pp tests $?"; tail -6 gpurun_out/t_pp.log

@@ -1,3 +1,4 @@
+# step, group and PP tests plus a short cfg2 bench
 mkdir -p gpurun_out
 python -m paper_conf_hotos_lipmk21_b200.build > gpurun_out/build.log 2>&1
 timeout 900 python -m pytest tests/test_gpu_step.py tests/test_gpu_group.py tests/test_gpu_pp.py -m gpu -x -q > gpurun_out/t_step.log 2>&1; echo "tests $?"; tail -2 gpurun_out/t_step.log

@@ -1,3 +1,4 @@
+# GEMM epilogue through LSU stores vs TMA stores (HARMONY_GEMM_DIAG=16)
 timeout 300 python tools/gemm_bench.py --graph --reps 20 > gpurun_out/gb_r02_tma.jsonl 2>&1
 HARMONY_GEMM_DIAG=16 timeout 300 python tools/gemm_bench.py --graph --reps 20 > gpurun_out/gb_r02_lsu.jsonl 2>&1
 timeout 300 python tools/gemm_bench.py --sweep --graph --reps 20 > gpurun_out/sw_r02_tma.jsonl 2>&1

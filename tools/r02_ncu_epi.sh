@@ -1,3 +1,4 @@
+# ncu --set full of the specialised FC1-forward / FC2-dgrad GEMM kernels
 mkdir -p gpurun_out
 python -m paper_conf_hotos_lipmk21_b200.build > gpurun_out/build.log 2>&1; echo "build $?"
 for k in fc1_fwd fc2_dgrad; do
