@@ -1093,6 +1093,7 @@ GroupPlan make_plan_pp(const harmony_config& cfg, int N, int L, const harmony_la
   // per-rank layout: the rank's layers as one stack of one rank (the update is not sharded: each layer
   // lives on one GPU), four activation buffers (A_in, A_out, G_in, G_out)
   HM_CHECK(cfg.groups <= 1, HARMONY_E_UNSUPPORTED, "microbatch groups are a Harmony-DP schedule");
+  HM_CHECK(cfg.fwd_pack <= 1, HARMONY_E_UNSUPPORTED, "forward packs are a Harmony-DP schedule");
   harmony_config rc = cfg;
   rc.world_size = 1; rc.rank = 0; rc.schedule = HARMONY_SCHED_HARMONY_DP; rc.groups = 1;
   for (int r = 0; r < N; ++r) {
