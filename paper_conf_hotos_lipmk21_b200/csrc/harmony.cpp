@@ -266,18 +266,26 @@ PtrKind ptr_kind(const void* p) {
   return PTR_PAGEABLE;
 }
 
-// Host copy on a few threads (pageable -> pinned staging of the step's inputs).
-void parallel_memcpy(void* dst, const void* src, size_t n) {
+// Host copy on the host's cores (pageable -> pinned staging of the step's inputs): every buffer of
+// the step cut into 16 MB pieces, the pieces dealt round-robin to min(cores, 16) threads.
+void parallel_memcpy_multi(void* const* dst, const void* const* src, const size_t* n, int count) {
   const size_t chunk = 16u << 20;
-  const int nt = (int)std::min<size_t>(8, (n + chunk - 1) / chunk);
-  if (nt <= 1) { memcpy(dst, src, n); return; }
-  std::vector<std::thread> th;
-  const size_t per = (n + nt - 1) / nt;
-  for (int i = 0; i < nt; ++i) {
-    const size_t lo = (size_t)i * per, hi = std::min(n, lo + per);
-    if (lo >= hi) break;
-    th.emplace_back([=] { memcpy(static_cast<char*>(dst) + lo, static_cast<const char*>(src) + lo, hi - lo); });
+  struct Piece { char* d; const char* s; size_t n; };
+  std::vector<Piece> pieces;
+  for (int b = 0; b < count; ++b)
+    for (size_t lo = 0; lo < n[b]; lo += chunk)
+      pieces.push_back({static_cast<char*>(dst[b]) + lo, static_cast<const char*>(src[b]) + lo, std::min(chunk, n[b] - lo)});
+  const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+  const int nt = (int)std::min<size_t>(std::min(16u, hw), pieces.size());
+  if (nt <= 1) {
+    for (const Piece& q : pieces) memcpy(q.d, q.s, q.n);
+    return;
   }
+  std::vector<std::thread> th;
+  for (int i = 0; i < nt; ++i)
+    th.emplace_back([&, i] {
+      for (size_t k = (size_t)i; k < pieces.size(); k += (size_t)nt) memcpy(pieces[k].d, pieces[k].s, pieces[k].n);
+    });
   for (auto& t : th) t.join();
 }
 
@@ -663,6 +671,10 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
     const float* src[2] = {x, tg};
     PtrKind* kinds[2] = {&xk, &tk};
     bool staged[2] = {false, false};
+    void* cd[2];
+    const void* cs[2];
+    size_t cn[2];
+    int nc = 0;
     for (int q = 0; q < 2 && stage; ++q) {
       if (*kinds[q] != PTR_PAGEABLE) continue;
       staged[q] = true;
@@ -672,9 +684,10 @@ void run_step(harmony_ctx* c, const float* x, const float* tg, double* loss_out,
         c->h_stage[q] = static_cast<uint8_t*>(alloc_host(nb[q]));
         c->h_stage_bytes[q] = nb[q];
       }
-      parallel_memcpy(c->h_stage[q], src[q], nb[q]);
+      cd[nc] = c->h_stage[q]; cs[nc] = src[q]; cn[nc] = nb[q]; ++nc;
       *kinds[q] = PTR_PINNED;
     }
+    if (nc) parallel_memcpy_multi(cd, cs, cn, nc);  // X and T together
     if (staged[0]) x = reinterpret_cast<const float*>(c->h_stage[0]);
     if (staged[1]) tg = reinterpret_cast<const float*>(c->h_stage[1]);
   }
